@@ -1,0 +1,124 @@
+"""Seeded synthetic workloads (numpy only).  Shared by tests, bench and smoke.
+
+Holds none of the method's arithmetic: it only draws inputs with the shapes and value
+structure of the paper's workloads (DESIGN.md §4 "input recipe"):
+
+* X: N(0, 1) activations, cast to float16 (bfloat16 bit patterns on request).
+* tags: n8 = round(f * nb) INT8 ("outlier") blocks (at least 1 if f > 0) at seeded random
+  block positions -- after COMET's channel permutation the outlier channels sit in a few
+  128-channel blocks; FMPQ leaves < 20 % of blocks INT8, ~16 % on
+  average and 8 % on LLaMA-1-30B.
+* outliers: in every INT8 block, 4 seeded channels are scaled by U(20, 100): outliers are
+  "< 1 %" of features with magnitudes "tenfold or even a hundredfold" the rest,
+  concentrated in specific channels (Fig. 3).
+* W: 4-bit weight codes uniform in [-8, 7] (stand-in for OmniQuant W4) and
+  per-output-channel scales s_w = U(0.5, 1.5) / (8 sqrt(K)) so outputs are O(1).
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass
+
+import numpy as np
+
+BLOCK = 128
+
+
+@dataclass(frozen=True)
+class Layer:
+    name: str
+    K: int   # input channels
+    N: int   # output channels
+
+
+# LLaMA linear-layer shapes named in BASELINE.json configs.
+LLAMA2_7B = (Layer("qkvo", 4096, 4096), Layer("gate_up", 4096, 11008), Layer("down", 11008, 4096))
+LLAMA3_8B = (Layer("up", 4096, 14336), Layer("down", 14336, 4096))
+LLAMA3_70B = (Layer("gate_up", 8192, 28672), Layer("down", 28672, 8192), Layer("qkv", 8192, 10240))
+
+
+def bf16_bits_from_f32(a: np.ndarray) -> np.ndarray:
+    """Round float32 -> bfloat16 (round-half-even) and return the uint16 bit patterns."""
+    u = np.ascontiguousarray(a, dtype=np.float32).view(np.uint32).astype(np.uint64)
+    lsb = (u >> 16) & 1
+    r = ((u + 0x7FFF + lsb) >> 16).astype(np.uint16)
+    return r
+
+
+def bf16_bits_to_f32(b: np.ndarray) -> np.ndarray:
+    return (np.ascontiguousarray(b, dtype=np.uint16).astype(np.uint32) << 16).view(np.float32)
+
+
+def make_tags(K: int, frac: float, rng: np.random.Generator, n8: int | None = None) -> np.ndarray:
+    nb = K // BLOCK
+    if n8 is None:
+        n8 = int(round(frac * nb))
+        if frac > 0 and n8 == 0:
+            n8 = 1
+    tags = np.zeros(nb, dtype=np.uint8)
+    if n8 > 0:
+        tags[rng.choice(nb, size=n8, replace=False)] = 1
+    return tags
+
+
+def make_activations(M: int, K: int, tags: np.ndarray, rng: np.random.Generator,
+                     *, bf16: bool = False, outliers_per_block: int = 4,
+                     lo: float = 20.0, hi: float = 100.0):
+    """X[M, K] ~ N(0,1) with `outliers_per_block` boosted channels in every INT8 block.
+    Returns float16 array, or uint16 bf16 bit patterns when bf16=True."""
+    x = rng.standard_normal((M, K), dtype=np.float32)
+    for b in np.nonzero(tags)[0]:
+        ch = b * BLOCK + rng.choice(BLOCK, size=outliers_per_block, replace=False)
+        x[:, ch] *= rng.uniform(lo, hi, size=outliers_per_block).astype(np.float32)
+    if bf16:
+        return bf16_bits_from_f32(x)
+    return x.astype(np.float16)
+
+
+def make_weights(N: int, K: int, rng: np.random.Generator):
+    """INT4 codes in [-8, 7] and per-output-channel scales."""
+    w = rng.integers(-8, 8, size=(N, K), dtype=np.int8)
+    s_w = (rng.uniform(0.5, 1.5, size=N) / (8.0 * np.sqrt(K))).astype(np.float32)
+    return w, s_w
+
+
+@dataclass
+class Problem:
+    x: np.ndarray        # [M,K] float16 (or uint16 bf16 bits if bf16)
+    tags: np.ndarray     # [K/128] uint8
+    w: np.ndarray        # [N,K] int8 codes in [-8,7]
+    s_w: np.ndarray      # [N] float32
+    bf16: bool = False
+
+    @property
+    def M(self): return self.x.shape[0]
+
+    @property
+    def K(self): return self.x.shape[1]
+
+    @property
+    def N(self): return self.w.shape[0]
+
+
+def make_problem(M: int, K: int, N: int, *, frac: float = 0.05, seed: int = 0,
+                 bf16: bool = False, n8: int | None = None) -> Problem:
+    rng = np.random.default_rng(seed)
+    tags = make_tags(K, frac, rng, n8=n8)
+    x = make_activations(M, K, tags, rng, bf16=bf16)
+    w, s_w = make_weights(N, K, rng)
+    return Problem(x=x, tags=tags, w=w, s_w=s_w, bf16=bf16)
+
+
+def config1(seed: int = 1) -> Problem:
+    """BASELINE config 1: single linear M=16 K=256 N=256, 2 blocks, 1 INT8 outlier block."""
+    return make_problem(16, 256, 256, seed=seed, n8=1)
+
+
+def sample_rows(M: int, n: int, x: np.ndarray, seed: int = 7) -> np.ndarray:
+    """Seeded sample of token rows that always contains the row holding max |x|."""
+    rng = np.random.default_rng(seed)
+    xf = x.astype(np.float32) if x.dtype == np.float16 else bf16_bits_to_f32(x)
+    top = int(np.unravel_index(np.argmax(np.abs(xf)), xf.shape)[0])
+    rows = set([top, 0, M - 1])
+    while len(rows) < min(n, M):
+        rows.add(int(rng.integers(0, M)))
+    return np.array(sorted(rows), dtype=np.int64)

@@ -1,0 +1,270 @@
+"""Pins for the CPU oracle (no GPU): the oracle is checked against things other than itself --
+brute force with exact rationals, library routines (numpy int64 / float64 matmul),
+closed forms, invariants and the paper's worked example -- chosen so that a plausible slip
+(dropped term, wrong qmax, floor instead of rint, swapped operand, wrong scale) fails one.
+"""
+from fractions import Fraction
+import json
+import os
+import struct
+
+import numpy as np
+import pytest
+
+import oracle
+from oracle import planner
+from paper_conf_asplos_liu0rxpwl0w25_b200 import synth
+
+BLOCK = 128
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+
+
+# ---------- exact helpers (independent of the oracle) -----------------------------------
+
+def f32_round(fr: Fraction) -> Fraction:
+    """Round an exact rational to the nearest binary32 (ties to even), exactly."""
+    if fr == 0:
+        return Fraction(0)
+    sign = -1 if fr < 0 else 1
+    a = abs(fr)
+    e = a.numerator.bit_length() - a.denominator.bit_length()
+    # find e with 2^e <= a < 2^(e+1)
+    while Fraction(2) ** e > a:
+        e -= 1
+    while Fraction(2) ** (e + 1) <= a:
+        e += 1
+    e = max(e, -126)                      # subnormal range shares the 2^-149 quantum
+    quantum = Fraction(2) ** (e - 23)
+    n = a / quantum
+    fl = n.numerator // n.denominator
+    rem = n - fl
+    if rem > Fraction(1, 2) or (rem == Fraction(1, 2) and fl % 2 == 1):
+        fl += 1
+    return sign * fl * quantum
+
+
+def test_f32_round_helper_matches_struct():
+    rng = np.random.default_rng(0)
+    for v in rng.standard_normal(200) * 1e3:
+        want = struct.unpack("f", struct.pack("f", float(v)))[0]
+        assert f32_round(Fraction(float(v))) == Fraction(want)
+
+
+def brute_quantize_block(xs, qmax):
+    """FMPQ quantisation of one block from the paper's description, in exact rationals with
+    explicit binary32 rounding of s, r and every product (reading R1-R5)."""
+    amax = max(abs(Fraction(float(v))) for v in xs)
+    if amax == 0:
+        return [0] * len(xs), Fraction(0)
+    s = f32_round(amax / qmax)
+    r = f32_round(Fraction(qmax) / amax)
+    codes = []
+    for v in xs:
+        t = f32_round(Fraction(float(v)) * r)
+        q = round(t)                 # Fraction.__round__ = round half to even
+        codes.append(max(-qmax, min(qmax, q)))
+    return codes, s
+
+
+# ---------- quantisation pins --------------------------------------------------------------
+
+def test_quantize_brute_force_config1():
+    p = synth.config1()
+    codes, scales = oracle.quantize(p.x, p.tags)
+    for m in range(p.M):
+        for b in range(p.K // BLOCK):
+            qmax = 127 if p.tags[b] else 7
+            xs = p.x[m, b * BLOCK:(b + 1) * BLOCK]
+            want_codes, want_s = brute_quantize_block(xs, qmax)
+            assert list(codes[m, b * BLOCK:(b + 1) * BLOCK]) == want_codes
+            assert Fraction(float(scales[m, b])) == want_s
+
+
+def test_quantize_roundtrip_error_bound_I2():
+    """|x - s q| <= s/2 (1 + 2^-20): min-max symmetric rounding never errs more than half a step."""
+    p = synth.make_problem(64, 1024, 128, frac=0.25, seed=3)
+    codes, scales = oracle.quantize(p.x, p.tags)
+    x = p.x.astype(np.float64).reshape(64, 8, BLOCK)
+    s = scales.astype(np.float64)[:, :, None]
+    err = np.abs(x - s * codes.reshape(64, 8, BLOCK))
+    assert np.all(err <= s / 2 * (1 + 2.0 ** -20))
+
+
+def test_quantize_maxabs_gets_qmax_I3_and_ranges():
+    p = synth.make_problem(32, 1024, 128, frac=0.25, seed=4)
+    codes, scales = oracle.quantize(p.x, p.tags)
+    xb = p.x.astype(np.float32).reshape(32, 8, BLOCK)
+    cb = codes.reshape(32, 8, BLOCK).astype(np.int32)
+    for b in range(8):
+        qmax = 127 if p.tags[b] else 7
+        assert np.abs(cb[:, b]).max() == qmax
+        idx = np.argmax(np.abs(xb[:, b]), axis=1)
+        top = cb[np.arange(32), b, idx]
+        assert np.all(np.abs(top) == qmax)
+        assert np.all(np.sign(top) == np.sign(xb[np.arange(32), b, idx]))
+    assert p.tags.sum() >= 1 and (p.tags == 0).sum() >= 1
+
+
+def test_quantize_round_half_even_special_case():
+    """amax = 7 on an INT4 block gives r = 1, s = 1: codes are rint(x) -> ties go to even."""
+    x = np.zeros((1, BLOCK), np.float16)
+    x[0, :6] = [7.0, 2.5, 3.5, -2.5, -0.5, 1.5]
+    codes, scales = oracle.quantize(x, np.array([0], np.uint8))
+    assert scales[0, 0] == 1.0
+    assert list(codes[0, :6]) == [7, 2, 4, -2, 0, 2]
+
+
+def test_quantize_odd_symmetry_and_power_of_two_I5():
+    p = synth.make_problem(16, 512, 128, frac=0.5, seed=5)
+    c0, s0 = oracle.quantize(p.x, p.tags)
+    c1, s1 = oracle.quantize(-p.x, p.tags)
+    assert np.array_equal(c1, -c0) and np.array_equal(s1, s0)
+    c2, s2 = oracle.quantize((p.x.astype(np.float32) * 0.25).astype(np.float16), p.tags)
+    # x/4 is exact in fp16 here (no underflow for N(0,1) data at this size) -> same codes
+    assert np.array_equal(c2, c0)
+    assert np.array_equal(s2, s0 * np.float32(0.25))
+
+
+def test_quantize_zero_block_I6_and_bf16_subnormal():
+    x = np.zeros((2, 256), np.float16)
+    x[1, 128:] = 1.0
+    codes, scales = oracle.quantize(x, np.array([0, 1], np.uint8))
+    assert np.all(codes[0] == 0) and np.all(scales[0] == 0)
+    assert np.all(codes[1, :128] == 0) and scales[1, 0] == 0
+    assert np.all(codes[1, 128:] == 127)
+    # bf16 binary32-subnormal block: r overflows to inf; zeros -> 0, nonzeros -> +-qmax
+    xb = np.zeros((1, 128), np.uint16)
+    xb[0, 0] = 0x0001   # 2^-133 (subnormal)
+    xb[0, 1] = 0x8001
+    c, s = oracle.quantize(xb, np.array([0], np.uint8), bf16_bits=True)
+    assert c[0, 0] == 7 and c[0, 1] == -7 and np.all(c[0, 2:] == 0)
+
+
+def test_quantize_bf16_matches_brute_force():
+    p = synth.make_problem(4, 256, 16, seed=11, bf16=True, n8=1)
+    codes, scales = oracle.quantize(p.x, p.tags, bf16_bits=True)
+    xf = synth.bf16_bits_to_f32(p.x)
+    for m in range(4):
+        for b in range(2):
+            want_c, want_s = brute_quantize_block(xf[m, b * BLOCK:(b + 1) * BLOCK],
+                                                  127 if p.tags[b] else 7)
+            assert list(codes[m, b * BLOCK:(b + 1) * BLOCK]) == want_c
+            assert Fraction(float(scales[m, b])) == want_s
+
+
+# ---------- integer GEMM pins --------------------------------------------------------------
+
+def test_gemm_blocks_sum_equals_numpy_int64_matmul_I8():
+    rng = np.random.default_rng(9)
+    q = rng.integers(-127, 128, size=(24, 640), dtype=np.int8)
+    w = rng.integers(-8, 8, size=(40, 640), dtype=np.int8)
+    acc = oracle.gemm_blocks(q, w)
+    assert acc.shape == (5, 24, 40)
+    ref = q.astype(np.int64) @ w.astype(np.int64).T
+    assert np.array_equal(acc.sum(0), ref)
+    for b in range(5):  # I1: every block is a plain INT8 GEMM of that block
+        sl = slice(b * BLOCK, (b + 1) * BLOCK)
+        assert np.array_equal(acc[b], q[:, sl].astype(np.int64) @ w[:, sl].astype(np.int64).T)
+
+
+def test_gemm_python_bigint_brute_force_config1():
+    p = synth.config1()
+    codes, _ = oracle.quantize(p.x, p.tags)
+    acc = oracle.gemm_blocks(codes, p.w)
+    rng = np.random.default_rng(2)
+    for _ in range(64):
+        m, n, b = int(rng.integers(16)), int(rng.integers(256)), int(rng.integers(2))
+        want = sum(int(codes[m, k]) * int(p.w[n, k]) for k in range(b * BLOCK, (b + 1) * BLOCK))
+        assert acc[b, m, n] == want
+
+
+def test_gemm_extreme_values_fit_int32():
+    q = np.full((1, BLOCK), -127, np.int8)
+    w = np.full((1, BLOCK), -8, np.int8)
+    acc = oracle.gemm_blocks(q, w)
+    assert acc[0, 0, 0] == 127 * 8 * BLOCK
+
+
+def test_gemm_rows_subset():
+    rng = np.random.default_rng(10)
+    q = rng.integers(-7, 8, size=(10, 256), dtype=np.int8)
+    w = rng.integers(-8, 8, size=(16, 256), dtype=np.int8)
+    full = oracle.gemm_blocks(q, w)
+    sub = oracle.gemm_blocks(q, w, rows=np.array([7, 2]))
+    assert np.array_equal(sub[:, 0], full[:, 7]) and np.array_equal(sub[:, 1], full[:, 2])
+
+
+# ---------- dequantisation pins ------------------------------------------------------------
+
+def test_dequant_closed_form_I4():
+    """y = (s_a q) (s_w w)^T by distributivity: compare with a numpy float64 matmul of the
+    dequantised operands (a library routine), relative 1e-12."""
+    p = synth.make_problem(32, 768, 96, frac=0.34, seed=12)
+    y, acc, codes, scales = oracle.w4ax(p.x, p.tags, p.w, p.s_w)
+    xd = codes.astype(np.float64) * np.repeat(scales.astype(np.float64), BLOCK, axis=1)
+    wd = p.w.astype(np.float64) * p.s_w.astype(np.float64)[:, None]
+    ref = xd @ wd.T
+    assert np.allclose(y, ref, rtol=1e-12, atol=1e-12 * np.abs(ref).max())
+
+
+def test_dequant_exact_rational_config1():
+    p = synth.config1()
+    y, acc, codes, scales = oracle.w4ax(p.x, p.tags, p.w, p.s_w)
+    for (m, n) in [(0, 0), (3, 17), (15, 255), (8, 128)]:
+        exact = Fraction(float(p.s_w[n])) * sum(
+            Fraction(float(scales[m, b])) * int(acc[b, m, n]) for b in range(2))
+        assert abs(Fraction(float(y[m, n])) - exact) <= abs(exact) * Fraction(1, 2 ** 50)
+
+
+def test_dequant_within_quantisation_error_bound():
+    """|y - x (s_w w)^T| <= sum_k |s_w w_k| s_a/2 (1+2^-20): the paper's min-max quantiser
+    bounds the GEMM error by half a step per activation element."""
+    p = synth.make_problem(16, 512, 64, frac=0.25, seed=13)
+    y, acc, codes, scales = oracle.w4ax(p.x, p.tags, p.w, p.s_w)
+    wd = p.w.astype(np.float64) * p.s_w.astype(np.float64)[:, None]
+    exact = p.x.astype(np.float64) @ wd.T
+    half_step = np.repeat(scales.astype(np.float64), BLOCK, axis=1) / 2 * (1 + 2.0 ** -20)
+    bound = half_step @ np.abs(wd).T
+    assert np.all(np.abs(y - exact) <= bound + 1e-12)
+
+
+def test_w4ax_rows_matches_full_path():
+    p = synth.make_problem(20, 384, 48, frac=0.34, seed=14)
+    y, acc, codes, scales = oracle.w4ax(p.x, p.tags, p.w, p.s_w)
+    rows = np.array([0, 5, 19])
+    y2, s2, c2, sc2 = oracle.w4ax_rows(p.x, p.tags, p.w, p.s_w, rows)
+    assert np.array_equal(y2, y[rows])
+    assert np.array_equal(s2, acc.sum(0)[rows])
+    assert np.array_equal(c2, codes[rows]) and np.array_equal(sc2, scales[rows])
+
+
+# ---------- planner (Fig. 8) pins -----------------------------------------------------------
+
+def _fig8():
+    with open(os.path.join(GOLDEN, "fig8_schedule.json")) as f:
+        return json.load(f)
+
+
+def test_fig8_naive_and_barrier_minimised():
+    g = _fig8()
+    tags, nb = g["tags"], len(g["tags"])
+    n_units = g["n_output_tiles"] * nb
+    cost = lambda u: planner.unit_cost(tags, u % nb, g["cost_int4"], g["cost_int8"])
+    assert planner.makespan_naive_barrier(n_units, g["n_sm"], cost) == Fraction(g["expected"]["naive_barrier_per_iteration"])
+    assert planner.makespan_round_robin(n_units, g["n_sm"], cost) == Fraction(g["expected"]["barrier_minimised_round_robin"])
+
+
+def test_fig8_remap_and_decomposition_bounds():
+    g = _fig8()
+    tags = g["tags"]
+    lb = planner.lower_bound(g["n_output_tiles"], tags, g["n_sm"], g["cost_int4"], g["cost_int8"])
+    assert lb == Fraction(g["expected"]["decomposed"])
+    # an explicit whole-unit remapping reaching 7: loads 7/7/7/6
+    segs = [[(0, 0, 2), (1, 0, 2), (2, 1, 2)],
+            [(2, 0, 1), (3, 0, 2), (4, 0, 1)],
+            [(4, 1, 2), (5, 0, 2), (6, 0, 2)],
+            [(7, 0, 2), (8, 0, 2)]]
+    planner.check_cover(segs, g["n_output_tiles"], len(tags))
+    assert planner.makespan(segs, tags, g["cost_int4"], g["cost_int8"]) == Fraction(g["expected"]["remapped_best_whole_tile"])
+    with pytest.raises(AssertionError):
+        planner.check_cover(segs[:3], g["n_output_tiles"], len(tags))
