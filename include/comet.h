@@ -1,0 +1,225 @@
+/*
+ * comet.h -- C ABI of libcomet.so, the B200 (sm_100a) W4Ax hot path of COMET
+ * (Liu et al., "COMET: Towards Practical W4A4KV4 LLMs Serving", ASPLOS'25).
+ * Citations "P:Lnnn" are lines of the paper text; DESIGN.md has the readings R*.
+ *
+ * The path ("O = WX"):   Y[M,N] = X[M,K] . W[N,K]^T
+ *   1. comet_quantize_act : FMPQ -- every 128-channel block of every token row is quantised
+ *      symmetric min-max to INT4 (qmax 7) or, for blocks tagged as outlier blocks, INT8
+ *      (qmax 127), one FP32 scale per (token, block)  (R1-R5).
+ *   2. comet_pack_weight  : INT4 weight codes [-8,7] -> packed nibbles (R14).
+ *   3. comet_plan_create  : the SM scheduler -- a persistent-CTA work list over
+ *      (output tile x K-block) units, either whole tiles balanced by cost (tile remapping,
+ *      P:L220) or a stream-K split of tiles across CTAs (tile decomposition).
+ *   4. comet_w4ax_gemm    : packed W4 x A4/A8 GEMM, exact integer per-block accumulation on
+ *      the tcgen05 tensor cores, per-block dequantisation into FP32 and the s_w epilogue
+ *      (P:L164-178).
+ *
+ * Conventions
+ *   - Every pointer named *_dev / documented "device" is a CUDA device pointer owned by the
+ *     caller; the library never frees caller memory.  *_host pointers are host memory read
+ *     synchronously during the call.
+ *   - Every launch is asynchronous on the given stream (cudaStream_t passed as void*; NULL =
+ *     legacy default stream).  No call allocates or synchronises on the hot path
+ *     (comet_quantize_act, comet_pack_weight, comet_w4ax_gemm).
+ *   - Errors: every function returns a comet_status_t; nothing throws or aborts across the
+ *     ABI.  Arguments are validated before any launch; on error nothing is launched.
+ *     comet_last_error() returns a thread-local detail string for the last failure.
+ *   - Shapes: K % 128 == 0 (FMPQ block k = 128); N % 128 == 0; M >= 1 (any value;
+ *     ragged tails are handled); K <= 131072, N <= 1048576, M <= 2^31-1.
+ *   - Alignment: every device pointer 16-byte aligned; ldx (elements) with ldx*2 % 16 == 0;
+ *     ldy (elements) with ldy*sizeof(y) % 16 == 0 (ldy >= N).
+ *   - Requires an sm_100a device (B200); otherwise COMET_ERR_NOT_SM100A.
+ */
+#ifndef COMET_H_
+#define COMET_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define COMET_BLOCK_K 128   /* FMPQ block: k = 128 channels */
+#define COMET_TILE_W  128   /* weight rows per output tile (MMA M) */
+#define COMET_SCALE_PAD 16  /* token dimension of per-token arrays is padded to Mp = roundup(M,16) */
+
+typedef enum {
+  COMET_OK = 0,
+  COMET_ERR_INVALID_ARG = 1,
+  COMET_ERR_UNSUPPORTED_SHAPE = 2,
+  COMET_ERR_MISALIGNED = 3,
+  COMET_ERR_NOT_SM100A = 4,
+  COMET_ERR_WORKSPACE_TOO_SMALL = 5,
+  COMET_ERR_CUDA = 6
+} comet_status_t;
+
+typedef enum { COMET_F16 = 0, COMET_BF16 = 1, COMET_F32 = 2 } comet_dtype_t;
+
+/* ------------------------------------------------------------------------------------------
+ * Activation packed layout ("mixed-precision data layout", reading R15)
+ *
+ * For X[M,K] with nb = K/128 blocks and Mp = roundup(M, 16), the buffer `act_packed`
+ * (comet_act_packed_bytes(M,K) bytes, 256-byte aligned) holds, at the byte offsets returned
+ * by comet_act_layout():
+ *
+ *   codes [M][K]  uint8, row-major (row stride K bytes).  Byte (m,k), block b = k/128:
+ *                   tags[b] == 0 (INT4 block): the E4M3 encoding of the INT4 code q in [-7,7]
+ *                     (every integer |q| <= 7 is exact in E4M3:  0 -> 0x00, 1 -> 0x38,
+ *                      2 -> 0x40, 3 -> 0x44, 4 -> 0x48, 5 -> 0x4A, 6 -> 0x4C, 7 -> 0x4E,
+ *                      negative = 0x80 | encoding of |q|; -0 is never produced);
+ *                   tags[b] == 1 (INT8 block): the two's-complement byte of q in [-127,127].
+ *   qsum  [nb][Mp] int16:  qsum[b][m] = sum_{k in block b} q[m,k]   (exact; 0 for m >= M)
+ *   corr  [Mp]     float:  corr[m] = 8 * sum_{b : tags[b]==0} scale[b][m] * qsum[b][m]
+ *                          (binary32 sum, order implementation-defined; used by the GEMM to
+ *                           undo the offset-binary weight encoding)
+ *
+ * act_scales [nb][Mp] float (separate buffer, 16-byte aligned):
+ *   act_scales[b*Mp + m] = s_a[m,b] = amax / qmax (binary32), 0 for an all-zero block and
+ *   for m >= M.
+ * ---------------------------------------------------------------------------------------- */
+typedef struct {
+  size_t codes_off;     /* always 0 */
+  size_t qsum_off;
+  size_t corr_off;
+  size_t total_bytes;
+  int64_t Mp;           /* padded token count */
+  int64_t nb;           /* K / 128 */
+} comet_act_layout_t;
+
+comet_status_t comet_act_layout(int64_t M, int64_t K, comet_act_layout_t* out);
+size_t comet_act_packed_bytes(int64_t M, int64_t K);
+/* number of floats of act_scales: nb * Mp */
+size_t comet_act_scales_count(int64_t M, int64_t K);
+
+/*
+ * FMPQ activation quantisation.
+ *   x          device, [M][ldx] float16 (xdt = COMET_F16) or bfloat16 (COMET_BF16), row-major.
+ *   tags_host  host, [K/128] uint8, nonzero = INT8 (outlier) block.  Read synchronously.
+ *   perm_dev   must be NULL (channel permutation P:L138-144 is applied offline to W and
+ *              upstream to X; a fused gather is not implemented -> COMET_ERR_UNSUPPORTED_SHAPE).
+ *   act_packed device, comet_act_packed_bytes(M,K) bytes, written completely.
+ *   act_scales device, comet_act_scales_count(M,K) floats, written completely.
+ * Per (m, b): amax = max|x|; qmax = 127 if tags[b] else 7; amax == 0 -> s = 0 and codes 0;
+ * else s = amax/qmax, r = qmax/amax (binary32, correctly rounded), q = clamp(rint(x*r))
+ * with rint = round-half-even and x*r one binary32 product (NaN -> 0).  Inputs must be
+ * finite.  Bit-exact with the CPU oracle.
+ */
+comet_status_t comet_quantize_act(const void* x, comet_dtype_t xdt, int64_t M, int64_t K,
+                                  int64_t ldx, const uint8_t* tags_host, const int32_t* perm_dev,
+                                  void* act_packed, float* act_scales, void* stream);
+
+/* ------------------------------------------------------------------------------------------
+ * Weight packed layout ("location switch" + "zero extension", reading R14)
+ *
+ * w_packed [N][K/2] uint8, row-major (row stride K/2 bytes).  For row n and every group of
+ * eight consecutive channels k = 8g .. 8g+7, the little-endian 32-bit word at byte offset
+ * n*K/2 + 4g has byte i (i = 0..3) equal to
+ *        (u[8g+i] & 0xF) | (u[8g+i+4] << 4),      u = w + 8  (offset binary, 0..15).
+ * Then (word & 0x0F0F0F0F) holds u[8g..8g+3] and ((word >> 4) & 0x0F0F0F0F) holds
+ * u[8g+4..8g+7], one per byte, in channel order: widening costs 3 instructions per 8 values.
+ * A byte 0x0u read as E4M3 is exactly u * 2^-9 (subnormal/first binade), so the widened
+ * bytes feed the FP8 tensor core directly; (u << 4) ^ 0x80 is the int8 16*w for INT8 blocks.
+ * ---------------------------------------------------------------------------------------- */
+size_t comet_weight_packed_bytes(int64_t N, int64_t K);
+/* w_codes_dev: device [N][K] int8 codes in [-8,7] (values outside are masked to 4 bits). */
+comet_status_t comet_pack_weight(const int8_t* w_codes_dev, int64_t N, int64_t K, void* w_packed,
+                                 void* stream);
+
+/* ------------------------------------------------------------------------------------------
+ * Tile scheduler ("fine-grained SM scheduling")
+ * ---------------------------------------------------------------------------------------- */
+typedef struct comet_plan_s* comet_plan_t;   /* opaque, library-owned, immutable after create */
+
+typedef struct {
+  int tile_n;          /* tokens per output tile (MMA N): 16..224, multiple of 16; 0 = auto */
+  int num_sms;         /* persistent CTAs (one per SM); 0 = query the current device */
+  int split_mode;      /* 0 = whole tiles onto the least-loaded CTA (no fix-up);
+                          1 = tile decomposition: stream-K contiguous K-ranges;
+                          2 = naive: (tile, K-block) units round-robin (Fig. 8b/c);
+                          3 = unit remapping: units longest-first onto the least-loaded CTA
+                              (Fig. 8d);
+                         -1 = auto (stream-K when whole tiles fill < 92 % of the last wave) */
+  float cost_int4;     /* planner cost of one INT4 K-block unit (default 1.0) */
+  float cost_int8;     /* planner cost of one INT8 K-block unit (default 1.0 on B200) */
+  int stages;          /* shared-memory ring depth; 0 = auto */
+  int device_plan;     /* 1 (default) = upload the work list to the device at create time;
+                          0 = host-only plan (comet_plan_describe only; CPU-safe) */
+  int reserved[6];
+} comet_sched_config;
+
+/* Fill *cfg with the defaults (tile_n 0, num_sms 0, split_mode -1, costs 1/1, stages 0,
+ * device_plan 1). */
+void comet_sched_config_default(comet_sched_config* cfg);
+
+/*
+ * Build the work list for Y[M,N] = X[M,K] W[N,K]^T with the given block tags.
+ *   tags_host  host [K/128] uint8 (copied into the plan).
+ *   cfg        NULL = defaults.
+ *   out        receives the plan.
+ *   workspace_bytes  receives the device workspace comet_w4ax_gemm needs (stream-K partials
+ *              and flags); may be 0.
+ * Not on the hot path: may allocate device memory (the work list) when device_plan = 1.
+ */
+comet_status_t comet_plan_create(int64_t M, int64_t N, int64_t K, const uint8_t* tags_host,
+                                 const comet_sched_config* cfg, comet_plan_t* out,
+                                 size_t* workspace_bytes);
+comet_status_t comet_plan_destroy(comet_plan_t plan);
+
+typedef struct {
+  int64_t M, N, K;
+  int tile_n, num_ctas, split_mode, stages;
+  int64_t n_tiles;         /* output tiles = (N/128) * ceil(M/tile_n) */
+  int64_t n_items;         /* work items in the list */
+  int64_t n_split_tiles;   /* tiles shared by more than one CTA */
+  double max_cta_cost;     /* planner makespan (sum of unit costs on the busiest CTA) */
+  double mean_cta_cost;
+} comet_plan_info_t;
+comet_status_t comet_plan_info(comet_plan_t plan, comet_plan_info_t* info);
+
+/* Export the work list: items[4*i + {0,1,2,3}] = {cta, tile, kb_begin, kb_end} for the
+ * i-th item (CTAs' items consecutive, in execution order).  *n_items = count written. */
+comet_status_t comet_plan_describe(comet_plan_t plan, int32_t* items, int64_t max_items,
+                                   int64_t* n_items);
+
+/*
+ * The W4Ax GEMM.   y[m, n] = s_w[n] * sum_b s_a[m,b] * acc_b[m,n]
+ *   act_packed, act_scales  from comet_quantize_act with the plan's M, K and tags.
+ *   w_packed                from comet_pack_weight, [N][K/2].
+ *   w_scales                device [N] float (per-output-channel, reading R7).
+ *   y                       device [M][ldy] of ydt (F16 / BF16 / F32), row-major.
+ *   debug_acc               NULL, or device [M][N] int32: sum_b acc_b[m,n] in code units
+ *                           (bit-exact integer accumulators; slower debug kernel).
+ *   debug_acc_blocks        NULL, or device [K/128][M][N] int32 per-block acc_b (tiny shapes).
+ *   workspace               device, >= the plan's workspace_bytes (may be NULL if 0).
+ */
+comet_status_t comet_w4ax_gemm(comet_plan_t plan, const void* act_packed, const float* act_scales,
+                               const void* w_packed, const float* w_scales, void* y,
+                               comet_dtype_t ydt, int64_t ldy, int32_t* debug_acc,
+                               int32_t* debug_acc_blocks, void* workspace, size_t ws_bytes,
+                               void* stream);
+
+/*
+ * Convenience: the whole hot path for one linear layer with HOST buffers (used for the
+ * end-to-end measurement).  Copies x_host (pinned recommended) to the device, quantises,
+ * runs the GEMM and copies y back to y_host, all on `stream`, then synchronises the stream.
+ * Device scratch (x, act, scales, y) is taken from `scratch` (comet_linear_scratch_bytes).
+ */
+size_t comet_linear_scratch_bytes(comet_plan_t plan, comet_dtype_t xdt, comet_dtype_t ydt);
+comet_status_t comet_w4ax_linear_host(comet_plan_t plan, const void* x_host, comet_dtype_t xdt,
+                                      const void* w_packed, const float* w_scales, void* y_host,
+                                      comet_dtype_t ydt, void* scratch, size_t scratch_bytes,
+                                      void* workspace, size_t ws_bytes, void* stream);
+
+const char* comet_status_string(comet_status_t s);
+const char* comet_last_error(void);
+/* Library version string and the number of kernels the last comet_w4ax_gemm /
+ * comet_quantize_act call launched (for launch accounting). */
+const char* comet_version(void);
+int comet_last_launch_count(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* COMET_H_ */

@@ -1,0 +1,276 @@
+"""comet-b200: the W4Ax hot path of COMET (ASPLOS'25) on B200 (sm_100a).
+
+Thin ctypes binding over ``lib/libcomet.so`` (C ABI in ``include/comet.h``).  Every step of
+the path runs in the library's CUDA kernels; this module only marshals torch tensors
+(device memory, streams) into the C calls and raises on error.  There is no CPU fallback:
+if the library is missing, importing the binding raises.
+
+Names follow the C ABI:  quantize_act, pack_weight, Plan (comet_plan_create),
+w4ax_gemm, w4ax_linear_host.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import re
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "lib", "libcomet.so")
+HEADER_PATH = os.path.join(os.path.dirname(_PKG), "include", "comet.h")
+
+COMET_F16, COMET_BF16, COMET_F32 = 0, 1, 2
+BLOCK_K = 128
+TILE_W = 128
+SCALE_PAD = 16
+
+
+class CometError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"{_STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+_STATUS = {0: "COMET_OK", 1: "COMET_ERR_INVALID_ARG", 2: "COMET_ERR_UNSUPPORTED_SHAPE",
+           3: "COMET_ERR_MISALIGNED", 4: "COMET_ERR_NOT_SM100A", 5: "COMET_ERR_WORKSPACE_TOO_SMALL",
+           6: "COMET_ERR_CUDA"}
+
+
+class ActLayout(ctypes.Structure):
+    _fields_ = [("codes_off", ctypes.c_size_t), ("qsum_off", ctypes.c_size_t),
+                ("corr_off", ctypes.c_size_t), ("total_bytes", ctypes.c_size_t),
+                ("Mp", ctypes.c_int64), ("nb", ctypes.c_int64)]
+
+
+class SchedConfig(ctypes.Structure):
+    _fields_ = [("tile_n", ctypes.c_int), ("num_sms", ctypes.c_int), ("split_mode", ctypes.c_int),
+                ("cost_int4", ctypes.c_float), ("cost_int8", ctypes.c_float),
+                ("stages", ctypes.c_int), ("device_plan", ctypes.c_int),
+                ("reserved", ctypes.c_int * 6)]
+
+
+class PlanInfo(ctypes.Structure):
+    _fields_ = [("M", ctypes.c_int64), ("N", ctypes.c_int64), ("K", ctypes.c_int64),
+                ("tile_n", ctypes.c_int), ("num_ctas", ctypes.c_int), ("split_mode", ctypes.c_int),
+                ("stages", ctypes.c_int), ("n_tiles", ctypes.c_int64), ("n_items", ctypes.c_int64),
+                ("n_split_tiles", ctypes.c_int64), ("max_cta_cost", ctypes.c_double),
+                ("mean_cta_cost", ctypes.c_double)]
+
+
+_lib = None
+
+
+def lib():
+    """Load libcomet.so (built in-tree by build.build()).  Raises if it is missing."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} not built: run `python -m paper_conf_asplos_liu0rxpwl0w25_b200.build`"
+                          " (there is no CPU fallback)")
+    L = ctypes.CDLL(LIB_PATH)
+    P, I64, I32, SZ = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int, ctypes.c_size_t
+    sig = {
+        "comet_act_layout": (I32, [I64, I64, ctypes.POINTER(ActLayout)]),
+        "comet_act_packed_bytes": (SZ, [I64, I64]),
+        "comet_act_scales_count": (SZ, [I64, I64]),
+        "comet_quantize_act": (I32, [P, I32, I64, I64, I64, P, P, P, P, P]),
+        "comet_weight_packed_bytes": (SZ, [I64, I64]),
+        "comet_pack_weight": (I32, [P, I64, I64, P, P]),
+        "comet_sched_config_default": (None, [ctypes.POINTER(SchedConfig)]),
+        "comet_plan_create": (I32, [I64, I64, I64, P, ctypes.POINTER(SchedConfig), ctypes.POINTER(P),
+                                    ctypes.POINTER(SZ)]),
+        "comet_plan_destroy": (I32, [P]),
+        "comet_plan_info": (I32, [P, ctypes.POINTER(PlanInfo)]),
+        "comet_plan_describe": (I32, [P, P, I64, ctypes.POINTER(I64)]),
+        "comet_w4ax_gemm": (I32, [P, P, P, P, P, P, I32, I64, P, P, P, SZ, P]),
+        "comet_linear_scratch_bytes": (SZ, [P, I32, I32]),
+        "comet_w4ax_linear_host": (I32, [P, P, I32, P, P, P, I32, P, SZ, P, SZ, P]),
+        "comet_status_string": (ctypes.c_char_p, [I32]),
+        "comet_last_error": (ctypes.c_char_p, []),
+        "comet_version": (ctypes.c_char_p, []),
+        "comet_last_launch_count": (I32, []),
+    }
+    for name, (res, args) in sig.items():
+        f = getattr(L, name)
+        f.restype = res
+        f.argtypes = args
+    _lib = L
+    return L
+
+
+def declared_symbols() -> list[str]:
+    """Function names declared in include/comet.h."""
+    with open(HEADER_PATH) as f:
+        txt = f.read()
+    txt = re.sub(r"/\*.*?\*/", "", txt, flags=re.S)
+    return sorted(set(re.findall(r"\b(comet_[a-z0-9_]+)\s*\(", txt)))
+
+
+def _check(st: int):
+    if st != 0:
+        raise CometError(st, lib().comet_last_error().decode())
+
+
+def _stream(stream=None):
+    import torch
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+def _dt(t) -> int:
+    import torch
+    return {torch.float16: COMET_F16, torch.bfloat16: COMET_BF16, torch.float32: COMET_F32}[t]
+
+
+def _tags_np(tags) -> np.ndarray:
+    return np.ascontiguousarray(np.asarray(tags, dtype=np.uint8))
+
+
+def act_layout(M: int, K: int) -> dict:
+    L = ActLayout()
+    _check(lib().comet_act_layout(M, K, ctypes.byref(L)))
+    return {f: getattr(L, f) for f, _ in ActLayout._fields_}
+
+
+def last_launch_count() -> int:
+    return int(lib().comet_last_launch_count())
+
+
+def quantize_act(x, tags, *, out=None, stream=None):
+    """FMPQ quantisation (comet_quantize_act).  x: [M, K] float16/bfloat16 CUDA tensor.
+    Returns (act_packed uint8 tensor, act_scales float32 tensor [nb*Mp])."""
+    import torch
+    assert x.is_cuda and x.dim() == 2 and x.stride(1) == 1
+    M, K = x.shape
+    t = _tags_np(tags)
+    lay = act_layout(M, K)
+    if out is None:
+        act = torch.empty(lay["total_bytes"], dtype=torch.uint8, device=x.device)
+        sc = torch.empty(lay["nb"] * lay["Mp"], dtype=torch.float32, device=x.device)
+    else:
+        act, sc = out
+    _check(lib().comet_quantize_act(ctypes.c_void_p(x.data_ptr()), _dt(x.dtype), M, K, x.stride(0),
+                                    t.ctypes.data_as(ctypes.c_void_p), None,
+                                    ctypes.c_void_p(act.data_ptr()), ctypes.c_void_p(sc.data_ptr()),
+                                    _stream(stream)))
+    return act, sc
+
+
+def pack_weight(w_codes, *, out=None, stream=None):
+    """comet_pack_weight: [N, K] int8 codes in [-8, 7] -> [N, K/2] packed uint8."""
+    import torch
+    assert w_codes.is_cuda and w_codes.dtype == torch.int8 and w_codes.is_contiguous()
+    N, K = w_codes.shape
+    wp = out if out is not None else torch.empty((N, K // 2), dtype=torch.uint8, device=w_codes.device)
+    _check(lib().comet_pack_weight(ctypes.c_void_p(w_codes.data_ptr()), N, K,
+                                   ctypes.c_void_p(wp.data_ptr()), _stream(stream)))
+    return wp
+
+
+class Plan:
+    """comet_plan_create: the persistent-CTA tile schedule for one GEMM shape and tag set."""
+
+    def __init__(self, M: int, N: int, K: int, tags, *, tile_n: int = 0, num_sms: int = 0,
+                 split_mode: int = -1, cost_int4: float = 1.0, cost_int8: float = 1.0,
+                 device_plan: bool = True):
+        L = lib()
+        cfg = SchedConfig()
+        L.comet_sched_config_default(ctypes.byref(cfg))
+        cfg.tile_n, cfg.num_sms, cfg.split_mode = tile_n, num_sms, split_mode
+        cfg.cost_int4, cfg.cost_int8 = cost_int4, cost_int8
+        cfg.device_plan = 1 if device_plan else 0
+        self.tags = _tags_np(tags)
+        h = ctypes.c_void_p()
+        ws = ctypes.c_size_t()
+        _check(L.comet_plan_create(M, N, K, self.tags.ctypes.data_as(ctypes.c_void_p), ctypes.byref(cfg),
+                                   ctypes.byref(h), ctypes.byref(ws)))
+        self._h = h
+        self.M, self.N, self.K = M, N, K
+        self.workspace_bytes = int(ws.value)
+        self._ws = None
+
+    @property
+    def handle(self):
+        return self._h
+
+    def info(self) -> dict:
+        i = PlanInfo()
+        _check(lib().comet_plan_info(self._h, ctypes.byref(i)))
+        return {f: getattr(i, f) for f, _ in PlanInfo._fields_}
+
+    def describe(self) -> np.ndarray:
+        """[n_items, 4] int32 rows (cta, tile, kb_begin, kb_end) in execution order."""
+        n = ctypes.c_int64()
+        _check(lib().comet_plan_describe(self._h, None, 0, ctypes.byref(n)))
+        buf = np.zeros((max(1, n.value), 4), dtype=np.int32)
+        _check(lib().comet_plan_describe(self._h, buf.ctypes.data_as(ctypes.c_void_p), n.value,
+                                         ctypes.byref(n)))
+        return buf[: n.value]
+
+    def workspace(self, device="cuda"):
+        """Zero-initialised workspace tensor (kept with the plan; one per plan)."""
+        import torch
+        if self._ws is None:
+            self._ws = torch.zeros(max(256, self.workspace_bytes), dtype=torch.uint8, device=device)
+        return self._ws
+
+    def close(self):
+        if self._h:
+            lib().comet_plan_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def w4ax_gemm(plan: Plan, act_packed, act_scales, w_packed, w_scales, *, out=None,
+              out_dtype=None, debug: bool = False, debug_blocks: bool = False, stream=None):
+    """comet_w4ax_gemm.  Returns y [M, N] (and debug int32 accumulators when requested)."""
+    import torch
+    dev = act_packed.device
+    if out is None:
+        out = torch.empty((plan.M, plan.N), dtype=out_dtype or torch.float16, device=dev)
+    dacc = torch.empty((plan.M, plan.N), dtype=torch.int32, device=dev) if (debug or debug_blocks) else None
+    dblk = (torch.empty((plan.K // BLOCK_K, plan.M, plan.N), dtype=torch.int32, device=dev)
+            if debug_blocks else None)
+    ws = plan.workspace(dev)
+    _check(lib().comet_w4ax_gemm(plan.handle, ctypes.c_void_p(act_packed.data_ptr()),
+                                 ctypes.c_void_p(act_scales.data_ptr()),
+                                 ctypes.c_void_p(w_packed.data_ptr()),
+                                 ctypes.c_void_p(w_scales.data_ptr()), ctypes.c_void_p(out.data_ptr()),
+                                 _dt(out.dtype), out.stride(0),
+                                 ctypes.c_void_p(dacc.data_ptr()) if dacc is not None else None,
+                                 ctypes.c_void_p(dblk.data_ptr()) if dblk is not None else None,
+                                 ctypes.c_void_p(ws.data_ptr()), ws.numel(), _stream(stream)))
+    if debug_blocks:
+        return out, dacc, dblk
+    if debug:
+        return out, dacc
+    return out
+
+
+def w4ax_linear(plan: Plan, x, w_packed, w_scales, *, out_dtype=None, stream=None):
+    """The whole hot path for one linear layer on device tensors: quantize_act + w4ax_gemm."""
+    act, sc = quantize_act(x, plan.tags, stream=stream)
+    return w4ax_gemm(plan, act, sc, w_packed, w_scales, out_dtype=out_dtype, stream=stream)
+
+
+def linear_scratch_bytes(plan: Plan, xdt: int, ydt: int) -> int:
+    return int(lib().comet_linear_scratch_bytes(plan.handle, xdt, ydt))
+
+
+def w4ax_linear_host(plan: Plan, x_host, w_packed, w_scales, y_host, scratch, *, stream=None):
+    """comet_w4ax_linear_host: host (pinned) x in, host y out; H2D, quantise, GEMM, D2H."""
+    ws = plan.workspace(w_packed.device)
+    _check(lib().comet_w4ax_linear_host(plan.handle, ctypes.c_void_p(x_host.data_ptr()), _dt(x_host.dtype),
+                                        ctypes.c_void_p(w_packed.data_ptr()),
+                                        ctypes.c_void_p(w_scales.data_ptr()),
+                                        ctypes.c_void_p(y_host.data_ptr()), _dt(y_host.dtype),
+                                        ctypes.c_void_p(scratch.data_ptr()), scratch.numel(),
+                                        ctypes.c_void_p(ws.data_ptr()), ws.numel(), _stream(stream)))
+    return y_host

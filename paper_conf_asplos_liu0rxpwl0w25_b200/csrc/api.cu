@@ -1,0 +1,340 @@
+// api.cu -- the C ABI of libcomet.so (include/comet.h): validation, layouts, planning, dispatch.
+#include <cstring>
+#include <cstdio>
+#include <mutex>
+#include <new>
+#include "internal.h"
+
+struct comet_plan_s {
+  comet::Plan p;
+};
+
+namespace comet {
+
+static thread_local std::string g_err;
+static thread_local int g_launches = 0;
+
+void set_error(const std::string& msg) { g_err = msg; }
+comet_status_t fail(comet_status_t st, const std::string& msg) {
+  g_err = msg;
+  return st;
+}
+comet_status_t cuda_status(cudaError_t e, const char* what) {
+  g_err = std::string(what) + ": " + cudaGetErrorString(e);
+  return COMET_ERR_CUDA;
+}
+void note_launches(int n) { g_launches = n; }
+
+static comet_status_t check_device(int* sms = nullptr) {
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return cuda_status(e, "cudaGetDevice");
+  int major = 0, minor = 0, nsm = 0;
+  cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev);
+  cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, dev);
+  cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+  if (major != 10 || minor != 0)
+    return fail(COMET_ERR_NOT_SM100A, "libcomet.so needs an sm_100a (B200) device; found sm_" +
+                                          std::to_string(major) + std::to_string(minor));
+  if (sms) *sms = nsm;
+  return COMET_OK;
+}
+
+static bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+
+static comet_status_t check_mk(int64_t M, int64_t K) {
+  if (M < 1 || M > INT32_MAX) return fail(COMET_ERR_UNSUPPORTED_SHAPE, "M must be in [1, 2^31-1]");
+  if (K < kBlockK || K % kBlockK != 0 || K > (int64_t)kBlockK * kMaxBlocks)
+    return fail(COMET_ERR_UNSUPPORTED_SHAPE, "K must be a positive multiple of 128, <= 131072");
+  return COMET_OK;
+}
+static comet_status_t check_n(int64_t N) {
+  if (N < kTileW || N % kTileW != 0 || N > (1 << 20))
+    return fail(COMET_ERR_UNSUPPORTED_SHAPE, "N must be a positive multiple of 128, <= 2^20");
+  return COMET_OK;
+}
+
+static TagMask mask_of(const uint8_t* tags, int64_t nb) {
+  TagMask m;
+  memset(&m, 0, sizeof(m));
+  for (int64_t b = 0; b < nb; ++b)
+    if (tags[b]) m.w[b >> 5] |= 1u << (b & 31);
+  return m;
+}
+
+}  // namespace comet
+
+using namespace comet;
+
+extern "C" {
+
+const char* comet_status_string(comet_status_t s) {
+  switch (s) {
+    case COMET_OK: return "COMET_OK";
+    case COMET_ERR_INVALID_ARG: return "COMET_ERR_INVALID_ARG";
+    case COMET_ERR_UNSUPPORTED_SHAPE: return "COMET_ERR_UNSUPPORTED_SHAPE";
+    case COMET_ERR_MISALIGNED: return "COMET_ERR_MISALIGNED";
+    case COMET_ERR_NOT_SM100A: return "COMET_ERR_NOT_SM100A";
+    case COMET_ERR_WORKSPACE_TOO_SMALL: return "COMET_ERR_WORKSPACE_TOO_SMALL";
+    case COMET_ERR_CUDA: return "COMET_ERR_CUDA";
+  }
+  return "COMET_ERR_UNKNOWN";
+}
+
+const char* comet_last_error(void) { return g_err.c_str(); }
+const char* comet_version(void) { return "comet-b200 0.1 (sm_100a; W4Ax = FP8-exact INT4 blocks + INT8 blocks)"; }
+int comet_last_launch_count(void) { return g_launches; }
+
+comet_status_t comet_act_layout(int64_t M, int64_t K, comet_act_layout_t* out) {
+  if (!out) return fail(COMET_ERR_INVALID_ARG, "out is NULL");
+  comet_status_t st = check_mk(M, K);
+  if (st != COMET_OK) return st;
+  act_layout(M, K, out);
+  return COMET_OK;
+}
+
+size_t comet_act_packed_bytes(int64_t M, int64_t K) {
+  if (check_mk(M, K) != COMET_OK) return 0;
+  comet_act_layout_t L;
+  act_layout(M, K, &L);
+  return L.total_bytes;
+}
+
+size_t comet_act_scales_count(int64_t M, int64_t K) {
+  if (check_mk(M, K) != COMET_OK) return 0;
+  return (size_t)(K / kBlockK) * (size_t)round_up(M, COMET_SCALE_PAD);
+}
+
+comet_status_t comet_quantize_act(const void* x, comet_dtype_t xdt, int64_t M, int64_t K,
+                                  int64_t ldx, const uint8_t* tags_host, const int32_t* perm_dev,
+                                  void* act_packed, float* act_scales, void* stream) {
+  g_launches = 0;
+  comet_status_t st = check_mk(M, K);
+  if (st != COMET_OK) return st;
+  if (!x || !tags_host || !act_packed || !act_scales) return fail(COMET_ERR_INVALID_ARG, "NULL pointer argument");
+  if (xdt != COMET_F16 && xdt != COMET_BF16) return fail(COMET_ERR_INVALID_ARG, "xdt must be COMET_F16 or COMET_BF16");
+  if (perm_dev) return fail(COMET_ERR_UNSUPPORTED_SHAPE, "fused channel permutation is not implemented (perm_dev must be NULL)");
+  if (ldx < K || (ldx * 2) % 16 != 0) return fail(COMET_ERR_MISALIGNED, "ldx must be >= K with ldx*2 % 16 == 0");
+  if (!aligned16(x) || !aligned16(act_packed) || !aligned16(act_scales))
+    return fail(COMET_ERR_MISALIGNED, "device pointers must be 16-byte aligned");
+  if ((reinterpret_cast<uintptr_t>(act_packed) & 255u) != 0)
+    return fail(COMET_ERR_MISALIGNED, "act_packed must be 256-byte aligned");
+  st = check_device();
+  if (st != COMET_OK) return st;
+  TagMask mask = mask_of(tags_host, K / kBlockK);
+  int launches = 0;
+  cudaError_t e = launch_quantize(x, xdt == COMET_BF16, M, K, ldx, mask, act_packed, act_scales,
+                                  static_cast<cudaStream_t>(stream), &launches);
+  if (e != cudaSuccess) return cuda_status(e, "quantize launch");
+  g_launches = launches;
+  return COMET_OK;
+}
+
+size_t comet_weight_packed_bytes(int64_t N, int64_t K) {
+  if (check_n(N) != COMET_OK || check_mk(1, K) != COMET_OK) return 0;
+  return (size_t)N * (size_t)K / 2;
+}
+
+comet_status_t comet_pack_weight(const int8_t* w_codes_dev, int64_t N, int64_t K, void* w_packed,
+                                 void* stream) {
+  g_launches = 0;
+  comet_status_t st = check_n(N);
+  if (st != COMET_OK) return st;
+  st = check_mk(1, K);
+  if (st != COMET_OK) return st;
+  if (!w_codes_dev || !w_packed) return fail(COMET_ERR_INVALID_ARG, "NULL pointer argument");
+  if (!aligned16(w_codes_dev) || !aligned16(w_packed)) return fail(COMET_ERR_MISALIGNED, "device pointers must be 16-byte aligned");
+  st = check_device();
+  if (st != COMET_OK) return st;
+  cudaError_t e = launch_pack_weight(w_codes_dev, N, K, w_packed, static_cast<cudaStream_t>(stream));
+  if (e != cudaSuccess) return cuda_status(e, "pack launch");
+  g_launches = 1;
+  return COMET_OK;
+}
+
+void comet_sched_config_default(comet_sched_config* cfg) {
+  if (!cfg) return;
+  memset(cfg, 0, sizeof(*cfg));
+  cfg->tile_n = 0;
+  cfg->num_sms = 0;
+  cfg->split_mode = -1;
+  cfg->cost_int4 = 1.0f;
+  cfg->cost_int8 = 1.0f;
+  cfg->stages = 0;
+  cfg->device_plan = 1;
+}
+
+comet_status_t comet_plan_create(int64_t M, int64_t N, int64_t K, const uint8_t* tags_host,
+                                 const comet_sched_config* cfg_in, comet_plan_t* out,
+                                 size_t* workspace_bytes) {
+  if (!out || !tags_host) return fail(COMET_ERR_INVALID_ARG, "NULL pointer argument");
+  *out = nullptr;
+  comet_status_t st = check_mk(M, K);
+  if (st != COMET_OK) return st;
+  st = check_n(N);
+  if (st != COMET_OK) return st;
+  comet_sched_config cfg;
+  if (cfg_in) cfg = *cfg_in;
+  else comet_sched_config_default(&cfg);
+  if (cfg.split_mode < -1 || cfg.split_mode > 3) return fail(COMET_ERR_INVALID_ARG, "split_mode must be -1, 0, 1, 2 or 3");
+  if (cfg.cost_int4 < 0 || cfg.cost_int8 < 0) return fail(COMET_ERR_INVALID_ARG, "costs must be >= 0");
+  if (cfg.num_sms <= 0) {
+    if (!cfg.device_plan) return fail(COMET_ERR_INVALID_ARG, "a host-only plan needs an explicit num_sms");
+    int sms = 0;
+    st = check_device(&sms);
+    if (st != COMET_OK) return st;
+    cfg.num_sms = sms;
+  } else if (cfg.device_plan) {
+    int sms = 0;
+    st = check_device(&sms);
+    if (st != COMET_OK) return st;
+    if (cfg.num_sms > sms) return fail(COMET_ERR_INVALID_ARG, "num_sms exceeds the device's SM count (persistent CTAs must be co-resident)");
+  }
+  comet_plan_s* h = new (std::nothrow) comet_plan_s();
+  if (!h) return fail(COMET_ERR_INVALID_ARG, "out of host memory");
+  Plan& p = h->p;
+  p.M = M; p.N = N; p.K = K;
+  p.tags.assign(tags_host, tags_host + K / kBlockK);
+  p.mask = mask_of(tags_host, K / kBlockK);
+  st = build_plan(p, cfg);
+  if (st != COMET_OK) { delete h; return st; }
+  if (cfg.device_plan) {
+    cudaGetDevice(&p.device);
+    cudaError_t e = cudaMalloc(&p.d_cta_begin, p.cta_begin.size() * sizeof(int32_t));
+    if (e == cudaSuccess) e = cudaMalloc(&p.d_items, std::max<size_t>(1, p.items.size()) * sizeof(WorkItem));
+    if (e == cudaSuccess) e = cudaMemcpy(p.d_cta_begin, p.cta_begin.data(), p.cta_begin.size() * sizeof(int32_t), cudaMemcpyHostToDevice);
+    if (e == cudaSuccess && !p.items.empty())
+      e = cudaMemcpy(p.d_items, p.items.data(), p.items.size() * sizeof(WorkItem), cudaMemcpyHostToDevice);
+    if (e != cudaSuccess) {
+      if (p.d_cta_begin) cudaFree(p.d_cta_begin);
+      if (p.d_items) cudaFree(p.d_items);
+      delete h;
+      return cuda_status(e, "plan upload");
+    }
+  }
+  if (workspace_bytes) *workspace_bytes = p.ws_bytes;
+  *out = h;
+  return COMET_OK;
+}
+
+comet_status_t comet_plan_destroy(comet_plan_t plan) {
+  if (!plan) return COMET_OK;
+  if (plan->p.d_cta_begin) cudaFree(plan->p.d_cta_begin);
+  if (plan->p.d_items) cudaFree(plan->p.d_items);
+  delete plan;
+  return COMET_OK;
+}
+
+comet_status_t comet_plan_info(comet_plan_t plan, comet_plan_info_t* info) {
+  if (!plan || !info) return fail(COMET_ERR_INVALID_ARG, "NULL pointer argument");
+  const Plan& p = plan->p;
+  info->M = p.M; info->N = p.N; info->K = p.K;
+  info->tile_n = p.tile_n; info->num_ctas = p.num_ctas; info->split_mode = p.split_mode;
+  info->stages = p.stages;
+  info->n_tiles = p.n_tiles;
+  info->n_items = (int64_t)p.items.size();
+  info->n_split_tiles = p.n_split_tiles;
+  info->max_cta_cost = p.max_cost;
+  info->mean_cta_cost = p.mean_cost;
+  return COMET_OK;
+}
+
+comet_status_t comet_plan_describe(comet_plan_t plan, int32_t* items, int64_t max_items, int64_t* n_items) {
+  if (!plan || !n_items) return fail(COMET_ERR_INVALID_ARG, "NULL pointer argument");
+  const Plan& p = plan->p;
+  int64_t n = 0;
+  for (int c = 0; c < p.num_ctas; ++c) {
+    for (int i = p.cta_begin[c]; i < p.cta_begin[c + 1]; ++i) {
+      if (items && n < max_items) {
+        items[4 * n + 0] = c;
+        items[4 * n + 1] = p.items[i].tile;
+        items[4 * n + 2] = p.items[i].kb_begin;
+        items[4 * n + 3] = p.items[i].kb_end;
+      }
+      ++n;
+    }
+  }
+  *n_items = items ? std::min(n, max_items) : n;
+  return COMET_OK;
+}
+
+comet_status_t comet_w4ax_gemm(comet_plan_t plan, const void* act_packed, const float* act_scales,
+                               const void* w_packed, const float* w_scales, void* y,
+                               comet_dtype_t ydt, int64_t ldy, int32_t* debug_acc,
+                               int32_t* debug_acc_blocks, void* workspace, size_t ws_bytes,
+                               void* stream) {
+  g_launches = 0;
+  if (!plan || !act_packed || !act_scales || !w_packed || !w_scales || !y)
+    return fail(COMET_ERR_INVALID_ARG, "NULL pointer argument");
+  Plan& p = plan->p;
+  if (ydt != COMET_F16 && ydt != COMET_BF16 && ydt != COMET_F32) return fail(COMET_ERR_INVALID_ARG, "bad ydt");
+  const int esz = ydt == COMET_F32 ? 4 : 2;
+  if (ldy < p.N || (ldy * esz) % 16 != 0) return fail(COMET_ERR_MISALIGNED, "ldy must be >= N with ldy*sizeof(y) % 16 == 0");
+  if ((reinterpret_cast<uintptr_t>(act_packed) & 255u) != 0) return fail(COMET_ERR_MISALIGNED, "act_packed must be 256-byte aligned");
+  if (!aligned16(act_scales) || !aligned16(w_packed) || !aligned16(w_scales) || !aligned16(y) ||
+      (debug_acc && !aligned16(debug_acc)) || (debug_acc_blocks && !aligned16(debug_acc_blocks)) ||
+      (workspace && !aligned16(workspace)))
+    return fail(COMET_ERR_MISALIGNED, "device pointers must be 16-byte aligned");
+  comet_status_t st = check_device();
+  if (st != COMET_OK) return st;
+  int launches = 0;
+  st = launch_gemm(p, act_packed, act_scales, w_packed, w_scales, y, ydt, ldy, debug_acc,
+                   debug_acc_blocks, workspace, ws_bytes, static_cast<cudaStream_t>(stream), &launches);
+  g_launches = launches;
+  return st;
+}
+
+static size_t scratch_layout(const Plan& p, comet_dtype_t xdt, comet_dtype_t ydt, size_t* x_off,
+                             size_t* act_off, size_t* sc_off, size_t* y_off) {
+  comet_act_layout_t L;
+  act_layout(p.M, p.K, &L);
+  size_t off = 0;
+  *x_off = off;
+  off += (size_t)round_up(p.M * p.K * 2, 256);
+  *act_off = off;
+  off += L.total_bytes;
+  *sc_off = off;
+  off += (size_t)round_up((int64_t)(L.nb * L.Mp * 4), 256);
+  *y_off = off;
+  off += (size_t)round_up(p.M * p.N * (ydt == COMET_F32 ? 4 : 2), 256);
+  (void)xdt;
+  return off;
+}
+
+size_t comet_linear_scratch_bytes(comet_plan_t plan, comet_dtype_t xdt, comet_dtype_t ydt) {
+  if (!plan) return 0;
+  size_t a, b, c, d;
+  return scratch_layout(plan->p, xdt, ydt, &a, &b, &c, &d);
+}
+
+comet_status_t comet_w4ax_linear_host(comet_plan_t plan, const void* x_host, comet_dtype_t xdt,
+                                      const void* w_packed, const float* w_scales, void* y_host,
+                                      comet_dtype_t ydt, void* scratch, size_t scratch_bytes,
+                                      void* workspace, size_t ws_bytes, void* stream) {
+  if (!plan || !x_host || !y_host || !scratch) return fail(COMET_ERR_INVALID_ARG, "NULL pointer argument");
+  Plan& p = plan->p;
+  size_t xo, ao, so, yo;
+  size_t need = scratch_layout(p, xdt, ydt, &xo, &ao, &so, &yo);
+  if (scratch_bytes < need) return fail(COMET_ERR_WORKSPACE_TOO_SMALL, "scratch smaller than comet_linear_scratch_bytes");
+  if ((reinterpret_cast<uintptr_t>(scratch) & 255u) != 0) return fail(COMET_ERR_MISALIGNED, "scratch must be 256-byte aligned");
+  uint8_t* s = static_cast<uint8_t*>(scratch);
+  cudaStream_t st_ = static_cast<cudaStream_t>(stream);
+  cudaError_t e = cudaMemcpyAsync(s + xo, x_host, (size_t)(p.M * p.K * 2), cudaMemcpyHostToDevice, st_);
+  if (e != cudaSuccess) return cuda_status(e, "H2D copy");
+  comet_status_t st = comet_quantize_act(s + xo, xdt, p.M, p.K, p.K, p.tags.data(), nullptr, s + ao,
+                                         reinterpret_cast<float*>(s + so), stream);
+  if (st != COMET_OK) return st;
+  int l1 = g_launches;
+  st = comet_w4ax_gemm(plan, s + ao, reinterpret_cast<float*>(s + so), w_packed, w_scales, s + yo, ydt,
+                       p.N, nullptr, nullptr, workspace, ws_bytes, stream);
+  if (st != COMET_OK) return st;
+  int l2 = g_launches;
+  e = cudaMemcpyAsync(y_host, s + yo, (size_t)(p.M * p.N * (ydt == COMET_F32 ? 4 : 2)), cudaMemcpyDeviceToHost, st_);
+  if (e != cudaSuccess) return cuda_status(e, "D2H copy");
+  e = cudaStreamSynchronize(st_);
+  if (e != cudaSuccess) return cuda_status(e, "stream synchronize");
+  g_launches = l1 + l2;
+  return COMET_OK;
+}
+
+}  // extern "C"

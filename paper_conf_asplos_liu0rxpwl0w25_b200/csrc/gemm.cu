@@ -1,0 +1,540 @@
+// gemm.cu -- the W4Ax GEMM on sm_100a (kernel 2), persistent and warp-specialised.
+//
+//   Y[m, n] = s_w[n] * sum_b s_a[m,b] * acc_b[m,n]
+//
+// One CTA per SM walks the planner's work list (tile, K-block range).  An output
+// tile is 128 weight rows (n) x NT tokens (m).  The MMA runs "transposed": the weight tile is
+// the A operand (M = 128 rows, held in TENSOR MEMORY after widening), the activation tile is
+// the B operand (N = NT tokens, TMA-staged in shared memory, 128-byte swizzle), so the tokens
+// become the MMA N dimension and decode-sized M still fills an instruction.
+//
+// Roles (512 threads, 16 warps):
+//   warp 0      TMA producer: activation tile [NT x 128 B], packed weight tile [128 x 64 B]
+//               and the block's scales s_a[b][m0 .. m0+NT) into a STAGES-deep mbarrier ring.
+//   warp 1      MMA issuer (one thread): per K-block 4 x tcgen05.mma (K = 32) into a fresh
+//               TMEM accumulator; INT4 blocks use kind::f8f6f4 (E4M3), INT8 blocks kind::i8.
+//   warp 2      TMEM allocator.
+//   warps 4-7   widen: packed INT4 weight row -> 128 bytes in 3 instructions per 8 values
+//               (the B200 form of the paper's location switch + zero extension),
+//               tcgen05.st into one of two TMEM A buffers.  INT4 block: byte = u = w+8, read by
+//               the FP8 tensor core as u * 2^-9 exactly.  INT8 block: byte = 16*w (s8).
+//   warps 8-15  promotion ("dequant"): per K-block, tcgen05.ld the accumulator and fold
+//               it into FP32 registers with the block's per-token scale (one FFMA2 per two
+//               elements for INT4 blocks, the accumulator is already FP32); at the end of the
+//               tile the FP32 result is scaled by s_w and stored (or, for a tile split across
+//               CTAs, exchanged through the stream-K workspace).
+//
+// Exactness: INT4 block: acc = 2^-9 * sum_k x_k (w_k + 8) with every term an integer multiple
+// of 2^-9 and |sum| < 2^14 -> exact in FP32 (checked bit-exactly against the oracle through the
+// debug accumulators); the +8 offset is removed with corr[m] = 8 sum_b s_a qsum (kernel 1).
+// INT8 block: acc = 16 * sum_k x_k w_k exactly in INT32.
+#include <cudaTypedefs.h>
+#include <cuda_fp16.h>
+#include <cuda_bf16.h>
+#include <algorithm>
+#include "internal.h"
+#include "sm100.cuh"
+
+namespace comet {
+namespace {
+
+using namespace sm100;
+
+constexpr int kThreads = 512;
+constexpr int kSRing = 8;            // scale ring depth
+constexpr uint32_t kAcol = 0;        // TMEM columns [0, 64): two widened-weight A buffers
+constexpr uint32_t kAccCol = 64;     // TMEM columns [64, 64 + 2 NT): two accumulators
+
+struct __align__(64) GemmParams {
+  CUtensorMap map_x;
+  CUtensorMap map_w;
+  const float* scales;       // [nb][Mp]
+  const float* corr;         // [Mp]
+  const int16_t* qsum;       // [nb][Mp]
+  const float* w_scales;     // [N]
+  void* y;
+  int64_t ldy;
+  int32_t* dbg_acc;          // [M][N] or null
+  int32_t* dbg_blocks;       // [nb][M][N] or null
+  float* ws_part;
+  uint32_t* ws_flags;
+  const int32_t* cta_begin;
+  const WorkItem* items;
+  int64_t M, N, Mp;
+  int nb, n_m_tiles, max_seg, ydt;
+  uint32_t epoch;
+  TagMask tags;
+};
+
+template <int NT>
+struct Cfg {
+  static constexpr int ACTIVE_WGS = NT >= 32 ? 2 : 1;          // promotion warpgroups in use
+  static constexpr int COLS = NT / ACTIVE_WGS;                 // accumulator columns per WG
+  static constexpr int X_BYTES = NT * 128;
+  static constexpr int W_BYTES = kTileW * 64;
+  static constexpr int STAGE_BYTES = X_BYTES + W_BYTES;
+  static constexpr int STAGES_RAW = (196 * 1024) / STAGE_BYTES;
+  static constexpr int STAGES = STAGES_RAW > 10 ? 10 : STAGES_RAW;
+  static constexpr int SMEM_DATA = STAGES * STAGE_BYTES + kSRing * NT * 4;
+  static constexpr int N_BARS = 2 * STAGES + 8 + 2 * kSRing;
+  static constexpr int SMEM_BYTES = 1024 + SMEM_DATA + N_BARS * 8 + 16 + kMaxBlocks;
+  static_assert(COLS % 16 == 0, "promotion chunks of 16 columns");
+  static_assert(2 * NT + 64 <= 512, "TMEM budget");
+};
+
+__device__ __forceinline__ void named_bar_sync(int id, int n) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
+}
+__device__ __forceinline__ void st_release_gpu(uint32_t* p, uint32_t v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ uint32_t ld_acquire_gpu(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ float ld_cg_f32(const float* p) {
+  float v;
+  asm volatile("ld.global.cg.f32 %0, [%1];" : "=f"(v) : "l"(p));
+  return v;
+}
+template <uint32_t N>
+__device__ __forceinline__ void setmaxnreg_dec() {
+  asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(N));
+}
+template <uint32_t N>
+__device__ __forceinline__ void setmaxnreg_inc() {
+  asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(N));
+}
+
+__device__ __forceinline__ WorkItem load_item(const GemmParams& P, int idx, bool debug) {
+  if (debug) {
+    WorkItem w{};
+    w.tile = blockIdx.x; w.kb_begin = 0; w.kb_end = P.nb; w.flags = 2; w.fix = -1;
+    return w;
+  }
+  const int4* src = reinterpret_cast<const int4*>(P.items + idx);
+  int4 a = __ldg(src);
+  int4 b = __ldg(src + 1);
+  WorkItem w;
+  w.tile = a.x; w.kb_begin = a.y; w.kb_end = a.z; w.flags = a.w;
+  w.fix = b.x; w.pad0 = b.y; w.pad1 = b.z; w.pad2 = b.w;
+  return w;
+}
+
+template <int NT, int DEBUG>
+__global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ GemmParams P) {
+  using C = Cfg<NT>;
+  constexpr int S = C::STAGES;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
+  uint8_t* sX = smem;
+  uint8_t* sW = sX + S * C::X_BYTES;
+  float* sS = reinterpret_cast<float*>(sW + S * C::W_BYTES);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + C::SMEM_DATA);
+  uint64_t* full = bars;                 // [S]  TMA -> (MMA, widen)
+  uint64_t* empty = bars + S;            // [S]  (MMA commit + 4 widen warps) -> TMA
+  uint64_t* a_full = bars + 2 * S;       // [2]  widen -> MMA
+  uint64_t* a_empty = a_full + 2;        // [2]  MMA commit -> widen
+  uint64_t* acc_full = a_full + 4;       // [2]  MMA commit -> promotion
+  uint64_t* acc_empty = a_full + 6;      // [2]  promotion -> MMA
+  uint64_t* s_full = a_full + 8;         // [kSRing] TMA -> promotion
+  uint64_t* s_empty = s_full + kSRing;   // [kSRing] promotion -> TMA
+  uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bars + C::N_BARS);
+  uint8_t* s_tags = reinterpret_cast<uint8_t*>(tmem_holder + 4);
+
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
+  const bool debug = DEBUG != 0;
+  const int it_begin = debug ? 0 : P.cta_begin[blockIdx.x];
+  const int it_end = debug ? 1 : P.cta_begin[blockIdx.x + 1];
+  const int nb = P.nb;
+
+  if (warp == 0 && lane == 0) {
+    tma_prefetch(&P.map_x);
+    tma_prefetch(&P.map_w);
+    for (int i = 0; i < S; ++i) {
+      mbar_init(&full[i], 1);
+      mbar_init(&empty[i], 1 + 4);
+    }
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&a_full[i], 4);
+      mbar_init(&a_empty[i], 1);
+      mbar_init(&acc_full[i], 1);
+      mbar_init(&acc_empty[i], 4 * C::ACTIVE_WGS);
+    }
+    for (int i = 0; i < kSRing; ++i) {
+      mbar_init(&s_full[i], 1);
+      mbar_init(&s_empty[i], 4 * C::ACTIVE_WGS);
+    }
+    fence_mbar_init();
+  }
+  if (warp == 2) {
+    tmem_alloc<512>(tmem_holder);
+    tmem_relinquish();
+  }
+  for (int i = threadIdx.x; i < nb; i += kThreads) s_tags[i] = P.tags.get(i) ? 1 : 0;
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tbase = *tmem_holder;
+
+  if (warp < 4) {
+    setmaxnreg_dec<40>();
+    if (warp == 0 && lane == 0) {
+      // ------------------------------------------------------------------ TMA producer
+      int stage = 0, ss = 0;
+      uint32_t ph = 0, sph = 0;
+      for (int it = it_begin; it < it_end; ++it) {
+        const WorkItem w = load_item(P, it, debug);
+        const int n_tile = w.tile / P.n_m_tiles, m_tile = w.tile % P.n_m_tiles;
+        const int m0 = m_tile * NT, n0 = n_tile * kTileW;
+        const int64_t srows = min((int64_t)NT, P.Mp - m0);
+        const uint32_t sbytes = (uint32_t)(srows * 4);
+        for (int kb = w.kb_begin; kb < w.kb_end; ++kb) {
+          mbar_wait(&empty[stage], ph ^ 1);
+          mbar_arrive_expect_tx(&full[stage], C::STAGE_BYTES);
+          tma_load_2d(sX + stage * C::X_BYTES, &P.map_x, &full[stage], kb * 128, m0);
+          tma_load_2d(sW + stage * C::W_BYTES, &P.map_w, &full[stage], kb * 64, n0);
+          mbar_wait(&s_empty[ss], sph ^ 1);
+          mbar_arrive_expect_tx(&s_full[ss], sbytes);
+          bulk_load(sS + ss * NT, P.scales + (int64_t)kb * P.Mp + m0, sbytes, &s_full[ss]);
+          if (++stage == S) { stage = 0; ph ^= 1; }
+          if (++ss == kSRing) { ss = 0; sph ^= 1; }
+        }
+      }
+    } else if (warp == 1 && lane == 0) {
+      // ------------------------------------------------------------------ MMA issuer
+      const uint32_t id_f8 = idesc_f8f6f4_e4m3(128, NT);
+      const uint32_t id_i8 = idesc_i8(128, NT);
+      int stage = 0, ab = 0;
+      uint32_t ph = 0, aph = 0, j = 0;
+      for (int it = it_begin; it < it_end; ++it) {
+        const WorkItem w = load_item(P, it, debug);
+        for (int kb = w.kb_begin; kb < w.kb_end; ++kb, ++j) {
+          const uint32_t accb = j & 1, accph = (j >> 1) & 1;
+          mbar_wait(&acc_empty[accb], accph ^ 1);
+          mbar_wait(&full[stage], ph);
+          mbar_wait(&a_full[ab], aph);
+          tc_fence_after();
+          const uint32_t d = tbase + kAccCol + accb * NT;
+          const uint32_t a = tbase + kAcol + ab * 32;
+          const uint32_t sx = smem_u32(sX + stage * C::X_BYTES);
+          if (s_tags[kb]) {
+#pragma unroll
+            for (int k = 0; k < 4; ++k) mma_i8_ts(d, a + 8 * k, sdesc_kmajor_sw128(sx + 32 * k), id_i8, k);
+          } else {
+#pragma unroll
+            for (int k = 0; k < 4; ++k) mma_f8_ts(d, a + 8 * k, sdesc_kmajor_sw128(sx + 32 * k), id_f8, k);
+          }
+          tc_commit(&empty[stage]);
+          tc_commit(&a_empty[ab]);
+          tc_commit(&acc_full[accb]);
+          if (++stage == S) { stage = 0; ph ^= 1; }
+          if (++ab == 2) { ab = 0; aph ^= 1; }
+        }
+      }
+    }
+  } else if (warp < 8) {
+    setmaxnreg_dec<88>();
+    // -------------------------------------------------------------------- widen (W -> TMEM A)
+    const int q = warp & 3;
+    const int r = q * 32 + lane;                  // TMEM lane = weight row within the tile
+    const uint32_t lane_addr = (uint32_t)(q * 32) << 16;
+    int stage = 0, ab = 0;
+    uint32_t ph = 0, aph = 0;
+    for (int it = it_begin; it < it_end; ++it) {
+      const WorkItem w = load_item(P, it, debug);
+      for (int kb = w.kb_begin; kb < w.kb_end; ++kb) {
+        mbar_wait(&full[stage], ph);
+        const uint8_t* wt = sW + stage * C::W_BYTES + r * 64;
+        const int sw = (r >> 1) & 3;              // TMA 64-byte swizzle: chunk ^= row bits [1:2]
+        uint4 c[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) c[j] = *reinterpret_cast<const uint4*>(wt + ((j ^ sw) << 4));
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&empty[stage]);
+        const bool is8 = s_tags[kb] != 0;
+        uint32_t o[32];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const uint32_t pw[4] = {c[j].x, c[j].y, c[j].z, c[j].w};
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            const uint32_t p = pw[i];
+            const int g = j * 4 + i;
+            if (is8) {
+              o[2 * g] = ((p << 4) & 0xF0F0F0F0u) ^ 0x80808080u;
+              o[2 * g + 1] = (p & 0xF0F0F0F0u) ^ 0x80808080u;
+            } else {
+              o[2 * g] = p & 0x0F0F0F0Fu;
+              o[2 * g + 1] = (p >> 4) & 0x0F0F0F0Fu;
+            }
+          }
+        }
+        mbar_wait(&a_empty[ab], aph ^ 1);
+        tc_fence_after();
+        tmem_st32(tbase + kAcol + ab * 32 + lane_addr, o);
+        tmem_wait_st();
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&a_full[ab]);
+        if (++stage == S) { stage = 0; ph ^= 1; }
+        if (++ab == 2) { ab = 0; aph ^= 1; }
+      }
+    }
+  } else {
+    setmaxnreg_inc<192>();
+    // -------------------------------------------------------------------- promotion + epilogue
+    const int pw = warp - 8;
+    const int wg = pw >> 2;
+    const int q = warp & 3;
+    const int r = q * 32 + lane;
+    const uint32_t lane_addr = (uint32_t)(q * 32) << 16;
+    const int col0 = wg * C::COLS;
+    const int n_promo_threads = 128 * C::ACTIVE_WGS;
+    if (wg < C::ACTIVE_WGS) {
+      int ss = 0;
+      uint32_t sph = 0, j = 0;
+      for (int it = it_begin; it < it_end; ++it) {
+        const WorkItem w = load_item(P, it, debug);
+        const int n_tile = w.tile / P.n_m_tiles, m_tile = w.tile % P.n_m_tiles;
+        const int m0 = m_tile * NT, n0 = n_tile * kTileW;
+        const bool owner = (w.flags & 2) != 0;
+        const bool split = (w.flags & 1) != 0;
+        float acc[C::COLS];
+        int32_t dacc[DEBUG ? C::COLS : 1];
+#pragma unroll
+        for (int c = 0; c < C::COLS; ++c) {
+          const int64_t m = m0 + col0 + c;
+          acc[c] = (owner && m < P.Mp) ? -__ldg(P.corr + m) * 0.001953125f : 0.f;   // 2^-9
+          if (DEBUG) dacc[c] = 0;
+        }
+        for (int kb = w.kb_begin; kb < w.kb_end; ++kb, ++j) {
+          const uint32_t accb = j & 1, accph = (j >> 1) & 1;
+          mbar_wait(&s_full[ss], sph);
+          mbar_wait(&acc_full[accb], accph);
+          tc_fence_after();
+          const bool is8 = s_tags[kb] != 0;
+          const float* sc = sS + ss * NT + col0;
+          const uint32_t taddr = tbase + kAccCol + accb * NT + col0 + lane_addr;
+#pragma unroll
+          for (int ch = 0; ch < C::COLS / 16; ++ch) {
+            uint32_t v[16];
+            tmem_ld16(taddr + ch * 16, v);
+            tmem_wait_ld();
+            float s[16];
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+              const float4 t4 = *reinterpret_cast<const float4*>(sc + ch * 16 + 4 * e);
+              s[4 * e] = t4.x; s[4 * e + 1] = t4.y; s[4 * e + 2] = t4.z; s[4 * e + 3] = t4.w;
+            }
+            if (!is8) {
+#pragma unroll
+              for (int e = 0; e < 8; ++e) {
+                const int c = ch * 16 + 2 * e;
+                float2 y2 = ffma2(make_float2(__uint_as_float(v[2 * e]), __uint_as_float(v[2 * e + 1])),
+                                  make_float2(s[2 * e], s[2 * e + 1]), make_float2(acc[c], acc[c + 1]));
+                acc[c] = y2.x;
+                acc[c + 1] = y2.y;
+              }
+            } else {
+#pragma unroll
+              for (int e = 0; e < 16; ++e) {
+                const int c = ch * 16 + e;
+                acc[c] = fmaf(__int2float_rn((int)v[e]), s[e] * 1.220703125e-04f, acc[c]);   // 2^-13
+              }
+            }
+            if (DEBUG) {
+#pragma unroll
+              for (int e = 0; e < 16; ++e) {
+                const int c = ch * 16 + e;
+                const int64_t m = m0 + col0 + c;
+                int32_t ab;
+                if (is8) {
+                  ab = ((int32_t)v[e]) >> 4;
+                } else {
+                  const int qs = (m < P.Mp) ? (int)P.qsum[(int64_t)kb * P.Mp + m] : 0;
+                  ab = (int32_t)(__uint_as_float(v[e]) * 512.f) - 8 * qs;
+                }
+                dacc[c] += ab;
+                if (DEBUG == 2 && m < P.M)
+                  P.dbg_blocks[((int64_t)kb * P.M + m) * P.N + n0 + r] = ab;
+              }
+            }
+          }
+          tc_fence_before();
+          __syncwarp();
+          if (lane == 0) {
+            mbar_arrive(&acc_empty[accb]);
+            mbar_arrive(&s_empty[ss]);
+          }
+          if (++ss == kSRing) { ss = 0; sph ^= 1; }
+        }
+        // ---------------------------------------------------------------- epilogue
+        if (split) {
+          const int seg = (w.flags >> 8) & 0xFF;
+          const int nseg = (w.flags >> 16) & 0xFF;
+          const int64_t part_tile = (int64_t)NT * kTileW;
+          if (!owner) {
+            float* dst = P.ws_part + ((int64_t)w.fix * (P.max_seg - 1) + (seg - 1)) * part_tile;
+#pragma unroll
+            for (int c = 0; c < C::COLS; ++c) dst[(int64_t)(col0 + c) * kTileW + r] = acc[c];
+            __threadfence();
+            named_bar_sync(1, n_promo_threads);
+            if (threadIdx.x == 256) st_release_gpu(P.ws_flags + (int64_t)w.fix * P.max_seg + seg, P.epoch);
+            continue;
+          }
+          if (threadIdx.x == 256) {
+            for (int sgi = 1; sgi < nseg; ++sgi) {
+              const uint32_t* f = P.ws_flags + (int64_t)w.fix * P.max_seg + sgi;
+              uint64_t t0 = globaltimer_ns();
+              while (ld_acquire_gpu(f) != P.epoch) {
+                if (globaltimer_ns() - t0 > COMET_MBAR_TIMEOUT_NS) {
+                  printf("comet: stream-K fix-up timeout (tile %d seg %d)\n", w.tile, sgi);
+                  __trap();
+                }
+              }
+            }
+          }
+          named_bar_sync(1, n_promo_threads);
+          for (int sgi = 1; sgi < nseg; ++sgi) {
+            const float* src = P.ws_part + ((int64_t)w.fix * (P.max_seg - 1) + (sgi - 1)) * part_tile;
+#pragma unroll
+            for (int c = 0; c < C::COLS; ++c) acc[c] += ld_cg_f32(src + (int64_t)(col0 + c) * kTileW + r);
+          }
+        }
+        const int n = n0 + r;
+        const float sw = __ldg(P.w_scales + n) * 512.f;
+#pragma unroll
+        for (int c = 0; c < C::COLS; ++c) {
+          const int64_t m = m0 + col0 + c;
+          if (m < P.M) {
+            const float yv = acc[c] * sw;
+            const int64_t off = m * P.ldy + n;
+            if (P.ydt == COMET_F16) reinterpret_cast<__half*>(P.y)[off] = __float2half_rn(yv);
+            else if (P.ydt == COMET_BF16) reinterpret_cast<__nv_bfloat16*>(P.y)[off] = __float2bfloat16_rn(yv);
+            else reinterpret_cast<float*>(P.y)[off] = yv;
+            if (DEBUG) P.dbg_acc[m * P.N + n] = dacc[c];
+          }
+        }
+      }
+    }
+  }
+
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 2) tmem_dealloc<512>(tbase);
+}
+
+// ------------------------------------------------------------------------------ host side
+PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  if (!fn) {
+    cudaDriverEntryPointQueryResult q;
+    void* p = nullptr;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+  }
+  return fn;
+}
+
+bool make_map_2d(CUtensorMap* map, const void* base, uint64_t inner, uint64_t outer,
+                 uint64_t row_bytes, uint32_t box_inner, uint32_t box_outer,
+                 CUtensorMapSwizzle swz) {
+  auto fn = encode_fn();
+  if (!fn) return false;
+  cuuint64_t dims[2] = {inner, outer};
+  cuuint64_t strides[1] = {row_bytes};
+  cuuint32_t box[2] = {box_inner, box_outer};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = fn(map, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, const_cast<void*>(base), dims, strides, box,
+                  estr, CU_TENSOR_MAP_INTERLEAVE_NONE, swz, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                  CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS;
+}
+
+template <int NT, int DEBUG>
+cudaError_t launch_nt(const GemmParams& prm, int grid, cudaStream_t stream) {
+  using C = Cfg<NT>;
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(k_w4ax<NT, DEBUG>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_BYTES);
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  k_w4ax<NT, DEBUG><<<grid, kThreads, C::SMEM_BYTES, stream>>>(prm);
+  return cudaGetLastError();
+}
+
+}  // namespace
+
+comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_scales,
+                           const void* w_packed, const float* w_scales, void* y,
+                           comet_dtype_t ydt, int64_t ldy, int32_t* debug_acc,
+                           int32_t* debug_acc_blocks, void* workspace, size_t ws_bytes,
+                           cudaStream_t stream, int* launches) {
+  *launches = 0;
+  const bool dbg = debug_acc != nullptr || debug_acc_blocks != nullptr;
+  const int NT = dbg ? 64 : p.tile_n;
+  comet_act_layout_t L;
+  act_layout(p.M, p.K, &L);
+  const uint8_t* base = static_cast<const uint8_t*>(act_packed);
+  GemmParams prm;
+  memset(&prm, 0, sizeof(prm));
+  if (!make_map_2d(&prm.map_x, base + L.codes_off, (uint64_t)p.K, (uint64_t)p.M, (uint64_t)p.K, 128,
+                   (uint32_t)NT, CU_TENSOR_MAP_SWIZZLE_128B))
+    return fail(COMET_ERR_CUDA, "cuTensorMapEncodeTiled failed for the activation codes");
+  if (!make_map_2d(&prm.map_w, w_packed, (uint64_t)(p.K / 2), (uint64_t)p.N, (uint64_t)(p.K / 2), 64,
+                   (uint32_t)kTileW, CU_TENSOR_MAP_SWIZZLE_64B))
+    return fail(COMET_ERR_CUDA, "cuTensorMapEncodeTiled failed for the packed weights");
+  prm.scales = act_scales;
+  prm.corr = reinterpret_cast<const float*>(base + L.corr_off);
+  prm.qsum = reinterpret_cast<const int16_t*>(base + L.qsum_off);
+  prm.w_scales = w_scales;
+  prm.y = y;
+  prm.ldy = ldy;
+  prm.dbg_acc = debug_acc;
+  prm.dbg_blocks = debug_acc_blocks;
+  prm.M = p.M;
+  prm.N = p.N;
+  prm.Mp = L.Mp;
+  prm.nb = (int)p.nb;
+  prm.ydt = (int)ydt;
+  prm.tags = p.mask;
+  cudaError_t e;
+  if (dbg) {
+    // whole tiles, one CTA each, NT = 64 (debug accumulators need the extra registers)
+    prm.n_m_tiles = (int)ceil_div(p.M, 64);
+    const int grid = (int)(prm.n_m_tiles * (p.N / kTileW));
+    prm.max_seg = 1;
+    e = debug_acc_blocks ? launch_nt<64, 2>(prm, grid, stream) : launch_nt<64, 1>(prm, grid, stream);
+  } else {
+    if (p.d_items == nullptr) return fail(COMET_ERR_INVALID_ARG, "plan was created with device_plan = 0");
+    if (p.ws_bytes > 0 && (workspace == nullptr || ws_bytes < p.ws_bytes))
+      return fail(COMET_ERR_WORKSPACE_TOO_SMALL, "workspace smaller than the plan's workspace_bytes");
+    prm.n_m_tiles = (int)p.n_m_tiles;
+    prm.cta_begin = p.d_cta_begin;
+    prm.items = p.d_items;
+    prm.max_seg = p.max_segments;
+    prm.ws_part = static_cast<float*>(workspace);
+    prm.ws_flags = reinterpret_cast<uint32_t*>(static_cast<uint8_t*>(workspace) + p.ws_flags_off);
+    prm.epoch = ++p.epoch;
+    const int grid = p.num_ctas;
+    switch (NT) {
+      case 16: e = launch_nt<16, 0>(prm, grid, stream); break;
+      case 32: e = launch_nt<32, 0>(prm, grid, stream); break;
+      case 64: e = launch_nt<64, 0>(prm, grid, stream); break;
+      case 128: e = launch_nt<128, 0>(prm, grid, stream); break;
+      case 192: e = launch_nt<192, 0>(prm, grid, stream); break;
+      case 224: e = launch_nt<224, 0>(prm, grid, stream); break;
+      default: return fail(COMET_ERR_UNSUPPORTED_SHAPE, "unsupported tile_n");
+    }
+  }
+  if (e != cudaSuccess) return cuda_status(e, "w4ax gemm launch");
+  *launches = 1;
+  return COMET_OK;
+}
+
+}  // namespace comet

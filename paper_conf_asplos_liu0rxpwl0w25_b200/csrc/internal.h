@@ -1,0 +1,82 @@
+// internal.h -- declarations shared by the libcomet.so translation units (not part of the ABI).
+#pragma once
+#include <cstdint>
+#include <cstddef>
+#include <string>
+#include <vector>
+#include <atomic>
+#include <cuda_runtime.h>
+
+#include "../../include/comet.h"
+
+namespace comet {
+
+constexpr int kBlockK = 128;       // FMPQ block
+constexpr int kTileW = 128;        // weight rows per output tile = MMA M (one CTA, cta_group::1)
+constexpr int kMaxBlocks = 1024;   // K <= 131072
+
+// 1024-bit tag mask passed by value to kernels.
+struct TagMask {
+  uint32_t w[kMaxBlocks / 32];
+  __host__ __device__ bool get(int b) const { return (w[b >> 5] >> (b & 31)) & 1u; }
+};
+
+inline int64_t round_up(int64_t a, int64_t b) { return (a + b - 1) / b * b; }
+inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+// Work item of the persistent GEMM: one output tile, a half-open K-block range.
+// flags: bit0 = tile is split across CTAs, bit1 = this item owns the tile (holds kb 0, does
+// the fix-up and the store); bits 8..15 = segment index within the tile (0 = owner);
+// bits 16..23 = number of segments of the tile.  fix = index of the tile among split tiles.
+struct WorkItem {
+  int32_t tile, kb_begin, kb_end, flags;
+  int32_t fix, pad0, pad1, pad2;
+};
+static_assert(sizeof(WorkItem) == 32, "work item layout");
+
+struct Plan {
+  int64_t M, N, K, nb, Mp;
+  int tile_n, num_ctas, split_mode, stages;
+  int64_t n_m_tiles, n_n_tiles, n_tiles;
+  std::vector<uint8_t> tags;
+  TagMask mask;
+  std::vector<int32_t> cta_begin;       // [num_ctas + 1] offsets into items
+  std::vector<WorkItem> items;
+  int64_t n_split_tiles = 0;
+  int max_segments = 1;
+  double max_cost = 0, mean_cost = 0;
+  // device copies
+  int32_t* d_cta_begin = nullptr;
+  WorkItem* d_items = nullptr;
+  size_t ws_bytes = 0;                  // stream-K partials + flags
+  size_t ws_flags_off = 0;
+  std::atomic<uint32_t> epoch{0};
+  int device = -1;
+};
+
+// thread-local error detail
+void set_error(const std::string& msg);
+comet_status_t fail(comet_status_t st, const std::string& msg);
+comet_status_t cuda_status(cudaError_t e, const char* what);
+void note_launches(int n);
+
+// planner.cpp
+comet_status_t build_plan(Plan& p, const comet_sched_config& cfg);
+
+// quantize.cu
+cudaError_t launch_quantize(const void* x, bool bf16, int64_t M, int64_t K, int64_t ldx,
+                            const TagMask& tags, void* act_packed, float* act_scales,
+                            cudaStream_t stream, int* launches);
+// pack.cu
+cudaError_t launch_pack_weight(const int8_t* w, int64_t N, int64_t K, void* w_packed,
+                               cudaStream_t stream);
+// gemm.cu
+comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_scales,
+                           const void* w_packed, const float* w_scales, void* y,
+                           comet_dtype_t ydt, int64_t ldy, int32_t* debug_acc,
+                           int32_t* debug_acc_blocks, void* workspace, size_t ws_bytes,
+                           cudaStream_t stream, int* launches);
+// act layout
+void act_layout(int64_t M, int64_t K, comet_act_layout_t* out);
+
+}  // namespace comet

@@ -1,0 +1,228 @@
+// quantize.cu -- kernel 1: FMPQ activation quantisation and the mixed-precision packed layout.
+//
+// Per (token m, 128-channel block b) (P:L136 blocks of k = 128 channels along the channel
+// dimension; P:L138 outlier blocks -> 8 bit, the rest 4 bit; P:L126 min-max; reading R1-R5):
+//   amax = max |x|, qmax = tags[b] ? 127 : 7, s = amax/qmax, r = qmax/amax (IEEE binary32,
+//   correctly rounded: __fdiv_rn), q = clamp(rint(x*r)) with x*r one binary32 product
+//   (__fmul_rn, never contracted) and rint = round-half-even (cvt.rni; NaN -> 0).
+// Layout written (include/comet.h): codes[M][K] bytes (E4M3 of q for INT4 blocks, s8 for INT8
+// blocks), scales[nb][Mp], qsum[nb][Mp] (int16), corr[Mp].
+//
+// HBM-bound: a block-row (128 halves = 256 B) is read by 16 lanes with one 128-bit load each;
+// block max-abs and code sum are 4-step xor-shuffle reductions inside the half-warp; codes
+// leave as one 64-bit store per lane.  A warp handles two blocks per step (one per half).
+#include <cuda_fp16.h>
+#include <cuda_bf16.h>
+#include "internal.h"
+
+namespace comet {
+namespace {
+
+__device__ __forceinline__ uint4 ldg_stream(const void* p) {
+  uint4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+               : "l"(p));
+  return r;
+}
+
+template <bool BF16>
+__device__ __forceinline__ void unpack8(const uint4& raw, float (&v)[8]) {
+  const uint32_t w[4] = {raw.x, raw.y, raw.z, raw.w};
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    if (BF16) {
+      v[2 * i] = __uint_as_float(w[i] << 16);
+      v[2 * i + 1] = __uint_as_float(w[i] & 0xFFFF0000u);
+    } else {
+      __half2 h = *reinterpret_cast<const __half2*>(&w[i]);
+      float2 f = __half22float2(h);
+      v[2 * i] = f.x;
+      v[2 * i + 1] = f.y;
+    }
+  }
+}
+
+// E4M3 byte of an integer q in [-7, 7]: |q| -> {00,38,40,44,48,4A,4C,4E}, sign in bit 7.
+__device__ __forceinline__ uint32_t e4m3_of_int4(int q) {
+  const uint32_t a = (uint32_t)(q < 0 ? -q : q);
+  const uint32_t e = __byte_perm(0x44403800u, 0x4E4C4A48u, a) & 0xFFu;
+  return e | (q < 0 ? 0x80u : 0u);
+}
+
+struct BlockOut {
+  uint32_t lo, hi;   // 8 code bytes
+  float s;
+  int q;             // code sum (full after the reduction)
+};
+
+// Quantise the 8 values of this lane for block b (16 lanes cooperate on 128 values).
+__device__ __forceinline__ BlockOut quantize8(const float (&v)[8], bool is8) {
+  float a = 0.f;
+#pragma unroll
+  for (int j = 0; j < 8; ++j) a = fmaxf(a, fabsf(v[j]));
+  a = fmaxf(a, __shfl_xor_sync(0xffffffffu, a, 8));
+  a = fmaxf(a, __shfl_xor_sync(0xffffffffu, a, 4));
+  a = fmaxf(a, __shfl_xor_sync(0xffffffffu, a, 2));
+  a = fmaxf(a, __shfl_xor_sync(0xffffffffu, a, 1));
+  const float qmax = is8 ? 127.f : 7.f;
+  const int iq = is8 ? 127 : 7;
+  BlockOut o;
+  o.s = (a == 0.f) ? 0.f : __fdiv_rn(a, qmax);
+  const float r = __fdiv_rn(qmax, a);          // +inf for an all-zero block -> t NaN -> code 0
+  uint32_t bytes[8];
+  int qs = 0;
+#pragma unroll
+  for (int j = 0; j < 8; ++j) {
+    const float t = __fmul_rn(v[j], r);
+    int q = __float2int_rn(t);                  // cvt.rni.s32.f32: half-even, NaN -> 0, saturating
+    q = min(max(q, -iq), iq);
+    qs += q;
+    bytes[j] = is8 ? ((uint32_t)q & 0xFFu) : e4m3_of_int4(q);
+  }
+  o.lo = bytes[0] | (bytes[1] << 8) | (bytes[2] << 16) | (bytes[3] << 24);
+  o.hi = bytes[4] | (bytes[5] << 8) | (bytes[6] << 16) | (bytes[7] << 24);
+  qs += __shfl_xor_sync(0xffffffffu, qs, 8);
+  qs += __shfl_xor_sync(0xffffffffu, qs, 4);
+  qs += __shfl_xor_sync(0xffffffffu, qs, 2);
+  qs += __shfl_xor_sync(0xffffffffu, qs, 1);
+  o.q = qs;
+  return o;
+}
+
+// WPR warps cooperate on one token row; a CTA of 8 warps covers 8/WPR rows.
+template <bool BF16, int WPR>
+__global__ void __launch_bounds__(256) k_quantize(const uint16_t* __restrict__ x, int64_t M,
+                                                  int64_t K, int64_t ldx, int64_t Mp, TagMask tags,
+                                                  uint8_t* __restrict__ codes,
+                                                  int16_t* __restrict__ qsum,
+                                                  float* __restrict__ corr,
+                                                  float* __restrict__ scales) {
+  constexpr int ROWS = 8 / WPR;
+  __shared__ float s_part[8][2];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int row_in_cta = warp / WPR, wi = warp % WPR;
+  const int64_t m = (int64_t)blockIdx.x * ROWS + row_in_cta;
+  const int half = lane >> 4, sub = lane & 15;
+  const int nb = (int)(K / kBlockK);
+  const int npairs = (nb + 1) / 2;
+  float cpart = 0.f;   // sum over this half's INT4 blocks of s * qsum (binary32)
+  if (m < Mp) {
+    const bool live = m < M;
+    const uint16_t* xrow = x + (live ? m : 0) * ldx;
+    uint8_t* crow = codes + (live ? m : 0) * K;
+    constexpr int U = 2;   // pairs in flight per warp
+    for (int p0 = wi; p0 < npairs; p0 += WPR * U) {
+      uint4 raw[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const int b = (p0 + u * WPR) * 2 + half;
+        raw[u] = make_uint4(0, 0, 0, 0);
+        if (live && (p0 + u * WPR) < npairs && b < nb)
+          raw[u] = ldg_stream(xrow + (int64_t)b * kBlockK + sub * 8);
+      }
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const int pp = p0 + u * WPR;
+        if (pp >= npairs) break;                 // warp-uniform
+        const int b = pp * 2 + half;
+        const bool bvalid = b < nb;
+        float v[8];
+        unpack8<BF16>(raw[u], v);
+        const bool is8 = bvalid ? tags.get(b) : false;
+        BlockOut o = quantize8(v, is8);
+        if (bvalid) {
+          if (live)
+            *reinterpret_cast<uint2*>(crow + (int64_t)b * kBlockK + sub * 8) = make_uint2(o.lo, o.hi);
+          if (sub == 0) {
+            scales[(int64_t)b * Mp + m] = o.s;
+            qsum[(int64_t)b * Mp + m] = (int16_t)o.q;
+            if (!is8) cpart = __fadd_rn(cpart, __fmul_rn(o.s, (float)o.q));
+          }
+        }
+      }
+    }
+  }
+  if (sub == 0) s_part[warp][half] = cpart;
+  __syncthreads();
+  if (wi == 0 && lane == 0 && m < Mp) {
+    float c = 0.f;
+    for (int i = 0; i < WPR; ++i) {
+      c = __fadd_rn(c, s_part[row_in_cta * WPR + i][0]);
+      c = __fadd_rn(c, s_part[row_in_cta * WPR + i][1]);
+    }
+    corr[m] = __fmul_rn(8.f, c);
+  }
+}
+
+template <bool BF16>
+cudaError_t launch_q(const void* x, int64_t M, int64_t K, int64_t ldx, const TagMask& tags,
+                     void* act_packed, float* act_scales, cudaStream_t stream) {
+  comet_act_layout_t L;
+  act_layout(M, K, &L);
+  uint8_t* base = static_cast<uint8_t*>(act_packed);
+  uint8_t* codes = base + L.codes_off;
+  int16_t* qsum = reinterpret_cast<int16_t*>(base + L.qsum_off);
+  float* corr = reinterpret_cast<float*>(base + L.corr_off);
+  const int64_t Mp = L.Mp;
+  const int64_t nb = L.nb;
+  const int64_t target = 2 * 148;
+  int wpr = 1;
+  if (Mp / 8 < target) wpr = 2;
+  if (Mp / 4 < target) wpr = 4;
+  if (Mp / 2 < target) wpr = 8;
+  while (wpr > 1 && (nb + 1) / 2 < wpr) wpr /= 2;
+  const int rows = 8 / wpr;
+  const dim3 grid((unsigned)ceil_div(Mp, rows));
+  const uint16_t* xp = static_cast<const uint16_t*>(x);
+  switch (wpr) {
+    case 1: k_quantize<BF16, 1><<<grid, 256, 0, stream>>>(xp, M, K, ldx, Mp, tags, codes, qsum, corr, act_scales); break;
+    case 2: k_quantize<BF16, 2><<<grid, 256, 0, stream>>>(xp, M, K, ldx, Mp, tags, codes, qsum, corr, act_scales); break;
+    case 4: k_quantize<BF16, 4><<<grid, 256, 0, stream>>>(xp, M, K, ldx, Mp, tags, codes, qsum, corr, act_scales); break;
+    default: k_quantize<BF16, 8><<<grid, 256, 0, stream>>>(xp, M, K, ldx, Mp, tags, codes, qsum, corr, act_scales); break;
+  }
+  return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------------------- weight packing
+// u = w + 8 = (w & 0xF) ^ 8 per nibble; word byte i = u[i] | u[i+4] << 4 (include/comet.h).
+__global__ void __launch_bounds__(256) k_pack_weight(const uint2* __restrict__ w, int64_t words,
+                                                     uint32_t* __restrict__ out) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < words;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const uint2 v = w[i];
+    const uint32_t lo = (v.x & 0x0F0F0F0Fu) ^ 0x08080808u;   // u[k0..k3]
+    const uint32_t hi = (v.y & 0x0F0F0F0Fu) ^ 0x08080808u;   // u[k4..k7]
+    out[i] = lo | (hi << 4);
+  }
+}
+
+}  // namespace
+
+void act_layout(int64_t M, int64_t K, comet_act_layout_t* L) {
+  L->nb = K / kBlockK;
+  L->Mp = round_up(M, COMET_SCALE_PAD);
+  L->codes_off = 0;
+  L->qsum_off = (size_t)round_up(M * K, 256);
+  L->corr_off = (size_t)round_up((int64_t)L->qsum_off + L->nb * L->Mp * 2, 256);
+  L->total_bytes = (size_t)round_up((int64_t)L->corr_off + L->Mp * 4, 256);
+}
+
+cudaError_t launch_quantize(const void* x, bool bf16, int64_t M, int64_t K, int64_t ldx,
+                            const TagMask& tags, void* act_packed, float* act_scales,
+                            cudaStream_t stream, int* launches) {
+  *launches = 1;
+  return bf16 ? launch_q<true>(x, M, K, ldx, tags, act_packed, act_scales, stream)
+              : launch_q<false>(x, M, K, ldx, tags, act_packed, act_scales, stream);
+}
+
+cudaError_t launch_pack_weight(const int8_t* w, int64_t N, int64_t K, void* w_packed,
+                               cudaStream_t stream) {
+  const int64_t words = N * K / 8;
+  const int64_t blocks = std::min<int64_t>(ceil_div(words, 256), 148 * 16);
+  k_pack_weight<<<(unsigned)blocks, 256, 0, stream>>>(reinterpret_cast<const uint2*>(w), words,
+                                                        static_cast<uint32_t*>(w_packed));
+  return cudaGetLastError();
+}
+
+}  // namespace comet

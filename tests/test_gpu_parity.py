@@ -1,0 +1,233 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle on the same seeded
+inputs.  Codes, tags, scales, qsum, weight packing and the INT32 debug accumulators are
+compared bit-exactly; the dequantised output within the north-star tolerance
+(rtol 1e-3 / atol 1e-2 for FP16/FP32 outputs, 1 BF16 ulp for BF16 outputs, R10)."""
+import numpy as np
+import pytest
+
+import oracle
+from paper_conf_asplos_liu0rxpwl0w25_b200 import synth
+from _layout import decode_act, unpack_weight
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+if not torch.cuda.is_available():
+    pytest.skip("no CUDA device", allow_module_level=True)
+
+import paper_conf_asplos_liu0rxpwl0w25_b200 as cb   # noqa: E402
+
+DEV = "cuda:0"
+
+
+def _x_dev(p: synth.Problem):
+    if p.bf16:
+        return torch.from_numpy(p.x.view(np.int16)).to(DEV).view(torch.bfloat16)
+    return torch.from_numpy(p.x).to(DEV)
+
+
+def _quant(p: synth.Problem):
+    act, sc = cb.quantize_act(_x_dev(p), p.tags)
+    torch.cuda.synchronize()
+    return act, sc
+
+
+def _check_quant(p, act, sc, rows=None):
+    codes, scales, qsum, corr = decode_act(act.cpu().numpy(), sc.cpu().numpy(), p.M, p.K, p.tags)
+    if rows is None:
+        ref_codes, ref_scales = oracle.quantize(p.x, p.tags, bf16_bits=p.bf16)
+        rows = np.arange(p.M)
+    else:
+        _, _, ref_codes, ref_scales = oracle.w4ax_rows(p.x, p.tags, np.zeros((128, p.K), np.int8),
+                                                       np.ones(128, np.float32), rows, bf16_bits=p.bf16)
+    assert np.array_equal(codes[rows], ref_codes), "codes differ"
+    assert np.array_equal(scales[rows].view(np.uint32), ref_scales.view(np.uint32)), "scales differ"
+    nb = p.K // 128
+    ref_q = ref_codes.reshape(len(rows), nb, 128).astype(np.int64).sum(2)
+    assert np.array_equal(qsum[:, rows].T.astype(np.int64), ref_q), "qsum differs"
+    Mp = qsum.shape[1]
+    assert np.all(qsum[:, p.M:] == 0) and np.all(sc.cpu().numpy().reshape(nb, Mp)[:, p.M:] == 0)
+    # corr = 8 sum_{INT4 blocks} s q  (binary32 sum; compare with the exact value)
+    terms = 8.0 * ref_scales.astype(np.float64) * ref_q * (p.tags == 0)[None, :]
+    # binary32 summation: error bounded by ~nb ulps of the running magnitude
+    bound = np.abs(terms).sum(1) * nb * 2.0 ** -23 + 1e-30
+    assert np.all(np.abs(corr[rows] - terms.sum(1)) <= bound)
+    return codes
+
+
+# ------------------------------------------------------------------------------- kernel 1
+
+@pytest.mark.parametrize("M,K,frac,bf16", [
+    (16, 256, None, False),            # config 1
+    (1, 4096, 0.05, False), (16, 4096, 0.05, False), (256, 11008, 0.05, False),   # config 2
+    (33, 1024, 0.5, True), (1000, 512, 0.25, False), (7, 14336, 0.05, True),
+])
+def test_quantize_parity(M, K, frac, bf16):
+    if frac is None:
+        p = synth.config1()
+    else:
+        p = synth.make_problem(M, K, 128, frac=frac, seed=M + K, bf16=bf16)
+    act, sc = _quant(p)
+    _check_quant(p, act, sc)
+
+
+def test_quantize_edge_cases():
+    # zero blocks, ties, bf16 binary32-subnormal block, all-INT8 and all-INT4
+    x = np.zeros((3, 512), np.float16)
+    x[1, :6] = [7.0, 2.5, 3.5, -2.5, -0.5, 1.5]
+    x[2, 128:256] = -1.0
+    x[2, 300] = 65504.0
+    for tags in (np.array([0, 1, 0, 1], np.uint8), np.zeros(4, np.uint8), np.ones(4, np.uint8)):
+        p = synth.Problem(x=x, tags=tags, w=np.zeros((128, 512), np.int8), s_w=np.ones(128, np.float32))
+        act, sc = _quant(p)
+        _check_quant(p, act, sc)
+    xb = np.zeros((2, 128), np.uint16)
+    xb[0, 0], xb[0, 1], xb[1, 5] = 0x0001, 0x8001, 0x3F80
+    p = synth.Problem(x=xb, tags=np.array([0], np.uint8), w=np.zeros((128, 128), np.int8),
+                      s_w=np.ones(128, np.float32), bf16=True)
+    act, sc = _quant(p)
+    _check_quant(p, act, sc)
+
+
+def test_quantize_full_size_sampled():
+    """LLaMA-3-8B down input at M=8192, K=14336 (config 3): sampled rows vs the oracle."""
+    p = synth.make_problem(8192, 14336, 128, frac=0.05, seed=3)
+    act, sc = _quant(p)
+    rows = synth.sample_rows(p.M, 24, p.x)
+    _check_quant(p, act, sc, rows=rows)
+
+
+# ------------------------------------------------------------------------------- weight pack
+
+@pytest.mark.parametrize("N,K", [(128, 128), (256, 4096), (1280, 8192)])
+def test_pack_weight_layout(N, K):
+    rng = np.random.default_rng(N + K)
+    w = rng.integers(-8, 8, size=(N, K), dtype=np.int8)
+    wp = cb.pack_weight(torch.from_numpy(w).to(DEV))
+    torch.cuda.synchronize()
+    assert np.array_equal(unpack_weight(wp.cpu().numpy(), N, K), w)
+
+
+# ------------------------------------------------------------------------------- GEMM
+
+def _run(p: synth.Problem, *, tile_n=0, split_mode=-1, out_dtype=torch.float32, debug=False,
+         debug_blocks=False, num_sms=0):
+    act, sc = _quant(p)
+    wp = cb.pack_weight(torch.from_numpy(p.w).to(DEV))
+    sw = torch.from_numpy(p.s_w).to(DEV)
+    plan = cb.Plan(p.M, p.N, p.K, p.tags, tile_n=tile_n, split_mode=split_mode, num_sms=num_sms)
+    res = cb.w4ax_gemm(plan, act, sc, wp, sw, out_dtype=out_dtype, debug=debug, debug_blocks=debug_blocks)
+    torch.cuda.synchronize()
+    return res, plan
+
+
+def _close(y, ref, dtype):
+    if dtype == torch.bfloat16:
+        got = y.float().cpu().numpy()
+        r = torch.from_numpy(ref).to(torch.bfloat16).float().numpy()
+        ulp = np.abs(r) * 2.0 ** -7 + 1e-30
+        assert np.all(np.abs(got - r) <= ulp * 1.0001 + 1e-6), "bf16 output off by more than 1 ulp"
+    else:
+        got = y.float().cpu().numpy().astype(np.float64)
+        bad = ~np.isclose(got, ref, rtol=1e-3, atol=1e-2)
+        assert not bad.any(), f"{bad.sum()} outputs outside rtol 1e-3 / atol 1e-2; max err {np.abs(got-ref).max()}"
+
+
+def test_gemm_config1_bit_exact_blocks():
+    p = synth.config1()
+    (y, dacc, dblk), _ = _run(p, debug_blocks=True)
+    yref, acc, _, _ = oracle.w4ax(p.x, p.tags, p.w, p.s_w)
+    assert np.array_equal(dblk.cpu().numpy().astype(np.int64), acc), "per-block INT32 accumulators differ"
+    assert np.array_equal(dacc.cpu().numpy().astype(np.int64), acc.sum(0))
+    _close(y, yref, torch.float32)
+
+
+@pytest.mark.parametrize("M,N,K,frac", [
+    (1, 256, 512, 0.5), (17, 384, 1024, 0.25), (100, 512, 2048, 0.05), (300, 256, 768, 1.0),
+    (64, 128, 256, 0.0),
+])
+def test_gemm_debug_accumulators_exact(M, N, K, frac):
+    p = synth.make_problem(M, K, N, frac=frac, seed=M * 7 + K)
+    (y, dacc), _ = _run(p, debug=True)
+    yref, acc, _, _ = oracle.w4ax(p.x, p.tags, p.w, p.s_w)
+    assert np.array_equal(dacc.cpu().numpy().astype(np.int64), acc.sum(0))
+    _close(y, yref, torch.float32)
+
+
+def test_gemm_all_int8_matches_torch_int_mm():
+    """I1 on the GPU: all tags INT8 -> per-block accumulators equal cuBLASLt's INT8 GEMM."""
+    p = synth.make_problem(64, 512, 256, frac=1.0, seed=5)
+    (y, dacc, dblk), _ = _run(p, debug_blocks=True)
+    codes, _ = oracle.quantize(p.x, p.tags)
+    for b in range(4):
+        a = torch.from_numpy(codes[:, b * 128:(b + 1) * 128].copy()).to(DEV)
+        w = torch.from_numpy(p.w[:, b * 128:(b + 1) * 128].copy()).to(DEV)
+        ref = torch._int_mm(a, w.t().contiguous())
+        assert torch.equal(dblk[b], ref)
+
+
+@pytest.mark.parametrize("tile_n", [16, 32, 64, 128, 192, 224])
+@pytest.mark.parametrize("split_mode", [0, 1])
+def test_gemm_tile_and_schedule_variants(tile_n, split_mode):
+    p = synth.make_problem(230, 2048, 1024, frac=0.25, seed=tile_n)
+    y, plan = _run(p, tile_n=tile_n, split_mode=split_mode, num_sms=37)
+    yref, _, _, _ = oracle.w4ax(p.x, p.tags, p.w, p.s_w)
+    _close(y, yref, torch.float32)
+
+
+@pytest.mark.parametrize("split_mode", [2, 3])
+def test_gemm_unit_schedules(split_mode):
+    p = synth.make_problem(96, 512, 1024, frac=0.25, seed=11)
+    y, plan = _run(p, split_mode=split_mode, num_sms=13)
+    assert plan.info()["n_split_tiles"] > 0
+    yref, _, _, _ = oracle.w4ax(p.x, p.tags, p.w, p.s_w)
+    _close(y, yref, torch.float32)
+
+
+@pytest.mark.parametrize("dtype", [torch.float16, torch.bfloat16, torch.float32])
+def test_gemm_output_dtypes(dtype):
+    p = synth.make_problem(48, 1024, 512, frac=0.25, seed=21)
+    y, _ = _run(p, out_dtype=dtype)
+    yref, _, _, _ = oracle.w4ax(p.x, p.tags, p.w, p.s_w)
+    _close(y, yref, dtype)
+
+
+@pytest.mark.parametrize("frac", [0.0, 0.05, 0.25, 1.0])
+def test_gemm_outlier_fraction_sweep(frac):
+    """Config 3's sweep shape class at reduced M (full size is in test_gemm_full_size)."""
+    p = synth.make_problem(200, 4096, 1024, frac=frac, seed=31)
+    y, _ = _run(p)
+    yref, _, _, _ = oracle.w4ax(p.x, p.tags, p.w, p.s_w)
+    _close(y, yref, torch.float32)
+
+
+def test_gemm_bf16_input():
+    p = synth.make_problem(40, 1024, 384, frac=0.34, seed=41, bf16=True)
+    (y, dacc), _ = _run(p, debug=True)
+    yref, acc, _, _ = oracle.w4ax(p.x, p.tags, p.w, p.s_w, bf16_bits=True)
+    assert np.array_equal(dacc.cpu().numpy().astype(np.int64), acc.sum(0))
+    _close(y, yref, torch.float32)
+
+
+FULL = [
+    ("l2_7b_qkvo_m1", 1, 4096, 4096, 0.05),
+    ("l2_7b_gateup_m16", 16, 4096, 11008, 0.05),
+    ("l2_7b_down_m256", 256, 11008, 4096, 0.05),
+    ("l2_7b_qkvo_m4096", 4096, 4096, 4096, 0.05),
+    ("l3_8b_down_m8192", 8192, 14336, 4096, 0.05),
+    ("l3_70b_gateup_m4096", 4096, 8192, 28672, 0.05),
+    ("l3_70b_down_m4096", 4096, 28672, 8192, 0.05),
+    ("l3_70b_qkv_m4096", 4096, 8192, 10240, 0.05),
+    ("l3_70b_gateup_tp8_m32", 32, 8192, 3584, 0.05),
+    ("l3_70b_down_tp8_m1", 1, 3584, 8192, 0.05),
+]
+
+
+@pytest.mark.parametrize("name,M,K,N,frac", FULL, ids=[f[0] for f in FULL])
+def test_gemm_full_size(name, M, K, N, frac):
+    """BASELINE sizes, the bench's launch configuration (auto plan), sampled rows vs oracle."""
+    p = synth.make_problem(M, K, N, frac=frac, seed=sum(map(ord, name)))
+    y, plan = _run(p, out_dtype=torch.float16)
+    rows = synth.sample_rows(M, 8, p.x)
+    yref, acc_sum, codes, scales = oracle.w4ax_rows(p.x, p.tags, p.w, p.s_w, rows)
+    _close(y[torch.from_numpy(rows).to(DEV)], yref, torch.float16)
