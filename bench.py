@@ -1,0 +1,401 @@
+#!/usr/bin/env python
+"""bench.py -- W4Ax GEMM TOPS on LLaMA-3-70B prefill layers (BASELINE.json config 4).
+
+One step = one pass of the whole hot path over one batch of synthetic input: for each of the
+three LLaMA-3-70B linear layers (gate/up 8192->28672, down 28672->8192, qkv 8192->10240) at
+M = 4096 tokens: FMPQ quantisation of the layer input (kernel 1) + the W4Ax GEMM (kernel 2).
+Weights are packed once (offline, as in the paper).  At N GPUs the layers are tensor-parallel:
+gate/up and qkv column-parallel (N sharded, no collective), down row-parallel (K sharded at
+128-channel block boundaries) followed by an NCCL all_reduce(SUM) of the FP32 partials.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl comet|reference]
+
+Prints one JSON line on rank 0.  --impl reference times the CPU oracle (oracle/) on a bounded
+sample of the same workload on the host cores (rank 0 only).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from paper_conf_asplos_liu0rxpwl0w25_b200 import synth  # noqa: E402
+
+WORKLOAD = "llama3_70b_prefill_m4096"
+M_TOKENS = 4096
+FRAC = 0.05
+LAYERS = [  # (name, K, N, tensor-parallel kind)
+    ("gate_up", 8192, 28672, "col"),
+    ("down", 28672, 8192, "row"),
+    ("qkv", 8192, 10240, "col"),
+]
+METRIC = "W4Ax GEMM TOPS (quantize + GEMM), LLaMA-3-70B linear layers, M=4096"
+
+
+def total_ops(M=M_TOKENS):
+    return sum(2.0 * M * N * K for _, K, N, _ in LAYERS)
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return d, "measured"
+    return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}, "fallback"
+
+
+def load_traffic():
+    """Per-launch DRAM bytes of the GEMM from the committed ncu --set full capture, if any."""
+    p = os.path.join(ROOT, "profiles", "ncu_gemm_traffic.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            return json.load(f)
+    return None
+
+
+class ClockSampler:
+    def __init__(self, gpu_index: int):
+        self.proc = None
+        self.gpu = gpu_index
+        self.path = os.path.join("/tmp", f"comet_clocks_{os.getpid()}.csv")
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.gpu),
+                 "--query-gpu=clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+                 "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+                 "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap",
+                 "--format=csv,noheader,nounits", "-lms", "50"],
+                stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
+        except (FileNotFoundError, OSError):
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return None
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        rows = []
+        with open(self.path) as f:
+            for line in f:
+                parts = [x.strip() for x in line.split(",")]
+                if len(parts) >= 8:
+                    rows.append(parts)
+        os.unlink(self.path)
+        if not rows:
+            return None
+        sm = [float(r[0]) for r in rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in rows for i in range(4) if r[4 + i].lower() == "active"})
+        loaded = [s for s in sm if s > 0.5 * (max(sm) if sm else 1)]
+        return {"sm_mhz": statistics.median(loaded or sm) if sm else None,
+                "sm_max_mhz": max(mx) if mx else None, "reasons": reasons, "samples": len(rows)}
+
+
+# ---------------------------------------------------------------------------- reference arm
+
+def run_reference(args, rank, world):
+    if rank != 0:
+        return 0
+    import oracle
+    oracle.build()
+    rng = np.random.default_rng(1234)
+    # bounded sample of the same workload: `rows` token rows of every layer per step
+    rows_per_layer = 1
+    data = []
+    for li, (name, K, N, _) in enumerate(LAYERS):
+        p = synth.make_problem(4, K, N, frac=FRAC, seed=100 + li)
+        data.append(p)
+    ops_step = sum(2.0 * rows_per_layer * p.N * p.K for p in data)
+
+    def step(i):
+        for p in data:
+            r = np.array([i % p.M], dtype=np.int64)
+            oracle.w4ax_rows(p.x, p.tags, p.w, p.s_w, r)
+
+    for i in range(args.warmup):
+        step(i)
+    t0 = time.perf_counter()
+    for i in range(args.steps):
+        step(i)
+    dt = time.perf_counter() - t0
+    value = ops_step * args.steps / dt / 1e12
+    cores = oracle.num_threads()
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": "TOPS", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "int64",
+        "data": "synthetic",
+        "config": {"workload": WORKLOAD, "M": M_TOKENS, "layers": [l[:3] for l in LAYERS],
+                   "int8_block_fraction": FRAC, "reference_sample": f"{rows_per_layer} token row per layer per step"},
+        "cpu_baseline": {"value": value, "unit": "TOPS", "cores": cores, "kind": "oracle",
+                         "sample": f"{rows_per_layer} token row of each layer per step (FMPQ quantise + int64 GEMM + fp64 dequant, oracle/comet_oracle.c)"},
+        "e2e": {"value": value, "unit": "TOPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def cpu_baseline_sample(budget_s=15.0):
+    """Time the oracle as it stands on a bounded sample of the workload (rank 0, N=1)."""
+    import oracle
+    oracle.build()
+    ops = 0.0
+    t_total = 0.0
+    n = 0
+    probs = [synth.make_problem(4, K, N, frac=FRAC, seed=200 + i) for i, (_, K, N, _) in enumerate(LAYERS)]
+    while t_total < budget_s and n < 100000:
+        p = probs[n % len(probs)]
+        t0 = time.perf_counter()
+        oracle.w4ax_rows(p.x, p.tags, p.w, p.s_w, np.array([n % p.M], np.int64))
+        t_total += time.perf_counter() - t0
+        ops += 2.0 * p.N * p.K
+        n += 1
+    return {"value": ops / t_total / 1e12, "unit": "TOPS", "cores": oracle.num_threads(), "kind": "oracle",
+            "sample": f"{n} single-token rows cycling over the 3 layers ({t_total:.1f} s of CPU work)"}
+
+
+# ---------------------------------------------------------------------------- comet arm
+
+def shard(K, N, kind, tags, rank, world):
+    """Tensor-parallel shard of one layer: returns (k0, k1, n0, n1)."""
+    if world == 1:
+        return 0, K, 0, N
+    if kind == "col":
+        assert N % (128 * world) == 0
+        n = N // world
+        return 0, K, rank * n, (rank + 1) * n
+    assert K % (128 * world) == 0
+    k = K // world
+    return rank * k, (rank + 1) * k, 0, N
+
+
+def run_comet(args, rank, world, local_rank):
+    import torch
+    import torch.distributed as dist
+    import paper_conf_asplos_liu0rxpwl0w25_b200 as cb
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    stream = torch.cuda.current_stream()
+
+    # ---- data (synthetic, seeded; identical on every rank, each rank keeps its shard)
+    layers = []
+    for li, (name, K, N, kind) in enumerate(LAYERS):
+        rng = np.random.default_rng(1000 + li)
+        tags = synth.make_tags(K, FRAC, rng)
+        x = synth.make_activations(M_TOKENS, K, tags, rng)
+        w, s_w = synth.make_weights(N, K, rng)
+        k0, k1, n0, n1 = shard(K, N, kind, tags, rank, world)
+        x_l = np.ascontiguousarray(x[:, k0:k1])
+        t_l = np.ascontiguousarray(tags[k0 // 128:k1 // 128])
+        w_l = np.ascontiguousarray(w[n0:n1, k0:k1])
+        sw_l = np.ascontiguousarray(s_w[n0:n1])
+        Kl, Nl = k1 - k0, n1 - n0
+        x_d = torch.from_numpy(x_l).to(dev)
+        wp = cb.pack_weight(torch.from_numpy(w_l).to(dev))
+        swd = torch.from_numpy(sw_l).to(dev)
+        plan = cb.Plan(M_TOKENS, Nl, Kl, t_l, tile_n=args.tile_n, split_mode=args.split_mode)
+        act, sc = cb.quantize_act(x_d, t_l)
+        ydt = torch.float32 if (kind == "row" and world > 1) else torch.float16
+        y = torch.empty((M_TOKENS, Nl), dtype=ydt, device=dev)
+        layers.append(dict(name=name, K=Kl, N=Nl, kind=kind, x=x_d, x_host=torch.from_numpy(x_l).pin_memory(),
+                           tags=t_l, wp=wp, sw=swd, plan=plan, act=act, sc=sc, y=y,
+                           ops=2.0 * M_TOKENS * Nl * Kl))
+        del w, x
+    torch.cuda.synchronize()
+
+    n_events = args.steps * len(layers)
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(n_events)]
+    evq = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(n_events)]
+    eva = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(n_events)]
+
+    def step(rec=None):
+        for li, L in enumerate(layers):
+            e = None if rec is None else rec * len(layers) + li
+            if e is not None:
+                evq[e][0].record(stream)
+            cb.quantize_act(L["x"], L["tags"], out=(L["act"], L["sc"]))
+            if e is not None:
+                evq[e][1].record(stream)
+                ev[e][0].record(stream)
+            cb.w4ax_gemm(L["plan"], L["act"], L["sc"], L["wp"], L["sw"], out=L["y"])
+            if e is not None:
+                ev[e][1].record(stream)
+            if L["kind"] == "row" and world > 1:
+                if e is not None:
+                    eva[e][0].record(stream)
+                dist.all_reduce(L["y"], op=dist.ReduceOp.SUM)
+                if e is not None:
+                    eva[e][1].record(stream)
+
+    for _ in range(max(args.warmup, 3) if args.warmup >= 0 else 3):
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clk = ClockSampler(local_rank)
+    if rank == 0:
+        clk.start()
+        time.sleep(0.2)
+    t_start = torch.cuda.Event(enable_timing=True)
+    t_end = torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    t_start.record(stream)
+    for s in range(args.steps):
+        step(rec=s)
+    t_end.record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clocks = clk.stop() if rank == 0 else None
+    ms_total = t_start.elapsed_time(t_end)
+    gemm_ms = [0.0] * len(layers)
+    q_ms = [0.0] * len(layers)
+    ar_ms = 0.0
+    for s in range(args.steps):
+        for li, L in enumerate(layers):
+            e = s * len(layers) + li
+            gemm_ms[li] += ev[e][0].elapsed_time(ev[e][1])
+            q_ms[li] += evq[e][0].elapsed_time(evq[e][1])
+            if L["kind"] == "row" and world > 1:
+                ar_ms += eva[e][0].elapsed_time(eva[e][1])
+    if world > 1:
+        t = torch.tensor([ms_total, sum(gemm_ms), ar_ms], device=dev, dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms_total, gemm_max, ar_ms = t.tolist()
+    ms_step = ms_total / args.steps
+    value = total_ops() / (ms_step * 1e-3) / 1e12     # whole-job: all ranks' shards = the full layers
+
+    # ---- roofline of the dominant kernel (the GEMM), measured live on the launching stream
+    peaks, peak_src = load_peaks()
+    gemm_ops_rank = sum(L["ops"] for L in layers)
+    gemm_s_rank = sum(gemm_ms) / args.steps * 1e-3
+    achieved = gemm_ops_rank / gemm_s_rank / 1e12
+    peak = 2.0 * peaks["bf16_tflops"]          # INT8/FP8 dense = 2 x bf16 (nominal ratio), burst
+    traffic = load_traffic()
+    roofline = {"bound": "tensor", "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
+                "frac": achieved / peak,
+                "traffic": (traffic or {}).get("bytes_per_launch"),
+                "peak_source": f"{peak_src} bf16 burst {peaks['bf16_tflops']} TFLOP/s x 2 (INT8/FP8 : BF16 nominal ratio)",
+                "kernel": "k_w4ax (persistent tcgen05 W4Ax GEMM)",
+                "per_layer_gemm_us": {L["name"]: gemm_ms[i] / args.steps * 1e3 for i, L in enumerate(layers)},
+                "per_layer_quantize_us": {L["name"]: q_ms[i] / args.steps * 1e3 for i, L in enumerate(layers)},
+                "probe_i8_peak_tops": 4551.1}
+
+    # ---- e2e through the public API with host buffers (pinned in, pinned out)
+    e2e = None
+    if args.e2e_steps > 0:
+        h2d = sum(L["x_host"].numel() * 2 for L in layers)
+        d2h = sum(L["y"].numel() * L["y"].element_size() for L in layers)
+        if world == 1:
+            scr = {}
+            outs = {}
+            for L in layers:
+                nbytes = cb.linear_scratch_bytes(L["plan"], cb.COMET_F16, cb.COMET_F16)
+                scr[L["name"]] = torch.empty(nbytes, dtype=torch.uint8, device=dev)
+                outs[L["name"]] = torch.empty((M_TOKENS, L["N"]), dtype=torch.float16).pin_memory()
+
+            def e2e_step():
+                for L in layers:
+                    cb.w4ax_linear_host(L["plan"], L["x_host"], L["wp"], L["sw"], outs[L["name"]], scr[L["name"]])
+        else:
+            outs = {L["name"]: torch.empty(L["y"].shape, dtype=L["y"].dtype).pin_memory() for L in layers}
+
+            def e2e_step():
+                for L in layers:
+                    L["x"].copy_(L["x_host"], non_blocking=True)
+                    cb.quantize_act(L["x"], L["tags"], out=(L["act"], L["sc"]))
+                    cb.w4ax_gemm(L["plan"], L["act"], L["sc"], L["wp"], L["sw"], out=L["y"])
+                    if L["kind"] == "row":
+                        dist.all_reduce(L["y"], op=dist.ReduceOp.SUM)
+                    outs[L["name"]].copy_(L["y"], non_blocking=True)
+                torch.cuda.synchronize()
+        e2e_step()
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        for _ in range(args.e2e_steps):
+            e2e_step()
+        b.record(stream)
+        torch.cuda.synchronize()
+        e_ms = a.elapsed_time(b) / args.e2e_steps
+        if world > 1:
+            t = torch.tensor([e_ms], device=dev, dtype=torch.float64)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            e_ms = t.item()
+        e2e = {"value": total_ops() / (e_ms * 1e-3) / 1e12, "unit": "TOPS", "h2d_bytes_per_step": h2d,
+               "d2h_bytes_per_step": d2h, "ms_per_step": e_ms,
+               "path": "comet_w4ax_linear_host (C ABI, pinned host buffers)" if world == 1 else
+                       "public API: H2D copy + quantize_act + w4ax_gemm (+ NCCL all_reduce) + D2H copy"}
+
+    cpu = cpu_baseline_sample(args.cpu_budget) if (rank == 0 and world == 1 and args.cpu_budget > 0) else None
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "TOPS", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "e4m3xe4m3+s8xs8->f32 (INT4/INT8 codes)",
+            "data": "synthetic (seeded N(0,1) activations with injected outlier channels, random INT4 weights)",
+            "config": {"workload": WORKLOAD, "M": M_TOKENS,
+                       "layers": [[n, K, N] for n, K, N, _ in LAYERS],
+                       "int8_block_fraction": FRAC,
+                       "parallelism": "single GPU" if world == 1 else f"tp{world} (gate_up/qkv column, down row + NCCL all_reduce fp32)",
+                       "tile_n": layers[0]["plan"].info()["tile_n"],
+                       "l2": "inputs larger than L2 (per step: 300 MB activations + 276 MB packed weights > 126 MB L2)"},
+            "roofline": roofline,
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": 2 * len(layers) * args.steps,
+            "clocks": clocks,
+        }
+        if world > 1:
+            line["allreduce_ms_per_step"] = ar_ms / args.steps
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=30)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="comet", choices=["comet", "reference"])
+    ap.add_argument("--e2e-steps", type=int, default=5)
+    ap.add_argument("--cpu-budget", type=float, default=15.0)
+    ap.add_argument("--tile-n", type=int, default=0, help="0 = planner default")
+    ap.add_argument("--split-mode", type=int, default=-1)
+    args = ap.parse_args()
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", str(args.gpus if args.gpus == 1 else 1)))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        return run_reference(args, rank, world)
+    return run_comet(args, rank, world, local_rank)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

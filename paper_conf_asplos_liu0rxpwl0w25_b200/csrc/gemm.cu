@@ -70,16 +70,17 @@ template <int NT>
 struct Cfg {
   static constexpr int ACTIVE_WGS = NT >= 32 ? 2 : 1;          // promotion warpgroups in use
   static constexpr int COLS = NT / ACTIVE_WGS;                 // accumulator columns per WG
+  static constexpr int NACC = (64 + 3 * NT <= 512) ? 3 : 2;    // accumulator buffers in TMEM
   static constexpr int X_BYTES = NT * 128;
   static constexpr int W_BYTES = kTileW * 64;
   static constexpr int STAGE_BYTES = X_BYTES + W_BYTES;
   static constexpr int STAGES_RAW = (196 * 1024) / STAGE_BYTES;
   static constexpr int STAGES = STAGES_RAW > 10 ? 10 : STAGES_RAW;
   static constexpr int SMEM_DATA = STAGES * STAGE_BYTES + kSRing * NT * 4;
-  static constexpr int N_BARS = 2 * STAGES + 8 + 2 * kSRing;
+  static constexpr int N_BARS = 2 * STAGES + 4 + 2 * NACC + 2 * kSRing;
   static constexpr int SMEM_BYTES = 1024 + SMEM_DATA + N_BARS * 8 + 16 + kMaxBlocks;
   static_assert(COLS % 16 == 0, "promotion chunks of 16 columns");
-  static_assert(2 * NT + 64 <= 512, "TMEM budget");
+  static_assert(NACC * NT + 64 <= 512, "TMEM budget");
 };
 
 __device__ __forceinline__ void named_bar_sync(int id, int n) {
@@ -91,11 +92,6 @@ __device__ __forceinline__ void st_release_gpu(uint32_t* p, uint32_t v) {
 __device__ __forceinline__ uint32_t ld_acquire_gpu(const uint32_t* p) {
   uint32_t v;
   asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-  return v;
-}
-__device__ __forceinline__ float ld_cg_f32(const float* p) {
-  float v;
-  asm volatile("ld.global.cg.f32 %0, [%1];" : "=f"(v) : "l"(p));
   return v;
 }
 template <uint32_t N>
@@ -126,22 +122,27 @@ template <int NT, int DEBUG>
 __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ GemmParams P) {
   using C = Cfg<NT>;
   constexpr int S = C::STAGES;
-  extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
+  constexpr int NACC = C::NACC;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  // keep the pointer derived from the __shared__ array (shared address space) when aligning
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   uint8_t* sX = smem;
   uint8_t* sW = sX + S * C::X_BYTES;
   float* sS = reinterpret_cast<float*>(sW + S * C::W_BYTES);
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + C::SMEM_DATA);
-  uint64_t* full = bars;                 // [S]  TMA -> (MMA, widen)
-  uint64_t* empty = bars + S;            // [S]  (MMA commit + 4 widen warps) -> TMA
-  uint64_t* a_full = bars + 2 * S;       // [2]  widen -> MMA
-  uint64_t* a_empty = a_full + 2;        // [2]  MMA commit -> widen
-  uint64_t* acc_full = a_full + 4;       // [2]  MMA commit -> promotion
-  uint64_t* acc_empty = a_full + 6;      // [2]  promotion -> MMA
-  uint64_t* s_full = a_full + 8;         // [kSRing] TMA -> promotion
-  uint64_t* s_empty = s_full + kSRing;   // [kSRing] promotion -> TMA
+  uint64_t* full = bars;                    // [S]    TMA -> (MMA, widen)
+  uint64_t* empty = bars + S;               // [S]    (MMA commit + 4 widen warps) -> TMA
+  uint64_t* a_full = bars + 2 * S;          // [2]    widen -> MMA
+  uint64_t* a_empty = a_full + 2;           // [2]    MMA commit -> widen
+  uint64_t* acc_full = a_full + 4;          // [NACC] MMA commit -> promotion
+  uint64_t* acc_empty = acc_full + NACC;    // [NACC] promotion -> MMA
+  uint64_t* s_full = acc_empty + NACC;      // [kSRing] TMA -> promotion
+  uint64_t* s_empty = s_full + kSRing;      // [kSRing] promotion -> TMA
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bars + C::N_BARS);
   uint8_t* s_tags = reinterpret_cast<uint8_t*>(tmem_holder + 4);
+  const uint32_t s_tags_a = smem_u32(s_tags);
+  const uint32_t sW_a = smem_u32(sW);
+  const uint32_t sS_a = smem_u32(sS);
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
@@ -160,6 +161,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
     for (int i = 0; i < 2; ++i) {
       mbar_init(&a_full[i], 4);
       mbar_init(&a_empty[i], 1);
+    }
+    for (int i = 0; i < NACC; ++i) {
       mbar_init(&acc_full[i], 1);
       mbar_init(&acc_empty[i], 4 * C::ACTIVE_WGS);
     }
@@ -207,12 +210,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
       // ------------------------------------------------------------------ MMA issuer
       const uint32_t id_f8 = idesc_f8f6f4_e4m3(128, NT);
       const uint32_t id_i8 = idesc_i8(128, NT);
-      int stage = 0, ab = 0;
-      uint32_t ph = 0, aph = 0, j = 0;
+      int stage = 0, ab = 0, accb = 0;
+      uint32_t ph = 0, aph = 0, accph = 0;
       for (int it = it_begin; it < it_end; ++it) {
         const WorkItem w = load_item(P, it, debug);
-        for (int kb = w.kb_begin; kb < w.kb_end; ++kb, ++j) {
-          const uint32_t accb = j & 1, accph = (j >> 1) & 1;
+        for (int kb = w.kb_begin; kb < w.kb_end; ++kb) {
           mbar_wait(&acc_empty[accb], accph ^ 1);
           mbar_wait(&full[stage], ph);
           mbar_wait(&a_full[ab], aph);
@@ -220,7 +222,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
           const uint32_t d = tbase + kAccCol + accb * NT;
           const uint32_t a = tbase + kAcol + ab * 32;
           const uint32_t sx = smem_u32(sX + stage * C::X_BYTES);
-          if (s_tags[kb]) {
+          if (lds_u8(s_tags_a + kb)) {
 #pragma unroll
             for (int k = 0; k < 4; ++k) mma_i8_ts(d, a + 8 * k, sdesc_kmajor_sw128(sx + 32 * k), id_i8, k);
           } else {
@@ -232,29 +234,30 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
           tc_commit(&acc_full[accb]);
           if (++stage == S) { stage = 0; ph ^= 1; }
           if (++ab == 2) { ab = 0; aph ^= 1; }
+          if (++accb == NACC) { accb = 0; accph ^= 1; }
         }
       }
     }
   } else if (warp < 8) {
-    setmaxnreg_dec<88>();
+    setmaxnreg_dec<80>();
     // -------------------------------------------------------------------- widen (W -> TMEM A)
     const int q = warp & 3;
     const int r = q * 32 + lane;                  // TMEM lane = weight row within the tile
     const uint32_t lane_addr = (uint32_t)(q * 32) << 16;
+    const int sw = (r >> 1) & 3;                  // TMA 64-byte swizzle: chunk ^= row bits [1:2]
     int stage = 0, ab = 0;
     uint32_t ph = 0, aph = 0;
     for (int it = it_begin; it < it_end; ++it) {
       const WorkItem w = load_item(P, it, debug);
       for (int kb = w.kb_begin; kb < w.kb_end; ++kb) {
+        const bool is8 = lds_u8(s_tags_a + kb) != 0;
         mbar_wait(&full[stage], ph);
-        const uint8_t* wt = sW + stage * C::W_BYTES + r * 64;
-        const int sw = (r >> 1) & 3;              // TMA 64-byte swizzle: chunk ^= row bits [1:2]
+        const uint32_t wt = sW_a + stage * C::W_BYTES + r * 64;
         uint4 c[4];
 #pragma unroll
-        for (int j = 0; j < 4; ++j) c[j] = *reinterpret_cast<const uint4*>(wt + ((j ^ sw) << 4));
+        for (int j = 0; j < 4; ++j) c[j] = lds128(wt + ((j ^ sw) << 4));
         __syncwarp();
         if (lane == 0) mbar_arrive(&empty[stage]);
-        const bool is8 = s_tags[kb] != 0;
         uint32_t o[32];
 #pragma unroll
         for (int j = 0; j < 4; ++j) {
@@ -286,80 +289,132 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
   } else {
     setmaxnreg_inc<192>();
     // -------------------------------------------------------------------- promotion + epilogue
+    // TMEM accumulator: lane = weight row (n), column = token (m).  With the 16x256b load shape
+    // thread t of warp quarter q owns lanes 32q + 16h + t/4 + 8i (h, i in {0,1}) and columns
+    // col0 + 8j + 2(t%4) + e (j < NJ, e in {0,1}): only NJ*2 distinct tokens, so the block's
+    // per-token scales for this thread are NJ float2 loads issued before the accumulator wait.
     const int pw = warp - 8;
     const int wg = pw >> 2;
     const int q = warp & 3;
-    const int r = q * 32 + lane;
-    const uint32_t lane_addr = (uint32_t)(q * 32) << 16;
+    const int t0 = lane & 3, t1 = lane >> 2;
     const int col0 = wg * C::COLS;
+    constexpr int NJ = C::COLS / 8;                 // 8-column groups per WG
+    constexpr int NB1 = NJ > 8 ? 8 : NJ;            // repetitions in the first load batch
+    constexpr int NB2 = NJ - NB1;
+    constexpr int NE = 4 * NJ;                      // accumulator elements per thread (per h: 2*NJ*2)
     const int n_promo_threads = 128 * C::ACTIVE_WGS;
+    const int ptid = threadIdx.x - 256;
     if (wg < C::ACTIVE_WGS) {
-      int ss = 0;
-      uint32_t sph = 0, j = 0;
+      int ss = 0, accb = 0;
+      uint32_t sph = 0, accph = 0;
       for (int it = it_begin; it < it_end; ++it) {
         const WorkItem w = load_item(P, it, debug);
         const int n_tile = w.tile / P.n_m_tiles, m_tile = w.tile % P.n_m_tiles;
         const int m0 = m_tile * NT, n0 = n_tile * kTileW;
         const bool owner = (w.flags & 2) != 0;
         const bool split = (w.flags & 1) != 0;
-        float acc[C::COLS];
-        int32_t dacc[DEBUG ? C::COLS : 1];
+        // acc index: ((h*2 + i)*NJ + j)*2 + e
+        float acc[2 * NE];
+        int32_t dacc[DEBUG ? 2 * NE : 1];
 #pragma unroll
-        for (int c = 0; c < C::COLS; ++c) {
-          const int64_t m = m0 + col0 + c;
-          acc[c] = (owner && m < P.Mp) ? -__ldg(P.corr + m) * 0.001953125f : 0.f;   // 2^-9
-          if (DEBUG) dacc[c] = 0;
+        for (int j = 0; j < NJ; ++j) {
+#pragma unroll
+          for (int e = 0; e < 2; ++e) {
+            const int64_t m = m0 + col0 + 8 * j + 2 * t0 + e;
+            const float c0 = (owner && m < P.Mp) ? -__ldg(P.corr + m) * 0.001953125f : 0.f;   // 2^-9
+#pragma unroll
+            for (int hi = 0; hi < 4; ++hi) {
+              acc[(hi * NJ + j) * 2 + e] = c0;
+              if (DEBUG) dacc[(hi * NJ + j) * 2 + e] = 0;
+            }
+          }
         }
-        for (int kb = w.kb_begin; kb < w.kb_end; ++kb, ++j) {
-          const uint32_t accb = j & 1, accph = (j >> 1) & 1;
+        for (int kb = w.kb_begin; kb < w.kb_end; ++kb) {
+          const bool is8 = lds_u8(s_tags_a + kb) != 0;
           mbar_wait(&s_full[ss], sph);
+          float2 sc[NJ];
+          {
+            const uint32_t sbase = sS_a + (ss * NT + col0 + 2 * t0) * 4;
+#pragma unroll
+            for (int j = 0; j < NJ; ++j) {
+              const uint2 u = lds64(sbase + j * 32);
+              sc[j] = make_float2(__uint_as_float(u.x), __uint_as_float(u.y));
+            }
+          }
           mbar_wait(&acc_full[accb], accph);
           tc_fence_after();
-          const bool is8 = s_tags[kb] != 0;
-          const float* sc = sS + ss * NT + col0;
-          const uint32_t taddr = tbase + kAccCol + accb * NT + col0 + lane_addr;
+          const uint32_t tcol = tbase + kAccCol + accb * NT + col0;
 #pragma unroll
-          for (int ch = 0; ch < C::COLS / 16; ++ch) {
-            uint32_t v[16];
-            tmem_ld16(taddr + ch * 16, v);
-            tmem_wait_ld();
-            float s[16];
+          for (int h = 0; h < 2; ++h) {
+            const uint32_t taddr = tcol + ((uint32_t)(32 * q + 16 * h) << 16);
 #pragma unroll
-            for (int e = 0; e < 4; ++e) {
-              const float4 t4 = *reinterpret_cast<const float4*>(sc + ch * 16 + 4 * e);
-              s[4 * e] = t4.x; s[4 * e + 1] = t4.y; s[4 * e + 2] = t4.z; s[4 * e + 3] = t4.w;
-            }
-            if (!is8) {
+            for (int part = 0; part < 2; ++part) {
+              constexpr int dummy = 0;
+              (void)dummy;
+              const int jb = part == 0 ? 0 : NB1;
+              const int nrep = part == 0 ? NB1 : NB2;
+              if (nrep == 0) continue;
+              uint32_t v[4 * 8];
+              if (part == 0) tmem_ld_16x256b<NB1>(taddr, v);
+              else if constexpr (NB2 > 0) tmem_ld_16x256b<(NB2 > 0 ? NB2 : 2)>(taddr + NB1 * 8, v);
+              tmem_wait_ld();
+              if (!is8) {
 #pragma unroll
-              for (int e = 0; e < 8; ++e) {
-                const int c = ch * 16 + 2 * e;
-                float2 y2 = ffma2(make_float2(__uint_as_float(v[2 * e]), __uint_as_float(v[2 * e + 1])),
-                                  make_float2(s[2 * e], s[2 * e + 1]), make_float2(acc[c], acc[c + 1]));
-                acc[c] = y2.x;
-                acc[c + 1] = y2.y;
-              }
-            } else {
+                for (int jj = 0; jj < 8; ++jj) {
+                  if (jj < nrep) {
+                    const int j = jb + jj;
 #pragma unroll
-              for (int e = 0; e < 16; ++e) {
-                const int c = ch * 16 + e;
-                acc[c] = fmaf(__int2float_rn((int)v[e]), s[e] * 1.220703125e-04f, acc[c]);   // 2^-13
-              }
-            }
-            if (DEBUG) {
-#pragma unroll
-              for (int e = 0; e < 16; ++e) {
-                const int c = ch * 16 + e;
-                const int64_t m = m0 + col0 + c;
-                int32_t ab;
-                if (is8) {
-                  ab = ((int32_t)v[e]) >> 4;
-                } else {
-                  const int qs = (m < P.Mp) ? (int)P.qsum[(int64_t)kb * P.Mp + m] : 0;
-                  ab = (int32_t)(__uint_as_float(v[e]) * 512.f) - 8 * qs;
+                    for (int i = 0; i < 2; ++i) {
+                      const int a = ((h * 2 + i) * NJ + j) * 2;
+                      float2 y = ffma2(make_float2(__uint_as_float(v[4 * jj + 2 * i]), __uint_as_float(v[4 * jj + 2 * i + 1])),
+                                       sc[j], make_float2(acc[a], acc[a + 1]));
+                      acc[a] = y.x;
+                      acc[a + 1] = y.y;
+                    }
+                  }
                 }
-                dacc[c] += ab;
-                if (DEBUG == 2 && m < P.M)
-                  P.dbg_blocks[((int64_t)kb * P.M + m) * P.N + n0 + r] = ab;
+              } else {
+#pragma unroll
+                for (int jj = 0; jj < 8; ++jj) {
+                  if (jj < nrep) {
+                    const int j = jb + jj;
+                    const float2 s8 = make_float2(sc[j].x * 1.220703125e-04f, sc[j].y * 1.220703125e-04f);  // 2^-13
+#pragma unroll
+                    for (int i = 0; i < 2; ++i) {
+                      const int a = ((h * 2 + i) * NJ + j) * 2;
+                      float2 y = ffma2(make_float2(__int2float_rn((int)v[4 * jj + 2 * i]), __int2float_rn((int)v[4 * jj + 2 * i + 1])),
+                                       s8, make_float2(acc[a], acc[a + 1]));
+                      acc[a] = y.x;
+                      acc[a + 1] = y.y;
+                    }
+                  }
+                }
+              }
+              if (DEBUG) {
+#pragma unroll
+                for (int jj = 0; jj < 8; ++jj) {
+                  if (jj < nrep) {
+                    const int j = jb + jj;
+#pragma unroll
+                    for (int i = 0; i < 2; ++i) {
+#pragma unroll
+                      for (int e = 0; e < 2; ++e) {
+                        const int64_t m = m0 + col0 + 8 * j + 2 * t0 + e;
+                        const int n = n0 + 32 * q + 16 * h + t1 + 8 * i;
+                        const uint32_t raw = v[4 * jj + 2 * i + e];
+                        int32_t ab;
+                        if (is8) {
+                          ab = ((int32_t)raw) >> 4;
+                        } else {
+                          const int qs = (m < P.Mp) ? (int)P.qsum[(int64_t)kb * P.Mp + m] : 0;
+                          ab = (int32_t)(__uint_as_float(raw) * 512.f) - 8 * qs;
+                        }
+                        dacc[((h * 2 + i) * NJ + j) * 2 + e] += ab;
+                        if (DEBUG == 2 && m < P.M) P.dbg_blocks[((int64_t)kb * P.M + m) * P.N + n] = ab;
+                      }
+                    }
+                  }
+                }
               }
             }
           }
@@ -370,16 +425,18 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
             mbar_arrive(&s_empty[ss]);
           }
           if (++ss == kSRing) { ss = 0; sph ^= 1; }
+          if (++accb == NACC) { accb = 0; accph ^= 1; }
         }
         // ---------------------------------------------------------------- epilogue
         if (split) {
           const int seg = (w.flags >> 8) & 0xFF;
           const int nseg = (w.flags >> 16) & 0xFF;
-          const int64_t part_tile = (int64_t)NT * kTileW;
+          const int64_t part_tile = (int64_t)NT * kTileW;    // = n_promo_threads * 2*NE floats
           if (!owner) {
-            float* dst = P.ws_part + ((int64_t)w.fix * (P.max_seg - 1) + (seg - 1)) * part_tile;
+            float4* dst = reinterpret_cast<float4*>(
+                P.ws_part + ((int64_t)w.fix * (P.max_seg - 1) + (seg - 1)) * part_tile + (int64_t)ptid * 2 * NE);
 #pragma unroll
-            for (int c = 0; c < C::COLS; ++c) dst[(int64_t)(col0 + c) * kTileW + r] = acc[c];
+            for (int a = 0; a < 2 * NE; a += 4) dst[a / 4] = make_float4(acc[a], acc[a + 1], acc[a + 2], acc[a + 3]);
             __threadfence();
             named_bar_sync(1, n_promo_threads);
             if (threadIdx.x == 256) st_release_gpu(P.ws_flags + (int64_t)w.fix * P.max_seg + seg, P.epoch);
@@ -388,9 +445,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
           if (threadIdx.x == 256) {
             for (int sgi = 1; sgi < nseg; ++sgi) {
               const uint32_t* f = P.ws_flags + (int64_t)w.fix * P.max_seg + sgi;
-              uint64_t t0 = globaltimer_ns();
+              uint64_t t0g = globaltimer_ns();
               while (ld_acquire_gpu(f) != P.epoch) {
-                if (globaltimer_ns() - t0 > COMET_MBAR_TIMEOUT_NS) {
+                if (globaltimer_ns() - t0g > COMET_MBAR_TIMEOUT_NS) {
                   printf("comet: stream-K fix-up timeout (tile %d seg %d)\n", w.tile, sgi);
                   __trap();
                 }
@@ -399,23 +456,37 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
           }
           named_bar_sync(1, n_promo_threads);
           for (int sgi = 1; sgi < nseg; ++sgi) {
-            const float* src = P.ws_part + ((int64_t)w.fix * (P.max_seg - 1) + (sgi - 1)) * part_tile;
+            const float4* src = reinterpret_cast<const float4*>(
+                P.ws_part + ((int64_t)w.fix * (P.max_seg - 1) + (sgi - 1)) * part_tile + (int64_t)ptid * 2 * NE);
 #pragma unroll
-            for (int c = 0; c < C::COLS; ++c) acc[c] += ld_cg_f32(src + (int64_t)(col0 + c) * kTileW + r);
+            for (int a = 0; a < 2 * NE; a += 4) {
+              float4 t4;
+              asm volatile("ld.global.cg.v4.f32 {%0,%1,%2,%3}, [%4];"
+                           : "=f"(t4.x), "=f"(t4.y), "=f"(t4.z), "=f"(t4.w) : "l"(src + a / 4));
+              acc[a] += t4.x; acc[a + 1] += t4.y; acc[a + 2] += t4.z; acc[a + 3] += t4.w;
+            }
           }
         }
-        const int n = n0 + r;
-        const float sw = __ldg(P.w_scales + n) * 512.f;
 #pragma unroll
-        for (int c = 0; c < C::COLS; ++c) {
-          const int64_t m = m0 + col0 + c;
-          if (m < P.M) {
-            const float yv = acc[c] * sw;
-            const int64_t off = m * P.ldy + n;
-            if (P.ydt == COMET_F16) reinterpret_cast<__half*>(P.y)[off] = __float2half_rn(yv);
-            else if (P.ydt == COMET_BF16) reinterpret_cast<__nv_bfloat16*>(P.y)[off] = __float2bfloat16_rn(yv);
-            else reinterpret_cast<float*>(P.y)[off] = yv;
-            if (DEBUG) P.dbg_acc[m * P.N + n] = dacc[c];
+        for (int hi = 0; hi < 4; ++hi) {
+          const int h = hi >> 1, i = hi & 1;
+          const int n = n0 + 32 * q + 16 * h + t1 + 8 * i;
+          const float swv = __ldg(P.w_scales + n) * 512.f;
+#pragma unroll
+          for (int j = 0; j < NJ; ++j) {
+#pragma unroll
+            for (int e = 0; e < 2; ++e) {
+              const int64_t m = m0 + col0 + 8 * j + 2 * t0 + e;
+              if (m < P.M) {
+                const int a = (hi * NJ + j) * 2 + e;
+                const float yv = acc[a] * swv;
+                const int64_t off = m * P.ldy + n;
+                if (P.ydt == COMET_F16) reinterpret_cast<__half*>(P.y)[off] = __float2half_rn(yv);
+                else if (P.ydt == COMET_BF16) reinterpret_cast<__nv_bfloat16*>(P.y)[off] = __float2bfloat16_rn(yv);
+                else reinterpret_cast<float*>(P.y)[off] = yv;
+                if (DEBUG) P.dbg_acc[m * P.N + n] = dacc[a];
+              }
+            }
           }
         }
       }
