@@ -146,7 +146,12 @@ typedef struct {
   int stages;          /* shared-memory ring depth; 0 = auto */
   int device_plan;     /* 1 (default) = upload the work list to the device at create time;
                           0 = host-only plan (comet_plan_describe only; CPU-safe) */
-  int reserved[6];
+  int orientation;     /* 0 = auto (2 when M >= 128, else 1);
+                          1 = weights on the MMA M side: tile = 128 weights x tile_n tokens
+                              (decode-sized M; weights widened into TMEM);
+                          2 = tokens on the MMA M side: tile = 128 tokens x 256 weights
+                              (prefill; weights widened into shared memory), tile_n ignored */
+  int reserved[5];
 } comet_sched_config;
 
 /* Fill *cfg with the defaults (tile_n 0, num_sms 0, split_mode -1, costs 1/1, stages 0,
@@ -170,7 +175,8 @@ comet_status_t comet_plan_destroy(comet_plan_t plan);
 typedef struct {
   int64_t M, N, K;
   int tile_n, num_ctas, split_mode, stages;
-  int64_t n_tiles;         /* output tiles = (N/128) * ceil(M/tile_n) */
+  int orientation, tile_w;  /* kernel orientation (1/2) and weights per output tile */
+  int64_t n_tiles;         /* output tiles = ceil(N/tile_w) * ceil(M/tile_n) */
   int64_t n_items;         /* work items in the list */
   int64_t n_split_tiles;   /* tiles shared by more than one CTA */
   double max_cta_cost;     /* planner makespan (sum of unit costs on the busiest CTA) */

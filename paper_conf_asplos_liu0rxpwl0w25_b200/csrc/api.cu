@@ -162,6 +162,7 @@ void comet_sched_config_default(comet_sched_config* cfg) {
   cfg->cost_int8 = 1.0f;
   cfg->stages = 0;
   cfg->device_plan = 1;
+  cfg->orientation = 0;
 }
 
 comet_status_t comet_plan_create(int64_t M, int64_t N, int64_t K, const uint8_t* tags_host,
@@ -178,6 +179,7 @@ comet_status_t comet_plan_create(int64_t M, int64_t N, int64_t K, const uint8_t*
   else comet_sched_config_default(&cfg);
   if (cfg.split_mode < -1 || cfg.split_mode > 3) return fail(COMET_ERR_INVALID_ARG, "split_mode must be -1, 0, 1, 2 or 3");
   if (cfg.cost_int4 < 0 || cfg.cost_int8 < 0) return fail(COMET_ERR_INVALID_ARG, "costs must be >= 0");
+  if (cfg.orientation < 0 || cfg.orientation > 2) return fail(COMET_ERR_INVALID_ARG, "orientation must be 0, 1 or 2");
   if (cfg.num_sms <= 0) {
     if (!cfg.device_plan) return fail(COMET_ERR_INVALID_ARG, "a host-only plan needs an explicit num_sms");
     int sms = 0;
@@ -231,6 +233,8 @@ comet_status_t comet_plan_info(comet_plan_t plan, comet_plan_info_t* info) {
   info->M = p.M; info->N = p.N; info->K = p.K;
   info->tile_n = p.tile_n; info->num_ctas = p.num_ctas; info->split_mode = p.split_mode;
   info->stages = p.stages;
+  info->orientation = p.orientation;
+  info->tile_w = p.tile_w;
   info->n_tiles = p.n_tiles;
   info->n_items = (int64_t)p.items.size();
   info->n_split_tiles = p.n_split_tiles;

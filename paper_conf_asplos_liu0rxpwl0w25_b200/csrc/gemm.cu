@@ -28,43 +28,14 @@
 // of 2^-9 and |sum| < 2^14 -> exact in FP32 (checked bit-exactly against the oracle through the
 // debug accumulators); the +8 offset is removed with corr[m] = 8 sum_b s_a qsum (kernel 1).
 // INT8 block: acc = 16 * sum_k x_k w_k exactly in INT32.
-#include <cudaTypedefs.h>
-#include <cuda_fp16.h>
-#include <cuda_bf16.h>
 #include <algorithm>
-#include "internal.h"
-#include "sm100.cuh"
+#include "gemm_common.cuh"
 
 namespace comet {
+namespace gemm {
 namespace {
-
-using namespace sm100;
-
-constexpr int kThreads = 512;
-constexpr int kSRing = 8;            // scale ring depth
 constexpr uint32_t kAcol = 0;        // TMEM columns [0, 64): two widened-weight A buffers
 constexpr uint32_t kAccCol = 64;     // TMEM columns [64, 64 + 2 NT): two accumulators
-
-struct __align__(64) GemmParams {
-  CUtensorMap map_x;
-  CUtensorMap map_w;
-  const float* scales;       // [nb][Mp]
-  const float* corr;         // [Mp]
-  const int16_t* qsum;       // [nb][Mp]
-  const float* w_scales;     // [N]
-  void* y;
-  int64_t ldy;
-  int32_t* dbg_acc;          // [M][N] or null
-  int32_t* dbg_blocks;       // [nb][M][N] or null
-  float* ws_part;
-  uint32_t* ws_flags;
-  const int32_t* cta_begin;
-  const WorkItem* items;
-  int64_t M, N, Mp;
-  int nb, n_m_tiles, max_seg, ydt;
-  uint32_t epoch;
-  TagMask tags;
-};
 
 template <int NT>
 struct Cfg {
@@ -82,41 +53,6 @@ struct Cfg {
   static_assert(COLS % 16 == 0, "promotion chunks of 16 columns");
   static_assert(NACC * NT + 64 <= 512, "TMEM budget");
 };
-
-__device__ __forceinline__ void named_bar_sync(int id, int n) {
-  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
-}
-__device__ __forceinline__ void st_release_gpu(uint32_t* p, uint32_t v) {
-  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
-__device__ __forceinline__ uint32_t ld_acquire_gpu(const uint32_t* p) {
-  uint32_t v;
-  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-  return v;
-}
-template <uint32_t N>
-__device__ __forceinline__ void setmaxnreg_dec() {
-  asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(N));
-}
-template <uint32_t N>
-__device__ __forceinline__ void setmaxnreg_inc() {
-  asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(N));
-}
-
-__device__ __forceinline__ WorkItem load_item(const GemmParams& P, int idx, bool debug) {
-  if (debug) {
-    WorkItem w{};
-    w.tile = blockIdx.x; w.kb_begin = 0; w.kb_end = P.nb; w.flags = 2; w.fix = -1;
-    return w;
-  }
-  const int4* src = reinterpret_cast<const int4*>(P.items + idx);
-  int4 a = __ldg(src);
-  int4 b = __ldg(src + 1);
-  WorkItem w;
-  w.tile = a.x; w.kb_begin = a.y; w.kb_end = a.z; w.flags = a.w;
-  w.fix = b.x; w.pad0 = b.y; w.pad1 = b.z; w.pad2 = b.w;
-  return w;
-}
 
 template <int NT, int DEBUG>
 __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ GemmParams P) {
@@ -498,7 +434,19 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
   if (warp == 2) tmem_dealloc<512>(tbase);
 }
 
-// ------------------------------------------------------------------------------ host side
+template <int NT, int DEBUG>
+cudaError_t launch_nt(const GemmParams& prm, int grid, cudaStream_t stream) {
+  using C = Cfg<NT>;
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(k_w4ax<NT, DEBUG>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_BYTES);
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  k_w4ax<NT, DEBUG><<<grid, kThreads, C::SMEM_BYTES, stream>>>(prm);
+  return cudaGetLastError();
+}
+
 PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
   static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
   if (!fn) {
@@ -511,6 +459,9 @@ PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
   return fn;
 }
 
+}  // namespace
+
+// ------------------------------------------------------------------------------ host side
 bool make_map_2d(CUtensorMap* map, const void* base, uint64_t inner, uint64_t outer,
                  uint64_t row_bytes, uint32_t box_inner, uint32_t box_outer,
                  CUtensorMapSwizzle swz) {
@@ -526,39 +477,32 @@ bool make_map_2d(CUtensorMap* map, const void* base, uint64_t inner, uint64_t ou
   return r == CUDA_SUCCESS;
 }
 
-template <int NT, int DEBUG>
-cudaError_t launch_nt(const GemmParams& prm, int grid, cudaStream_t stream) {
-  using C = Cfg<NT>;
-  static bool attr_set = false;
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(k_w4ax<NT, DEBUG>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_BYTES);
-    if (e != cudaSuccess) return e;
-    attr_set = true;
-  }
-  k_w4ax<NT, DEBUG><<<grid, kThreads, C::SMEM_BYTES, stream>>>(prm);
-  return cudaGetLastError();
-}
-
-}  // namespace
+}  // namespace gemm
 
 comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_scales,
                            const void* w_packed, const float* w_scales, void* y,
                            comet_dtype_t ydt, int64_t ldy, int32_t* debug_acc,
                            int32_t* debug_acc_blocks, void* workspace, size_t ws_bytes,
                            cudaStream_t stream, int* launches) {
+  using namespace gemm;
   *launches = 0;
   const bool dbg = debug_acc != nullptr || debug_acc_blocks != nullptr;
-  const int NT = dbg ? 64 : p.tile_n;
+  const int debug = debug_acc_blocks ? 2 : (dbg ? 1 : 0);
+  const bool normal = p.orientation == 2;
+  // token-tile (box rows of the activation TMA) and weight-tile (box rows of the weight TMA)
+  int tile_m, tile_w;
+  if (normal) { tile_m = 128; tile_w = dbg ? 128 : 256; }
+  else { tile_m = dbg ? 64 : p.tile_n; tile_w = kTileW; }
   comet_act_layout_t L;
   act_layout(p.M, p.K, &L);
   const uint8_t* base = static_cast<const uint8_t*>(act_packed);
   GemmParams prm;
   memset(&prm, 0, sizeof(prm));
   if (!make_map_2d(&prm.map_x, base + L.codes_off, (uint64_t)p.K, (uint64_t)p.M, (uint64_t)p.K, 128,
-                   (uint32_t)NT, CU_TENSOR_MAP_SWIZZLE_128B))
+                   (uint32_t)tile_m, CU_TENSOR_MAP_SWIZZLE_128B))
     return fail(COMET_ERR_CUDA, "cuTensorMapEncodeTiled failed for the activation codes");
   if (!make_map_2d(&prm.map_w, w_packed, (uint64_t)(p.K / 2), (uint64_t)p.N, (uint64_t)(p.K / 2), 64,
-                   (uint32_t)kTileW, CU_TENSOR_MAP_SWIZZLE_64B))
+                   (uint32_t)tile_w, CU_TENSOR_MAP_SWIZZLE_64B))
     return fail(COMET_ERR_CUDA, "cuTensorMapEncodeTiled failed for the packed weights");
   prm.scales = act_scales;
   prm.corr = reinterpret_cast<const float*>(base + L.corr_off);
@@ -575,12 +519,12 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
   prm.ydt = (int)ydt;
   prm.tags = p.mask;
   cudaError_t e;
+  int grid;
   if (dbg) {
-    // whole tiles, one CTA each, NT = 64 (debug accumulators need the extra registers)
-    prm.n_m_tiles = (int)ceil_div(p.M, 64);
-    const int grid = (int)(prm.n_m_tiles * (p.N / kTileW));
+    // whole tiles, one CTA each, narrower tiles (the debug accumulators need the registers)
+    prm.n_m_tiles = (int)ceil_div(p.M, tile_m);
+    grid = (int)(prm.n_m_tiles * ceil_div(p.N, tile_w));
     prm.max_seg = 1;
-    e = debug_acc_blocks ? launch_nt<64, 2>(prm, grid, stream) : launch_nt<64, 1>(prm, grid, stream);
   } else {
     if (p.d_items == nullptr) return fail(COMET_ERR_INVALID_ARG, "plan was created with device_plan = 0");
     if (p.ws_bytes > 0 && (workspace == nullptr || ws_bytes < p.ws_bytes))
@@ -592,8 +536,14 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
     prm.ws_part = static_cast<float*>(workspace);
     prm.ws_flags = reinterpret_cast<uint32_t*>(static_cast<uint8_t*>(workspace) + p.ws_flags_off);
     prm.epoch = ++p.epoch;
-    const int grid = p.num_ctas;
-    switch (NT) {
+    grid = p.num_ctas;
+  }
+  if (normal) {
+    e = launch_gemm_n(prm, grid, tile_w, debug, stream);
+  } else if (dbg) {
+    e = debug == 2 ? launch_nt<64, 2>(prm, grid, stream) : launch_nt<64, 1>(prm, grid, stream);
+  } else {
+    switch (tile_m) {
       case 16: e = launch_nt<16, 0>(prm, grid, stream); break;
       case 32: e = launch_nt<32, 0>(prm, grid, stream); break;
       case 64: e = launch_nt<64, 0>(prm, grid, stream); break;

@@ -1,0 +1,82 @@
+// gemm_common.cuh -- pieces shared by the two W4Ax GEMM kernels (gemm.cu: weights on the MMA M
+// side, for decode-sized token counts; gemm_n.cu: tokens on the MMA M side, for prefill).
+#pragma once
+#include <cudaTypedefs.h>
+#include <cuda_fp16.h>
+#include <cuda_bf16.h>
+#include "internal.h"
+#include "sm100.cuh"
+
+namespace comet {
+namespace gemm {
+
+using namespace sm100;
+
+constexpr int kThreads = 512;
+constexpr int kSRing = 8;            // scale ring depth
+
+struct __align__(64) GemmParams {
+  CUtensorMap map_x;
+  CUtensorMap map_w;
+  const float* scales;       // [nb][Mp]
+  const float* corr;         // [Mp]
+  const int16_t* qsum;       // [nb][Mp]
+  const float* w_scales;     // [N]
+  void* y;
+  int64_t ldy;
+  int32_t* dbg_acc;          // [M][N] or null
+  int32_t* dbg_blocks;       // [nb][M][N] or null
+  float* ws_part;
+  uint32_t* ws_flags;
+  const int32_t* cta_begin;
+  const WorkItem* items;
+  int64_t M, N, Mp;
+  int nb, n_m_tiles, max_seg, ydt;
+  uint32_t epoch;
+  TagMask tags;
+};
+
+__device__ __forceinline__ void named_bar_sync(int id, int n) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
+}
+__device__ __forceinline__ void st_release_gpu(uint32_t* p, uint32_t v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ uint32_t ld_acquire_gpu(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+template <uint32_t N>
+__device__ __forceinline__ void setmaxnreg_dec() {
+  asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(N));
+}
+template <uint32_t N>
+__device__ __forceinline__ void setmaxnreg_inc() {
+  asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(N));
+}
+
+__device__ __forceinline__ WorkItem load_item(const GemmParams& P, int idx, bool debug) {
+  if (debug) {
+    WorkItem w{};
+    w.tile = blockIdx.x; w.kb_begin = 0; w.kb_end = P.nb; w.flags = 2; w.fix = -1;
+    return w;
+  }
+  const int4* src = reinterpret_cast<const int4*>(P.items + idx);
+  int4 a = __ldg(src);
+  int4 b = __ldg(src + 1);
+  WorkItem w;
+  w.tile = a.x; w.kb_begin = a.y; w.kb_end = a.z; w.flags = a.w;
+  w.fix = b.x; w.pad0 = b.y; w.pad1 = b.z; w.pad2 = b.w;
+  return w;
+}
+
+// Host: TMA descriptor helper (gemm.cu).
+bool make_map_2d(CUtensorMap* map, const void* base, uint64_t inner, uint64_t outer,
+                 uint64_t row_bytes, uint32_t box_inner, uint32_t box_outer, CUtensorMapSwizzle swz);
+
+// Normal-orientation launcher (gemm_n.cu).  BN = weights per tile (256, or 128 for debug).
+cudaError_t launch_gemm_n(const GemmParams& prm, int grid, int bn, int debug, cudaStream_t stream);
+
+}  // namespace gemm
+}  // namespace comet

@@ -37,6 +37,8 @@ static_assert(sizeof(WorkItem) == 32, "work item layout");
 struct Plan {
   int64_t M, N, K, nb, Mp;
   int tile_n, num_ctas, split_mode, stages;
+  int orientation = 1;   // 1: weights on MMA M (gemm.cu), 2: tokens on MMA M (gemm_n.cu)
+  int tile_w = 128;      // weights per output tile
   int64_t n_m_tiles, n_n_tiles, n_tiles;
   std::vector<uint8_t> tags;
   TagMask mask;

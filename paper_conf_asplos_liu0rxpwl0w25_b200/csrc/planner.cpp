@@ -83,13 +83,20 @@ static std::vector<int64_t> best_contiguous_cuts(const std::vector<double>& cost
 comet_status_t build_plan(Plan& p, const comet_sched_config& cfg) {
   p.nb = p.K / kBlockK;
   p.Mp = round_up(p.M, COMET_SCALE_PAD);
-  p.tile_n = cfg.tile_n > 0 ? cfg.tile_n : auto_tile_n(p.M);
-  if (!valid_tile_n(p.tile_n))
-    return fail(COMET_ERR_UNSUPPORTED_SHAPE, "tile_n must be one of 16, 32, 64, 128, 192, 224");
+  p.orientation = cfg.orientation > 0 ? cfg.orientation : (p.M >= 128 ? 2 : 1);
+  if (p.orientation == 2) {
+    p.tile_n = 128;          // tokens per tile = MMA M
+    p.tile_w = 256;          // weights per tile = MMA N
+  } else {
+    p.tile_n = cfg.tile_n > 0 ? cfg.tile_n : auto_tile_n(p.M);
+    p.tile_w = kTileW;
+    if (!valid_tile_n(p.tile_n))
+      return fail(COMET_ERR_UNSUPPORTED_SHAPE, "tile_n must be one of 16, 32, 64, 128, 192, 224");
+  }
   p.num_ctas = cfg.num_sms;
   if (p.num_ctas <= 0) return fail(COMET_ERR_INVALID_ARG, "num_sms must be resolved before planning");
   p.n_m_tiles = ceil_div(p.M, p.tile_n);
-  p.n_n_tiles = p.N / kTileW;
+  p.n_n_tiles = ceil_div(p.N, p.tile_w);
   p.n_tiles = p.n_m_tiles * p.n_n_tiles;
   const int P = p.num_ctas;
   const int64_t T = p.n_tiles;
@@ -216,7 +223,7 @@ comet_status_t build_plan(Plan& p, const comet_sched_config& cfg) {
   p.cta_begin[P] = (int32_t)p.items.size();
   p.max_cost = *std::max_element(load.begin(), load.end());
   p.mean_cost = std::accumulate(load.begin(), load.end(), 0.0) / P;
-  const size_t part = (size_t)p.tile_n * kTileW * sizeof(float);
+  const size_t part = (size_t)p.tile_n * p.tile_w * sizeof(float);
   const size_t n_part = (size_t)p.n_split_tiles * (size_t)(p.max_segments - 1);
   p.ws_flags_off = n_part * part;
   p.ws_bytes = p.n_split_tiles ? p.ws_flags_off + (size_t)p.n_split_tiles * p.max_segments * sizeof(uint32_t) : 0;

@@ -90,7 +90,8 @@ def test_fig8_product_planner_matches_paper(mode, key, expect):
     g = _fig8()
     M, N, K = g["gemm_mnk"]
     plan = cb.Plan(M, N, K, g["tags"], tile_n=128, num_sms=g["n_sm"], split_mode=mode,
-                   cost_int4=g["cost_int4"], cost_int8=g["cost_int8"], device_plan=False)
+                   cost_int4=g["cost_int4"], cost_int8=g["cost_int8"], device_plan=False,
+                   orientation=1)   # 128 x 128 output tiles, as in Fig. 8
     assert plan.info()["n_tiles"] == g["n_output_tiles"]
     segs = _segments(plan, g["n_sm"])
     oplan.check_cover(segs, g["n_output_tiles"], len(g["tags"]))
@@ -108,7 +109,7 @@ def test_fig8_decomposition_ordering():
     ms = {}
     for mode in (0, 1, 2, 3):
         plan = cb.Plan(M, N, K, g["tags"], tile_n=128, num_sms=4, split_mode=mode,
-                       cost_int4=1, cost_int8=2, device_plan=False)
+                       cost_int4=1, cost_int8=2, device_plan=False, orientation=1)
         segs = _segments(plan, 4)
         oplan.check_cover(segs, 9, 2)
         ms[mode] = oplan.makespan(segs, g["tags"], 1, 2)
@@ -123,6 +124,7 @@ def test_fig8_decomposition_ordering():
     assert best == 8
 
 
+@pytest.mark.parametrize("orientation", [0, 1, 2])
 @pytest.mark.parametrize("M,N,K,frac,P,mode", [
     (4096, 28672 // 8, 8192, 0.05, 148, 1),
     (4096, 1280, 8192, 0.05, 148, 1),
@@ -133,12 +135,13 @@ def test_fig8_decomposition_ordering():
     (300, 1024, 1024, 0.5, 13, 3),
     (77, 512, 768, 0.34, 7, 2),
 ])
-def test_planner_cover_order_and_balance(M, N, K, frac, P, mode):
+def test_planner_cover_order_and_balance(M, N, K, frac, P, mode, orientation):
     from paper_conf_asplos_liu0rxpwl0w25_b200 import synth
     rng = np.random.default_rng(M + N + K)
     tags = synth.make_tags(K, frac, rng)
     c8 = 1.5 if mode == 3 else 1.0
-    plan = cb.Plan(M, N, K, tags, num_sms=P, split_mode=mode, cost_int8=c8, device_plan=False)
+    plan = cb.Plan(M, N, K, tags, num_sms=P, split_mode=mode, cost_int8=c8, device_plan=False,
+                   orientation=orientation)
     info = plan.info()
     segs = _segments(plan, P)
     oplan.check_cover(segs, info["n_tiles"], K // 128)

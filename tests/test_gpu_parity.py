@@ -111,11 +111,12 @@ def test_pack_weight_layout(N, K):
 # ------------------------------------------------------------------------------- GEMM
 
 def _run(p: synth.Problem, *, tile_n=0, split_mode=-1, out_dtype=torch.float32, debug=False,
-         debug_blocks=False, num_sms=0):
+         debug_blocks=False, num_sms=0, orientation=0):
     act, sc = _quant(p)
     wp = cb.pack_weight(torch.from_numpy(p.w).to(DEV))
     sw = torch.from_numpy(p.s_w).to(DEV)
-    plan = cb.Plan(p.M, p.N, p.K, p.tags, tile_n=tile_n, split_mode=split_mode, num_sms=num_sms)
+    plan = cb.Plan(p.M, p.N, p.K, p.tags, tile_n=tile_n, split_mode=split_mode, num_sms=num_sms,
+                   orientation=orientation)
     res = cb.w4ax_gemm(plan, act, sc, wp, sw, out_dtype=out_dtype, debug=debug, debug_blocks=debug_blocks)
     torch.cuda.synchronize()
     return res, plan
@@ -133,9 +134,10 @@ def _close(y, ref, dtype):
         assert not bad.any(), f"{bad.sum()} outputs outside rtol 1e-3 / atol 1e-2; max err {np.abs(got-ref).max()}"
 
 
-def test_gemm_config1_bit_exact_blocks():
+@pytest.mark.parametrize("orientation", [1, 2])
+def test_gemm_config1_bit_exact_blocks(orientation):
     p = synth.config1()
-    (y, dacc, dblk), _ = _run(p, debug_blocks=True)
+    (y, dacc, dblk), _ = _run(p, debug_blocks=True, orientation=orientation)
     yref, acc, _, _ = oracle.w4ax(p.x, p.tags, p.w, p.s_w)
     assert np.array_equal(dblk.cpu().numpy().astype(np.int64), acc), "per-block INT32 accumulators differ"
     assert np.array_equal(dacc.cpu().numpy().astype(np.int64), acc.sum(0))
@@ -146,18 +148,20 @@ def test_gemm_config1_bit_exact_blocks():
     (1, 256, 512, 0.5), (17, 384, 1024, 0.25), (100, 512, 2048, 0.05), (300, 256, 768, 1.0),
     (64, 128, 256, 0.0),
 ])
-def test_gemm_debug_accumulators_exact(M, N, K, frac):
+@pytest.mark.parametrize("orientation", [1, 2])
+def test_gemm_debug_accumulators_exact(M, N, K, frac, orientation):
     p = synth.make_problem(M, K, N, frac=frac, seed=M * 7 + K)
-    (y, dacc), _ = _run(p, debug=True)
+    (y, dacc), _ = _run(p, debug=True, orientation=orientation)
     yref, acc, _, _ = oracle.w4ax(p.x, p.tags, p.w, p.s_w)
     assert np.array_equal(dacc.cpu().numpy().astype(np.int64), acc.sum(0))
     _close(y, yref, torch.float32)
 
 
-def test_gemm_all_int8_matches_torch_int_mm():
+@pytest.mark.parametrize("orientation", [1, 2])
+def test_gemm_all_int8_matches_torch_int_mm(orientation):
     """I1 on the GPU: all tags INT8 -> per-block accumulators equal cuBLASLt's INT8 GEMM."""
     p = synth.make_problem(64, 512, 256, frac=1.0, seed=5)
-    (y, dacc, dblk), _ = _run(p, debug_blocks=True)
+    (y, dacc, dblk), _ = _run(p, debug_blocks=True, orientation=orientation)
     codes, _ = oracle.quantize(p.x, p.tags)
     for b in range(4):
         a = torch.from_numpy(codes[:, b * 128:(b + 1) * 128].copy()).to(DEV)
@@ -170,24 +174,36 @@ def test_gemm_all_int8_matches_torch_int_mm():
 @pytest.mark.parametrize("split_mode", [0, 1])
 def test_gemm_tile_and_schedule_variants(tile_n, split_mode):
     p = synth.make_problem(230, 2048, 1024, frac=0.25, seed=tile_n)
-    y, plan = _run(p, tile_n=tile_n, split_mode=split_mode, num_sms=37)
+    y, plan = _run(p, tile_n=tile_n, split_mode=split_mode, num_sms=37, orientation=1)
     yref, _, _, _ = oracle.w4ax(p.x, p.tags, p.w, p.s_w)
     _close(y, yref, torch.float32)
 
 
+@pytest.mark.parametrize("M,N", [(230, 2048), (300, 1152), (129, 256), (1000, 384)])
+@pytest.mark.parametrize("split_mode", [0, 1])
+def test_gemm_normal_orientation_schedules(M, N, split_mode):
+    """Tokens on the MMA M side (prefill kernel): ragged M, N % 256 == 128, stream-K."""
+    p = synth.make_problem(M, 1024, N, frac=0.25, seed=M + N)
+    y, plan = _run(p, split_mode=split_mode, num_sms=23, orientation=2)
+    yref, _, _, _ = oracle.w4ax(p.x, p.tags, p.w, p.s_w)
+    _close(y, yref, torch.float32)
+
+
+@pytest.mark.parametrize("orientation", [1, 2])
 @pytest.mark.parametrize("split_mode", [2, 3])
-def test_gemm_unit_schedules(split_mode):
+def test_gemm_unit_schedules(split_mode, orientation):
     p = synth.make_problem(96, 512, 1024, frac=0.25, seed=11)
-    y, plan = _run(p, split_mode=split_mode, num_sms=13)
+    y, plan = _run(p, split_mode=split_mode, num_sms=13, orientation=orientation)
     assert plan.info()["n_split_tiles"] > 0
     yref, _, _, _ = oracle.w4ax(p.x, p.tags, p.w, p.s_w)
     _close(y, yref, torch.float32)
 
 
+@pytest.mark.parametrize("orientation", [1, 2])
 @pytest.mark.parametrize("dtype", [torch.float16, torch.bfloat16, torch.float32])
-def test_gemm_output_dtypes(dtype):
+def test_gemm_output_dtypes(dtype, orientation):
     p = synth.make_problem(48, 1024, 512, frac=0.25, seed=21)
-    y, _ = _run(p, out_dtype=dtype)
+    y, _ = _run(p, out_dtype=dtype, orientation=orientation)
     yref, _, _, _ = oracle.w4ax(p.x, p.tags, p.w, p.s_w)
     _close(y, yref, dtype)
 
@@ -201,9 +217,10 @@ def test_gemm_outlier_fraction_sweep(frac):
     _close(y, yref, torch.float32)
 
 
-def test_gemm_bf16_input():
+@pytest.mark.parametrize("orientation", [1, 2])
+def test_gemm_bf16_input(orientation):
     p = synth.make_problem(40, 1024, 384, frac=0.34, seed=41, bf16=True)
-    (y, dacc), _ = _run(p, debug=True)
+    (y, dacc), _ = _run(p, debug=True, orientation=orientation)
     yref, acc, _, _ = oracle.w4ax(p.x, p.tags, p.w, p.s_w, bf16_bits=True)
     assert np.array_equal(dacc.cpu().numpy().astype(np.int64), acc.sum(0))
     _close(y, yref, torch.float32)
