@@ -146,11 +146,13 @@ typedef struct {
   int stages;          /* shared-memory ring depth; 0 = auto */
   int device_plan;     /* 1 (default) = upload the work list to the device at create time;
                           0 = host-only plan (comet_plan_describe only; CPU-safe) */
-  int orientation;     /* 0 = auto (2 when M >= 128, else 1);
+  int orientation;     /* 0 = auto (3 when M >= 256, 2 when M >= 128, else 1);
                           1 = weights on the MMA M side: tile = 128 weights x tile_n tokens
                               (decode-sized M; weights widened into TMEM);
                           2 = tokens on the MMA M side: tile = 128 tokens x 256 weights
-                              (prefill; weights widened into shared memory), tile_n ignored */
+                              (prefill; weights widened into shared memory), tile_n ignored;
+                          3 = as 2 on a tcgen05 CTA pair: tile = 256 tokens x 256 weights,
+                              each SM widens half the weights; num_ctas counts pairs */
   int reserved[5];
 } comet_sched_config;
 

@@ -83,8 +83,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
   const bool debug = DEBUG != 0;
-  const int it_begin = debug ? 0 : P.cta_begin[blockIdx.x];
-  const int it_end = debug ? 1 : P.cta_begin[blockIdx.x + 1];
+  const int it_begin = debug ? (int)blockIdx.x : P.cta_begin[blockIdx.x];
+  const int it_end = debug ? (int)blockIdx.x + 1 : P.cta_begin[blockIdx.x + 1];
   const int nb = P.nb;
 
   if (warp == 0 && lane == 0) {
@@ -488,21 +488,23 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
   *launches = 0;
   const bool dbg = debug_acc != nullptr || debug_acc_blocks != nullptr;
   const int debug = debug_acc_blocks ? 2 : (dbg ? 1 : 0);
-  const bool normal = p.orientation == 2;
-  // token-tile (box rows of the activation TMA) and weight-tile (box rows of the weight TMA)
-  int tile_m, tile_w;
-  if (normal) { tile_m = 128; tile_w = dbg ? 128 : 256; }
-  else { tile_m = dbg ? 64 : p.tile_n; tile_w = kTileW; }
+  const bool normal = p.orientation >= 2;
+  const int cg = p.orientation == 3 ? 2 : 1;
+  // token-tile and weight-tile of one CTA (= box rows of the two TMA maps) and of the tile
+  int tile_m, tile_w, cta_rows_w;
+  if (normal) { tile_m = 128 * cg; tile_w = dbg ? 128 : 256; cta_rows_w = tile_w / cg; }
+  else { tile_m = dbg ? 64 : p.tile_n; tile_w = kTileW; cta_rows_w = kTileW; }
+  const int box_m = normal ? 128 : tile_m;
   comet_act_layout_t L;
   act_layout(p.M, p.K, &L);
   const uint8_t* base = static_cast<const uint8_t*>(act_packed);
   GemmParams prm;
   memset(&prm, 0, sizeof(prm));
   if (!make_map_2d(&prm.map_x, base + L.codes_off, (uint64_t)p.K, (uint64_t)p.M, (uint64_t)p.K, 128,
-                   (uint32_t)tile_m, CU_TENSOR_MAP_SWIZZLE_128B))
+                   (uint32_t)box_m, CU_TENSOR_MAP_SWIZZLE_128B))
     return fail(COMET_ERR_CUDA, "cuTensorMapEncodeTiled failed for the activation codes");
   if (!make_map_2d(&prm.map_w, w_packed, (uint64_t)(p.K / 2), (uint64_t)p.N, (uint64_t)(p.K / 2), 64,
-                   (uint32_t)tile_w, CU_TENSOR_MAP_SWIZZLE_64B))
+                   (uint32_t)cta_rows_w, CU_TENSOR_MAP_SWIZZLE_64B))
     return fail(COMET_ERR_CUDA, "cuTensorMapEncodeTiled failed for the packed weights");
   prm.scales = act_scales;
   prm.corr = reinterpret_cast<const float*>(base + L.corr_off);
@@ -523,7 +525,7 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
   if (dbg) {
     // whole tiles, one CTA each, narrower tiles (the debug accumulators need the registers)
     prm.n_m_tiles = (int)ceil_div(p.M, tile_m);
-    grid = (int)(prm.n_m_tiles * ceil_div(p.N, tile_w));
+    grid = (int)(prm.n_m_tiles * ceil_div(p.N, tile_w)) * cg;
     prm.max_seg = 1;
   } else {
     if (p.d_items == nullptr) return fail(COMET_ERR_INVALID_ARG, "plan was created with device_plan = 0");
@@ -536,10 +538,10 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
     prm.ws_part = static_cast<float*>(workspace);
     prm.ws_flags = reinterpret_cast<uint32_t*>(static_cast<uint8_t*>(workspace) + p.ws_flags_off);
     prm.epoch = ++p.epoch;
-    grid = p.num_ctas;
+    grid = p.num_ctas * cg;
   }
   if (normal) {
-    e = launch_gemm_n(prm, grid, tile_w, debug, stream);
+    e = launch_gemm_n(prm, grid, tile_w, cg, debug, stream);
   } else if (dbg) {
     e = debug == 2 ? launch_nt<64, 2>(prm, grid, stream) : launch_nt<64, 1>(prm, grid, stream);
   } else {

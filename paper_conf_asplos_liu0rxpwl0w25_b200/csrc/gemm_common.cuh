@@ -59,7 +59,7 @@ __device__ __forceinline__ void setmaxnreg_inc() {
 __device__ __forceinline__ WorkItem load_item(const GemmParams& P, int idx, bool debug) {
   if (debug) {
     WorkItem w{};
-    w.tile = blockIdx.x; w.kb_begin = 0; w.kb_end = P.nb; w.flags = 2; w.fix = -1;
+    w.tile = idx; w.kb_begin = 0; w.kb_end = P.nb; w.flags = 2; w.fix = -1;
     return w;
   }
   const int4* src = reinterpret_cast<const int4*>(P.items + idx);
@@ -75,8 +75,9 @@ __device__ __forceinline__ WorkItem load_item(const GemmParams& P, int idx, bool
 bool make_map_2d(CUtensorMap* map, const void* base, uint64_t inner, uint64_t outer,
                  uint64_t row_bytes, uint32_t box_inner, uint32_t box_outer, CUtensorMapSwizzle swz);
 
-// Normal-orientation launcher (gemm_n.cu).  BN = weights per tile (256, or 128 for debug).
-cudaError_t launch_gemm_n(const GemmParams& prm, int grid, int bn, int debug, cudaStream_t stream);
+// Normal-orientation launcher (gemm_n.cu).  BN = weights per tile (256, or 128 for debug);
+// cg = CTAs per tile (1, or 2 for the tcgen05 CTA pair; grid must then be even).
+cudaError_t launch_gemm_n(const GemmParams& prm, int grid, int bn, int cg, int debug, cudaStream_t stream);
 
 }  // namespace gemm
 }  // namespace comet

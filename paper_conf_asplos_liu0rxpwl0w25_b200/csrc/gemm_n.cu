@@ -14,25 +14,31 @@
 // its registers with FFMA2 (two columns per instruction).
 //
 // Roles (512 threads): warp 0 TMA producer, warp 1 MMA issuer, warp 2 TMEM allocator,
-// warps 4-7 widen (each thread 2 weight rows per K-block), warps 8-15 promotion + epilogue
-// (two warpgroups, BN/2 columns each).
+// warps 4-7 widen, warps 8-15 promotion + epilogue (two warpgroups, BN/2 columns each).
+//
+// CG = 2 (CTA pair, tcgen05 cta_group::2): the tile is 256 tokens x BN weights; CTA r of the
+// pair holds tokens m0 + 128 r (its half of A, its TMEM lanes) and widens weights
+// n0 + r BN/2 .. (its half of B), so each SM widens half as many weight rows per MMA FLOP.
+// The even CTA issues the pair MMA; both CTAs' widen / promotion warps arrive on the even
+// CTA's b_full / acc_empty barriers, MMA completion is multicast to both CTAs.
 #include "gemm_common.cuh"
 
 namespace comet {
 namespace gemm {
 namespace {
 
-template <int BN>
+template <int BN, int CG>
 struct CfgN {
-  static constexpr int BM = 128;                          // tokens per tile
+  static constexpr int BM = 128;                          // tokens per CTA (TMEM lanes)
+  static constexpr int WROWS = BN / CG;                   // weight rows widened by this CTA
   static constexpr int X_BYTES = BM * 128;                // activation tile (one K-block)
-  static constexpr int WP_BYTES = BN * 64;                // packed weight tile
+  static constexpr int WP_BYTES = WROWS * 64;             // packed weight rows
   static constexpr int STAGE_BYTES = X_BYTES + WP_BYTES;
-  static constexpr int B_BYTES = BN * 128;                // widened weight tile (MMA B)
+  static constexpr int B_BYTES = WROWS * 128;             // widened weight rows (MMA B half)
   static constexpr int NBUF = 2;                          // widened-weight ring
   static constexpr int COLS = BN / 2;                     // accumulator columns per promotion WG
   static constexpr int NACC = (3 * BN <= 512) ? 3 : 2;    // accumulators in TMEM
-  static constexpr int ROWS_PER_THREAD = BN / 128;        // widen rows per thread
+  static constexpr int ROWS_PER_THREAD = (WROWS + 127) / 128;   // widen rows per thread
   static constexpr int STAGES_RAW = (200 * 1024 - NBUF * B_BYTES - kSRing * BM * 4) / STAGE_BYTES;
   static constexpr int STAGES = STAGES_RAW > 8 ? 8 : STAGES_RAW;
   static constexpr int SMEM_DATA = STAGES * STAGE_BYTES + NBUF * B_BYTES + kSRing * BM * 4;
@@ -43,9 +49,9 @@ struct CfgN {
   static_assert(COLS % 32 == 0, "promotion batches");
 };
 
-template <int BN, int DEBUG>
+template <int BN, int CG, int DEBUG>
 __global__ void __launch_bounds__(kThreads, 1) k_w4ax_n(const __grid_constant__ GemmParams P) {
-  using C = CfgN<BN>;
+  using C = CfgN<BN, CG>;
   constexpr int S = C::STAGES;
   constexpr int NACC = C::NACC;
   constexpr int BM = C::BM;
@@ -71,8 +77,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax_n(const __grid_constant__ 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
   const bool debug = DEBUG != 0;
-  const int it_begin = debug ? 0 : P.cta_begin[blockIdx.x];
-  const int it_end = debug ? 1 : P.cta_begin[blockIdx.x + 1];
+  const uint32_t rank = CG == 2 ? cluster_ctarank() : 0;   // CTA rank within the pair
+  const int unit = blockIdx.x / CG;                          // work list index (pair or CTA)
+  const int it_begin = debug ? unit : P.cta_begin[unit];
+  const int it_end = debug ? unit + 1 : P.cta_begin[unit + 1];
   const int nb = P.nb;
 
   if (warp == 0 && lane == 0) {
@@ -83,12 +91,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax_n(const __grid_constant__ 
       mbar_init(&empty[i], 1 + 4);
     }
     for (int i = 0; i < C::NBUF; ++i) {
-      mbar_init(&b_full[i], 4);
+      mbar_init(&b_full[i], 4 * CG);
       mbar_init(&b_empty[i], 1);
     }
     for (int i = 0; i < NACC; ++i) {
       mbar_init(&acc_full[i], 1);
-      mbar_init(&acc_empty[i], 8);
+      mbar_init(&acc_empty[i], 8 * CG);
     }
     for (int i = 0; i < kSRing; ++i) {
       mbar_init(&s_full[i], 1);
@@ -97,14 +105,19 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax_n(const __grid_constant__ 
     fence_mbar_init();
   }
   if (warp == 2) {
-    tmem_alloc<512>(tmem_holder);
-    tmem_relinquish();
+    if (CG == 2) { tmem_alloc_cg2<512>(tmem_holder); tmem_relinquish_cg2(); }
+    else { tmem_alloc<512>(tmem_holder); tmem_relinquish(); }
   }
   for (int i = threadIdx.x; i < nb; i += kThreads) s_tags[i] = P.tags.get(i) ? 1 : 0;
   tc_fence_before();
   __syncthreads();
+  if (CG == 2) cluster_sync();                 // peer barriers initialised before remote arrives
   tc_fence_after();
   const uint32_t tbase = *tmem_holder;
+  // the even CTA's barriers that both CTAs arrive on (shared::cluster addresses)
+  const uint32_t b_full_lead = CG == 2 ? mapa_shared(smem_u32(b_full), 0) : smem_u32(b_full);
+  const uint32_t acc_empty_lead = CG == 2 ? mapa_shared(smem_u32(acc_empty), 0) : smem_u32(acc_empty);
+  auto wait_x = [&](uint64_t* bar, uint32_t par) { mbar_wait(bar, par); };
 
   if (warp < 4) {
     setmaxnreg_dec<32>();
@@ -115,48 +128,62 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax_n(const __grid_constant__ 
       for (int it = it_begin; it < it_end; ++it) {
         const WorkItem w = load_item(P, it, debug);
         const int n_tile = w.tile / P.n_m_tiles, m_tile = w.tile % P.n_m_tiles;
-        const int m0 = m_tile * BM, n0 = n_tile * BN;
-        const uint32_t sbytes = (uint32_t)(min((int64_t)BM, P.Mp - m0) * 4);
+        const int m0 = m_tile * (BM * CG) + BM * rank, n0 = n_tile * BN + C::WROWS * rank;
+        const uint32_t sbytes = m0 < P.Mp ? (uint32_t)(min((int64_t)BM, P.Mp - m0) * 4) : 0u;
         for (int kb = w.kb_begin; kb < w.kb_end; ++kb) {
-          mbar_wait(&empty[stage], ph ^ 1);
+          wait_x(&empty[stage], ph ^ 1);
           mbar_arrive_expect_tx(&full[stage], C::STAGE_BYTES);
           tma_load_2d(sX + stage * C::X_BYTES, &P.map_x, &full[stage], kb * 128, m0);
           tma_load_2d(sWp + stage * C::WP_BYTES, &P.map_w, &full[stage], kb * 64, n0);
           mbar_wait(&s_empty[ss], sph ^ 1);
-          mbar_arrive_expect_tx(&s_full[ss], sbytes);
-          bulk_load(sS + ss * BM, P.scales + (int64_t)kb * P.Mp + m0, sbytes, &s_full[ss]);
+          if (sbytes) {
+            mbar_arrive_expect_tx(&s_full[ss], sbytes);
+            bulk_load(sS + ss * BM, P.scales + (int64_t)kb * P.Mp + m0, sbytes, &s_full[ss]);
+          } else {
+            mbar_arrive(&s_full[ss]);        // this CTA's tokens are all padding
+          }
           if (++stage == S) { stage = 0; ph ^= 1; }
           if (++ss == kSRing) { ss = 0; sph ^= 1; }
         }
       }
-    } else if (warp == 1 && lane == 0) {
+    } else if (warp == 1 && lane == 0 && rank == 0) {
       // ------------------------------------------------------------------ MMA issuer
-      const uint32_t id_f8 = idesc_f8f6f4_e4m3(BM, BN);
-      const uint32_t id_i8 = idesc_i8(BM, BN);
+      const uint32_t id_f8 = idesc_f8f6f4_e4m3(BM * CG, BN);
+      const uint32_t id_i8 = idesc_i8(BM * CG, BN);
       int stage = 0, bb = 0, accb = 0;
       uint32_t ph = 0, bph = 0, accph = 0;
       for (int it = it_begin; it < it_end; ++it) {
         const WorkItem w = load_item(P, it, debug);
         for (int kb = w.kb_begin; kb < w.kb_end; ++kb) {
-          mbar_wait(&acc_empty[accb], accph ^ 1);
-          mbar_wait(&full[stage], ph);
-          mbar_wait(&b_full[bb], bph);
+          wait_x(&acc_empty[accb], accph ^ 1);
+          // b_full covers the stage too: every widen warp waited on its CTA's full[stage]
+          wait_x(&b_full[bb], bph);
           tc_fence_after();
           const uint32_t d = tbase + accb * BN;
           const uint32_t sa = smem_u32(sX + stage * C::X_BYTES);
           const uint32_t sbv = smem_u32(sB + bb * C::B_BYTES);
           if (lds_u8(s_tags_a + kb)) {
 #pragma unroll
-            for (int k = 0; k < 4; ++k)
-              mma_i8_ss(d, sdesc_kmajor_sw128(sa + 32 * k), sdesc_kmajor_sw128(sbv + 32 * k), id_i8, k);
+            for (int k = 0; k < 4; ++k) {
+              const uint64_t ad = sdesc_kmajor_sw128(sa + 32 * k), bd = sdesc_kmajor_sw128(sbv + 32 * k);
+              if (CG == 2) mma_i8_ss_cg2(d, ad, bd, id_i8, k); else mma_i8_ss(d, ad, bd, id_i8, k);
+            }
           } else {
 #pragma unroll
-            for (int k = 0; k < 4; ++k)
-              mma_f8_ss(d, sdesc_kmajor_sw128(sa + 32 * k), sdesc_kmajor_sw128(sbv + 32 * k), id_f8, k);
+            for (int k = 0; k < 4; ++k) {
+              const uint64_t ad = sdesc_kmajor_sw128(sa + 32 * k), bd = sdesc_kmajor_sw128(sbv + 32 * k);
+              if (CG == 2) mma_f8_ss_cg2(d, ad, bd, id_f8, k); else mma_f8_ss(d, ad, bd, id_f8, k);
+            }
           }
-          tc_commit(&empty[stage]);
-          tc_commit(&b_empty[bb]);
-          tc_commit(&acc_full[accb]);
+          if (CG == 2) {
+            tc_commit_mc(&empty[stage], 3);
+            tc_commit_mc(&b_empty[bb], 3);
+            tc_commit_mc(&acc_full[accb], 3);
+          } else {
+            tc_commit(&empty[stage]);
+            tc_commit(&b_empty[bb]);
+            tc_commit(&acc_full[accb]);
+          }
           if (++stage == S) { stage = 0; ph ^= 1; }
           if (++bb == C::NBUF) { bb = 0; bph ^= 1; }
           if (++accb == NACC) { accb = 0; accph ^= 1; }
@@ -167,6 +194,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax_n(const __grid_constant__ 
     setmaxnreg_dec<64>();
     // -------------------------------------------------------------------- widen (W -> smem B)
     const int t = threadIdx.x - 128;                      // weight row t (and t + 128)
+    const bool has_row = t < C::WROWS;
     const uint32_t sWp_a = smem_u32(sWp), sB_a = smem_u32(sB);
     int stage = 0, bb = 0;
     uint32_t ph = 0, bph = 0;
@@ -174,7 +202,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax_n(const __grid_constant__ 
       const WorkItem w = load_item(P, it, debug);
       for (int kb = w.kb_begin; kb < w.kb_end; ++kb) {
         const bool is8 = lds_u8(s_tags_a + kb) != 0;
-        mbar_wait(&full[stage], ph);
+        wait_x(&full[stage], ph);
         uint4 c[C::ROWS_PER_THREAD][4];
 #pragma unroll
         for (int rr = 0; rr < C::ROWS_PER_THREAD; ++rr) {
@@ -182,13 +210,14 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax_n(const __grid_constant__ 
           const uint32_t src = sWp_a + stage * C::WP_BYTES + row * 64;
           const int sw = (row >> 1) & 3;                  // TMA 64-byte swizzle
 #pragma unroll
-          for (int j = 0; j < 4; ++j) c[rr][j] = lds128(src + ((j ^ sw) << 4));
+          for (int j = 0; j < 4; ++j) c[rr][j] = has_row ? lds128(src + ((j ^ sw) << 4)) : make_uint4(0, 0, 0, 0);
         }
         __syncwarp();
         if (lane == 0) mbar_arrive(&empty[stage]);
-        mbar_wait(&b_empty[bb], bph ^ 1);
+        wait_x(&b_empty[bb], bph ^ 1);
 #pragma unroll
         for (int rr = 0; rr < C::ROWS_PER_THREAD; ++rr) {
+          if (!has_row) break;
           const int row = t + 128 * rr;
           const uint32_t dst = sB_a + bb * C::B_BYTES + row * 128;
           const int sw = row & 7;                         // UMMA/TMA 128-byte swizzle
@@ -216,7 +245,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax_n(const __grid_constant__ 
         }
         fence_proxy_async_smem();                         // generic-proxy stores -> tensor core
         __syncwarp();
-        if (lane == 0) mbar_arrive(&b_full[bb]);
+        if (lane == 0) mbar_arrive_cluster(b_full_lead + bb * 8);
         if (++stage == S) { stage = 0; ph ^= 1; }
         if (++bb == C::NBUF) { bb = 0; bph ^= 1; }
       }
@@ -239,7 +268,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax_n(const __grid_constant__ 
     for (int it = it_begin; it < it_end; ++it) {
       const WorkItem w = load_item(P, it, debug);
       const int n_tile = w.tile / P.n_m_tiles, m_tile = w.tile % P.n_m_tiles;
-      const int m0 = m_tile * BM, n0 = n_tile * BN;
+      const int m0 = m_tile * (BM * CG) + BM * rank, n0 = n_tile * BN;
       const int64_t m = m0 + r;
       const bool owner = (w.flags & 2) != 0;
       const bool split = (w.flags & 1) != 0;
@@ -260,7 +289,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax_n(const __grid_constant__ 
         const float2 s2 = make_float2(s, s);
         int qs = 0;
         if (DEBUG && !is8 && m < P.Mp) qs = P.qsum[(int64_t)kb * P.Mp + m];
-        mbar_wait(&acc_full[accb], accph);
+        wait_x(&acc_full[accb], accph);
         tc_fence_after();
         const uint32_t taddr = tbase + accb * BN + col0 + lane_addr;
 #pragma unroll
@@ -293,7 +322,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax_n(const __grid_constant__ 
         tc_fence_before();
         __syncwarp();
         if (lane == 0) {
-          mbar_arrive(&acc_empty[accb]);
+          mbar_arrive_cluster(acc_empty_lead + accb * 8);
           mbar_arrive(&s_empty[ss]);
         }
         if (++ss == kSRing) { ss = 0; sph ^= 1; }
@@ -306,17 +335,17 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax_n(const __grid_constant__ 
         const int64_t part_tile = (int64_t)BM * BN;        // = 256 threads * COLS floats
         if (!owner) {
           float4* dst = reinterpret_cast<float4*>(
-              P.ws_part + ((int64_t)w.fix * (P.max_seg - 1) + (seg - 1)) * part_tile + (int64_t)ptid * COLS);
+              P.ws_part + (((int64_t)w.fix * (P.max_seg - 1) + (seg - 1)) * CG + rank) * part_tile + (int64_t)ptid * COLS);
 #pragma unroll
           for (int a = 0; a < COLS; a += 4) dst[a / 4] = make_float4(acc[a], acc[a + 1], acc[a + 2], acc[a + 3]);
           __threadfence();
           named_bar_sync(1, 256);
-          if (threadIdx.x == 256) st_release_gpu(P.ws_flags + (int64_t)w.fix * P.max_seg + seg, P.epoch);
+          if (threadIdx.x == 256) st_release_gpu(P.ws_flags + ((int64_t)w.fix * P.max_seg + seg) * CG + rank, P.epoch);
           continue;
         }
         if (threadIdx.x == 256) {
           for (int sgi = 1; sgi < nseg; ++sgi) {
-            const uint32_t* f = P.ws_flags + (int64_t)w.fix * P.max_seg + sgi;
+            const uint32_t* f = P.ws_flags + ((int64_t)w.fix * P.max_seg + sgi) * CG + rank;
             uint64_t t0g = globaltimer_ns();
             while (ld_acquire_gpu(f) != P.epoch) {
               if (globaltimer_ns() - t0g > COMET_MBAR_TIMEOUT_NS) {
@@ -329,7 +358,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax_n(const __grid_constant__ 
         named_bar_sync(1, 256);
         for (int sgi = 1; sgi < nseg; ++sgi) {
           const float4* src = reinterpret_cast<const float4*>(
-              P.ws_part + ((int64_t)w.fix * (P.max_seg - 1) + (sgi - 1)) * part_tile + (int64_t)ptid * COLS);
+              P.ws_part + (((int64_t)w.fix * (P.max_seg - 1) + (sgi - 1)) * CG + rank) * part_tile + (int64_t)ptid * COLS);
 #pragma unroll
           for (int a = 0; a < COLS; a += 4) {
             float4 t4;
@@ -384,29 +413,48 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax_n(const __grid_constant__ 
 
   tc_fence_before();
   __syncthreads();
-  if (warp == 2) tmem_dealloc<512>(tbase);
+  if (CG == 2) cluster_sync();                 // the pair is done with each other's smem / TMEM
+  if (warp == 2) {
+    if (CG == 2) tmem_dealloc_cg2<512>(tbase); else tmem_dealloc<512>(tbase);
+  }
 }
 
-template <int BN, int DEBUG>
+template <int BN, int CG, int DEBUG>
 cudaError_t launch_bn(const GemmParams& prm, int grid, cudaStream_t stream) {
-  using C = CfgN<BN>;
+  using C = CfgN<BN, CG>;
   static bool attr_set = false;
   if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(k_w4ax_n<BN, DEBUG>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_BYTES);
+    cudaError_t e = cudaFuncSetAttribute(k_w4ax_n<BN, CG, DEBUG>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_BYTES);
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
-  k_w4ax_n<BN, DEBUG><<<grid, kThreads, C::SMEM_BYTES, stream>>>(prm);
-  return cudaGetLastError();
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)grid);
+  cfg.blockDim = dim3(kThreads);
+  cfg.dynamicSmemBytes = C::SMEM_BYTES;
+  cfg.stream = stream;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = CG;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, k_w4ax_n<BN, CG, DEBUG>, prm);
 }
 
 }  // namespace
 
-cudaError_t launch_gemm_n(const GemmParams& prm, int grid, int bn, int debug, cudaStream_t stream) {
-  if (debug == 2) return launch_bn<128, 2>(prm, grid, stream);
-  if (debug == 1) return launch_bn<128, 1>(prm, grid, stream);
-  if (bn == 128) return launch_bn<128, 0>(prm, grid, stream);
-  return launch_bn<256, 0>(prm, grid, stream);
+cudaError_t launch_gemm_n(const GemmParams& prm, int grid, int bn, int cg, int debug, cudaStream_t stream) {
+  if (cg == 2) {
+    if (debug == 2) return launch_bn<128, 2, 2>(prm, grid, stream);
+    if (debug == 1) return launch_bn<128, 2, 1>(prm, grid, stream);
+    return launch_bn<256, 2, 0>(prm, grid, stream);
+  }
+  if (debug == 2) return launch_bn<128, 1, 2>(prm, grid, stream);
+  if (debug == 1) return launch_bn<128, 1, 1>(prm, grid, stream);
+  if (bn == 128) return launch_bn<128, 1, 0>(prm, grid, stream);
+  return launch_bn<256, 1, 0>(prm, grid, stream);
 }
 
 }  // namespace gemm

@@ -83,18 +83,19 @@ static std::vector<int64_t> best_contiguous_cuts(const std::vector<double>& cost
 comet_status_t build_plan(Plan& p, const comet_sched_config& cfg) {
   p.nb = p.K / kBlockK;
   p.Mp = round_up(p.M, COMET_SCALE_PAD);
-  p.orientation = cfg.orientation > 0 ? cfg.orientation : (p.M >= 128 ? 2 : 1);
-  if (p.orientation == 2) {
-    p.tile_n = 128;          // tokens per tile = MMA M
-    p.tile_w = 256;          // weights per tile = MMA N
+  p.orientation = cfg.orientation > 0 ? cfg.orientation : (p.M >= 256 ? 3 : (p.M >= 128 ? 2 : 1));
+  if (p.orientation >= 2) {
+    p.tile_n = p.orientation == 3 ? 256 : 128;   // tokens per tile = MMA M (CTA pair: 2 x 128)
+    p.tile_w = 256;                              // weights per tile = MMA N
   } else {
     p.tile_n = cfg.tile_n > 0 ? cfg.tile_n : auto_tile_n(p.M);
     p.tile_w = kTileW;
     if (!valid_tile_n(p.tile_n))
       return fail(COMET_ERR_UNSUPPORTED_SHAPE, "tile_n must be one of 16, 32, 64, 128, 192, 224");
   }
-  p.num_ctas = cfg.num_sms;
-  if (p.num_ctas <= 0) return fail(COMET_ERR_INVALID_ARG, "num_sms must be resolved before planning");
+  // scheduling units: CTAs, or CTA pairs for the pair kernel
+  p.num_ctas = p.orientation == 3 ? cfg.num_sms / 2 : cfg.num_sms;
+  if (p.num_ctas <= 0) return fail(COMET_ERR_INVALID_ARG, "num_sms must be resolved before planning (>= 2 for CTA pairs)");
   p.n_m_tiles = ceil_div(p.M, p.tile_n);
   p.n_n_tiles = ceil_div(p.N, p.tile_w);
   p.n_tiles = p.n_m_tiles * p.n_n_tiles;
@@ -226,7 +227,7 @@ comet_status_t build_plan(Plan& p, const comet_sched_config& cfg) {
   const size_t part = (size_t)p.tile_n * p.tile_w * sizeof(float);
   const size_t n_part = (size_t)p.n_split_tiles * (size_t)(p.max_segments - 1);
   p.ws_flags_off = n_part * part;
-  p.ws_bytes = p.n_split_tiles ? p.ws_flags_off + (size_t)p.n_split_tiles * p.max_segments * sizeof(uint32_t) : 0;
+  p.ws_bytes = p.n_split_tiles ? p.ws_flags_off + (size_t)p.n_split_tiles * p.max_segments * 2 * sizeof(uint32_t) : 0;
   p.ws_bytes = (p.ws_bytes + 255) / 256 * 256;
   if (p.ws_bytes > ((size_t)8 << 30)) return fail(COMET_ERR_UNSUPPORTED_SHAPE, "schedule needs more than 8 GiB of fix-up workspace");
   return COMET_OK;

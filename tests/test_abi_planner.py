@@ -143,6 +143,7 @@ def test_planner_cover_order_and_balance(M, N, K, frac, P, mode, orientation):
     plan = cb.Plan(M, N, K, tags, num_sms=P, split_mode=mode, cost_int8=c8, device_plan=False,
                    orientation=orientation)
     info = plan.info()
+    P = info["num_ctas"]          # scheduling units: CTAs, or CTA pairs (orientation 3)
     segs = _segments(plan, P)
     oplan.check_cover(segs, info["n_tiles"], K // 128)
     ms = oplan.makespan(segs, tags, 1, Fraction(c8).limit_denominator())
