@@ -212,7 +212,8 @@ def run_comet(args, rank, world, local_rank):
         x_d = torch.from_numpy(x_l).to(dev)
         wp = cb.pack_weight(torch.from_numpy(w_l).to(dev))
         swd = torch.from_numpy(sw_l).to(dev)
-        plan = cb.Plan(M_TOKENS, Nl, Kl, t_l, tile_n=args.tile_n, split_mode=args.split_mode)
+        plan = cb.Plan(M_TOKENS, Nl, Kl, t_l, tile_n=args.tile_n, split_mode=args.split_mode,
+                       orientation=args.orientation)
         act, sc = cb.quantize_act(x_d, t_l)
         ydt = torch.float32 if (kind == "row" and world > 1) else torch.float16
         y = torch.empty((M_TOKENS, Nl), dtype=ydt, device=dev)
@@ -388,6 +389,7 @@ def main():
     ap.add_argument("--cpu-budget", type=float, default=15.0)
     ap.add_argument("--tile-n", type=int, default=0, help="0 = planner default")
     ap.add_argument("--split-mode", type=int, default=-1)
+    ap.add_argument("--orientation", type=int, default=0, help="0 = planner default")
     args = ap.parse_args()
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", str(args.gpus if args.gpus == 1 else 1)))

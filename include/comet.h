@@ -149,9 +149,9 @@ typedef struct {
   int orientation;     /* 0 = auto (3 when M >= 256, 2 when M >= 128, else 1);
                           1 = weights on the MMA M side: tile = 128 weights x tile_n tokens
                               (decode-sized M; weights widened into TMEM);
-                          2 = tokens on the MMA M side: tile = 128 tokens x 256 weights
+                          2 = tokens on the MMA M side: tile = 128 tokens x 192 weights
                               (prefill; weights widened into shared memory), tile_n ignored;
-                          3 = as 2 on a tcgen05 CTA pair: tile = 256 tokens x 256 weights,
+                          3 = as 2 on a tcgen05 CTA pair: tile = 256 tokens x 192 weights,
                               each SM widens half the weights; num_ctas counts pairs */
   int reserved[5];
 } comet_sched_config;

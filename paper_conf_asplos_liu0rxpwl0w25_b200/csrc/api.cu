@@ -4,6 +4,7 @@
 #include <mutex>
 #include <new>
 #include "internal.h"
+#include "gemm_common.cuh"
 
 struct comet_plan_s {
   comet::Plan p;
@@ -84,6 +85,10 @@ const char* comet_status_string(comet_status_t s) {
 const char* comet_last_error(void) { return g_err.c_str(); }
 const char* comet_version(void) { return "comet-b200 0.1 (sm_100a; W4Ax = FP8-exact INT4 blocks + INT8 blocks)"; }
 int comet_last_launch_count(void) { return g_launches; }
+
+/* Diagnostic (not part of comet.h): subsequent GEMM launches record a clock64 timeline of the
+ * first two CTAs into buf ([2][8][1024] uint64, device memory); NULL disables. */
+void comet_debug_set_trace(void* buf) { comet::gemm::g_trace = static_cast<unsigned long long*>(buf); }
 
 comet_status_t comet_act_layout(int64_t M, int64_t K, comet_act_layout_t* out) {
   if (!out) return fail(COMET_ERR_INVALID_ARG, "out is NULL");

@@ -29,6 +29,7 @@
 // debug accumulators); the +8 offset is removed with corr[m] = 8 sum_b s_a qsum (kernel 1).
 // INT8 block: acc = 16 * sum_k x_k w_k exactly in INT32.
 #include <algorithm>
+#include <cstdlib>
 #include "gemm_common.cuh"
 
 namespace comet {
@@ -477,6 +478,8 @@ bool make_map_2d(CUtensorMap* map, const void* base, uint64_t inner, uint64_t ou
   return r == CUDA_SUCCESS;
 }
 
+unsigned long long* g_trace = nullptr;
+
 }  // namespace gemm
 
 comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_scales,
@@ -492,7 +495,7 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
   const int cg = p.orientation == 3 ? 2 : 1;
   // token-tile and weight-tile of one CTA (= box rows of the two TMA maps) and of the tile
   int tile_m, tile_w, cta_rows_w;
-  if (normal) { tile_m = 128 * cg; tile_w = dbg ? 128 : 256; cta_rows_w = tile_w / cg; }
+  if (normal) { tile_m = 128 * cg; tile_w = dbg ? 96 : 192; cta_rows_w = tile_w / cg; }
   else { tile_m = dbg ? 64 : p.tile_n; tile_w = kTileW; cta_rows_w = kTileW; }
   const int box_m = normal ? 128 : tile_m;
   comet_act_layout_t L;
@@ -520,6 +523,11 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
   prm.nb = (int)p.nb;
   prm.ydt = (int)ydt;
   prm.tags = p.mask;
+  {
+    const char* ab = getenv("COMET_ABLATE");
+    prm.ablate = ab ? atoi(ab) : 0;
+    prm.trace = g_trace;
+  }
   cudaError_t e;
   int grid;
   if (dbg) {

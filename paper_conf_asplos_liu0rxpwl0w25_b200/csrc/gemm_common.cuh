@@ -33,6 +33,9 @@ struct __align__(64) GemmParams {
   int64_t M, N, Mp;
   int nb, n_m_tiles, max_seg, ydt;
   uint32_t epoch;
+  unsigned long long* trace;  // diagnostic only (comet_debug_set_trace): [cta<2][event<8][kb<1024] clock64
+  int ablate;                // diagnostic only (env COMET_ABLATE): 4 skip widening, 8 skip MMAs
+                             // (prefill kernel); the output is invalid under it
   TagMask tags;
 };
 
@@ -71,9 +74,26 @@ __device__ __forceinline__ WorkItem load_item(const GemmParams& P, int idx, bool
   return w;
 }
 
+// Diagnostic hooks (timeline trace, stage ablation) exist only in a COMET_DIAG=1 build.
+#ifndef COMET_DIAG
+#define COMET_DIAG 0
+#endif
+__device__ __forceinline__ int diag_ablate(const GemmParams& P) { return COMET_DIAG ? P.ablate : 0; }
+
+// Diagnostic timeline: CTA c < 2, event e < 8, K-block index i < 1024 (per-CTA running count).
+__device__ __forceinline__ void trace_ev(const GemmParams& P, int e, int i) {
+  if (COMET_DIAG && P.trace != nullptr && blockIdx.x < 2 && i < 1024) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%clock64;" : "=l"(t));
+    P.trace[((int)blockIdx.x * 8 + e) * 1024 + i] = t;
+  }
+}
+
 // Host: TMA descriptor helper (gemm.cu).
 bool make_map_2d(CUtensorMap* map, const void* base, uint64_t inner, uint64_t outer,
                  uint64_t row_bytes, uint32_t box_inner, uint32_t box_outer, CUtensorMapSwizzle swz);
+
+extern unsigned long long* g_trace;   // diagnostic timeline buffer (comet_debug_set_trace)
 
 // Normal-orientation launcher (gemm_n.cu).  BN = weights per tile (256, or 128 for debug);
 // cg = CTAs per tile (1, or 2 for the tcgen05 CTA pair; grid must then be even).

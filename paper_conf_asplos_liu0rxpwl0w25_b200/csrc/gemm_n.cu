@@ -2,7 +2,7 @@
 //
 //   Y[m, n] = s_w[n] * sum_b s_a[m,b] * acc_b[m,n]
 //
-// Output tile: 128 tokens (MMA M = TMEM lanes) x BN weights (MMA N = TMEM columns, BN = 256).
+// Output tile: 128 tokens (MMA M = TMEM lanes) x BN weights (MMA N = TMEM columns, BN = 192).
 // A operand = the activation tile, TMA-staged straight from the mixed-precision code plane
 // (E4M3 bytes for INT4 blocks, s8 for INT8 blocks; 128-byte swizzle, no conversion).
 // B operand = the weight tile, widened from packed INT4 by CUDA cores into a 128-byte-swizzled
@@ -33,43 +33,63 @@ struct CfgN {
   static constexpr int WROWS = BN / CG;                   // weight rows widened by this CTA
   static constexpr int X_BYTES = BM * 128;                // activation tile (one K-block)
   static constexpr int WP_BYTES = WROWS * 64;             // packed weight rows
-  static constexpr int STAGE_BYTES = X_BYTES + WP_BYTES;
   static constexpr int B_BYTES = WROWS * 128;             // widened weight rows (MMA B half)
-  static constexpr int NBUF = 2;                          // widened-weight ring
-  static constexpr int COLS = BN / 2;                     // accumulator columns per promotion WG
+  static constexpr int SLOT_BYTES = X_BYTES + WP_BYTES + B_BYTES;
+  static constexpr int NPW = 3;                           // promotion warpgroups
+  static constexpr int COLS = BN / NPW;                   // accumulator columns per promotion WG
   static constexpr int NACC = (3 * BN <= 512) ? 3 : 2;    // accumulators in TMEM
-  static constexpr int ROWS_PER_THREAD = (WROWS + 127) / 128;   // widen rows per thread
-  static constexpr int STAGES_RAW = (200 * 1024 - NBUF * B_BYTES - kSRing * BM * 4) / STAGE_BYTES;
-  static constexpr int STAGES = STAGES_RAW > 8 ? 8 : STAGES_RAW;
-  static constexpr int SMEM_DATA = STAGES * STAGE_BYTES + NBUF * B_BYTES + kSRing * BM * 4;
-  static constexpr int N_BARS = 2 * STAGES + 2 * NBUF + 2 * NACC + 2 * kSRing;
+  // S pipeline slots, each holding one K-block's activation tile, packed and widened weights;
+  // the scale ring has S + NACC slots (reuse is implied by the slot-free barrier, see below).
+  static constexpr int S_RAW = (200 * 1024) / (SLOT_BYTES + BM * 4);
+  static constexpr int S = S_RAW > 8 ? 8 : S_RAW;
+  static constexpr int SS = S + NACC;
+  static constexpr int SMEM_DATA = S * SLOT_BYTES + SS * BM * 4;
+  static constexpr int N_BARS = 3 * S + NACC;
   static constexpr int SMEM_BYTES = 1024 + SMEM_DATA + N_BARS * 8 + 16 + kMaxBlocks;
-  static_assert(STAGES >= 2, "pipeline depth");
+  static_assert(S >= 3, "pipeline depth");
+  static_assert(S >= NACC + 1, "mma_ready ring must outlast the accumulator ring");
+  static_assert(NACC % 2 == 0 || true, "");
   static_assert(NACC * BN <= 512, "TMEM budget");
-  static_assert(COLS % 32 == 0, "promotion batches");
+  static_assert(COLS % 16 == 0, "promotion batches");
 };
 
+// Synchronisation (every role waits on exactly ONE mbarrier per K-block; a satisfied
+// try_wait still costs ~180 clk on B200, see profiles/r01/probe_sync.json):
+//   full[s]       TMA (activations, packed weights, scales) -> widen          [local]
+//   slot_free[s]  MMA completion (multicast) + 4 local widen warps (packed W read) -> producer
+//   mma_ready[s]  widen done for K-block kb (4 warps per CTA) + promotion done for K-block
+//                 kb - NACC (8 warps per CTA, frees the accumulator kb reuses) -> MMA [even CTA]
+//   acc_full[a]   MMA completion (multicast) -> promotion
+// Implied orders: widen(kb) may overwrite widened slot s because the producer issued full[s] for
+// kb only after slot_free[s] for kb - S; the scales of kb have landed when acc_full(kb) fires
+// (MMA(kb) waited mma_ready(kb) which waited widen(kb) which waited full[s]); the producer may
+// reuse scale slot kb % (S+NACC) because slot_free(kb-S) => MMA(kb-S) => promotion(kb-S-NACC).
+// WG0 producer/MMA, WG1-2 widen (alternate K-blocks), WG3-5 promotion.  768
+// threads launch with 80 registers each; setmaxnreg redistributes that pool
+// (40 + 2 x 40 + 3 x 120 = 480 = 6 x 80).
+constexpr int kWidenWarps = 8;
+constexpr int kPromoWarp0 = 4 + kWidenWarps;          // first promotion warp
+constexpr int kThreadsN = 128 * (1 + kWidenWarps / 4 + 3);
+
 template <int BN, int CG, int DEBUG>
-__global__ void __launch_bounds__(kThreads, 1) k_w4ax_n(const __grid_constant__ GemmParams P) {
+__global__ void __launch_bounds__(kThreadsN, 1) k_w4ax_n(const __grid_constant__ GemmParams P) {
   using C = CfgN<BN, CG>;
-  constexpr int S = C::STAGES;
+  constexpr int S = C::S;
+  constexpr int SS = C::SS;
   constexpr int NACC = C::NACC;
   constexpr int BM = C::BM;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
-  uint8_t* sX = smem;                                     // [S][BM x 128 B]   (A)
-  uint8_t* sWp = sX + S * C::X_BYTES;                     // [S][BN x 64 B]    packed W
-  uint8_t* sB = sWp + S * C::WP_BYTES;                    // [NBUF][BN x 128 B] widened W (B)
-  float* sS = reinterpret_cast<float*>(sB + C::NBUF * C::B_BYTES);   // [kSRing][BM]
+  // slot s: [X: BM x 128 B][B: WROWS x 128 B][Wp: WROWS x 64 B]  (X and B 1024-aligned)
+  auto sX = [&](int s) { return smem + s * C::SLOT_BYTES; };
+  auto sB = [&](int s) { return smem + s * C::SLOT_BYTES + C::X_BYTES; };
+  auto sWp = [&](int s) { return smem + s * C::SLOT_BYTES + C::X_BYTES + C::B_BYTES; };
+  float* sS = reinterpret_cast<float*>(smem + S * C::SLOT_BYTES);   // [SS][BM]
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + C::SMEM_DATA);
-  uint64_t* full = bars;                     // [S]     TMA -> MMA, widen
-  uint64_t* empty = full + S;                // [S]     MMA commit + 4 widen warps -> TMA
-  uint64_t* b_full = empty + S;              // [NBUF]  widen -> MMA
-  uint64_t* b_empty = b_full + C::NBUF;      // [NBUF]  MMA commit -> widen
-  uint64_t* acc_full = b_empty + C::NBUF;    // [NACC]  MMA commit -> promotion
-  uint64_t* acc_empty = acc_full + NACC;     // [NACC]  promotion -> MMA
-  uint64_t* s_full = acc_empty + NACC;       // [kSRing]
-  uint64_t* s_empty = s_full + kSRing;       // [kSRing]
+  uint64_t* full = bars;                     // [S]
+  uint64_t* slot_free = full + S;            // [S]
+  uint64_t* mma_ready = slot_free + S;       // [S]   (used in the even CTA)
+  uint64_t* acc_full = mma_ready + S;        // [NACC]
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bars + C::N_BARS);
   uint8_t* s_tags = reinterpret_cast<uint8_t*>(tmem_holder + 4);
   const uint32_t s_tags_a = smem_u32(s_tags);
@@ -82,87 +102,83 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax_n(const __grid_constant__ 
   const int it_begin = debug ? unit : P.cta_begin[unit];
   const int it_end = debug ? unit + 1 : P.cta_begin[unit + 1];
   const int nb = P.nb;
+  constexpr int NPROMO_WARPS = 4 * C::NPW;
+  constexpr uint32_t kReadyCount = (kWidenWarps / 2) * CG + NPROMO_WARPS * CG;   // one widen group
 
   if (warp == 0 && lane == 0) {
     tma_prefetch(&P.map_x);
     tma_prefetch(&P.map_w);
     for (int i = 0; i < S; ++i) {
       mbar_init(&full[i], 1);
-      mbar_init(&empty[i], 1 + 4);
+      mbar_init(&slot_free[i], 1 + kWidenWarps / 2);
+      mbar_init(&mma_ready[i], kReadyCount);
     }
-    for (int i = 0; i < C::NBUF; ++i) {
-      mbar_init(&b_full[i], 4 * CG);
-      mbar_init(&b_empty[i], 1);
-    }
-    for (int i = 0; i < NACC; ++i) {
-      mbar_init(&acc_full[i], 1);
-      mbar_init(&acc_empty[i], 8 * CG);
-    }
-    for (int i = 0; i < kSRing; ++i) {
-      mbar_init(&s_full[i], 1);
-      mbar_init(&s_empty[i], 8);
-    }
+    for (int i = 0; i < NACC; ++i) mbar_init(&acc_full[i], 1);
+    // the first NACC K-blocks have no promotion predecessor
+    for (int i = 0; i < NACC; ++i) mbar_arrive_count(&mma_ready[i], NPROMO_WARPS * CG);
     fence_mbar_init();
   }
   if (warp == 2) {
     if (CG == 2) { tmem_alloc_cg2<512>(tmem_holder); tmem_relinquish_cg2(); }
     else { tmem_alloc<512>(tmem_holder); tmem_relinquish(); }
   }
-  for (int i = threadIdx.x; i < nb; i += kThreads) s_tags[i] = P.tags.get(i) ? 1 : 0;
+  for (int i = threadIdx.x; i < nb; i += kThreadsN) s_tags[i] = P.tags.get(i) ? 1 : 0;
   tc_fence_before();
   __syncthreads();
   if (CG == 2) cluster_sync();                 // peer barriers initialised before remote arrives
   tc_fence_after();
   const uint32_t tbase = *tmem_holder;
-  // the even CTA's barriers that both CTAs arrive on (shared::cluster addresses)
-  const uint32_t b_full_lead = CG == 2 ? mapa_shared(smem_u32(b_full), 0) : smem_u32(b_full);
-  const uint32_t acc_empty_lead = CG == 2 ? mapa_shared(smem_u32(acc_empty), 0) : smem_u32(acc_empty);
-  auto wait_x = [&](uint64_t* bar, uint32_t par) { mbar_wait(bar, par); };
+  // the even CTA's mma_ready barriers (shared::cluster addresses), arrived on by both CTAs
+  const uint32_t ready_lead = CG == 2 ? mapa_shared(smem_u32(mma_ready), 0) : smem_u32(mma_ready);
 
   if (warp < 4) {
-    setmaxnreg_dec<32>();
+    setmaxnreg_dec<40>();
     if (warp == 0 && lane == 0) {
       // ------------------------------------------------------------------ TMA producer
-      int stage = 0, ss = 0;
-      uint32_t ph = 0, sph = 0;
+      int s = 0, sc = 0, tr = 0;
+      uint32_t ph = 0;
       for (int it = it_begin; it < it_end; ++it) {
         const WorkItem w = load_item(P, it, debug);
         const int n_tile = w.tile / P.n_m_tiles, m_tile = w.tile % P.n_m_tiles;
         const int m0 = m_tile * (BM * CG) + BM * rank, n0 = n_tile * BN + C::WROWS * rank;
         const uint32_t sbytes = m0 < P.Mp ? (uint32_t)(min((int64_t)BM, P.Mp - m0) * 4) : 0u;
         for (int kb = w.kb_begin; kb < w.kb_end; ++kb) {
-          wait_x(&empty[stage], ph ^ 1);
-          mbar_arrive_expect_tx(&full[stage], C::STAGE_BYTES);
-          tma_load_2d(sX + stage * C::X_BYTES, &P.map_x, &full[stage], kb * 128, m0);
-          tma_load_2d(sWp + stage * C::WP_BYTES, &P.map_w, &full[stage], kb * 64, n0);
-          mbar_wait(&s_empty[ss], sph ^ 1);
-          if (sbytes) {
-            mbar_arrive_expect_tx(&s_full[ss], sbytes);
-            bulk_load(sS + ss * BM, P.scales + (int64_t)kb * P.Mp + m0, sbytes, &s_full[ss]);
-          } else {
-            mbar_arrive(&s_full[ss]);        // this CTA's tokens are all padding
-          }
-          if (++stage == S) { stage = 0; ph ^= 1; }
-          if (++ss == kSRing) { ss = 0; sph ^= 1; }
+          mbar_wait(&slot_free[s], ph ^ 1);
+          mbar_arrive_expect_tx(&full[s], C::X_BYTES + C::WP_BYTES + sbytes);
+          tma_load_2d(sX(s), &P.map_x, &full[s], kb * 128, m0);
+          tma_load_2d(sWp(s), &P.map_w, &full[s], kb * 64, n0);
+          if (sbytes) bulk_load(sS + sc * BM, P.scales + (int64_t)kb * P.Mp + m0, sbytes, &full[s]);
+          trace_ev(P, 0, tr++);
+          if (++s == S) { s = 0; ph ^= 1; }
+          if (++sc == SS) sc = 0;
         }
       }
-    } else if (warp == 1 && lane == 0 && rank == 0) {
-      // ------------------------------------------------------------------ MMA issuer
+    } else if ((warp == 1 || warp == 3) && lane == 0 && rank == 0) {
+      // ------------------------------------------------------------------ MMA issuers
+      // Two issuing threads: warp 1 takes the even K-blocks of the CTA's sequence, warp 3 the
+      // odd ones (different accumulators and slots), so one thread's barrier wait and commits
+      // overlap the MMAs the other has queued.  tcgen05.commit tracks the issuing thread's own
+      // MMAs, so each thread commits exactly the K-blocks it issued.
+      const int parity = warp == 1 ? 0 : 1;
       const uint32_t id_f8 = idesc_f8f6f4_e4m3(BM * CG, BN);
       const uint32_t id_i8 = idesc_i8(BM * CG, BN);
-      int stage = 0, bb = 0, accb = 0;
-      uint32_t ph = 0, bph = 0, accph = 0;
+      int j = 0, tr = 0;
       for (int it = it_begin; it < it_end; ++it) {
         const WorkItem w = load_item(P, it, debug);
-        for (int kb = w.kb_begin; kb < w.kb_end; ++kb) {
-          wait_x(&acc_empty[accb], accph ^ 1);
-          // b_full covers the stage too: every widen warp waited on its CTA's full[stage]
-          wait_x(&b_full[bb], bph);
+        for (int kb = w.kb_begin; kb < w.kb_end; ++kb, ++j) {
+          if ((j & 1) != parity) continue;
+          const int s = j % S, accb = j % NACC;
+          const uint32_t ph = (uint32_t)(j / S) & 1u;
+          if (parity == 0) trace_ev(P, 1, tr);
+          mbar_wait(&mma_ready[s], ph);
+          if (parity == 0) trace_ev(P, 3, tr++);
           tc_fence_after();
           const uint32_t d = tbase + accb * BN;
-          const uint32_t sa = smem_u32(sX + stage * C::X_BYTES);
-          const uint32_t sbv = smem_u32(sB + bb * C::B_BYTES);
-          if (lds_u8(s_tags_a + kb)) {
+          const uint32_t sa = smem_u32(sX(s));
+          const uint32_t sbv = smem_u32(sB(s));
+          if (diag_ablate(P) & 8) {
+            // diagnostic: no MMA
+          } else if (lds_u8(s_tags_a + kb)) {
 #pragma unroll
             for (int k = 0; k < 4; ++k) {
               const uint64_t ad = sdesc_kmajor_sw128(sa + 32 * k), bd = sdesc_kmajor_sw128(sbv + 32 * k);
@@ -176,95 +192,94 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax_n(const __grid_constant__ 
             }
           }
           if (CG == 2) {
-            tc_commit_mc(&empty[stage], 3);
-            tc_commit_mc(&b_empty[bb], 3);
             tc_commit_mc(&acc_full[accb], 3);
+            tc_commit_mc(&slot_free[s], 3);
           } else {
-            tc_commit(&empty[stage]);
-            tc_commit(&b_empty[bb]);
             tc_commit(&acc_full[accb]);
+            tc_commit(&slot_free[s]);
           }
-          if (++stage == S) { stage = 0; ph ^= 1; }
-          if (++bb == C::NBUF) { bb = 0; bph ^= 1; }
-          if (++accb == NACC) { accb = 0; accph ^= 1; }
         }
       }
     }
-  } else if (warp < 8) {
-    setmaxnreg_dec<64>();
+  } else if (warp < kPromoWarp0) {
+    setmaxnreg_dec<40>();
     // -------------------------------------------------------------------- widen (W -> smem B)
-    const int t = threadIdx.x - 128;                      // weight row t (and t + 128)
-    const bool has_row = t < C::WROWS;
-    const uint32_t sWp_a = smem_u32(sWp), sB_a = smem_u32(sB);
-    int stage = 0, bb = 0;
-    uint32_t ph = 0, bph = 0;
+    // Two widen warpgroups take alternate K-blocks; thread t of a group converts weight rows
+    // t, t + 128, ... of its K-blocks.  INT4 block: byte = u (E4M3 u * 2^-9); INT8 block:
+    // byte = 16 u - 128 = 16 w (s8), derived from the INT4-block form with one shift + xor.
+    constexpr int RPT = (C::WROWS + 127) / 128;           // rows per thread
+    const int grp = (warp - 4) >> 2;                      // 0: even K-blocks, 1: odd
+    const int t = threadIdx.x - 128 - 128 * grp;
+    int s = 0, tr = 0, j = 0;
+    uint32_t ph = 0;
     for (int it = it_begin; it < it_end; ++it) {
       const WorkItem w = load_item(P, it, debug);
-      for (int kb = w.kb_begin; kb < w.kb_end; ++kb) {
-        const bool is8 = lds_u8(s_tags_a + kb) != 0;
-        wait_x(&full[stage], ph);
-        uint4 c[C::ROWS_PER_THREAD][4];
+      for (int kb = w.kb_begin; kb < w.kb_end; ++kb, ++j) {
+        if ((j & 1) == grp) {
+          const bool is8 = lds_u8(s_tags_a + kb) != 0;
+          mbar_wait(&full[s], ph);
+          if (warp == 4 && lane == 0) trace_ev(P, 5, tr);
+          uint4 c[RPT][4];
 #pragma unroll
-        for (int rr = 0; rr < C::ROWS_PER_THREAD; ++rr) {
-          const int row = t + 128 * rr;
-          const uint32_t src = sWp_a + stage * C::WP_BYTES + row * 64;
-          const int sw = (row >> 1) & 3;                  // TMA 64-byte swizzle
+          for (int i = 0; i < RPT; ++i) {
+            const int row = t + 128 * i;
+            if (row < C::WROWS) {
+              const uint32_t src = smem_u32(sWp(s)) + row * 64;
+              const int sw64 = (row >> 1) & 3;            // TMA 64-byte swizzle of the packed row
 #pragma unroll
-          for (int j = 0; j < 4; ++j) c[rr][j] = has_row ? lds128(src + ((j ^ sw) << 4)) : make_uint4(0, 0, 0, 0);
-        }
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&empty[stage]);
-        wait_x(&b_empty[bb], bph ^ 1);
-#pragma unroll
-        for (int rr = 0; rr < C::ROWS_PER_THREAD; ++rr) {
-          if (!has_row) break;
-          const int row = t + 128 * rr;
-          const uint32_t dst = sB_a + bb * C::B_BYTES + row * 128;
-          const int sw = row & 7;                         // UMMA/TMA 128-byte swizzle
-#pragma unroll
-          for (int j = 0; j < 4; ++j) {
-            const uint32_t pw[4] = {c[rr][j].x, c[rr][j].y, c[rr][j].z, c[rr][j].w};
-            uint32_t o[8];
-#pragma unroll
-            for (int i = 0; i < 4; ++i) {
-              const uint32_t p = pw[i];
-              if (is8) {
-                o[2 * i] = ((p << 4) & 0xF0F0F0F0u) ^ 0x80808080u;
-                o[2 * i + 1] = (p & 0xF0F0F0F0u) ^ 0x80808080u;
-              } else {
-                o[2 * i] = p & 0x0F0F0F0Fu;
-                o[2 * i + 1] = (p >> 4) & 0x0F0F0F0Fu;
-              }
+              for (int q4 = 0; q4 < 4; ++q4) c[i][q4] = lds128(src + ((q4 ^ sw64) << 4));
             }
-            // logical 16-byte chunks 2j and 2j+1 (channels 32j .. 32j+31)
-            asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(dst + (((2 * j) ^ sw) << 4)),
-                         "r"(o[0]), "r"(o[1]), "r"(o[2]), "r"(o[3]) : "memory");
-            asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(dst + (((2 * j + 1) ^ sw) << 4)),
-                         "r"(o[4]), "r"(o[5]), "r"(o[6]), "r"(o[7]) : "memory");
           }
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&slot_free[s]);     // packed weights of slot s consumed
+#pragma unroll
+          for (int i = 0; i < RPT; ++i) {
+            const int row = t + 128 * i;
+            if (row >= C::WROWS || (diag_ablate(P) & 4)) break;
+            const uint32_t dst = smem_u32(sB(s)) + row * 128;
+            const int sw128 = row & 7;                    // UMMA 128-byte swizzle of the widened row
+#pragma unroll
+            for (int q4 = 0; q4 < 4; ++q4) {
+              const uint32_t pw[4] = {c[i][q4].x, c[i][q4].y, c[i][q4].z, c[i][q4].w};
+              uint32_t o[8];
+#pragma unroll
+              for (int k = 0; k < 4; ++k) {
+                o[2 * k] = pw[k] & 0x0F0F0F0Fu;           // u[8g .. 8g+3]
+                o[2 * k + 1] = (pw[k] >> 4) & 0x0F0F0F0Fu; // u[8g+4 .. 8g+7]
+              }
+              if (is8) {                                  // warp-uniform: 5 % of blocks
+#pragma unroll
+                for (int k = 0; k < 8; ++k) o[k] = (o[k] << 4) ^ 0x80808080u;
+              }
+              const int oc = 2 * q4;                      // logical 16-byte output chunk
+              asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(dst + ((oc ^ sw128) << 4)),
+                           "r"(o[0]), "r"(o[1]), "r"(o[2]), "r"(o[3]) : "memory");
+              asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(dst + (((oc + 1) ^ sw128) << 4)),
+                           "r"(o[4]), "r"(o[5]), "r"(o[6]), "r"(o[7]) : "memory");
+            }
+          }
+          if (warp == 4 && lane == 0) trace_ev(P, 2, tr);
+          fence_proxy_async_smem();                       // generic-proxy stores -> tensor core
+          __syncwarp();
+          if (lane == 0) mbar_arrive_cluster(ready_lead + s * 8);
+          if (warp == 4 && lane == 0) trace_ev(P, 4, tr);
+          ++tr;
         }
-        fence_proxy_async_smem();                         // generic-proxy stores -> tensor core
-        __syncwarp();
-        if (lane == 0) mbar_arrive_cluster(b_full_lead + bb * 8);
-        if (++stage == S) { stage = 0; ph ^= 1; }
-        if (++bb == C::NBUF) { bb = 0; bph ^= 1; }
+        if (++s == S) { s = 0; ph ^= 1; }
       }
     }
   } else {
-    setmaxnreg_inc<208>();
+    setmaxnreg_inc<120>();
     // -------------------------------------------------------------------- promotion + epilogue
-    const int wg = (warp - 8) >> 2;
+    const int wg = (warp - kPromoWarp0) >> 2;
     const int q = warp & 3;
     const int r = q * 32 + lane;                          // TMEM lane = token row within the tile
     const uint32_t lane_addr = (uint32_t)(q * 32) << 16;
     constexpr int COLS = C::COLS;
-    constexpr int BC = COLS > 64 ? 64 : COLS;             // columns per TMEM load batch
-    constexpr int NBATCH = COLS / BC;
     const int col0 = wg * COLS;
-    const int ptid = threadIdx.x - 256;
-    const uint32_t sS_a = smem_u32(sS);
-    int ss = 0, accb = 0;
-    uint32_t sph = 0, accph = 0;
+    const int ptid = threadIdx.x - kPromoWarp0 * 32;
+    int accb = 0, sc = 0, rs = NACC % S, tr = 0;           // rs: mma_ready slot of kb + NACC
+    uint32_t accph = 0;
     for (int it = it_begin; it < it_end; ++it) {
       const WorkItem w = load_item(P, it, debug);
       const int n_tile = w.tile / P.n_m_tiles, m_tile = w.tile % P.n_m_tiles;
@@ -282,68 +297,95 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax_n(const __grid_constant__ 
       }
       for (int kb = w.kb_begin; kb < w.kb_end; ++kb) {
         const bool is8 = lds_u8(s_tags_a + kb) != 0;
-        mbar_wait(&s_full[ss], sph);
-        float s;
-        asm volatile("ld.shared.f32 %0, [%1];" : "=f"(s) : "r"(sS_a + (ss * BM + r) * 4));
-        if (is8) s *= 1.220703125e-04f;                   // 2^-13: INT8 block acc = 16 sum x w
-        const float2 s2 = make_float2(s, s);
         int qs = 0;
         if (DEBUG && !is8 && m < P.Mp) qs = P.qsum[(int64_t)kb * P.Mp + m];
-        wait_x(&acc_full[accb], accph);
+        mbar_wait(&acc_full[accb], accph);
+        if (threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 6, tr);
         tc_fence_after();
+        if (diag_ablate(P) & 16) {                              // diagnostic: no promotion work
+          tc_fence_before();
+          __syncwarp();
+          if (lane == 0) mbar_arrive_cluster(ready_lead + rs * 8);
+          ++tr;
+          if (++accb == NACC) { accb = 0; accph ^= 1; }
+          if (++sc == SS) sc = 0;
+          if (++rs == S) rs = 0;
+          continue;
+        }
+        float s;
+        asm volatile("ld.shared.f32 %0, [%1];" : "=f"(s) : "r"(smem_u32(sS + sc * BM + r)));
+        if (is8) s *= 1.220703125e-04f;                   // 2^-13: INT8 block acc = 16 sum x w
+        const float2 s2 = make_float2(s, s);
         const uint32_t taddr = tbase + accb * BN + col0 + lane_addr;
+        // software-pipelined over 32-column batches: the load of batch b+1 is in flight while
+        // batch b is folded in; the accumulator is released once the last load has landed.
+        constexpr int PB = 16;                            // columns per TMEM load batch
+        constexpr int NB_ = COLS / PB;
+        uint32_t vb[2][PB];
+        tmem_ld_32x32b_x16(taddr, vb[0]);
+        tmem_wait_ld();
 #pragma unroll
-        for (int b = 0; b < NBATCH; ++b) {
-          uint32_t v[BC];
-          tmem_ld_32x32b<BC>(taddr + b * BC, v);
-          tmem_wait_ld();
+        for (int b = 0; b < NB_; ++b) {
+          uint32_t* v = vb[b & 1];
+          if (b + 1 < NB_) tmem_ld_32x32b_x16(taddr + (b + 1) * PB, vb[(b + 1) & 1]);
           if (DEBUG) {
 #pragma unroll
-            for (int c = 0; c < BC; ++c) {
+            for (int c = 0; c < PB; ++c) {
               const int32_t ab = is8 ? (((int32_t)v[c]) >> 4) : ((int32_t)(__uint_as_float(v[c]) * 512.f) - 8 * qs);
-              dacc[b * BC + c] += ab;
-              if (DEBUG == 2 && m < P.M && n0 + col0 + b * BC + c < P.N)
-                P.dbg_blocks[((int64_t)kb * P.M + m) * P.N + n0 + col0 + b * BC + c] = ab;
+              dacc[b * PB + c] += ab;
+              if (DEBUG == 2 && m < P.M && n0 + col0 + b * PB + c < P.N)
+                P.dbg_blocks[((int64_t)kb * P.M + m) * P.N + n0 + col0 + b * PB + c] = ab;
             }
           }
           if (is8) {
 #pragma unroll
-            for (int c = 0; c < BC; ++c) v[c] = __float_as_uint(__int2float_rn((int)v[c]));
+            for (int c = 0; c < PB; ++c) v[c] = __float_as_uint(__int2float_rn((int)v[c]));
           }
 #pragma unroll
-          for (int c = 0; c < BC; c += 2) {
-            const int a = b * BC + c;
+          for (int c = 0; c < PB; c += 2) {
+            const int a = b * PB + c;
             float2 y = ffma2(make_float2(__uint_as_float(v[c]), __uint_as_float(v[c + 1])), s2,
                              make_float2(acc[a], acc[a + 1]));
             acc[a] = y.x;
             acc[a + 1] = y.y;
           }
+          if (b + 1 < NB_) {
+            tmem_wait_ld();
+            if (b + 2 == NB_) {
+              // every accumulator column of this thread is now in registers: release the TMEM
+              // buffer (the MMA for kb + NACC may start) before the last batch's math
+              tc_fence_before();
+              __syncwarp();
+              if (lane == 0) mbar_arrive_cluster(ready_lead + rs * 8);
+            }
+          } else if (NB_ == 1) {
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) mbar_arrive_cluster(ready_lead + rs * 8);
+          }
         }
-        tc_fence_before();
-        __syncwarp();
-        if (lane == 0) {
-          mbar_arrive_cluster(acc_empty_lead + accb * 8);
-          mbar_arrive(&s_empty[ss]);
-        }
-        if (++ss == kSRing) { ss = 0; sph ^= 1; }
+        if (threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 7, tr);
+        ++tr;
         if (++accb == NACC) { accb = 0; accph ^= 1; }
+        if (++sc == SS) sc = 0;
+        if (++rs == S) rs = 0;
       }
       // ---------------------------------------------------------------- epilogue
       if (split) {
         const int seg = (w.flags >> 8) & 0xFF;
         const int nseg = (w.flags >> 16) & 0xFF;
-        const int64_t part_tile = (int64_t)BM * BN;        // = 256 threads * COLS floats
+        const int64_t part_tile = (int64_t)BM * BN;        // = 512 promotion threads * COLS floats
         if (!owner) {
           float4* dst = reinterpret_cast<float4*>(
               P.ws_part + (((int64_t)w.fix * (P.max_seg - 1) + (seg - 1)) * CG + rank) * part_tile + (int64_t)ptid * COLS);
 #pragma unroll
           for (int a = 0; a < COLS; a += 4) dst[a / 4] = make_float4(acc[a], acc[a + 1], acc[a + 2], acc[a + 3]);
           __threadfence();
-          named_bar_sync(1, 256);
-          if (threadIdx.x == 256) st_release_gpu(P.ws_flags + ((int64_t)w.fix * P.max_seg + seg) * CG + rank, P.epoch);
+          named_bar_sync(1, 128 * C::NPW);
+          if (threadIdx.x == kPromoWarp0 * 32) st_release_gpu(P.ws_flags + ((int64_t)w.fix * P.max_seg + seg) * CG + rank, P.epoch);
           continue;
         }
-        if (threadIdx.x == 256) {
+        if (threadIdx.x == kPromoWarp0 * 32) {
           for (int sgi = 1; sgi < nseg; ++sgi) {
             const uint32_t* f = P.ws_flags + ((int64_t)w.fix * P.max_seg + sgi) * CG + rank;
             uint64_t t0g = globaltimer_ns();
@@ -355,7 +397,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax_n(const __grid_constant__ 
             }
           }
         }
-        named_bar_sync(1, 256);
+        named_bar_sync(1, 128 * C::NPW);
         for (int sgi = 1; sgi < nseg; ++sgi) {
           const float4* src = reinterpret_cast<const float4*>(
               P.ws_part + (((int64_t)w.fix * (P.max_seg - 1) + (sgi - 1)) * CG + rank) * part_tile + (int64_t)ptid * COLS);
@@ -430,7 +472,7 @@ cudaError_t launch_bn(const GemmParams& prm, int grid, cudaStream_t stream) {
   }
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)grid);
-  cfg.blockDim = dim3(kThreads);
+  cfg.blockDim = dim3(kThreadsN);
   cfg.dynamicSmemBytes = C::SMEM_BYTES;
   cfg.stream = stream;
   cudaLaunchAttribute attr[1];
@@ -446,15 +488,15 @@ cudaError_t launch_bn(const GemmParams& prm, int grid, cudaStream_t stream) {
 }  // namespace
 
 cudaError_t launch_gemm_n(const GemmParams& prm, int grid, int bn, int cg, int debug, cudaStream_t stream) {
+  (void)bn;   // BN = 192 (normal) or 96 (debug accumulators)
   if (cg == 2) {
-    if (debug == 2) return launch_bn<128, 2, 2>(prm, grid, stream);
-    if (debug == 1) return launch_bn<128, 2, 1>(prm, grid, stream);
-    return launch_bn<256, 2, 0>(prm, grid, stream);
+    if (debug == 2) return launch_bn<96, 2, 2>(prm, grid, stream);
+    if (debug == 1) return launch_bn<96, 2, 1>(prm, grid, stream);
+    return launch_bn<192, 2, 0>(prm, grid, stream);
   }
-  if (debug == 2) return launch_bn<128, 1, 2>(prm, grid, stream);
-  if (debug == 1) return launch_bn<128, 1, 1>(prm, grid, stream);
-  if (bn == 128) return launch_bn<128, 1, 0>(prm, grid, stream);
-  return launch_bn<256, 1, 0>(prm, grid, stream);
+  if (debug == 2) return launch_bn<96, 1, 2>(prm, grid, stream);
+  if (debug == 1) return launch_bn<96, 1, 1>(prm, grid, stream);
+  return launch_bn<192, 1, 0>(prm, grid, stream);
 }
 
 }  // namespace gemm

@@ -86,7 +86,7 @@ comet_status_t build_plan(Plan& p, const comet_sched_config& cfg) {
   p.orientation = cfg.orientation > 0 ? cfg.orientation : (p.M >= 256 ? 3 : (p.M >= 128 ? 2 : 1));
   if (p.orientation >= 2) {
     p.tile_n = p.orientation == 3 ? 256 : 128;   // tokens per tile = MMA M (CTA pair: 2 x 128)
-    p.tile_w = 256;                              // weights per tile = MMA N
+    p.tile_w = 192;                              // weights per tile = MMA N
   } else {
     p.tile_n = cfg.tile_n > 0 ? cfg.tile_n : auto_tile_n(p.M);
     p.tile_w = kTileW;
