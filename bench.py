@@ -213,7 +213,7 @@ def run_comet(args, rank, world, local_rank):
         wp = cb.pack_weight(torch.from_numpy(w_l).to(dev))
         swd = torch.from_numpy(sw_l).to(dev)
         plan = cb.Plan(M_TOKENS, Nl, Kl, t_l, tile_n=args.tile_n, split_mode=args.split_mode,
-                       orientation=args.orientation)
+                       orientation=args.orientation, tile_w=args.tile_w)
         act, sc = cb.quantize_act(x_d, t_l)
         ydt = torch.float32 if (kind == "row" and world > 1) else torch.float16
         y = torch.empty((M_TOKENS, Nl), dtype=ydt, device=dev)
@@ -363,7 +363,7 @@ def run_comet(args, rank, world, local_rank):
                        "layers": [[n, K, N] for n, K, N, _ in LAYERS],
                        "int8_block_fraction": FRAC,
                        "parallelism": "single GPU" if world == 1 else f"tp{world} (gate_up/qkv column, down row + NCCL all_reduce fp32)",
-                       "tile_n": layers[0]["plan"].info()["tile_n"],
+                       "tile": [layers[0]["plan"].info()["tile_n"], layers[0]["plan"].info()["tile_w"]],
                        "l2": "inputs larger than L2 (per step: 300 MB activations + 276 MB packed weights > 126 MB L2)"},
             "roofline": roofline,
             "cpu_baseline": cpu,
@@ -390,6 +390,7 @@ def main():
     ap.add_argument("--tile-n", type=int, default=0, help="0 = planner default")
     ap.add_argument("--split-mode", type=int, default=-1)
     ap.add_argument("--orientation", type=int, default=0, help="0 = planner default")
+    ap.add_argument("--tile-w", type=int, default=0, help="weights per tile (192/256); 0 = planner default")
     args = ap.parse_args()
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", str(args.gpus if args.gpus == 1 else 1)))

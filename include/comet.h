@@ -149,11 +149,15 @@ typedef struct {
   int orientation;     /* 0 = auto (3 when M >= 256, 2 when M >= 128, else 1);
                           1 = weights on the MMA M side: tile = 128 weights x tile_n tokens
                               (decode-sized M; weights widened into TMEM);
-                          2 = tokens on the MMA M side: tile = 128 tokens x 192 weights
+                          2 = tokens on the MMA M side: tile = 128 tokens x tile_w weights
                               (prefill; weights widened into shared memory), tile_n ignored;
-                          3 = as 2 on a tcgen05 CTA pair: tile = 256 tokens x 192 weights,
+                          3 = as 2 on a tcgen05 CTA pair: tile = 256 tokens x tile_w weights,
                               each SM widens half the weights; num_ctas counts pairs */
-  int reserved[5];
+  int tile_w;          /* orientations 2/3: weights per output tile (MMA N): 128, 160, 192, or
+                          256 (orientation 3 only);
+                          0 = auto (256 for orientation 3, 192 for 2).  Ignored for
+                          orientation 1 (always 128). */
+  int reserved[4];
 } comet_sched_config;
 
 /* Fill *cfg with the defaults (tile_n 0, num_sms 0, split_mode -1, costs 1/1, stages 0,

@@ -47,7 +47,8 @@ class SchedConfig(ctypes.Structure):
     _fields_ = [("tile_n", ctypes.c_int), ("num_sms", ctypes.c_int), ("split_mode", ctypes.c_int),
                 ("cost_int4", ctypes.c_float), ("cost_int8", ctypes.c_float),
                 ("stages", ctypes.c_int), ("device_plan", ctypes.c_int),
-                ("orientation", ctypes.c_int), ("reserved", ctypes.c_int * 5)]
+                ("orientation", ctypes.c_int), ("tile_w", ctypes.c_int),
+                ("reserved", ctypes.c_int * 4)]
 
 
 class PlanInfo(ctypes.Structure):
@@ -175,7 +176,7 @@ class Plan:
 
     def __init__(self, M: int, N: int, K: int, tags, *, tile_n: int = 0, num_sms: int = 0,
                  split_mode: int = -1, cost_int4: float = 1.0, cost_int8: float = 1.0,
-                 device_plan: bool = True, orientation: int = 0):
+                 device_plan: bool = True, orientation: int = 0, tile_w: int = 0):
         L = lib()
         cfg = SchedConfig()
         L.comet_sched_config_default(ctypes.byref(cfg))
@@ -183,6 +184,7 @@ class Plan:
         cfg.cost_int4, cfg.cost_int8 = cost_int4, cost_int8
         cfg.device_plan = 1 if device_plan else 0
         cfg.orientation = orientation
+        cfg.tile_w = tile_w
         self.tags = _tags_np(tags)
         h = ctypes.c_void_p()
         ws = ctypes.c_size_t()

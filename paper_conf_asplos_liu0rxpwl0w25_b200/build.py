@@ -36,7 +36,8 @@ def _run(cmd):
 def build(force: bool = False, verbose: bool = False) -> str:
     """COMET_DIAG=1 in the environment builds the diagnostic variant (timeline trace and
     stage-ablation hooks, tools/trace_gemm.py); normal builds compile them out.  Switching
-    between the two needs force=True."""
+    between the two needs force=True.  COMET_NVCC_DEFS="-DNAME=V ..." adds defines (kernel
+    variant experiments only)."""
     os.makedirs(BUILD, exist_ok=True)
     os.makedirs(os.path.dirname(LIB), exist_ok=True)
     hdrs = [os.path.join(CSRC, h) for h in HEADERS] + [os.path.join(ROOT, "include", "comet.h")]
@@ -48,6 +49,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
         if force or _newer([src] + hdrs, obj):
             jobs.append([NVCC, *ARCH, "-O3", "-std=c++17", "-lineinfo", "-Xptxas", "-v",
                          f"-DCOMET_DIAG={1 if os.environ.get('COMET_DIAG') == '1' else 0}",
+                         *os.environ.get("COMET_NVCC_DEFS", "").split(),
                          "-Xcompiler", "-fPIC", "-I", CSRC, "-I", os.path.join(ROOT, "include"),
                          "-c", src, "-o", obj])
     for s in CPP_SOURCES:

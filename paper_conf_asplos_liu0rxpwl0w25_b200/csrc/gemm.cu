@@ -385,7 +385,6 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
               uint64_t t0g = globaltimer_ns();
               while (ld_acquire_gpu(f) != P.epoch) {
                 if (globaltimer_ns() - t0g > COMET_MBAR_TIMEOUT_NS) {
-                  printf("comet: stream-K fix-up timeout (tile %d seg %d)\n", w.tile, sgi);
                   __trap();
                 }
               }
@@ -495,7 +494,7 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
   const int cg = p.orientation == 3 ? 2 : 1;
   // token-tile and weight-tile of one CTA (= box rows of the two TMA maps) and of the tile
   int tile_m, tile_w, cta_rows_w;
-  if (normal) { tile_m = 128 * cg; tile_w = dbg ? 96 : 192; cta_rows_w = tile_w / cg; }
+  if (normal) { tile_m = 128 * cg; tile_w = dbg ? 96 : p.tile_w; cta_rows_w = tile_w / cg; }
   else { tile_m = dbg ? 64 : p.tile_n; tile_w = kTileW; cta_rows_w = kTileW; }
   const int box_m = normal ? 128 : tile_m;
   comet_act_layout_t L;
@@ -509,6 +508,12 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
   if (!make_map_2d(&prm.map_w, w_packed, (uint64_t)(p.K / 2), (uint64_t)p.N, (uint64_t)(p.K / 2), 64,
                    (uint32_t)cta_rows_w, CU_TENSOR_MAP_SWIZZLE_64B))
     return fail(COMET_ERR_CUDA, "cuTensorMapEncodeTiled failed for the packed weights");
+  if (normal && !dbg) {
+    const int esz = ydt == COMET_F32 ? 4 : 2;
+    if (!make_map_2d(&prm.map_y, y, (uint64_t)p.N * esz, (uint64_t)p.M, (uint64_t)ldy * esz, 64, 128,
+                     CU_TENSOR_MAP_SWIZZLE_64B))
+      return fail(COMET_ERR_CUDA, "cuTensorMapEncodeTiled failed for the output");
+  }
   prm.scales = act_scales;
   prm.corr = reinterpret_cast<const float*>(base + L.corr_off);
   prm.qsum = reinterpret_cast<const int16_t*>(base + L.qsum_off);

@@ -18,6 +18,7 @@ constexpr int kSRing = 8;            // scale ring depth
 struct __align__(64) GemmParams {
   CUtensorMap map_x;
   CUtensorMap map_w;
+  CUtensorMap map_y;         // prefill kernel: Y as bytes [M][N*esz], box 64 B x 128 rows, 64B swizzle
   const float* scales;       // [nb][Mp]
   const float* corr;         // [Mp]
   const int16_t* qsum;       // [nb][Mp]
@@ -78,14 +79,22 @@ __device__ __forceinline__ WorkItem load_item(const GemmParams& P, int idx, bool
 #ifndef COMET_DIAG
 #define COMET_DIAG 0
 #endif
-__device__ __forceinline__ int diag_ablate(const GemmParams& P) { return COMET_DIAG ? P.ablate : 0; }
+#ifndef COMET_TRACE
+#define COMET_TRACE 0       // 1: timeline trace only (tools/trace_gemm.py), no ablation hooks
+#endif
+#ifndef COMET_ABLATE_CT
+#define COMET_ABLATE_CT 0   // compile-time ablation bits (timing experiments only; wrong results)
+#endif
+__device__ __forceinline__ int diag_ablate(const GemmParams& P) {
+  return (COMET_DIAG ? P.ablate : 0) | COMET_ABLATE_CT;
+}
 
 // Diagnostic timeline: CTA c < 2, event e < 8, K-block index i < 1024 (per-CTA running count).
 __device__ __forceinline__ void trace_ev(const GemmParams& P, int e, int i) {
-  if (COMET_DIAG && P.trace != nullptr && blockIdx.x < 2 && i < 1024) {
+  if ((COMET_DIAG || COMET_TRACE) && P.trace != nullptr && blockIdx.x < 2 && i < 1024) {
     unsigned long long t;
     asm volatile("mov.u64 %0, %%clock64;" : "=l"(t));
-    P.trace[((int)blockIdx.x * 8 + e) * 1024 + i] = t;
+    P.trace[((int)blockIdx.x * 16 + e) * 1024 + i] = t;
   }
 }
 

@@ -2,7 +2,8 @@
 //
 //   Y[m, n] = s_w[n] * sum_b s_a[m,b] * acc_b[m,n]
 //
-// Output tile: 128 tokens (MMA M = TMEM lanes) x BN weights (MMA N = TMEM columns, BN = 192).
+// Output tile: 128 tokens (MMA M = TMEM lanes) x BN weights (MMA N = TMEM columns, BN = 192
+// or 256).
 // A operand = the activation tile, TMA-staged straight from the mixed-precision code plane
 // (E4M3 bytes for INT4 blocks, s8 for INT8 blocks; 128-byte swizzle, no conversion).
 // B operand = the weight tile, widened from packed INT4 by CUDA cores into a 128-byte-swizzled
@@ -13,8 +14,9 @@
 // activation scale s_a[m,b] per K-block and folds the 32x32b-loaded FP32 accumulator row into
 // its registers with FFMA2 (two columns per instruction).
 //
-// Roles (512 threads): warp 0 TMA producer, warp 1 MMA issuer, warp 2 TMEM allocator,
-// warps 4-7 widen, warps 8-15 promotion + epilogue (two warpgroups, BN/2 columns each).
+// Roles: warpgroup 0 = TMA producer (warp 0), two MMA issuers (warps 1, 3), TMEM allocator
+// (warp 2); NWG widen warpgroups (taking K-blocks in turn); NPW promotion + epilogue
+// warpgroups (BN / NPW accumulator columns each).
 //
 // CG = 2 (CTA pair, tcgen05 cta_group::2): the tile is 256 tokens x BN weights; CTA r of the
 // pair holds tokens m0 + 128 r (its half of A, its TMEM lanes) and widens weights
@@ -23,11 +25,27 @@
 // CTA's b_full / acc_empty barriers, MMA completion is multicast to both CTAs.
 #include "gemm_common.cuh"
 
+#ifndef COMET_ISSUERS
+#define COMET_ISSUERS 2   // MMA issuing threads (K-blocks alternate between them)
+#endif
+#ifndef COMET_NSUB
+#define COMET_NSUB 1   // 2: split each K-block's MMA into two sub-MMAs (experimental, slower)
+#endif
+#ifndef COMET_SMEM_BUDGET_KB
+#define COMET_SMEM_BUDGET_KB 216   // pipeline slots + output staging + scale ring
+#endif
+#ifndef COMET_N256_NPW
+#define COMET_N256_NPW 2   // promotion warpgroups of the 256-wide tile
+#endif
+#ifndef COMET_N256_NWG
+#define COMET_N256_NWG 2   // widen warpgroups of the 256-wide tile
+#endif
+
 namespace comet {
 namespace gemm {
 namespace {
 
-template <int BN, int CG>
+template <int BN, int CG, int NPW_, int NWG_, int DEBUG_>
 struct CfgN {
   static constexpr int BM = 128;                          // tokens per CTA (TMEM lanes)
   static constexpr int WROWS = BN / CG;                   // weight rows widened by this CTA
@@ -35,22 +53,55 @@ struct CfgN {
   static constexpr int WP_BYTES = WROWS * 64;             // packed weight rows
   static constexpr int B_BYTES = WROWS * 128;             // widened weight rows (MMA B half)
   static constexpr int SLOT_BYTES = X_BYTES + WP_BYTES + B_BYTES;
-  static constexpr int NPW = 3;                           // promotion warpgroups
+  static constexpr int NPW = NPW_;                        // promotion warpgroups
+  static constexpr int NWG = NWG_;                        // widen warpgroups (K-blocks in turn)
+  static constexpr int THREADS = 128 * (1 + NWG + NPW);
   static constexpr int COLS = BN / NPW;                   // accumulator columns per promotion WG
-  static constexpr int NACC = (3 * BN <= 512) ? 3 : 2;    // accumulators in TMEM
+  // setmaxnreg only redistributes the launch-time pool (THREADS x floor8(65536 / THREADS)):
+  // the producer/MMA and widen warpgroups get REG_LOW (40, or 32 when that lets promotion fit
+  // its working set), promotion the rest.
+  static constexpr int REG_LAUNCH = ((65536 / THREADS) / 8) * 8;
+  static constexpr int REG_POOL = REG_LAUNCH * (1 + NWG + NPW);
+  static constexpr int promo_regs(int low) {
+    return ((REG_POOL - low * (1 + NWG)) / NPW / 8) * 8 > 248 ? 248 : ((REG_POOL - low * (1 + NWG)) / NPW / 8) * 8;
+  }
+  static constexpr int ACC_REGS = COLS * (DEBUG_ ? 2 : 1);  // FP32 sums (+ debug int sums)
+  // LOADALL: every column of the K-block is loaded with one wait, the accumulator released at
+  // once, and the FFMA2 folding done afterwards; else 16/32-column batches double-buffered.
+  static constexpr bool LOADALL = COLS <= 120 && promo_regs(32) >= ACC_REGS + COLS + 24;
+  static constexpr int NEED = LOADALL ? ACC_REGS + COLS + 24 : ACC_REGS + 2 * 16 + 24;
+  static constexpr int REG_LOW = promo_regs(40) >= NEED ? 40 : 32;
+  static constexpr int REG_PROMO = promo_regs(REG_LOW);
+  static constexpr int PB = LOADALL ? COLS
+                          : ((REG_PROMO >= ACC_REGS + 2 * 32 + 24 && COLS % 32 == 0) ? 32 : 16);
+  static constexpr int NACC_TMEM = 512 / BN >= 4 ? 4 : 512 / BN;   // accumulators TMEM holds
+  // NSUB = 2: each K-block is issued as two N = BN/2 sub-MMAs, one per promotion warpgroup, each
+  // with its own ready / full barriers and issuing thread, so promotion of one half overlaps the
+  // other half's MMAs and the accumulator ring is four half-units deep (BN = 256, NPW = 2).
+  static constexpr int NSUB = (COMET_NSUB == 2 && NPW == 2 && BN / 2 >= 128) ? 2 : 1;
   // S pipeline slots, each holding one K-block's activation tile, packed and widened weights;
   // the scale ring has S + NACC slots (reuse is implied by the slot-free barrier, see below).
-  static constexpr int S_RAW = (200 * 1024) / (SLOT_BYTES + BM * 4);
+  // output staging for the TMA-store epilogue: per promotion WG two [128 rows][64 B] buffers
+  static constexpr int STAGE_BYTES = NPW * 2 * 8192;
+  static constexpr int S_RAW = (COMET_SMEM_BUDGET_KB * 1024 - STAGE_BYTES) / (SLOT_BYTES + BM * 4);
   static constexpr int S = S_RAW > 8 ? 8 : S_RAW;
+  // accumulators in TMEM; fewer than the slots (the promotion's release of K-block kb + NACC
+  // lands on the mma_ready barrier of slot (kb + NACC) % S)
+  static constexpr int NACC = NACC_TMEM < S ? NACC_TMEM : S - 1;
   static constexpr int SS = S + NACC;
-  static constexpr int SMEM_DATA = S * SLOT_BYTES + SS * BM * 4;
-  static constexpr int N_BARS = 3 * S + NACC;
+  // [slots][output staging][scale ring SS x BM][w_scales 2 x BN][barriers][tmem][tags]
+  static constexpr int SMEM_DATA = S * SLOT_BYTES + STAGE_BYTES + SS * BM * 4 + 2 * BN * 4;
+  static constexpr int N_BARS = 2 * S + NSUB * S + NSUB * NACC;
   static constexpr int SMEM_BYTES = 1024 + SMEM_DATA + N_BARS * 8 + 16 + kMaxBlocks;
   static_assert(S >= 3, "pipeline depth");
+  static_assert(SMEM_BYTES <= 232448, "shared memory per CTA");
   static_assert(S >= NACC + 1, "mma_ready ring must outlast the accumulator ring");
   static_assert(NACC % 2 == 0 || true, "");
   static_assert(NACC * BN <= 512, "TMEM budget");
   static_assert(COLS % 16 == 0, "promotion batches");
+  static_assert(THREADS <= 1024, "threads per CTA");
+  static_assert(REG_PROMO >= NEED, "promotion registers");
+  static_assert(!(DEBUG_ && NSUB == 2), "debug kernels use whole-tile MMAs");
 };
 
 // Synchronisation (every role waits on exactly ONE mbarrier per K-block; a satisfied
@@ -64,16 +115,11 @@ struct CfgN {
 // kb only after slot_free[s] for kb - S; the scales of kb have landed when acc_full(kb) fires
 // (MMA(kb) waited mma_ready(kb) which waited widen(kb) which waited full[s]); the producer may
 // reuse scale slot kb % (S+NACC) because slot_free(kb-S) => MMA(kb-S) => promotion(kb-S-NACC).
-// WG0 producer/MMA, WG1-2 widen (alternate K-blocks), WG3-5 promotion.  768
-// threads launch with 80 registers each; setmaxnreg redistributes that pool
-// (40 + 2 x 40 + 3 x 120 = 480 = 6 x 80).
-constexpr int kWidenWarps = 8;
-constexpr int kPromoWarp0 = 4 + kWidenWarps;          // first promotion warp
-constexpr int kThreadsN = 128 * (1 + kWidenWarps / 4 + 3);
-
-template <int BN, int CG, int DEBUG>
-__global__ void __launch_bounds__(kThreadsN, 1) k_w4ax_n(const __grid_constant__ GemmParams P) {
-  using C = CfgN<BN, CG>;
+template <int BN, int CG, int NPW, int NWG, int DEBUG>
+__global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w4ax_n(const __grid_constant__ GemmParams P) {
+  using C = CfgN<BN, CG, NPW, NWG, DEBUG>;
+  constexpr int kThreadsN = C::THREADS;
+  constexpr int kPromoWarp0 = 4 + 4 * NWG;              // first promotion warp
   constexpr int S = C::S;
   constexpr int SS = C::SS;
   constexpr int NACC = C::NACC;
@@ -84,12 +130,14 @@ __global__ void __launch_bounds__(kThreadsN, 1) k_w4ax_n(const __grid_constant__
   auto sX = [&](int s) { return smem + s * C::SLOT_BYTES; };
   auto sB = [&](int s) { return smem + s * C::SLOT_BYTES + C::X_BYTES; };
   auto sWp = [&](int s) { return smem + s * C::SLOT_BYTES + C::X_BYTES + C::B_BYTES; };
-  float* sS = reinterpret_cast<float*>(smem + S * C::SLOT_BYTES);   // [SS][BM]
+  uint8_t* sY = smem + S * C::SLOT_BYTES;                                       // [NPW][2][8 KB]
+  float* sS = reinterpret_cast<float*>(sY + C::STAGE_BYTES);                     // [SS][BM]
+  float* sWs = sS + SS * BM;                                                     // [2][BN]
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + C::SMEM_DATA);
   uint64_t* full = bars;                     // [S]
   uint64_t* slot_free = full + S;            // [S]
-  uint64_t* mma_ready = slot_free + S;       // [S]   (used in the even CTA)
-  uint64_t* acc_full = mma_ready + S;        // [NACC]
+  uint64_t* mma_ready = slot_free + S;       // [NSUB][S]   (used in the even CTA)
+  uint64_t* acc_full = mma_ready + C::NSUB * S;   // [NSUB][NACC]
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bars + C::N_BARS);
   uint8_t* s_tags = reinterpret_cast<uint8_t*>(tmem_holder + 4);
   const uint32_t s_tags_a = smem_u32(s_tags);
@@ -103,19 +151,22 @@ __global__ void __launch_bounds__(kThreadsN, 1) k_w4ax_n(const __grid_constant__
   const int it_end = debug ? unit + 1 : P.cta_begin[unit + 1];
   const int nb = P.nb;
   constexpr int NPROMO_WARPS = 4 * C::NPW;
-  constexpr uint32_t kReadyCount = (kWidenWarps / 2) * CG + NPROMO_WARPS * CG;   // one widen group
+  constexpr int NSUB = C::NSUB;
+  // per sub-MMA: one widen group + the promotion warps that fold that sub-accumulator
+  constexpr uint32_t kReadyCount = 4 * CG + (NPROMO_WARPS / NSUB) * CG;
 
   if (warp == 0 && lane == 0) {
     tma_prefetch(&P.map_x);
     tma_prefetch(&P.map_w);
     for (int i = 0; i < S; ++i) {
       mbar_init(&full[i], 1);
-      mbar_init(&slot_free[i], 1 + kWidenWarps / 2);
-      mbar_init(&mma_ready[i], kReadyCount);
+      mbar_init(&slot_free[i], NSUB + 4);        // MMA commit(s) + 4 widen warps
+      for (int h = 0; h < NSUB; ++h) mbar_init(&mma_ready[h * S + i], kReadyCount);
     }
-    for (int i = 0; i < NACC; ++i) mbar_init(&acc_full[i], 1);
+    for (int i = 0; i < NSUB * NACC; ++i) mbar_init(&acc_full[i], 1);
     // the first NACC K-blocks have no promotion predecessor
-    for (int i = 0; i < NACC; ++i) mbar_arrive_count(&mma_ready[i], NPROMO_WARPS * CG);
+    for (int h = 0; h < NSUB; ++h)
+      for (int i = 0; i < NACC; ++i) mbar_arrive_count(&mma_ready[h * S + i], (NPROMO_WARPS / NSUB) * CG);
     fence_mbar_init();
   }
   if (warp == 2) {
@@ -132,7 +183,7 @@ __global__ void __launch_bounds__(kThreadsN, 1) k_w4ax_n(const __grid_constant__
   const uint32_t ready_lead = CG == 2 ? mapa_shared(smem_u32(mma_ready), 0) : smem_u32(mma_ready);
 
   if (warp < 4) {
-    setmaxnreg_dec<40>();
+    setmaxnreg_dec<C::REG_LOW>();
     if (warp == 0 && lane == 0) {
       // ------------------------------------------------------------------ TMA producer
       int s = 0, sc = 0, tr = 0;
@@ -143,39 +194,48 @@ __global__ void __launch_bounds__(kThreadsN, 1) k_w4ax_n(const __grid_constant__
         const int m0 = m_tile * (BM * CG) + BM * rank, n0 = n_tile * BN + C::WROWS * rank;
         const uint32_t sbytes = m0 < P.Mp ? (uint32_t)(min((int64_t)BM, P.Mp - m0) * 4) : 0u;
         for (int kb = w.kb_begin; kb < w.kb_end; ++kb) {
+          trace_ev(P, 14, tr);
           mbar_wait(&slot_free[s], ph ^ 1);
-          mbar_arrive_expect_tx(&full[s], C::X_BYTES + C::WP_BYTES + sbytes);
-          tma_load_2d(sX(s), &P.map_x, &full[s], kb * 128, m0);
-          tma_load_2d(sWp(s), &P.map_w, &full[s], kb * 64, n0);
-          if (sbytes) bulk_load(sS + sc * BM, P.scales + (int64_t)kb * P.Mp + m0, sbytes, &full[s]);
+          if (diag_ablate(P) & 32) {                       // diagnostic: no global loads
+            mbar_arrive(&full[s]);
+          } else {
+            mbar_arrive_expect_tx(&full[s], C::X_BYTES + C::WP_BYTES + sbytes);
+            tma_load_2d(sX(s), &P.map_x, &full[s], kb * 128, m0);
+            tma_load_2d(sWp(s), &P.map_w, &full[s], kb * 64, n0);
+            if (sbytes) bulk_load(sS + sc * BM, P.scales + (int64_t)kb * P.Mp + m0, sbytes, &full[s]);
+          }
           trace_ev(P, 0, tr++);
           if (++s == S) { s = 0; ph ^= 1; }
           if (++sc == SS) sc = 0;
         }
       }
-    } else if ((warp == 1 || warp == 3) && lane == 0 && rank == 0) {
+    } else if ((warp == 1 || (COMET_ISSUERS == 2 && warp == 3)) && lane == 0 && rank == 0) {
       // ------------------------------------------------------------------ MMA issuers
       // Two issuing threads: warp 1 takes the even K-blocks of the CTA's sequence, warp 3 the
       // odd ones (different accumulators and slots), so one thread's barrier wait and commits
       // overlap the MMAs the other has queued.  tcgen05.commit tracks the issuing thread's own
       // MMAs, so each thread commits exactly the K-blocks it issued.
+      // NSUB = 2: warp 1 issues sub-MMA 0 (accumulator columns [0, BN/2)) of every K-block and
+      // warp 3 sub-MMA 1; each sub-MMA reads its half of every CTA's widened B rows.
       const int parity = warp == 1 ? 0 : 1;
-      const uint32_t id_f8 = idesc_f8f6f4_e4m3(BM * CG, BN);
-      const uint32_t id_i8 = idesc_i8(BM * CG, BN);
+      const int h = NSUB == 2 ? parity : 0;
+      constexpr int NMMA = BN / NSUB;
+      const uint32_t id_f8 = idesc_f8f6f4_e4m3(BM * CG, NMMA);
+      const uint32_t id_i8 = idesc_i8(BM * CG, NMMA);
       int j = 0, tr = 0;
       for (int it = it_begin; it < it_end; ++it) {
         const WorkItem w = load_item(P, it, debug);
         for (int kb = w.kb_begin; kb < w.kb_end; ++kb, ++j) {
-          if ((j & 1) != parity) continue;
+          if (NSUB == 1 && COMET_ISSUERS == 2 && (j & 1) != parity) continue;
           const int s = j % S, accb = j % NACC;
           const uint32_t ph = (uint32_t)(j / S) & 1u;
-          if (parity == 0) trace_ev(P, 1, tr);
-          mbar_wait(&mma_ready[s], ph);
-          if (parity == 0) trace_ev(P, 3, tr++);
+          trace_ev(P, parity ? 13 : 1, tr);
+          mbar_wait(&mma_ready[h * S + s], ph);
+          trace_ev(P, parity ? 11 : 3, tr++);
           tc_fence_after();
-          const uint32_t d = tbase + accb * BN;
+          const uint32_t d = tbase + accb * BN + h * NMMA;
           const uint32_t sa = smem_u32(sX(s));
-          const uint32_t sbv = smem_u32(sB(s));
+          const uint32_t sbv = smem_u32(sB(s)) + h * (C::WROWS / NSUB) * 128;
           if (diag_ablate(P) & 8) {
             // diagnostic: no MMA
           } else if (lds_u8(s_tags_a + kb)) {
@@ -192,30 +252,30 @@ __global__ void __launch_bounds__(kThreadsN, 1) k_w4ax_n(const __grid_constant__
             }
           }
           if (CG == 2) {
-            tc_commit_mc(&acc_full[accb], 3);
+            tc_commit_mc(&acc_full[h * NACC + accb], 3);
             tc_commit_mc(&slot_free[s], 3);
           } else {
-            tc_commit(&acc_full[accb]);
+            tc_commit(&acc_full[h * NACC + accb]);
             tc_commit(&slot_free[s]);
           }
         }
       }
     }
   } else if (warp < kPromoWarp0) {
-    setmaxnreg_dec<40>();
+    setmaxnreg_dec<C::REG_LOW>();
     // -------------------------------------------------------------------- widen (W -> smem B)
-    // Two widen warpgroups take alternate K-blocks; thread t of a group converts weight rows
+    // The NWG widen warpgroups take K-blocks in turn; thread t of a group converts weight rows
     // t, t + 128, ... of its K-blocks.  INT4 block: byte = u (E4M3 u * 2^-9); INT8 block:
     // byte = 16 u - 128 = 16 w (s8), derived from the INT4-block form with one shift + xor.
     constexpr int RPT = (C::WROWS + 127) / 128;           // rows per thread
-    const int grp = (warp - 4) >> 2;                      // 0: even K-blocks, 1: odd
+    const int grp = (warp - 4) >> 2;                      // K-blocks j with j % NWG == grp
     const int t = threadIdx.x - 128 - 128 * grp;
     int s = 0, tr = 0, j = 0;
     uint32_t ph = 0;
     for (int it = it_begin; it < it_end; ++it) {
       const WorkItem w = load_item(P, it, debug);
       for (int kb = w.kb_begin; kb < w.kb_end; ++kb, ++j) {
-        if ((j & 1) == grp) {
+        if (NWG == 1 || j % NWG == grp) {
           const bool is8 = lds_u8(s_tags_a + kb) != 0;
           mbar_wait(&full[s], ph);
           if (warp == 4 && lane == 0) trace_ev(P, 5, tr);
@@ -261,7 +321,8 @@ __global__ void __launch_bounds__(kThreadsN, 1) k_w4ax_n(const __grid_constant__
           if (warp == 4 && lane == 0) trace_ev(P, 2, tr);
           fence_proxy_async_smem();                       // generic-proxy stores -> tensor core
           __syncwarp();
-          if (lane == 0) mbar_arrive_cluster(ready_lead + s * 8);
+          if (lane == 0)
+            for (int h = 0; h < NSUB; ++h) mbar_arrive_cluster(ready_lead + (h * S + s) * 8);
           if (warp == 4 && lane == 0) trace_ev(P, 4, tr);
           ++tr;
         }
@@ -269,7 +330,7 @@ __global__ void __launch_bounds__(kThreadsN, 1) k_w4ax_n(const __grid_constant__
       }
     }
   } else {
-    setmaxnreg_inc<120>();
+    setmaxnreg_inc<C::REG_PROMO>();
     // -------------------------------------------------------------------- promotion + epilogue
     const int wg = (warp - kPromoWarp0) >> 2;
     const int q = warp & 3;
@@ -278,56 +339,92 @@ __global__ void __launch_bounds__(kThreadsN, 1) k_w4ax_n(const __grid_constant__
     constexpr int COLS = C::COLS;
     const int col0 = wg * COLS;
     const int ptid = threadIdx.x - kPromoWarp0 * 32;
+    const uint32_t s_scale_r = smem_u32(sS) + 4u * r;     // this row's scale in ring slot 0
+    const uint32_t t_cols = tbase + col0 + lane_addr;     // this warp's columns in accumulator 0
+    const int sub = NSUB == 2 ? wg : 0;                   // the sub-MMA whose columns this WG folds
+    const uint32_t ready_rel = ready_lead + sub * S * 8;  // its mma_ready ring (even CTA)
     int accb = 0, sc = 0, rs = NACC % S, tr = 0;           // rs: mma_ready slot of kb + NACC
     uint32_t accph = 0;
+    int tpar = 0;                                         // w_scales buffer of the current tile
+    uint32_t ych = 0;                                     // output chunks this WG has staged
+    // Accumulator column c of this WG -> weight row n of the tile (see the epilogue)
+    constexpr int RUNS = (CG == 2 && NSUB == 2) ? 2 : 1;
+    constexpr int RUN = COLS / RUNS;
+    auto col_n = [&](int wgi, int c) -> int {             // offset from n0 (tile's first weight)
+      return RUNS == 2 ? (c / RUN) * C::WROWS + wgi * RUN + (c % RUN) : wgi * COLS + c;
+    };
+    WorkItem wn = it_begin < it_end ? load_item(P, it_begin, debug) : WorkItem{};
     for (int it = it_begin; it < it_end; ++it) {
-      const WorkItem w = load_item(P, it, debug);
+      const WorkItem w = wn;
+      if (it + 1 < it_end) wn = load_item(P, it + 1, debug);   // in flight during this tile
+      const int tp = tpar;                                // w_scales buffer of this tile
+      tpar ^= 1;
       const int n_tile = w.tile / P.n_m_tiles, m_tile = w.tile % P.n_m_tiles;
       const int m0 = m_tile * (BM * CG) + BM * rank, n0 = n_tile * BN;
       const int64_t m = m0 + r;
       const bool owner = (w.flags & 2) != 0;
       const bool split = (w.flags & 1) != 0;
-      const float init = (owner && m < P.Mp) ? -__ldg(P.corr + m) * 0.001953125f : 0.f;   // 2^-9
+      // -corr * 2^-9 (offset-binary weight correction, owner segment only); loaded now, used
+      // in the epilogue, so the load latency is off the K-loop's critical path
+      const float init = (owner && m < P.Mp) ? -__ldg(P.corr + m) * 0.001953125f : 0.f;
+      if (!DEBUG) {
+        // this tile's per-output-channel weight scales -> shared memory (read in the epilogue)
+        for (int i = ptid; i < BN; i += 128 * C::NPW) {
+          const int wgi = i / COLS, c = i % COLS;
+          const int64_t n = (int64_t)n0 + col_n(wgi, c);
+          sWs[tp * BN + i] = n < P.N ? __ldg(P.w_scales + n) : 0.f;
+        }
+      }
       float acc[COLS];
       int32_t dacc[DEBUG ? COLS : 1];
 #pragma unroll
       for (int c = 0; c < COLS; ++c) {
-        acc[c] = init;
+        acc[c] = 0.f;
         if (DEBUG) dacc[c] = 0;
       }
       for (int kb = w.kb_begin; kb < w.kb_end; ++kb) {
         const bool is8 = lds_u8(s_tags_a + kb) != 0;
         int qs = 0;
         if (DEBUG && !is8 && m < P.Mp) qs = P.qsum[(int64_t)kb * P.Mp + m];
-        mbar_wait(&acc_full[accb], accph);
+        if (threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 12, tr);
+        mbar_wait(&acc_full[sub * NACC + accb], accph);
         if (threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 6, tr);
         tc_fence_after();
         if (diag_ablate(P) & 16) {                              // diagnostic: no promotion work
           tc_fence_before();
           __syncwarp();
-          if (lane == 0) mbar_arrive_cluster(ready_lead + rs * 8);
+          if (lane == 0) mbar_arrive_cluster(ready_rel + rs * 8);
           ++tr;
           if (++accb == NACC) { accb = 0; accph ^= 1; }
           if (++sc == SS) sc = 0;
           if (++rs == S) rs = 0;
           continue;
         }
+        const uint32_t taddr = t_cols + accb * BN;
+        // LOADALL: one load of all COLS columns, release, then fold.  Otherwise software-
+        // pipelined over PB-column batches: the load of batch b+1 is in flight while batch b is
+        // folded in; the accumulator is released once the last load has landed.
+        constexpr int PB = C::PB;                         // columns per TMEM load batch
+        constexpr int NB_ = COLS / PB;
+        uint32_t vb[NB_ > 1 ? 2 : 1][PB];
+        tmem_ld_32x32b<PB>(taddr, vb[0]);
+        if (threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 8, tr);
         float s;
-        asm volatile("ld.shared.f32 %0, [%1];" : "=f"(s) : "r"(smem_u32(sS + sc * BM + r)));
+        asm volatile("ld.shared.f32 %0, [%1];" : "=f"(s) : "r"(s_scale_r + 4u * BM * sc));
         if (is8) s *= 1.220703125e-04f;                   // 2^-13: INT8 block acc = 16 sum x w
         const float2 s2 = make_float2(s, s);
-        const uint32_t taddr = tbase + accb * BN + col0 + lane_addr;
-        // software-pipelined over 32-column batches: the load of batch b+1 is in flight while
-        // batch b is folded in; the accumulator is released once the last load has landed.
-        constexpr int PB = 16;                            // columns per TMEM load batch
-        constexpr int NB_ = COLS / PB;
-        uint32_t vb[2][PB];
-        tmem_ld_32x32b_x16(taddr, vb[0]);
         tmem_wait_ld();
+        if (threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 9, tr);
+        if (NB_ == 1) {
+          // every accumulator column of this thread is in registers: release the TMEM buffer
+          tc_fence_before();
+          __syncwarp();
+          if (lane == 0) mbar_arrive_cluster(ready_rel + rs * 8);
+        }
 #pragma unroll
         for (int b = 0; b < NB_; ++b) {
-          uint32_t* v = vb[b & 1];
-          if (b + 1 < NB_) tmem_ld_32x32b_x16(taddr + (b + 1) * PB, vb[(b + 1) & 1]);
+          uint32_t* v = vb[NB_ > 1 ? (b & 1) : 0];
+          if (b + 1 < NB_) tmem_ld_32x32b<PB>(taddr + (b + 1) * PB, vb[NB_ > 1 ? ((b + 1) & 1) : 0]);
           if (DEBUG) {
 #pragma unroll
             for (int c = 0; c < PB; ++c) {
@@ -356,12 +453,9 @@ __global__ void __launch_bounds__(kThreadsN, 1) k_w4ax_n(const __grid_constant__
               // buffer (the MMA for kb + NACC may start) before the last batch's math
               tc_fence_before();
               __syncwarp();
-              if (lane == 0) mbar_arrive_cluster(ready_lead + rs * 8);
+              if (lane == 0) mbar_arrive_cluster(ready_rel + rs * 8);
+              if (threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 10, tr);
             }
-          } else if (NB_ == 1) {
-            tc_fence_before();
-            __syncwarp();
-            if (lane == 0) mbar_arrive_cluster(ready_lead + rs * 8);
           }
         }
         if (threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 7, tr);
@@ -374,12 +468,14 @@ __global__ void __launch_bounds__(kThreadsN, 1) k_w4ax_n(const __grid_constant__
       if (split) {
         const int seg = (w.flags >> 8) & 0xFF;
         const int nseg = (w.flags >> 16) & 0xFF;
-        const int64_t part_tile = (int64_t)BM * BN;        // = 512 promotion threads * COLS floats
+        // partial tile: float4 (a/4, ptid) at [(a/4) * NT + ptid] -- a warp's stores are contiguous
+        const int64_t part_tile = (int64_t)BM * BN;        // = NT promotion threads * COLS floats
+        constexpr int NT = 128 * C::NPW;
         if (!owner) {
           float4* dst = reinterpret_cast<float4*>(
-              P.ws_part + (((int64_t)w.fix * (P.max_seg - 1) + (seg - 1)) * CG + rank) * part_tile + (int64_t)ptid * COLS);
+              P.ws_part + (((int64_t)w.fix * (P.max_seg - 1) + (seg - 1)) * CG + rank) * part_tile) + ptid;
 #pragma unroll
-          for (int a = 0; a < COLS; a += 4) dst[a / 4] = make_float4(acc[a], acc[a + 1], acc[a + 2], acc[a + 3]);
+          for (int a = 0; a < COLS; a += 4) dst[(a / 4) * NT] = make_float4(acc[a], acc[a + 1], acc[a + 2], acc[a + 3]);
           __threadfence();
           named_bar_sync(1, 128 * C::NPW);
           if (threadIdx.x == kPromoWarp0 * 32) st_release_gpu(P.ws_flags + ((int64_t)w.fix * P.max_seg + seg) * CG + rank, P.epoch);
@@ -391,7 +487,6 @@ __global__ void __launch_bounds__(kThreadsN, 1) k_w4ax_n(const __grid_constant__
             uint64_t t0g = globaltimer_ns();
             while (ld_acquire_gpu(f) != P.epoch) {
               if (globaltimer_ns() - t0g > COMET_MBAR_TIMEOUT_NS) {
-                printf("comet: stream-K fix-up timeout (tile %d seg %d)\n", w.tile, sgi);
                 __trap();
               }
             }
@@ -400,57 +495,95 @@ __global__ void __launch_bounds__(kThreadsN, 1) k_w4ax_n(const __grid_constant__
         named_bar_sync(1, 128 * C::NPW);
         for (int sgi = 1; sgi < nseg; ++sgi) {
           const float4* src = reinterpret_cast<const float4*>(
-              P.ws_part + (((int64_t)w.fix * (P.max_seg - 1) + (sgi - 1)) * CG + rank) * part_tile + (int64_t)ptid * COLS);
+              P.ws_part + (((int64_t)w.fix * (P.max_seg - 1) + (sgi - 1)) * CG + rank) * part_tile) + ptid;
 #pragma unroll
           for (int a = 0; a < COLS; a += 4) {
             float4 t4;
             asm volatile("ld.global.cg.v4.f32 {%0,%1,%2,%3}, [%4];"
-                         : "=f"(t4.x), "=f"(t4.y), "=f"(t4.z), "=f"(t4.w) : "l"(src + a / 4));
+                         : "=f"(t4.x), "=f"(t4.y), "=f"(t4.z), "=f"(t4.w) : "l"(src + (a / 4) * NT));
             acc[a] += t4.x; acc[a + 1] += t4.y; acc[a + 2] += t4.z; acc[a + 3] += t4.w;
           }
         }
       }
-      const int nbase = n0 + col0;
-      if (m < P.M && nbase < P.N) {
-        const float* swp = P.w_scales + nbase;
-        if (P.ydt == COMET_F32) {
-          float* yrow = reinterpret_cast<float*>(P.y) + m * P.ldy + nbase;
+      if (DEBUG) {
+        // Debug kernels: direct stores (plus the exact integer accumulators).
+        if (m < P.M) {
+          const int nbase = n0 + col0;
+          if (nbase < P.N) {
+            const int nvalid = (int)min((int64_t)COLS, (int64_t)P.N - nbase);
 #pragma unroll
-          for (int c = 0; c < COLS; c += 4) {
-            const float4 sw4 = __ldg(reinterpret_cast<const float4*>(swp + c));
-            reinterpret_cast<float4*>(yrow)[c / 4] = make_float4(acc[c] * sw4.x * 512.f, acc[c + 1] * sw4.y * 512.f,
-                                                                 acc[c + 2] * sw4.z * 512.f, acc[c + 3] * sw4.w * 512.f);
-          }
-        } else {
-          uint16_t* yrow = reinterpret_cast<uint16_t*>(P.y) + m * P.ldy + nbase;
-          const bool bf = P.ydt == COMET_BF16;
-#pragma unroll
-          for (int c = 0; c < COLS; c += 8) {
-            const float4 sa = __ldg(reinterpret_cast<const float4*>(swp + c));
-            const float4 sb = __ldg(reinterpret_cast<const float4*>(swp + c + 4));
-            const float f[8] = {acc[c] * sa.x * 512.f, acc[c + 1] * sa.y * 512.f, acc[c + 2] * sa.z * 512.f,
-                                acc[c + 3] * sa.w * 512.f, acc[c + 4] * sb.x * 512.f, acc[c + 5] * sb.y * 512.f,
-                                acc[c + 6] * sb.z * 512.f, acc[c + 7] * sb.w * 512.f};
-            uint32_t pk[4];
-#pragma unroll
-            for (int i = 0; i < 4; ++i) {
-              if (bf) {
-                __nv_bfloat162 h = __floats2bfloat162_rn(f[2 * i], f[2 * i + 1]);
-                pk[i] = *reinterpret_cast<uint32_t*>(&h);
-              } else {
-                __half2 h = __floats2half2_rn(f[2 * i], f[2 * i + 1]);
-                pk[i] = *reinterpret_cast<uint32_t*>(&h);
-              }
+            for (int c = 0; c < COLS; ++c) {
+              if (c >= nvalid) continue;
+              const float f = (acc[c] + init) * __ldg(P.w_scales + nbase + c) * 512.f;
+              if (P.ydt == COMET_F32) reinterpret_cast<float*>(P.y)[m * P.ldy + nbase + c] = f;
+              else if (P.ydt == COMET_BF16) reinterpret_cast<__nv_bfloat16*>(P.y)[m * P.ldy + nbase + c] = __float2bfloat16_rn(f);
+              else reinterpret_cast<__half*>(P.y)[m * P.ldy + nbase + c] = __float2half_rn(f);
+              P.dbg_acc[m * P.N + nbase + c] = dacc[c];
             }
-            reinterpret_cast<uint4*>(yrow)[c / 8] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
           }
         }
-        if (DEBUG) {
+      } else {
+        // TMA-store epilogue.  y = (acc - corr 2^-9) * s_w * 512 (R7).  The
+        // WG's COLS columns leave in chunks of 64 bytes per row (32 half / 16 float columns),
+        // staged in a double-buffered, 64B-swizzled [128 rows][64 B] shared tile and written by
+        // one TMA tensor store each (coalesced; rows >= M and columns >= N are clipped).
+        named_bar_sync(1, 128 * C::NPW);                  // this tile's w_scales are in smem
+        const float* sw = sWs + tp * BN + wg * COLS;
+        uint8_t* stage = sY + wg * 2 * 8192;
+        const uint32_t swz = (uint32_t)((r >> 1) & 3);
+        const bool leader = (threadIdx.x & 127) == 0;     // thread 0 of the WG (row 0)
+        auto stage_and_store = [&](const uint32_t (&pk)[16], int ncol_off, int esz) {
+          // caller: buffer (ych & 1) is free (see the wait below)
+          const uint32_t rowa = smem_u32(stage + (ych & 1) * 8192) + r * 64;
 #pragma unroll
-          for (int c = 0; c < COLS; ++c) P.dbg_acc[m * P.N + nbase + c] = dacc[c];
+          for (int k = 0; k < 4; ++k)
+            asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(rowa + ((k ^ swz) << 4)),
+                         "r"(pk[4 * k]), "r"(pk[4 * k + 1]), "r"(pk[4 * k + 2]), "r"(pk[4 * k + 3]) : "memory");
+          fence_proxy_async_smem();
+          named_bar_sync(2 + wg, 128);
+          if (leader) {
+            tma_store_2d(&P.map_y, stage + (ych & 1) * 8192, (n0 + col_n(wg, ncol_off)) * esz, m0);
+            bulk_commit_group();
+          }
+          ++ych;
+        };
+        auto wait_buffer = [&]() {                        // the store 2 chunks ago has read its buffer
+          if (leader) bulk_wait_group_read<1>();
+          named_bar_sync(2 + wg, 128);
+        };
+        if (P.ydt == COMET_F32) {
+#pragma unroll
+          for (int q = 0; q < COLS / 16; ++q) {
+            wait_buffer();
+            uint32_t pk[16];
+#pragma unroll
+            for (int i = 0; i < 16; ++i) pk[i] = __float_as_uint((acc[q * 16 + i] + init) * sw[q * 16 + i] * 512.f);
+            stage_and_store(pk, q * 16, 4);
+          }
+        } else {
+          const bool bf = P.ydt == COMET_BF16;
+#pragma unroll
+          for (int q = 0; q < COLS / 32; ++q) {
+            wait_buffer();
+            uint32_t pk[16];
+#pragma unroll
+            for (int i = 0; i < 16; ++i) {
+              const int c = q * 32 + 2 * i;
+              const float f0 = (acc[c] + init) * sw[c] * 512.f, f1 = (acc[c + 1] + init) * sw[c + 1] * 512.f;
+              if (bf) {
+                __nv_bfloat162 hv = __floats2bfloat162_rn(f0, f1);
+                pk[i] = *reinterpret_cast<uint32_t*>(&hv);
+              } else {
+                __half2 hv = __floats2half2_rn(f0, f1);
+                pk[i] = *reinterpret_cast<uint32_t*>(&hv);
+              }
+            }
+            stage_and_store(pk, q * 32, 2);
+          }
         }
       }
     }
+    if (!DEBUG && (threadIdx.x & 127) == 0) bulk_wait_group<0>();   // all output stores done
   }
 
   tc_fence_before();
@@ -461,18 +594,18 @@ __global__ void __launch_bounds__(kThreadsN, 1) k_w4ax_n(const __grid_constant__
   }
 }
 
-template <int BN, int CG, int DEBUG>
+template <int BN, int CG, int NPW, int NWG, int DEBUG>
 cudaError_t launch_bn(const GemmParams& prm, int grid, cudaStream_t stream) {
-  using C = CfgN<BN, CG>;
+  using C = CfgN<BN, CG, NPW, NWG, DEBUG>;
   static bool attr_set = false;
   if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(k_w4ax_n<BN, CG, DEBUG>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_BYTES);
+    cudaError_t e = cudaFuncSetAttribute(k_w4ax_n<BN, CG, NPW, NWG, DEBUG>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_BYTES);
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)grid);
-  cfg.blockDim = dim3(kThreadsN);
+  cfg.blockDim = dim3(C::THREADS);
   cfg.dynamicSmemBytes = C::SMEM_BYTES;
   cfg.stream = stream;
   cudaLaunchAttribute attr[1];
@@ -482,21 +615,27 @@ cudaError_t launch_bn(const GemmParams& prm, int grid, cudaStream_t stream) {
   attr[0].val.clusterDim.z = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  return cudaLaunchKernelEx(&cfg, k_w4ax_n<BN, CG, DEBUG>, prm);
+  return cudaLaunchKernelEx(&cfg, k_w4ax_n<BN, CG, NPW, NWG, DEBUG>, prm);
 }
 
 }  // namespace
 
+// bn = 128, 160, 192 or 256; 96 for the debug-accumulator kernels (they need the registers).
 cudaError_t launch_gemm_n(const GemmParams& prm, int grid, int bn, int cg, int debug, cudaStream_t stream) {
-  (void)bn;   // BN = 192 (normal) or 96 (debug accumulators)
   if (cg == 2) {
-    if (debug == 2) return launch_bn<96, 2, 2>(prm, grid, stream);
-    if (debug == 1) return launch_bn<96, 2, 1>(prm, grid, stream);
-    return launch_bn<192, 2, 0>(prm, grid, stream);
+    if (debug == 2) return launch_bn<96, 2, 3, 2, 2>(prm, grid, stream);
+    if (debug == 1) return launch_bn<96, 2, 3, 2, 1>(prm, grid, stream);
+    if (bn == 192) return launch_bn<192, 2, 3, 2, 0>(prm, grid, stream);
+    if (bn == 160) return launch_bn<160, 2, 2, 2, 0>(prm, grid, stream);
+    if (bn == 128) return launch_bn<128, 2, 2, 2, 0>(prm, grid, stream);
+    return launch_bn<256, 2, COMET_N256_NPW, COMET_N256_NWG, 0>(prm, grid, stream);
   }
-  if (debug == 2) return launch_bn<96, 1, 2>(prm, grid, stream);
-  if (debug == 1) return launch_bn<96, 1, 1>(prm, grid, stream);
-  return launch_bn<192, 1, 0>(prm, grid, stream);
+  if (debug == 2) return launch_bn<96, 1, 3, 2, 2>(prm, grid, stream);
+  if (debug == 1) return launch_bn<96, 1, 3, 2, 1>(prm, grid, stream);
+  if (bn == 192) return launch_bn<192, 1, 3, 2, 0>(prm, grid, stream);
+  if (bn == 160) return launch_bn<160, 1, 2, 2, 0>(prm, grid, stream);
+  if (bn == 128) return launch_bn<128, 1, 2, 2, 0>(prm, grid, stream);
+  return cudaErrorInvalidValue;   // the single-CTA kernel has no 256-wide variant (planner rejects it)
 }
 
 }  // namespace gemm

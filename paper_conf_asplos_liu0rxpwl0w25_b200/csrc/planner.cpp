@@ -86,7 +86,9 @@ comet_status_t build_plan(Plan& p, const comet_sched_config& cfg) {
   p.orientation = cfg.orientation > 0 ? cfg.orientation : (p.M >= 256 ? 3 : (p.M >= 128 ? 2 : 1));
   if (p.orientation >= 2) {
     p.tile_n = p.orientation == 3 ? 256 : 128;   // tokens per tile = MMA M (CTA pair: 2 x 128)
-    p.tile_w = 192;                              // weights per tile = MMA N
+    p.tile_w = cfg.tile_w > 0 ? cfg.tile_w : (p.orientation == 3 ? 256 : 192);  // weights per tile = MMA N
+    if (p.tile_w != 128 && p.tile_w != 160 && p.tile_w != 192 && !(p.tile_w == 256 && p.orientation == 3))
+      return fail(COMET_ERR_UNSUPPORTED_SHAPE, "tile_w must be 128, 160 or 192 (or 256 with orientation 3)");
   } else {
     p.tile_n = cfg.tile_n > 0 ? cfg.tile_n : auto_tile_n(p.M);
     p.tile_w = kTileW;

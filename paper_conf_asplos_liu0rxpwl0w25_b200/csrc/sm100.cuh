@@ -70,18 +70,52 @@ __device__ __forceinline__ uint64_t globaltimer_ns() {
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
   return t;
 }
+// Blocking wait on phase `parity`.  First a non-suspending test_wait: on a phase that has
+// already completed it returns in ~21 clk, where try_wait costs ~165 clk even then
+// (profiles/r01/probe_lat.json).  Otherwise a loop of try_wait with a suspend hint: the thread
+// sleeps in hardware until the phase completes instead of spinning on issue slots.  The whole
+// loop is one PTX block so the compiler cannot hoist the hang guard into it; the global timer is
+// read once every 64 unsuccessful suspensions, and a wait longer than COMET_MBAR_TIMEOUT_NS
+// traps (the launch fails with an error) instead of hanging the GPU.
+#ifndef COMET_WAIT_MODE
+#define COMET_WAIT_MODE 0
+#endif
+#if COMET_WAIT_MODE == 0        // try_wait with a suspend-time hint (hardware sleep)
+#define COMET_WAIT_INSTR "mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1, %2;\n\t"
+#elif COMET_WAIT_MODE == 1      // try_wait, system-dependent suspend window
+#define COMET_WAIT_INSTR "mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1;\n\t"
+#else                           // spin on test_wait
+#define COMET_WAIT_INSTR "mbarrier.test_wait.parity.shared::cta.b64 P, [%0], %1;\n\t"
+#endif
+__device__ __forceinline__ void mbar_wait_addr(uint32_t a, uint32_t parity) {
+  asm volatile(
+      "{\n\t"
+      ".reg .pred P, Q;\n\t"
+      ".reg .u32 c;\n\t"
+      ".reg .u64 t0, t1;\n\t"
+      "mbarrier.test_wait.parity.shared::cta.b64 P, [%0], %1;\n\t"
+      "@P bra.uni WAIT_DONE;\n\t"
+      "mov.u64 t0, %%globaltimer;\n"
+      "WAIT_OUTER:\n\t"
+      "mov.u32 c, 64;\n"
+      "WAIT_LOOP:\n\t"
+      COMET_WAIT_INSTR
+      "@P bra.uni WAIT_DONE;\n\t"
+      "sub.u32 c, c, 1;\n\t"
+      "setp.ne.u32 Q, c, 0;\n\t"
+      "@Q bra.uni WAIT_LOOP;\n\t"
+      "mov.u64 t1, %%globaltimer;\n\t"
+      "sub.u64 t1, t1, t0;\n\t"
+      "setp.lt.u64 Q, t1, %3;\n\t"
+      "@Q bra.uni WAIT_OUTER;\n\t"
+      "trap;\n"
+      "WAIT_DONE:\n\t"
+      "}\n" ::"r"(a),
+      "r"(parity), "n"(1000000), "l"((uint64_t)COMET_MBAR_TIMEOUT_NS)
+      : "memory");
+}
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
-  const uint32_t a = smem_u32(bar);
-  if (mbar_try_wait(a, parity)) return;
-  uint64_t t0 = globaltimer_ns();
-  uint32_t spins = 0;
-  while (!mbar_try_wait(a, parity)) {
-    if ((++spins & 255u) == 0 && globaltimer_ns() - t0 > COMET_MBAR_TIMEOUT_NS) {
-      printf("comet: mbarrier wait timeout (block %d thread %d parity %u)\n", blockIdx.x,
-             threadIdx.x, parity);
-      __trap();
-    }
-  }
+  mbar_wait_addr(smem_u32(bar), parity);
 }
 
 // ------------------------------------------------------------------ explicit shared loads
@@ -130,6 +164,24 @@ __device__ __forceinline__ void tma_load_2d_hint(void* dst, const CUtensorMap* m
       " [%0], [%1, {%3, %4}], [%2], %5;" ::"r"(smem_u32(dst)),
       "l"(map), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "l"(policy)
       : "memory");
+}
+// 2D tiled store shared -> global (bulk-group completion; clipped at the tensor bounds).
+__device__ __forceinline__ void tma_store_2d(const CUtensorMap* map, const void* src, int32_t c0, int32_t c1) {
+  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(map),
+               "r"(smem_u32(src)), "r"(c0), "r"(c1)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_commit_group() {
+  asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+// wait until at most N of this thread's committed bulk groups still read shared memory
+template <int N>
+__device__ __forceinline__ void bulk_wait_group_read() {
+  asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
+}
+template <int N>
+__device__ __forceinline__ void bulk_wait_group() {
+  asm volatile("cp.async.bulk.wait_group %0;" ::"n"(N) : "memory");
 }
 // 1D bulk copy global -> shared (bytes % 16 == 0, both addresses 16B aligned).
 __device__ __forceinline__ void bulk_load(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
@@ -388,31 +440,6 @@ __device__ __forceinline__ uint32_t mapa_shared(uint32_t saddr, uint32_t rank) {
 // (MEMBAR.ALL + ERRBAR) is needed on this hot path.
 __device__ __forceinline__ void mbar_arrive_cluster(uint32_t cluster_addr) {
   asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
-}
-__device__ __forceinline__ bool mbar_try_wait_cluster(uint32_t bar, uint32_t parity) {
-  uint32_t ok;
-  asm volatile(
-      "{\n\t.reg .pred P;\n\t"
-      "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 P, [%1], %2;\n\t"
-      "selp.b32 %0, 1, 0, P;\n\t}\n"
-      : "=r"(ok)
-      : "r"(bar), "r"(parity)
-      : "memory");
-  return ok != 0;
-}
-// Wait on a local mbarrier whose arrivals may come from the peer CTA (acquire at cluster scope).
-__device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity) {
-  const uint32_t a = smem_u32(bar);
-  if (mbar_try_wait_cluster(a, parity)) return;
-  uint64_t t0 = globaltimer_ns();
-  uint32_t spins = 0;
-  while (!mbar_try_wait_cluster(a, parity)) {
-    if ((++spins & 255u) == 0 && globaltimer_ns() - t0 > COMET_MBAR_TIMEOUT_NS) {
-      printf("comet: cluster mbarrier wait timeout (block %d thread %d parity %u)\n", blockIdx.x,
-             threadIdx.x, parity);
-      __trap();
-    }
-  }
 }
 // TMEM management for a CTA pair (executed by the same warp in both CTAs).
 template <uint32_t NCOLS>

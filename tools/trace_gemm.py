@@ -26,7 +26,7 @@ act, sc = cb.quantize_act(x, tags)
 wp = cb.pack_weight(w)
 plan = cb.Plan(M, N, K, tags, orientation=orient)
 y = cb.w4ax_gemm(plan, act, sc, wp, sw)
-buf = torch.zeros(2 * 8 * 1024, dtype=torch.int64, device="cuda")
+buf = torch.zeros(2 * 16 * 1024, dtype=torch.int64, device="cuda")
 L = cb.lib()
 L.comet_debug_set_trace.argtypes = [ctypes.c_void_p]
 L.comet_debug_set_trace(ctypes.c_void_p(buf.data_ptr()))
@@ -34,5 +34,5 @@ for _ in range(2):
     cb.w4ax_gemm(plan, act, sc, wp, sw, out=y)
 torch.cuda.synchronize()
 L.comet_debug_set_trace(None)
-t = buf.view(2, 8, 1024).cpu().numpy()
+t = buf.view(2, 16, 1024).cpu().numpy()
 print(json.dumps({"info": plan.info(), "trace": t.tolist()}))
