@@ -172,6 +172,44 @@ def cpu_baseline_sample(budget_s=15.0):
 
 # ---------------------------------------------------------------------------- comet arm
 
+def decode_sweep(cb, torch, dev, peaks, Ms=(1, 4, 8, 32), iters=20):
+    """BASELINE config 5: decode-regime W4Ax GEMM on the LLaMA-3-70B layers (TP1), HBM-bound.
+    Each timed GEMM is preceded by a 256 MiB write that evicts L2, so the packed weights are
+    read from HBM.  Bytes = packed weights + weight scales + activation codes/scales + output."""
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    out = {}
+    hbm = peaks["hbm_gbs"]
+    for name, K, N, _ in LAYERS:
+        rng = np.random.default_rng(7)
+        tags = synth.make_tags(K, FRAC, rng)
+        w, s_w = synth.make_weights(N, K, rng)
+        wp = cb.pack_weight(torch.from_numpy(w).to(dev))
+        swd = torch.from_numpy(s_w).to(dev)
+        del w
+        for M in Ms:
+            x = torch.from_numpy(synth.make_activations(M, K, tags, rng)).to(dev)
+            plan = cb.Plan(M, N, K, tags)
+            act, sc = cb.quantize_act(x, tags)
+            y = torch.empty((M, N), dtype=torch.float16, device=dev)
+            ws = []
+            for i in range(iters + 3):
+                flush.fill_(i & 0xFF)
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record()
+                cb.w4ax_gemm(plan, act, sc, wp, swd, out=y)
+                b.record()
+                ws.append((a, b))
+            torch.cuda.synchronize()
+            us = statistics.median(a.elapsed_time(b) for a, b in ws[3:]) * 1e3
+            nbytes = N * K // 2 + N * 4 + act.numel() + sc.numel() * 4 + M * N * 2
+            gbs = nbytes / (us * 1e-6) / 1e9
+            out[f"{name}_M{M}"] = {"us": round(us, 2), "GB/s": round(gbs, 1), "frac_hbm": round(gbs / hbm, 3),
+                                   "orientation": plan.info()["orientation"], "tile_n": plan.info()["tile_n"]}
+        del wp
+    del flush
+    return {"unit": "GB/s", "peak_gbs": hbm, "l2": "256 MiB write before every timed GEMM", "layers": out}
+
+
 def shard(K, N, kind, tags, rank, world):
     """Tensor-parallel shard of one layer: returns (k0, k1, n0, n1)."""
     if world == 1:
@@ -296,6 +334,7 @@ def run_comet(args, rank, world, local_rank):
     traffic = load_traffic()
     roofline = {"bound": "tensor", "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
                 "frac": achieved / peak,
+                "frac_spec_4500": achieved / 4500.0,
                 "traffic": (traffic or {}).get("bytes_per_launch"),
                 "peak_source": f"{peak_src} bf16 burst {peaks['bf16_tflops']} TFLOP/s x 2 (INT8/FP8 : BF16 nominal ratio)",
                 "kernel": "k_w4ax (persistent tcgen05 W4Ax GEMM)",
@@ -352,6 +391,7 @@ def run_comet(args, rank, world, local_rank):
                        "public API: H2D copy + quantize_act + w4ax_gemm (+ NCCL all_reduce) + D2H copy"}
 
     cpu = cpu_baseline_sample(args.cpu_budget) if (rank == 0 and world == 1 and args.cpu_budget > 0) else None
+    decode = decode_sweep(cb, torch, dev, peaks) if (rank == 0 and world == 1 and args.decode) else None
 
     if rank == 0:
         line = {
@@ -370,6 +410,7 @@ def run_comet(args, rank, world, local_rank):
             "e2e": e2e,
             "gpu_launches": 2 * len(layers) * args.steps,
             "clocks": clocks,
+            "decode": decode,
         }
         if world > 1:
             line["allreduce_ms_per_step"] = ar_ms / args.steps
@@ -391,6 +432,7 @@ def main():
     ap.add_argument("--split-mode", type=int, default=-1)
     ap.add_argument("--orientation", type=int, default=0, help="0 = planner default")
     ap.add_argument("--tile-w", type=int, default=0, help="weights per tile (192/256); 0 = planner default")
+    ap.add_argument("--decode", type=int, default=1, help="1 = add the decode (M<=32) HBM sweep (N=1)")
     args = ap.parse_args()
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", str(args.gpus if args.gpus == 1 else 1)))
