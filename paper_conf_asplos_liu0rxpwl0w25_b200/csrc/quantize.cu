@@ -50,6 +50,38 @@ __device__ __forceinline__ uint32_t e4m3_of_int4(int q) {
   return e | (q < 0 ? 0x80u : 0u);
 }
 
+// Packed binary32 pairs (FMUL2 / FADD2 on sm_100a), round-to-nearest-even, never contracted.
+__device__ __forceinline__ float2 fmul2_rn(float2 a, float2 b) {
+  float2 d;
+  asm("{\n\t.reg .b64 ra, rb, rd;\n\tmov.b64 ra, {%2, %3};\n\tmov.b64 rb, {%4, %5};\n\t"
+      "mul.rn.f32x2 rd, ra, rb;\n\tmov.b64 {%0, %1}, rd;\n\t}\n"
+      : "=f"(d.x), "=f"(d.y) : "f"(a.x), "f"(a.y), "f"(b.x), "f"(b.y));
+  return d;
+}
+// a + b as fma(a, 1, b): one rounding, so exactly RN(a + b).  (ptxas contracts a preceding
+// mul.rn.f32x2 with add.rn.f32x2 into one FFMA2 -- a single rounding of a*r + b, which breaks
+// the tie cases of the definition -- but leaves FMUL2 followed by this FFMA2 alone.)
+__device__ __forceinline__ float2 fadd2_rn(float2 a, float2 b) {
+  float2 d;
+  asm("{\n\t.reg .b64 ra, rb, rc, rd;\n\tmov.b64 ra, {%2, %3};\n\tmov.b64 rb, {%6, %6};\n\t"
+      "mov.b64 rc, {%4, %5};\n\tfma.rn.f32x2 rd, ra, rb, rc;\n\tmov.b64 {%0, %1}, rd;\n\t}\n"
+      : "=f"(d.x), "=f"(d.y) : "f"(a.x), "f"(a.y), "f"(b.x), "f"(b.y), "f"(1.0f));
+  return d;
+}
+// E4M3 bytes of two floats (exact for the integers |q| <= 7): low byte <- lo, high byte <- hi.
+__device__ __forceinline__ uint32_t e4m3x2(float lo, float hi) {
+  uint16_t d;
+  asm("cvt.rn.satfinite.e4m3x2.f32 %0, %1, %2;" : "=h"(d) : "f"(hi), "f"(lo));
+  return d;
+}
+
+// Rounding by the magic constant 1.5 * 2^23: for |t| < 2^22, RN(t + 1.5 * 2^23) =
+// 1.5 * 2^23 + rint(t) with rint = round half to even (reading R3), so the low bits of its
+// binary32 pattern are the two's-complement integer rint(t) and RN(that - 1.5 * 2^23) is
+// rint(t) as a float, exactly.
+constexpr float kMagic = 12582912.0f;
+constexpr uint32_t kMagicBits = 0x4B400000u;
+
 struct BlockOut {
   uint32_t lo, hi;   // 8 code bytes
   float s;
@@ -57,6 +89,11 @@ struct BlockOut {
 };
 
 // Quantise the 8 values of this lane for block b (16 lanes cooperate on 128 values).
+//   Fast path (every finite r = qmax/amax, and amax == 0): t = x * r as one binary32 product,
+//   q = rint(t) by the magic constant.  |x| <= amax gives |t| <= qmax (1 + 2^-24)^2, so
+//   rint(t) never exceeds qmax and the clamp of the definition is a no-op.
+//   Slow path (a binary32-subnormal amax, where qmax/amax overflows to inf, reading R5):
+//   the definition written out with a saturating conversion and the clamp.
 __device__ __forceinline__ BlockOut quantize8(const float (&v)[8], bool is8) {
   float a = 0.f;
 #pragma unroll
@@ -66,22 +103,53 @@ __device__ __forceinline__ BlockOut quantize8(const float (&v)[8], bool is8) {
   a = fmaxf(a, __shfl_xor_sync(0xffffffffu, a, 2));
   a = fmaxf(a, __shfl_xor_sync(0xffffffffu, a, 1));
   const float qmax = is8 ? 127.f : 7.f;
-  const int iq = is8 ? 127 : 7;
   BlockOut o;
   o.s = (a == 0.f) ? 0.f : __fdiv_rn(a, qmax);
-  const float r = __fdiv_rn(qmax, a);          // +inf for an all-zero block -> t NaN -> code 0
-  uint32_t bytes[8];
+  const float r = __fdiv_rn(qmax, a);          // +inf for an all-zero block
   int qs = 0;
+  if (a == 0.f || r <= 3.0e38f) {              // uniform per half-warp
+    const float rr = a == 0.f ? 0.f : r;       // zero block: every code 0
+    float2 y[4];
+    uint32_t bsum = 0;
 #pragma unroll
-  for (int j = 0; j < 8; ++j) {
-    const float t = __fmul_rn(v[j], r);
-    int q = __float2int_rn(t);                  // cvt.rni.s32.f32: half-even, NaN -> 0, saturating
-    q = min(max(q, -iq), iq);
-    qs += q;
-    bytes[j] = is8 ? ((uint32_t)q & 0xFFu) : e4m3_of_int4(q);
+    for (int i = 0; i < 4; ++i) {
+      y[i] = fadd2_rn(fmul2_rn(make_float2(v[2 * i], v[2 * i + 1]), make_float2(rr, rr)),
+                      make_float2(kMagic, kMagic));
+      bsum += __float_as_uint(y[i].x) + __float_as_uint(y[i].y);
+    }
+    qs = (int)(bsum - 8u * kMagicBits);        // sum of the 8 codes (mod 2^32, exact)
+    if (is8) {
+      // two's-complement byte of rint(t) = low byte of the biased pattern
+      const uint32_t p01 = __byte_perm(__float_as_uint(y[0].x), __float_as_uint(y[0].y), 0x0040);
+      const uint32_t p23 = __byte_perm(__float_as_uint(y[1].x), __float_as_uint(y[1].y), 0x0040);
+      const uint32_t p45 = __byte_perm(__float_as_uint(y[2].x), __float_as_uint(y[2].y), 0x0040);
+      const uint32_t p67 = __byte_perm(__float_as_uint(y[3].x), __float_as_uint(y[3].y), 0x0040);
+      o.lo = __byte_perm(p01, p23, 0x5410);
+      o.hi = __byte_perm(p45, p67, 0x5410);
+    } else {
+      uint32_t e[4];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const float2 f = fadd2_rn(y[i], make_float2(-kMagic, -kMagic));   // rint(t), +0 for 0
+        e[i] = e4m3x2(f.x, f.y);
+      }
+      o.lo = e[0] | (e[1] << 16);
+      o.hi = e[2] | (e[3] << 16);
+    }
+  } else {
+    const int iq = is8 ? 127 : 7;
+    uint32_t bytes[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const float t = __fmul_rn(v[j], r);
+      int q = __float2int_rn(t);                // cvt.rni.s32.f32: half-even, NaN -> 0, saturating
+      q = min(max(q, -iq), iq);
+      qs += q;
+      bytes[j] = is8 ? ((uint32_t)q & 0xFFu) : e4m3_of_int4(q);
+    }
+    o.lo = bytes[0] | (bytes[1] << 8) | (bytes[2] << 16) | (bytes[3] << 24);
+    o.hi = bytes[4] | (bytes[5] << 8) | (bytes[6] << 16) | (bytes[7] << 24);
   }
-  o.lo = bytes[0] | (bytes[1] << 8) | (bytes[2] << 16) | (bytes[3] << 24);
-  o.hi = bytes[4] | (bytes[5] << 8) | (bytes[6] << 16) | (bytes[7] << 24);
   qs += __shfl_xor_sync(0xffffffffu, qs, 8);
   qs += __shfl_xor_sync(0xffffffffu, qs, 4);
   qs += __shfl_xor_sync(0xffffffffu, qs, 2);
@@ -111,7 +179,7 @@ __global__ void __launch_bounds__(256) k_quantize(const uint16_t* __restrict__ x
     const bool live = m < M;
     const uint16_t* xrow = x + (live ? m : 0) * ldx;
     uint8_t* crow = codes + (live ? m : 0) * K;
-    constexpr int U = 2;   // pairs in flight per warp
+    constexpr int U = 4;   // block pairs in flight per warp (64 B per lane)
     for (int p0 = wi; p0 < npairs; p0 += WPR * U) {
       uint4 raw[U];
 #pragma unroll
@@ -166,12 +234,10 @@ cudaError_t launch_q(const void* x, int64_t M, int64_t K, int64_t ldx, const Tag
   float* corr = reinterpret_cast<float*>(base + L.corr_off);
   const int64_t Mp = L.Mp;
   const int64_t nb = L.nb;
-  const int64_t target = 2 * 148;
+  // enough CTAs for ~16 per SM (memory-level parallelism), warps of a row sharing its pairs
+  const int64_t target = 16 * 148;
   int wpr = 1;
-  if (Mp / 8 < target) wpr = 2;
-  if (Mp / 4 < target) wpr = 4;
-  if (Mp / 2 < target) wpr = 8;
-  while (wpr > 1 && (nb + 1) / 2 < wpr) wpr /= 2;
+  while (wpr < 8 && ceil_div(Mp, 8 / wpr) < target && (nb + 1) / 2 >= 2 * wpr) wpr *= 2;
   const int rows = 8 / wpr;
   const dim3 grid((unsigned)ceil_div(Mp, rows));
   const uint16_t* xp = static_cast<const uint16_t*>(x);
