@@ -133,7 +133,7 @@ comet_status_t comet_pack_weight(const int8_t* w_codes_dev, int64_t N, int64_t K
 typedef struct comet_plan_s* comet_plan_t;   /* opaque, library-owned, immutable after create */
 
 typedef struct {
-  int tile_n;          /* tokens per output tile (MMA N): 16..224, multiple of 16; 0 = auto */
+  int tile_n;          /* orientation 1: tokens per output tile (MMA N): 16, 32, 64 or 128; 0 = auto */
   int num_sms;         /* persistent CTAs (one per SM); 0 = query the current device */
   int split_mode;      /* 0 = whole tiles onto the least-loaded CTA (no fix-up);
                           1 = tile decomposition: stream-K contiguous K-ranges;

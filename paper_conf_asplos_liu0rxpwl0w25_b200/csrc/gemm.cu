@@ -1,4 +1,5 @@
-// gemm.cu -- the W4Ax GEMM on sm_100a (kernel 2), persistent and warp-specialised.
+// gemm.cu -- the W4Ax GEMM for decode-sized token counts on sm_100a (kernel 2, orientation 1),
+// persistent, warp-specialised, HBM-streaming; plus the host-side launcher of both GEMM kernels.
 //
 //   Y[m, n] = s_w[n] * sum_b s_a[m,b] * acc_b[m,n]
 //
@@ -8,21 +9,27 @@
 // the B operand (N = NT tokens, TMA-staged in shared memory, 128-byte swizzle), so the tokens
 // become the MMA N dimension and decode-sized M still fills an instruction.
 //
+// At decode sizes the kernel is a weight stream: the packed weights (N*K/2 bytes) dominate the
+// traffic.  A pipeline stage therefore carries TWO K-blocks: a 128-row x 128-byte box of packed
+// weights (16 KB; 128-byte rows stream from HBM at ~4.6 TB/s where 64-byte rows reach ~3.8,
+// profiles/r01/probe_stream.txt), the two K-blocks' activation codes and their scales.
+//
 // Roles (512 threads, 16 warps):
-//   warp 0      TMA producer: activation tile [NT x 128 B], packed weight tile [128 x 64 B]
-//               and the block's scales s_a[b][m0 .. m0+NT) into a STAGES-deep mbarrier ring.
-//   warp 1      MMA issuer (one thread): per K-block 4 x tcgen05.mma (K = 32) into a fresh
-//               TMEM accumulator; INT4 blocks use kind::f8f6f4 (E4M3), INT8 blocks kind::i8.
-//   warp 2      TMEM allocator.
-//   warps 4-7   widen: packed INT4 weight row -> 128 bytes in 3 instructions per 8 values
-//               (the B200 form of the paper's location switch + zero extension),
-//               tcgen05.st into one of two TMEM A buffers.  INT4 block: byte = u = w+8, read by
-//               the FP8 tensor core as u * 2^-9 exactly.  INT8 block: byte = 16*w (s8).
-//   warps 8-15  promotion ("dequant"): per K-block, tcgen05.ld the accumulator and fold
-//               it into FP32 registers with the block's per-token scale (one FFMA2 per two
-//               elements for INT4 blocks, the accumulator is already FP32); at the end of the
-//               tile the FP32 result is scaled by s_w and stored (or, for a tile split across
-//               CTAs, exchanged through the stream-K workspace).
+//   warp 0       TMA producer: W box [128 rows x 128 B], X boxes [NT x 128 B] per K-block, and
+//                each K-block's scales s_a[b][m0 .. m0+NT) (own ring).
+//   warp 1       MMA issuer (one thread): per K-block 4 x tcgen05.mma (K = 32) into its own TMEM
+//                accumulator; INT4 blocks use kind::f8f6f4 (E4M3), INT8 blocks kind::i8.
+//   warp 2       TMEM allocator.
+//   warps 4-11   widen, two groups of 4 warps taking alternate stages: a packed INT4 weight row
+//                -> 256 bytes in 3 instructions per 8 values (the B200 form of the paper's
+//                location switch + zero extension), tcgen05.st into a TMEM A buffer.
+//                INT4 block: byte = u = w+8, read by the FP8 tensor core as u * 2^-9 exactly.
+//                INT8 block: byte = 16*w (s8).
+//   warps 12-15  promotion ("dequant"): per K-block, tcgen05.ld the accumulator (thread =
+//                weight row, columns = tokens) and fold it into FP32 registers with the block's
+//                per-token scale (FFMA2); at the end of the tile the FP32 result is scaled by s_w
+//                and stored (or, for a tile split across CTAs, exchanged through the stream-K
+//                workspace in a fixed order).
 //
 // Exactness: INT4 block: acc = 2^-9 * sum_k x_k (w_k + 8) with every term an integer multiple
 // of 2^-9 and |sum| < 2^14 -> exact in FP32 (checked bit-exactly against the oracle through the
@@ -35,55 +42,91 @@
 namespace comet {
 namespace gemm {
 namespace {
-constexpr uint32_t kAcol = 0;        // TMEM columns [0, 64): two widened-weight A buffers
-constexpr uint32_t kAccCol = 64;     // TMEM columns [64, 64 + 2 NT): two accumulators
+#ifndef COMET_DEC_ABLATE
+#define COMET_DEC_ABLATE 0      // timing experiments only (wrong results): bit 0 no MMAs, bit 1 no
+#endif                          // TMEM stores of widened weights, bit 2 no accumulator loads
+#ifndef COMET_DEC_ISSUERS
+#define COMET_DEC_ISSUERS 2     // MMA-issuing threads (warps 1 and 3 alternate stages)
+#endif
 
+constexpr int kWidenWarp0 = 4;
+constexpr int kPromoWarp0 = 12;
+
+// One pipeline stage = KS consecutive K-blocks of one tile (KS = 4 for NT <= 32, else 2):
+//   W   KS/2 boxes of 128 weight rows x 128 B (two K-blocks of packed nibbles per row), SW128
+//   X   one 3D box [KS K-blocks][NT tokens][128 B] of activation codes, SW128 (UMMA B operand)
+//   S   one 2D box [KS][NT] of per-token scales s_a
+// all on one mbarrier.  The stage is released by the MMA commit, the 4 widen warps and the 4
+// promotion warps (which read the scales from it).
+// TMEM columns: [0, NA * 32 KS) widened-weight A buffers (one per widen group), then NACC
+// accumulator sets of KS x NT columns (one accumulator per K-block of a stage).
 template <int NT>
 struct Cfg {
-  static constexpr int ACTIVE_WGS = NT >= 32 ? 2 : 1;          // promotion warpgroups in use
-  static constexpr int COLS = NT / ACTIVE_WGS;                 // accumulator columns per WG
-  static constexpr int NACC = (64 + 3 * NT <= 512) ? 3 : 2;    // accumulator buffers in TMEM
-  static constexpr int X_BYTES = NT * 128;
-  static constexpr int W_BYTES = kTileW * 64;
-  static constexpr int STAGE_BYTES = X_BYTES + W_BYTES;
-  static constexpr int STAGES_RAW = (196 * 1024) / STAGE_BYTES;
-  static constexpr int STAGES = STAGES_RAW > 10 ? 10 : STAGES_RAW;
-  static constexpr int SMEM_DATA = STAGES * STAGE_BYTES + kSRing * NT * 4;
-  static constexpr int N_BARS = 2 * STAGES + 4 + 2 * NACC + 2 * kSRing;
+  static constexpr int KS = NT <= 32 ? 4 : 2;                  // K-blocks per stage
+  static constexpr int NA = 2;                                 // = widen groups
+  static constexpr int A_COLS = 32 * KS;
+  static constexpr int ACC_SET = KS * NT;                      // accumulator columns per stage
+  static constexpr int NACC_RAW = (512 - NA * A_COLS) / ACC_SET;
+  // Two MMA issuers and two widen groups take alternate stages.  An mbarrier wait is only sound
+  // if the waiter observes every phase of that barrier (a parity wait cannot tell phase k+2 from
+  // phase k), so each alternating role must always land on the same barriers: the stage count
+  // and the accumulator-set count are even (or there is a single issuer).
+  static constexpr int ISSUERS = (COMET_DEC_ISSUERS == 2 && NACC_RAW >= 2) ? 2 : 1;
+  static constexpr int NACC_C = NACC_RAW > 4 ? 4 : NACC_RAW;
+  static constexpr int NACC = ISSUERS == 2 ? (NACC_C & ~1) : NACC_C;
+  static constexpr uint32_t ACC_COL = NA * A_COLS;
+  static constexpr int XKB_BYTES = NT * 128;                   // one K-block of codes
+  static constexpr int W_BYTES = KS * kTileW * 64;             // KS K-blocks of packed weights
+  static constexpr int S_BYTES = KS * NT * 4;
+  static constexpr int STAGE_RAW = W_BYTES + KS * XKB_BYTES + S_BYTES;
+  static constexpr int STAGE_BYTES = (STAGE_RAW + 1023) / 1024 * 1024;
+  static constexpr int STAGES_RAW = (222 * 1024) / STAGE_BYTES;
+  static constexpr int STAGES = (STAGES_RAW > 8 ? 8 : STAGES_RAW) & ~1;   // even (see ISSUERS)
+  static constexpr int SMEM_DATA = STAGES * STAGE_BYTES;
+  static constexpr int N_BARS = 2 * STAGES + 2 * NA + 2 * NACC;
   static constexpr int SMEM_BYTES = 1024 + SMEM_DATA + N_BARS * 8 + 16 + kMaxBlocks;
-  static_assert(COLS % 16 == 0, "promotion chunks of 16 columns");
-  static_assert(NACC * NT + 64 <= 512, "TMEM budget");
+  static constexpr int CH = NT < 32 ? NT : 32;                 // promotion column chunk
+  static_assert(NT % 16 == 0 && NT <= 128, "decode tile");
+  static_assert(NACC >= 1 && NACC * ACC_SET + NA * A_COLS <= 512, "TMEM budget");
+  static_assert(STAGES >= 2 && (ISSUERS == 1 || NACC % 2 == 0), "alternating roles");
+  static_assert(SMEM_BYTES <= 227 * 1024, "shared memory budget");
 };
+
+template <int NCOL>
+__device__ __forceinline__ void tmem_ld_cols(uint32_t taddr, uint32_t* r) {
+  if constexpr (NCOL == 32) tmem_ld_32x32b_x32(taddr, r);
+  else tmem_ld_32x32b_x16(taddr, r);
+}
 
 template <int NT, int DEBUG>
 __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ GemmParams P) {
   using C = Cfg<NT>;
   constexpr int S = C::STAGES;
+  constexpr int NA = C::NA;
   constexpr int NACC = C::NACC;
+  constexpr int KS = C::KS;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   // keep the pointer derived from the __shared__ array (shared address space) when aligning
   uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
-  uint8_t* sX = smem;
-  uint8_t* sW = sX + S * C::X_BYTES;
-  float* sS = reinterpret_cast<float*>(sW + S * C::W_BYTES);
+  auto sW = [&](int st) { return smem + st * C::STAGE_BYTES; };
+  auto sX = [&](int st) { return smem + st * C::STAGE_BYTES + C::W_BYTES; };
+  auto sS = [&](int st) { return smem + st * C::STAGE_BYTES + C::W_BYTES + KS * C::XKB_BYTES; };
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + C::SMEM_DATA);
-  uint64_t* full = bars;                    // [S]    TMA -> (MMA, widen)
-  uint64_t* empty = bars + S;               // [S]    (MMA commit + 4 widen warps) -> TMA
-  uint64_t* a_full = bars + 2 * S;          // [2]    widen -> MMA
-  uint64_t* a_empty = a_full + 2;           // [2]    MMA commit -> widen
-  uint64_t* acc_full = a_full + 4;          // [NACC] MMA commit -> promotion
+  uint64_t* full = bars;                    // [S]    TMA -> (MMA, widen, promotion)
+  uint64_t* empty = bars + S;               // [S]    MMA commit + 4 widen + 4 promotion warps -> TMA
+  uint64_t* a_full = bars + 2 * S;          // [NA]   widen group -> MMA
+  uint64_t* a_empty = a_full + NA;          // [NA]   MMA commit -> widen group
+  uint64_t* acc_full = a_empty + NA;        // [NACC] MMA commit -> promotion
   uint64_t* acc_empty = acc_full + NACC;    // [NACC] promotion -> MMA
-  uint64_t* s_full = acc_empty + NACC;      // [kSRing] TMA -> promotion
-  uint64_t* s_empty = s_full + kSRing;      // [kSRing] promotion -> TMA
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bars + C::N_BARS);
   uint8_t* s_tags = reinterpret_cast<uint8_t*>(tmem_holder + 4);
   const uint32_t s_tags_a = smem_u32(s_tags);
-  const uint32_t sW_a = smem_u32(sW);
-  const uint32_t sS_a = smem_u32(sS);
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
   const bool debug = DEBUG != 0;
+  const bool tracing = (COMET_DIAG || COMET_TRACE) && P.trace != nullptr;
+  if (tracing && threadIdx.x == 0) P.trace[32768 + blockIdx.x * 4 + 0] = globaltimer_ns();
   const int it_begin = debug ? (int)blockIdx.x : P.cta_begin[blockIdx.x];
   const int it_end = debug ? (int)blockIdx.x + 1 : P.cta_begin[blockIdx.x + 1];
   const int nb = P.nb;
@@ -91,21 +134,18 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
   if (warp == 0 && lane == 0) {
     tma_prefetch(&P.map_x);
     tma_prefetch(&P.map_w);
+    tma_prefetch(&P.map_s);
     for (int i = 0; i < S; ++i) {
       mbar_init(&full[i], 1);
-      mbar_init(&empty[i], 1 + 4);
+      mbar_init(&empty[i], 1 + 4 + 4);
     }
-    for (int i = 0; i < 2; ++i) {
+    for (int i = 0; i < NA; ++i) {
       mbar_init(&a_full[i], 4);
       mbar_init(&a_empty[i], 1);
     }
     for (int i = 0; i < NACC; ++i) {
       mbar_init(&acc_full[i], 1);
-      mbar_init(&acc_empty[i], 4 * C::ACTIVE_WGS);
-    }
-    for (int i = 0; i < kSRing; ++i) {
-      mbar_init(&s_full[i], 1);
-      mbar_init(&s_empty[i], 4 * C::ACTIVE_WGS);
+      mbar_init(&acc_empty[i], 4);
     }
     fence_mbar_init();
   }
@@ -118,319 +158,314 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
   __syncthreads();
   tc_fence_after();
   const uint32_t tbase = *tmem_holder;
+  if (tracing && threadIdx.x == 0) P.trace[32768 + blockIdx.x * 4 + 1] = globaltimer_ns();
+  int tr = 0;   // trace index (per role)
 
-  if (warp < 4) {
+  if (warp < kWidenWarp0) {
     setmaxnreg_dec<40>();
     if (warp == 0 && lane == 0) {
       // ------------------------------------------------------------------ TMA producer
-      int stage = 0, ss = 0;
-      uint32_t ph = 0, sph = 0;
+      int stage = 0;
+      uint32_t ph = 0;
       for (int it = it_begin; it < it_end; ++it) {
         const WorkItem w = load_item(P, it, debug);
         const int n_tile = w.tile / P.n_m_tiles, m_tile = w.tile % P.n_m_tiles;
         const int m0 = m_tile * NT, n0 = n_tile * kTileW;
-        const int64_t srows = min((int64_t)NT, P.Mp - m0);
-        const uint32_t sbytes = (uint32_t)(srows * 4);
-        for (int kb = w.kb_begin; kb < w.kb_end; ++kb) {
+        for (int kb = w.kb_begin; kb < w.kb_end; kb += KS) {
+          const int npair = (min(KS, w.kb_end - kb) + 1) >> 1;
           mbar_wait(&empty[stage], ph ^ 1);
-          mbar_arrive_expect_tx(&full[stage], C::STAGE_BYTES);
-          tma_load_2d(sX + stage * C::X_BYTES, &P.map_x, &full[stage], kb * 128, m0);
-          tma_load_2d(sW + stage * C::W_BYTES, &P.map_w, &full[stage], kb * 64, n0);
-          mbar_wait(&s_empty[ss], sph ^ 1);
-          mbar_arrive_expect_tx(&s_full[ss], sbytes);
-          bulk_load(sS + ss * NT, P.scales + (int64_t)kb * P.Mp + m0, sbytes, &s_full[ss]);
+          mbar_arrive_expect_tx(&full[stage], npair * 2 * kTileW * 64 + KS * C::XKB_BYTES + C::S_BYTES);
+          for (int p = 0; p < npair; ++p)
+            tma_load_2d(sW(stage) + p * 2 * kTileW * 64, &P.map_w, &full[stage], (kb + 2 * p) * 64, n0);
+          tma_load_3d(sX(stage), &P.map_x, &full[stage], 0, m0, kb);
+          tma_load_2d(sS(stage), &P.map_s, &full[stage], m0, kb);
+          trace_ev(P, 0, tr++);
           if (++stage == S) { stage = 0; ph ^= 1; }
-          if (++ss == kSRing) { ss = 0; sph ^= 1; }
         }
       }
-    } else if (warp == 1 && lane == 0) {
-      // ------------------------------------------------------------------ MMA issuer
+    } else if ((warp == 1 || (C::ISSUERS == 2 && warp == 3)) && lane == 0) {
+      // ------------------------------------------------------------------ MMA issuer(s)
+      // With two issuers, warp 1 takes the even stages and warp 3 the odd ones; tcgen05.commit
+      // tracks the issuing thread's own MMAs, so each commits exactly the stages it issued.
+      const int par = warp == 1 ? 0 : 1;
       const uint32_t id_f8 = idesc_f8f6f4_e4m3(128, NT);
       const uint32_t id_i8 = idesc_i8(128, NT);
-      int stage = 0, ab = 0, accb = 0;
+      int stage = 0, ab = 0, accs = 0, seq = 0;
       uint32_t ph = 0, aph = 0, accph = 0;
       for (int it = it_begin; it < it_end; ++it) {
         const WorkItem w = load_item(P, it, debug);
-        for (int kb = w.kb_begin; kb < w.kb_end; ++kb) {
-          mbar_wait(&acc_empty[accb], accph ^ 1);
-          mbar_wait(&full[stage], ph);
-          mbar_wait(&a_full[ab], aph);
-          tc_fence_after();
-          const uint32_t d = tbase + kAccCol + accb * NT;
-          const uint32_t a = tbase + kAcol + ab * 32;
-          const uint32_t sx = smem_u32(sX + stage * C::X_BYTES);
-          if (lds_u8(s_tags_a + kb)) {
+        for (int kb = w.kb_begin; kb < w.kb_end; kb += KS, ++seq) {
+          if (C::ISSUERS == 1 || (seq & 1) == par) {
+            const int nk = min(KS, w.kb_end - kb);
+            mbar_wait(&full[stage], ph);
+            mbar_wait(&a_full[ab], aph);
+            mbar_wait(&acc_empty[accs], accph ^ 1);
+            if (par == 0) trace_ev(P, 1, tr++);
+            tc_fence_after();
+            const uint32_t d0 = tbase + C::ACC_COL + accs * C::ACC_SET;
+            const uint32_t a0 = tbase + ab * C::A_COLS;
+            const uint64_t b0 = sdesc_kmajor_sw128(smem_u32(sX(stage)));
+            for (int c = 0; c < nk; ++c) {
+              const uint32_t d = d0 + c * NT, a = a0 + c * 32;
+              const uint64_t bd = b0 + (uint64_t)((c * C::XKB_BYTES) >> 4);
+              if (COMET_DEC_ABLATE & 1) {
+              } else if (lds_u8(s_tags_a + kb + c)) {
 #pragma unroll
-            for (int k = 0; k < 4; ++k) mma_i8_ts(d, a + 8 * k, sdesc_kmajor_sw128(sx + 32 * k), id_i8, k);
-          } else {
+                for (int k = 0; k < 4; ++k) mma_i8_ts(d, a + 8 * k, bd + 2 * k, id_i8, k);
+              } else {
 #pragma unroll
-            for (int k = 0; k < 4; ++k) mma_f8_ts(d, a + 8 * k, sdesc_kmajor_sw128(sx + 32 * k), id_f8, k);
+                for (int k = 0; k < 4; ++k) mma_f8_ts(d, a + 8 * k, bd + 2 * k, id_f8, k);
+              }
+            }
+            tc_commit(&acc_full[accs]);
+            tc_commit(&empty[stage]);
+            tc_commit(&a_empty[ab]);
+            if (par == 0) trace_ev(P, 2, tr - 1);
           }
-          tc_commit(&empty[stage]);
-          tc_commit(&a_empty[ab]);
-          tc_commit(&acc_full[accb]);
           if (++stage == S) { stage = 0; ph ^= 1; }
-          if (++ab == 2) { ab = 0; aph ^= 1; }
-          if (++accb == NACC) { accb = 0; accph ^= 1; }
+          if (++ab == NA) { ab = 0; aph ^= 1; }
+          if (++accs == NACC) { accs = 0; accph ^= 1; }
         }
       }
     }
-  } else if (warp < 8) {
-    setmaxnreg_dec<80>();
+  } else if (warp < kPromoWarp0) {
+    setmaxnreg_dec<112>();
     // -------------------------------------------------------------------- widen (W -> TMEM A)
+    const int grp = (warp - kWidenWarp0) >> 2;    // this group takes stages with seq % 2 == grp
     const int q = warp & 3;
     const int r = q * 32 + lane;                  // TMEM lane = weight row within the tile
     const uint32_t lane_addr = (uint32_t)(q * 32) << 16;
-    const int sw = (r >> 1) & 3;                  // TMA 64-byte swizzle: chunk ^= row bits [1:2]
-    int stage = 0, ab = 0;
+    const int sw = r & 7;                         // TMA 128-byte swizzle: chunk ^= row bits [0:2]
+    int stage = 0, seq = 0;
     uint32_t ph = 0, aph = 0;
     for (int it = it_begin; it < it_end; ++it) {
       const WorkItem w = load_item(P, it, debug);
-      for (int kb = w.kb_begin; kb < w.kb_end; ++kb) {
-        const bool is8 = lds_u8(s_tags_a + kb) != 0;
-        mbar_wait(&full[stage], ph);
-        const uint32_t wt = sW_a + stage * C::W_BYTES + r * 64;
-        uint4 c[4];
-#pragma unroll
-        for (int j = 0; j < 4; ++j) c[j] = lds128(wt + ((j ^ sw) << 4));
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&empty[stage]);
-        uint32_t o[32];
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-          const uint32_t pw[4] = {c[j].x, c[j].y, c[j].z, c[j].w};
-#pragma unroll
-          for (int i = 0; i < 4; ++i) {
-            const uint32_t p = pw[i];
-            const int g = j * 4 + i;
-            if (is8) {
-              o[2 * g] = ((p << 4) & 0xF0F0F0F0u) ^ 0x80808080u;
-              o[2 * g + 1] = (p & 0xF0F0F0F0u) ^ 0x80808080u;
-            } else {
-              o[2 * g] = p & 0x0F0F0F0Fu;
-              o[2 * g + 1] = (p >> 4) & 0x0F0F0F0Fu;
-            }
-          }
-        }
-        mbar_wait(&a_empty[ab], aph ^ 1);
-        tc_fence_after();
-        tmem_st32(tbase + kAcol + ab * 32 + lane_addr, o);
-        tmem_wait_st();
-        tc_fence_before();
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&a_full[ab]);
-        if (++stage == S) { stage = 0; ph ^= 1; }
-        if (++ab == 2) { ab = 0; aph ^= 1; }
-      }
-    }
-  } else {
-    setmaxnreg_inc<192>();
-    // -------------------------------------------------------------------- promotion + epilogue
-    // TMEM accumulator: lane = weight row (n), column = token (m).  With the 16x256b load shape
-    // thread t of warp quarter q owns lanes 32q + 16h + t/4 + 8i (h, i in {0,1}) and columns
-    // col0 + 8j + 2(t%4) + e (j < NJ, e in {0,1}): only NJ*2 distinct tokens, so the block's
-    // per-token scales for this thread are NJ float2 loads issued before the accumulator wait.
-    const int pw = warp - 8;
-    const int wg = pw >> 2;
-    const int q = warp & 3;
-    const int t0 = lane & 3, t1 = lane >> 2;
-    const int col0 = wg * C::COLS;
-    constexpr int NJ = C::COLS / 8;                 // 8-column groups per WG
-    constexpr int NB1 = NJ > 8 ? 8 : NJ;            // repetitions in the first load batch
-    constexpr int NB2 = NJ - NB1;
-    constexpr int NE = 4 * NJ;                      // accumulator elements per thread (per h: 2*NJ*2)
-    const int n_promo_threads = 128 * C::ACTIVE_WGS;
-    const int ptid = threadIdx.x - 256;
-    if (wg < C::ACTIVE_WGS) {
-      int ss = 0, accb = 0;
-      uint32_t sph = 0, accph = 0;
-      for (int it = it_begin; it < it_end; ++it) {
-        const WorkItem w = load_item(P, it, debug);
-        const int n_tile = w.tile / P.n_m_tiles, m_tile = w.tile % P.n_m_tiles;
-        const int m0 = m_tile * NT, n0 = n_tile * kTileW;
-        const bool owner = (w.flags & 2) != 0;
-        const bool split = (w.flags & 1) != 0;
-        // acc index: ((h*2 + i)*NJ + j)*2 + e
-        float acc[2 * NE];
-        int32_t dacc[DEBUG ? 2 * NE : 1];
-#pragma unroll
-        for (int j = 0; j < NJ; ++j) {
-#pragma unroll
-          for (int e = 0; e < 2; ++e) {
-            const int64_t m = m0 + col0 + 8 * j + 2 * t0 + e;
-            const float c0 = (owner && m < P.Mp) ? -__ldg(P.corr + m) * 0.001953125f : 0.f;   // 2^-9
-#pragma unroll
-            for (int hi = 0; hi < 4; ++hi) {
-              acc[(hi * NJ + j) * 2 + e] = c0;
-              if (DEBUG) dacc[(hi * NJ + j) * 2 + e] = 0;
-            }
-          }
-        }
-        for (int kb = w.kb_begin; kb < w.kb_end; ++kb) {
-          const bool is8 = lds_u8(s_tags_a + kb) != 0;
-          mbar_wait(&s_full[ss], sph);
-          float2 sc[NJ];
-          {
-            const uint32_t sbase = sS_a + (ss * NT + col0 + 2 * t0) * 4;
-#pragma unroll
-            for (int j = 0; j < NJ; ++j) {
-              const uint2 u = lds64(sbase + j * 32);
-              sc[j] = make_float2(__uint_as_float(u.x), __uint_as_float(u.y));
-            }
-          }
-          mbar_wait(&acc_full[accb], accph);
+      for (int kb = w.kb_begin; kb < w.kb_end; kb += KS, ++seq) {
+        if ((seq & 1) == grp) {
+          const int nk = min(KS, w.kb_end - kb);
+          mbar_wait(&full[stage], ph);
+          if (lane == 0 && q == 0) trace_ev(P, 3 + grp, seq);
+          mbar_wait(&a_empty[grp], aph ^ 1);
           tc_fence_after();
-          const uint32_t tcol = tbase + kAccCol + accb * NT + col0;
+          const uint32_t wbase = smem_u32(sW(stage)) + r * 128;
 #pragma unroll
-          for (int h = 0; h < 2; ++h) {
-            const uint32_t taddr = tcol + ((uint32_t)(32 * q + 16 * h) << 16);
+          for (int p = 0; p < KS / 2; ++p) {
+            if (2 * p < nk) {
+              uint4 c[8];
 #pragma unroll
-            for (int part = 0; part < 2; ++part) {
-              constexpr int dummy = 0;
-              (void)dummy;
-              const int jb = part == 0 ? 0 : NB1;
-              const int nrep = part == 0 ? NB1 : NB2;
-              if (nrep == 0) continue;
-              uint32_t v[4 * 8];
-              if (part == 0) tmem_ld_16x256b<NB1>(taddr, v);
-              else if constexpr (NB2 > 0) tmem_ld_16x256b<(NB2 > 0 ? NB2 : 2)>(taddr + NB1 * 8, v);
-              tmem_wait_ld();
-              if (!is8) {
+              for (int j = 0; j < 8; ++j) c[j] = lds128(wbase + p * 2 * kTileW * 64 + ((j ^ sw) << 4));
 #pragma unroll
-                for (int jj = 0; jj < 8; ++jj) {
-                  if (jj < nrep) {
-                    const int j = jb + jj;
+              for (int h = 0; h < 2; ++h) {
+                if (2 * p + h < nk) {
+                  const bool is8 = lds_u8(s_tags_a + kb + 2 * p + h) != 0;
+                  uint32_t o[32];
 #pragma unroll
-                    for (int i = 0; i < 2; ++i) {
-                      const int a = ((h * 2 + i) * NJ + j) * 2;
-                      float2 y = ffma2(make_float2(__uint_as_float(v[4 * jj + 2 * i]), __uint_as_float(v[4 * jj + 2 * i + 1])),
-                                       sc[j], make_float2(acc[a], acc[a + 1]));
-                      acc[a] = y.x;
-                      acc[a + 1] = y.y;
-                    }
-                  }
-                }
-              } else {
+                  for (int j = 0; j < 4; ++j) {
+                    const uint32_t pw[4] = {c[4 * h + j].x, c[4 * h + j].y, c[4 * h + j].z, c[4 * h + j].w};
 #pragma unroll
-                for (int jj = 0; jj < 8; ++jj) {
-                  if (jj < nrep) {
-                    const int j = jb + jj;
-                    const float2 s8 = make_float2(sc[j].x * 1.220703125e-04f, sc[j].y * 1.220703125e-04f);  // 2^-13
-#pragma unroll
-                    for (int i = 0; i < 2; ++i) {
-                      const int a = ((h * 2 + i) * NJ + j) * 2;
-                      float2 y = ffma2(make_float2(__int2float_rn((int)v[4 * jj + 2 * i]), __int2float_rn((int)v[4 * jj + 2 * i + 1])),
-                                       s8, make_float2(acc[a], acc[a + 1]));
-                      acc[a] = y.x;
-                      acc[a + 1] = y.y;
-                    }
-                  }
-                }
-              }
-              if (DEBUG) {
-#pragma unroll
-                for (int jj = 0; jj < 8; ++jj) {
-                  if (jj < nrep) {
-                    const int j = jb + jj;
-#pragma unroll
-                    for (int i = 0; i < 2; ++i) {
-#pragma unroll
-                      for (int e = 0; e < 2; ++e) {
-                        const int64_t m = m0 + col0 + 8 * j + 2 * t0 + e;
-                        const int n = n0 + 32 * q + 16 * h + t1 + 8 * i;
-                        const uint32_t raw = v[4 * jj + 2 * i + e];
-                        int32_t ab;
-                        if (is8) {
-                          ab = ((int32_t)raw) >> 4;
-                        } else {
-                          const int qs = (m < P.Mp) ? (int)P.qsum[(int64_t)kb * P.Mp + m] : 0;
-                          ab = (int32_t)(__uint_as_float(raw) * 512.f) - 8 * qs;
-                        }
-                        dacc[((h * 2 + i) * NJ + j) * 2 + e] += ab;
-                        if (DEBUG == 2 && m < P.M) P.dbg_blocks[((int64_t)kb * P.M + m) * P.N + n] = ab;
+                    for (int i = 0; i < 4; ++i) {
+                      const uint32_t pv = pw[i];
+                      const int g = 2 * (j * 4 + i);
+                      if (is8) {
+                        o[g] = ((pv << 4) & 0xF0F0F0F0u) ^ 0x80808080u;
+                        o[g + 1] = (pv & 0xF0F0F0F0u) ^ 0x80808080u;
+                      } else {
+                        o[g] = pv & 0x0F0F0F0Fu;
+                        o[g + 1] = (pv >> 4) & 0x0F0F0F0Fu;
                       }
                     }
                   }
+                  if (!(COMET_DEC_ABLATE & 2)) tmem_st32(tbase + grp * C::A_COLS + (2 * p + h) * 32 + lane_addr, o);
                 }
               }
             }
           }
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&empty[stage]);
+          if (!(COMET_DEC_ABLATE & 2)) tmem_wait_st();
           tc_fence_before();
           __syncwarp();
-          if (lane == 0) {
-            mbar_arrive(&acc_empty[accb]);
-            mbar_arrive(&s_empty[ss]);
-          }
-          if (++ss == kSRing) { ss = 0; sph ^= 1; }
-          if (++accb == NACC) { accb = 0; accph ^= 1; }
+          if (lane == 0) mbar_arrive(&a_full[grp]);
+          if (lane == 0 && q == 0) trace_ev(P, 5 + grp, seq);
+#if COMET_HANG_PRINT
+          if (blockIdx.x == 0 && lane == 0) printf("widen warp %d seq %d done\n", warp, seq);
+#endif
+          aph ^= 1;
         }
-        // ---------------------------------------------------------------- epilogue
-        if (split) {
-          const int seg = (w.flags >> 8) & 0xFF;
-          const int nseg = (w.flags >> 16) & 0xFF;
-          const int64_t part_tile = (int64_t)NT * kTileW;    // = n_promo_threads * 2*NE floats
-          if (!owner) {
-            float4* dst = reinterpret_cast<float4*>(
-                P.ws_part + ((int64_t)w.fix * (P.max_seg - 1) + (seg - 1)) * part_tile + (int64_t)ptid * 2 * NE);
+        if (++stage == S) { stage = 0; ph ^= 1; }
+      }
+    }
+  } else {
+    setmaxnreg_inc<208>();
+#if COMET_HANG_PRINT
+    if (blockIdx.x == 0 && (threadIdx.x & 31) == 0) printf("promo warp %d started\n", warp);
+#endif
+    // -------------------------------------------------------------------- promotion + epilogue
+    // TMEM accumulator: lane = weight row (n), column = token (m); 32x32b loads give thread t of
+    // warp quarter q the row 32q + t and every token column of the tile.
+    constexpr int CH = C::CH;
+    const int q = warp & 3;
+    const int row = q * 32 + lane;
+    const uint32_t lane_addr = (uint32_t)(q * 32) << 16;
+    const int ptid = threadIdx.x - kPromoWarp0 * 32;
+    int stage = 0, accs = 0;
+    uint32_t ph = 0, accph = 0;
+    for (int it = it_begin; it < it_end; ++it) {
+      const WorkItem w = load_item(P, it, debug);
+      const int n_tile = w.tile / P.n_m_tiles, m_tile = w.tile % P.n_m_tiles;
+      const int m0 = m_tile * NT, n0 = n_tile * kTileW;
+      const bool owner = (w.flags & 2) != 0;
+      const bool split = (w.flags & 1) != 0;
+      const int n = n0 + row;
+      float acc[NT];
+      int32_t dacc[DEBUG ? NT : 1];
 #pragma unroll
-            for (int a = 0; a < 2 * NE; a += 4) dst[a / 4] = make_float4(acc[a], acc[a + 1], acc[a + 2], acc[a + 3]);
-            __threadfence();
-            named_bar_sync(1, n_promo_threads);
-            if (threadIdx.x == 256) st_release_gpu(P.ws_flags + (int64_t)w.fix * P.max_seg + seg, P.epoch);
-            continue;
-          }
-          if (threadIdx.x == 256) {
-            for (int sgi = 1; sgi < nseg; ++sgi) {
-              const uint32_t* f = P.ws_flags + (int64_t)w.fix * P.max_seg + sgi;
-              uint64_t t0g = globaltimer_ns();
-              while (ld_acquire_gpu(f) != P.epoch) {
-                if (globaltimer_ns() - t0g > COMET_MBAR_TIMEOUT_NS) {
-                  __trap();
+      for (int j = 0; j < NT; ++j) {
+        const int64_t m = m0 + j;
+        acc[j] = (owner && m < P.Mp) ? -__ldg(P.corr + m) * 0.001953125f : 0.f;   // 2^-9
+        if (DEBUG) dacc[j] = 0;
+      }
+      for (int kb0 = w.kb_begin; kb0 < w.kb_end; kb0 += KS) {
+        const int nk = min(KS, w.kb_end - kb0);
+        mbar_wait(&full[stage], ph);
+        mbar_wait(&acc_full[accs], accph);
+        if (ptid == 0) trace_ev(P, 7, tr);
+        tc_fence_after();
+        const uint32_t sbase = smem_u32(sS(stage));
+        for (int c = 0; c < nk; ++c) {
+          const int kb = kb0 + c;
+          const bool is8 = lds_u8(s_tags_a + kb) != 0;
+          const uint32_t tcol = tbase + C::ACC_COL + accs * C::ACC_SET + c * NT + lane_addr;
+#pragma unroll
+          for (int ch = 0; ch < NT / CH; ++ch) {
+            uint32_t v[CH];
+            if (COMET_DEC_ABLATE & 4) {
+#pragma unroll
+              for (int z = 0; z < CH; ++z) v[z] = 0;
+            } else {
+              tmem_ld_cols<CH>(tcol + ch * CH, v);
+            }
+            float sc[CH];
+#pragma unroll
+            for (int j = 0; j < CH; j += 4) {
+              const float4 f = lds128f(sbase + (c * NT + ch * CH + j) * 4);
+              sc[j] = f.x; sc[j + 1] = f.y; sc[j + 2] = f.z; sc[j + 3] = f.w;
+            }
+            tmem_wait_ld();
+            if (!is8) {
+#pragma unroll
+              for (int j = 0; j < CH; j += 2) {
+                const int a = ch * CH + j;
+                const float2 y = ffma2(make_float2(__uint_as_float(v[j]), __uint_as_float(v[j + 1])),
+                                       make_float2(sc[j], sc[j + 1]), make_float2(acc[a], acc[a + 1]));
+                acc[a] = y.x;
+                acc[a + 1] = y.y;
+              }
+            } else {
+#pragma unroll
+              for (int j = 0; j < CH; j += 2) {
+                const int a = ch * CH + j;
+                const float2 s8 = make_float2(sc[j] * 1.220703125e-04f, sc[j + 1] * 1.220703125e-04f);  // 2^-13
+                const float2 y = ffma2(make_float2(__int2float_rn((int)v[j]), __int2float_rn((int)v[j + 1])),
+                                       s8, make_float2(acc[a], acc[a + 1]));
+                acc[a] = y.x;
+                acc[a + 1] = y.y;
+              }
+            }
+            if (DEBUG) {
+#pragma unroll
+              for (int j = 0; j < CH; ++j) {
+                const int64_t m = m0 + ch * CH + j;
+                int32_t ab;
+                if (is8) {
+                  ab = ((int32_t)v[j]) >> 4;
+                } else {
+                  const int qs = (m < P.Mp) ? (int)P.qsum[(int64_t)kb * P.Mp + m] : 0;
+                  ab = (int32_t)(__uint_as_float(v[j]) * 512.f) - 8 * qs;
                 }
+                dacc[ch * CH + j] += ab;
+                if (DEBUG == 2 && m < P.M && n < P.N) P.dbg_blocks[((int64_t)kb * P.M + m) * P.N + n] = ab;
               }
-            }
-          }
-          named_bar_sync(1, n_promo_threads);
-          for (int sgi = 1; sgi < nseg; ++sgi) {
-            const float4* src = reinterpret_cast<const float4*>(
-                P.ws_part + ((int64_t)w.fix * (P.max_seg - 1) + (sgi - 1)) * part_tile + (int64_t)ptid * 2 * NE);
-#pragma unroll
-            for (int a = 0; a < 2 * NE; a += 4) {
-              float4 t4;
-              asm volatile("ld.global.cg.v4.f32 {%0,%1,%2,%3}, [%4];"
-                           : "=f"(t4.x), "=f"(t4.y), "=f"(t4.z), "=f"(t4.w) : "l"(src + a / 4));
-              acc[a] += t4.x; acc[a + 1] += t4.y; acc[a + 2] += t4.z; acc[a + 3] += t4.w;
             }
           }
         }
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) {
+          mbar_arrive(&acc_empty[accs]);
+          mbar_arrive(&empty[stage]);
+        }
+        if (ptid == 0) trace_ev(P, 8, tr++);
+#if COMET_HANG_PRINT
+        if (blockIdx.x == 0 && lane == 0) printf("promo warp %d kb0 %d done\n", warp, kb0);
+#endif
+        if (++stage == S) { stage = 0; ph ^= 1; }
+        if (++accs == NACC) { accs = 0; accph ^= 1; }
+      }
+      // ---------------------------------------------------------------- epilogue
+      if (ptid == 0) trace_ev(P, 10, it - it_begin);
+      if (split) {
+        const int seg = (w.flags >> 8) & 0xFF;
+        const int nseg = (w.flags >> 16) & 0xFF;
+        const int64_t part_tile = (int64_t)NT * kTileW;
+        if (!owner) {
+          float4* dst = reinterpret_cast<float4*>(
+              P.ws_part + ((int64_t)w.fix * (P.max_seg - 1) + (seg - 1)) * part_tile);
 #pragma unroll
-        for (int hi = 0; hi < 4; ++hi) {
-          const int h = hi >> 1, i = hi & 1;
-          const int n = n0 + 32 * q + 16 * h + t1 + 8 * i;
-          const float swv = __ldg(P.w_scales + n) * 512.f;
-#pragma unroll
-          for (int j = 0; j < NJ; ++j) {
-#pragma unroll
-            for (int e = 0; e < 2; ++e) {
-              const int64_t m = m0 + col0 + 8 * j + 2 * t0 + e;
-              if (m < P.M) {
-                const int a = (hi * NJ + j) * 2 + e;
-                const float yv = acc[a] * swv;
-                const int64_t off = m * P.ldy + n;
-                if (P.ydt == COMET_F16) reinterpret_cast<__half*>(P.y)[off] = __float2half_rn(yv);
-                else if (P.ydt == COMET_BF16) reinterpret_cast<__nv_bfloat16*>(P.y)[off] = __float2bfloat16_rn(yv);
-                else reinterpret_cast<float*>(P.y)[off] = yv;
-                if (DEBUG) P.dbg_acc[m * P.N + n] = dacc[a];
+          for (int j = 0; j < NT; j += 4) dst[(j / 4) * 128 + ptid] = make_float4(acc[j], acc[j + 1], acc[j + 2], acc[j + 3]);
+          __threadfence();
+          named_bar_sync(1, 128);
+          if (ptid == 0) st_release_gpu(P.ws_flags + (int64_t)w.fix * P.max_seg + seg, P.epoch);
+          if (ptid == 0) trace_ev(P, 12, it - it_begin);
+          continue;
+        }
+        if (ptid == 0) {
+          for (int sgi = 1; sgi < nseg; ++sgi) {
+            const uint32_t* f = P.ws_flags + (int64_t)w.fix * P.max_seg + sgi;
+            uint64_t t0g = globaltimer_ns();
+            while (ld_acquire_gpu(f) != P.epoch) {
+              if (globaltimer_ns() - t0g > COMET_MBAR_TIMEOUT_NS) {
+                __trap();
               }
             }
+          }
+        }
+        named_bar_sync(1, 128);
+        if (ptid == 0) trace_ev(P, 11, it - it_begin);
+        for (int sgi = 1; sgi < nseg; ++sgi) {
+          const float4* src = reinterpret_cast<const float4*>(
+              P.ws_part + ((int64_t)w.fix * (P.max_seg - 1) + (sgi - 1)) * part_tile);
+#pragma unroll
+          for (int j = 0; j < NT; j += 4) {
+            float4 t4;
+            asm volatile("ld.global.cg.v4.f32 {%0,%1,%2,%3}, [%4];"
+                         : "=f"(t4.x), "=f"(t4.y), "=f"(t4.z), "=f"(t4.w) : "l"(src + (j / 4) * 128 + ptid));
+            acc[j] += t4.x; acc[j + 1] += t4.y; acc[j + 2] += t4.z; acc[j + 3] += t4.w;
           }
         }
       }
+      if (n < P.N) {
+        const float swv = __ldg(P.w_scales + n) * 512.f;
+#pragma unroll
+        for (int j = 0; j < NT; ++j) {
+          const int64_t m = m0 + j;
+          if (m < P.M) {
+            const float yv = acc[j] * swv;
+            const int64_t off = m * P.ldy + n;
+            if (P.ydt == COMET_F16) reinterpret_cast<__half*>(P.y)[off] = __float2half_rn(yv);
+            else if (P.ydt == COMET_BF16) reinterpret_cast<__nv_bfloat16*>(P.y)[off] = __float2bfloat16_rn(yv);
+            else reinterpret_cast<float*>(P.y)[off] = yv;
+            if (DEBUG) P.dbg_acc[m * P.N + n] = dacc[j];
+          }
+        }
+      }
+      if (ptid == 0) trace_ev(P, 12, it - it_begin);
     }
   }
 
   tc_fence_before();
   __syncthreads();
+  if (tracing && threadIdx.x == 0) P.trace[32768 + blockIdx.x * 4 + 2] = globaltimer_ns();
   if (warp == 2) tmem_dealloc<512>(tbase);
 }
 
@@ -462,6 +497,21 @@ PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
 }  // namespace
 
 // ------------------------------------------------------------------------------ host side
+bool make_map(CUtensorMap* map, CUtensorMapDataType dt, int rank, const void* base,
+              const uint64_t* dims, const uint64_t* stride_bytes, const uint32_t* box,
+              CUtensorMapSwizzle swz) {
+  auto fn = encode_fn();
+  if (!fn) return false;
+  cuuint64_t d[5], st[4];
+  cuuint32_t bx[5], es[5];
+  for (int i = 0; i < rank; ++i) { d[i] = dims[i]; bx[i] = box[i]; es[i] = 1; }
+  for (int i = 0; i + 1 < rank; ++i) st[i] = stride_bytes[i];
+  CUresult r = fn(map, dt, (cuuint32_t)rank, const_cast<void*>(base), d, st, bx, es,
+                  CU_TENSOR_MAP_INTERLEAVE_NONE, swz, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                  CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS;
+}
+
 bool make_map_2d(CUtensorMap* map, const void* base, uint64_t inner, uint64_t outer,
                  uint64_t row_bytes, uint32_t box_inner, uint32_t box_outer,
                  CUtensorMapSwizzle swz) {
@@ -495,18 +545,39 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
   // token-tile and weight-tile of one CTA (= box rows of the two TMA maps) and of the tile
   int tile_m, tile_w, cta_rows_w;
   if (normal) { tile_m = 128 * cg; tile_w = dbg ? 96 : p.tile_w; cta_rows_w = tile_w / cg; }
-  else { tile_m = dbg ? 64 : p.tile_n; tile_w = kTileW; cta_rows_w = kTileW; }
+  else { tile_m = dbg ? 32 : p.tile_n; tile_w = kTileW; cta_rows_w = kTileW; }
   const int box_m = normal ? 128 : tile_m;
   comet_act_layout_t L;
   act_layout(p.M, p.K, &L);
   const uint8_t* base = static_cast<const uint8_t*>(act_packed);
   GemmParams prm;
   memset(&prm, 0, sizeof(prm));
-  if (!make_map_2d(&prm.map_x, base + L.codes_off, (uint64_t)p.K, (uint64_t)p.M, (uint64_t)p.K, 128,
-                   (uint32_t)box_m, CU_TENSOR_MAP_SWIZZLE_128B))
-    return fail(COMET_ERR_CUDA, "cuTensorMapEncodeTiled failed for the activation codes");
-  if (!make_map_2d(&prm.map_w, w_packed, (uint64_t)(p.K / 2), (uint64_t)p.N, (uint64_t)(p.K / 2), 64,
-                   (uint32_t)cta_rows_w, CU_TENSOR_MAP_SWIZZLE_64B))
+  if (normal) {
+    if (!make_map_2d(&prm.map_x, base + L.codes_off, (uint64_t)p.K, (uint64_t)p.M, (uint64_t)p.K, 128,
+                     (uint32_t)box_m, CU_TENSOR_MAP_SWIZZLE_128B))
+      return fail(COMET_ERR_CUDA, "cuTensorMapEncodeTiled failed for the activation codes");
+  } else {
+    // decode: codes as [nb][M][128 B] (dims innermost first: byte in block, token, block) so
+    // one box brings a stage's KS K-blocks as KS UMMA-ready [NT][128 B] SW128 tiles; scales
+    // [nb][Mp] f32, one box of KS x NT per stage.
+    const uint32_t ks = tile_m <= 32 ? 4 : 2;
+    const uint64_t xd[3] = {128, (uint64_t)p.M, (uint64_t)p.nb};
+    const uint64_t xs[2] = {(uint64_t)p.K, 128};
+    const uint32_t xb[3] = {128, (uint32_t)tile_m, ks};
+    if (!make_map(&prm.map_x, CU_TENSOR_MAP_DATA_TYPE_UINT8, 3, base + L.codes_off, xd, xs, xb,
+                  CU_TENSOR_MAP_SWIZZLE_128B))
+      return fail(COMET_ERR_CUDA, "cuTensorMapEncodeTiled failed for the activation codes (3D)");
+    const uint64_t sd[2] = {(uint64_t)L.Mp, (uint64_t)p.nb};
+    const uint64_t ss[1] = {(uint64_t)L.Mp * 4};
+    const uint32_t sb[2] = {(uint32_t)tile_m, ks};
+    if (!make_map(&prm.map_s, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, act_scales, sd, ss, sb,
+                  CU_TENSOR_MAP_SWIZZLE_NONE))
+      return fail(COMET_ERR_CUDA, "cuTensorMapEncodeTiled failed for the activation scales");
+  }
+  // prefill: 64-byte rows (one K-block) with 64B swizzle; decode: 128-byte rows (two K-blocks)
+  if (!make_map_2d(&prm.map_w, w_packed, (uint64_t)(p.K / 2), (uint64_t)p.N, (uint64_t)(p.K / 2),
+                   normal ? 64 : 128, (uint32_t)cta_rows_w,
+                   normal ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B))
     return fail(COMET_ERR_CUDA, "cuTensorMapEncodeTiled failed for the packed weights");
   if (normal && !dbg) {
     const int esz = ydt == COMET_F32 ? 4 : 2;
@@ -556,15 +627,13 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
   if (normal) {
     e = launch_gemm_n(prm, grid, tile_w, cg, debug, stream);
   } else if (dbg) {
-    e = debug == 2 ? launch_nt<64, 2>(prm, grid, stream) : launch_nt<64, 1>(prm, grid, stream);
+    e = debug == 2 ? launch_nt<32, 2>(prm, grid, stream) : launch_nt<32, 1>(prm, grid, stream);
   } else {
     switch (tile_m) {
       case 16: e = launch_nt<16, 0>(prm, grid, stream); break;
       case 32: e = launch_nt<32, 0>(prm, grid, stream); break;
       case 64: e = launch_nt<64, 0>(prm, grid, stream); break;
       case 128: e = launch_nt<128, 0>(prm, grid, stream); break;
-      case 192: e = launch_nt<192, 0>(prm, grid, stream); break;
-      case 224: e = launch_nt<224, 0>(prm, grid, stream); break;
       default: return fail(COMET_ERR_UNSUPPORTED_SHAPE, "unsupported tile_n");
     }
   }

@@ -13,12 +13,12 @@ namespace gemm {
 using namespace sm100;
 
 constexpr int kThreads = 512;
-constexpr int kSRing = 8;            // scale ring depth
 
 struct __align__(64) GemmParams {
   CUtensorMap map_x;
   CUtensorMap map_w;
   CUtensorMap map_y;         // prefill kernel: Y as bytes [M][N*esz], box 64 B x 128 rows, 64B swizzle
+  CUtensorMap map_s;         // decode kernel: act_scales [nb][Mp] f32, box NT x KS
   const float* scales;       // [nb][Mp]
   const float* corr;         // [Mp]
   const int16_t* qsum;       // [nb][Mp]
@@ -98,9 +98,13 @@ __device__ __forceinline__ void trace_ev(const GemmParams& P, int e, int i) {
   }
 }
 
-// Host: TMA descriptor helper (gemm.cu).
+// Host: TMA descriptor helpers (gemm.cu).
 bool make_map_2d(CUtensorMap* map, const void* base, uint64_t inner, uint64_t outer,
                  uint64_t row_bytes, uint32_t box_inner, uint32_t box_outer, CUtensorMapSwizzle swz);
+// General tiled map: `rank` dims (innermost first), byte strides of dims 1.. , box sizes.
+bool make_map(CUtensorMap* map, CUtensorMapDataType dt, int rank, const void* base,
+              const uint64_t* dims, const uint64_t* stride_bytes, const uint32_t* box,
+              CUtensorMapSwizzle swz);
 
 extern unsigned long long* g_trace;   // diagnostic timeline buffer (comet_debug_set_trace)
 

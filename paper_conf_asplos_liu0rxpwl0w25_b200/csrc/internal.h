@@ -39,6 +39,7 @@ struct Plan {
   int tile_n, num_ctas, split_mode, stages;
   int orientation = 1;   // 1: weights on MMA M (gemm.cu), 2: tokens on MMA M (gemm_n.cu)
   int tile_w = 128;      // weights per output tile
+  int kgran = 1;         // K-blocks per scheduling unit (4 for the decode kernel's stream-K)
   int64_t n_m_tiles, n_n_tiles, n_tiles;
   std::vector<uint8_t> tags;
   TagMask mask;

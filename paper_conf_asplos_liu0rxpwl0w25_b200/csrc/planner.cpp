@@ -31,19 +31,11 @@ static int auto_tile_n(int64_t M) {
   if (M <= 16) return 16;
   if (M <= 32) return 32;
   if (M <= 64) return 64;
-  if (M <= 128) return 128;
-  static const int cands[] = {224, 192, 128};   // minimise padded tokens; prefer larger tiles
-  int best = 224;
-  int64_t best_pad = INT64_MAX;
-  for (int nt : cands) {
-    const int64_t pad = ceil_div(M, nt) * nt;
-    if (pad < best_pad) { best_pad = pad; best = nt; }
-  }
-  return best;
+  return 128;
 }
 
 static bool valid_tile_n(int nt) {
-  return nt == 16 || nt == 32 || nt == 64 || nt == 128 || nt == 192 || nt == 224;
+  return nt == 16 || nt == 32 || nt == 64 || nt == 128;
 }
 
 // Smallest max-part cost when cutting `cost` (a sequence) into at most P contiguous parts;
@@ -93,7 +85,7 @@ comet_status_t build_plan(Plan& p, const comet_sched_config& cfg) {
     p.tile_n = cfg.tile_n > 0 ? cfg.tile_n : auto_tile_n(p.M);
     p.tile_w = kTileW;
     if (!valid_tile_n(p.tile_n))
-      return fail(COMET_ERR_UNSUPPORTED_SHAPE, "tile_n must be one of 16, 32, 64, 128, 192, 224");
+      return fail(COMET_ERR_UNSUPPORTED_SHAPE, "tile_n must be one of 16, 32, 64, 128");
   }
   // scheduling units: CTAs, or CTA pairs for the pair kernel
   p.num_ctas = p.orientation == 3 ? cfg.num_sms / 2 : cfg.num_sms;
@@ -103,12 +95,9 @@ comet_status_t build_plan(Plan& p, const comet_sched_config& cfg) {
   p.n_tiles = p.n_m_tiles * p.n_n_tiles;
   const int P = p.num_ctas;
   const int64_t T = p.n_tiles;
-  const int nb = (int)p.nb;
+  const int nkb = (int)p.nb;
   const double c4 = cfg.cost_int4 > 0 ? cfg.cost_int4 : 1.0;
   const double c8 = cfg.cost_int8 > 0 ? cfg.cost_int8 : 1.0;
-  std::vector<double> ucost(nb);
-  for (int b = 0; b < nb; ++b) ucost[b] = p.tags[b] ? c8 : c4;
-  const double tile_cost = std::accumulate(ucost.begin(), ucost.end(), 0.0);
 
   int mode = cfg.split_mode;
   if (mode < 0) {
@@ -117,6 +106,16 @@ comet_status_t build_plan(Plan& p, const comet_sched_config& cfg) {
   }
   if (mode < 0 || mode > 3) return fail(COMET_ERR_INVALID_ARG, "split_mode must be -1..3");
   p.split_mode = mode;
+  // Scheduling granularity: the decode kernel streams 4 K-blocks per pipeline stage at
+  // tile_n <= 32, so its stream-K / whole-tile cuts fall on 4-K-block boundaries (a cut
+  // elsewhere would load weights another CTA also loads).  The paper's unit-level modes 2/3
+  // (Fig. 8) keep single K-blocks.
+  const int kgran = (p.orientation == 1 && p.tile_n <= 32 && (mode == 0 || mode == 1)) ? 4 : 1;
+  p.kgran = kgran;
+  const int nb = (int)ceil_div(nkb, kgran);          // scheduling units per tile
+  std::vector<double> ucost(nb, 0.0);
+  for (int b = 0; b < nkb; ++b) ucost[b / kgran] += p.tags[b] ? c8 : c4;
+  const double tile_cost = std::accumulate(ucost.begin(), ucost.end(), 0.0);
 
   // ---- assignment: for every CTA an ordered list of (tile, kb) runs
   struct Run { int64_t tile; int kb0, kb1; };
@@ -208,7 +207,7 @@ comet_status_t build_plan(Plan& p, const comet_sched_config& cfg) {
     for (int s = 0; s < nseg; ++s) {
       const Run& r = runs[segs[s].cta][segs[s].idx];
       WorkItem w{};
-      w.tile = (int32_t)tile; w.kb_begin = r.kb0; w.kb_end = r.kb1;
+      w.tile = (int32_t)tile; w.kb_begin = r.kb0 * kgran; w.kb_end = std::min(r.kb1 * kgran, nkb);
       w.flags = (split ? 1 : 0) | (s == 0 ? 2 : 0) | (s << 8) | (nseg << 16);
       w.fix = split ? fix : -1;
       per[segs[s].cta][segs[s].idx] = w;

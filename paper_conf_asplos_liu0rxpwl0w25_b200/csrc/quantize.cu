@@ -8,9 +8,9 @@
 // Layout written (include/comet.h): codes[M][K] bytes (E4M3 of q for INT4 blocks, s8 for INT8
 // blocks), scales[nb][Mp], qsum[nb][Mp] (int16), corr[Mp].
 //
-// HBM-bound: a block-row (128 halves = 256 B) is read by 16 lanes with one 128-bit load each;
-// block max-abs and code sum are 4-step xor-shuffle reductions inside the half-warp; codes
-// leave as one 64-bit store per lane.  A warp handles two blocks per step (one per half).
+// HBM-bound: a block-row (128 halves = 256 B) is read by 4 lanes with four 128-bit loads each
+// (a warp step covers 8 blocks, sector-coalesced); block max-abs and code sum are 2-step
+// xor-shuffle reductions inside the lane quad; codes leave as four 64-bit stores per lane.
 #include <cuda_fp16.h>
 #include <cuda_bf16.h>
 #include "internal.h"
@@ -80,85 +80,94 @@ __device__ __forceinline__ uint32_t e4m3x2(float lo, float hi) {
 // binary32 pattern are the two's-complement integer rint(t) and RN(that - 1.5 * 2^23) is
 // rint(t) as a float, exactly.
 constexpr float kMagic = 12582912.0f;
-constexpr uint32_t kMagicBits = 0x4B400000u;
 
-struct BlockOut {
-  uint32_t lo, hi;   // 8 code bytes
-  float s;
-  int q;             // code sum (full after the reduction)
-};
-
-// Quantise the 8 values of this lane for block b (16 lanes cooperate on 128 values).
+// One lane's share of one block: 32 channels (four runs of 8 consecutive channels at
+// 32 j + 8 sub, j = 0..3) -- four lanes (sub = 0..3) cover the block's 128 channels.
 //   Fast path (every finite r = qmax/amax, and amax == 0): t = x * r as one binary32 product,
 //   q = rint(t) by the magic constant.  |x| <= amax gives |t| <= qmax (1 + 2^-24)^2, so
 //   rint(t) never exceeds qmax and the clamp of the definition is a no-op.
 //   Slow path (a binary32-subnormal amax, where qmax/amax overflows to inf, reading R5):
 //   the definition written out with a saturating conversion and the clamp.
-__device__ __forceinline__ BlockOut quantize8(const float (&v)[8], bool is8) {
+struct LaneOut {
+  uint2 c[4];        // 4 x 8 code bytes
+  float s;           // block scale (same in the 4 lanes)
+  int q;             // block code sum (same in the 4 lanes, after the reduction)
+};
+
+__device__ __forceinline__ LaneOut quantize32(const float (&v)[32], bool is8) {
   float a = 0.f;
 #pragma unroll
-  for (int j = 0; j < 8; ++j) a = fmaxf(a, fabsf(v[j]));
-  a = fmaxf(a, __shfl_xor_sync(0xffffffffu, a, 8));
-  a = fmaxf(a, __shfl_xor_sync(0xffffffffu, a, 4));
-  a = fmaxf(a, __shfl_xor_sync(0xffffffffu, a, 2));
+  for (int j = 0; j < 32; ++j) a = fmaxf(a, fabsf(v[j]));
   a = fmaxf(a, __shfl_xor_sync(0xffffffffu, a, 1));
+  a = fmaxf(a, __shfl_xor_sync(0xffffffffu, a, 2));
   const float qmax = is8 ? 127.f : 7.f;
-  BlockOut o;
+  LaneOut o;
   o.s = (a == 0.f) ? 0.f : __fdiv_rn(a, qmax);
   const float r = __fdiv_rn(qmax, a);          // +inf for an all-zero block
-  int qs = 0;
-  if (a == 0.f || r <= 3.0e38f) {              // uniform per half-warp
+  float qsf = 0.f;
+  int qsi = 0;
+  if (a == 0.f || r <= 3.0e38f) {
     const float rr = a == 0.f ? 0.f : r;       // zero block: every code 0
-    float2 y[4];
-    uint32_t bsum = 0;
-#pragma unroll
-    for (int i = 0; i < 4; ++i) {
-      y[i] = fadd2_rn(fmul2_rn(make_float2(v[2 * i], v[2 * i + 1]), make_float2(rr, rr)),
-                      make_float2(kMagic, kMagic));
-      bsum += __float_as_uint(y[i].x) + __float_as_uint(y[i].y);
-    }
-    qs = (int)(bsum - 8u * kMagicBits);        // sum of the 8 codes (mod 2^32, exact)
+    float2 acc = make_float2(0.f, 0.f);
     if (is8) {
-      // two's-complement byte of rint(t) = low byte of the biased pattern
-      const uint32_t p01 = __byte_perm(__float_as_uint(y[0].x), __float_as_uint(y[0].y), 0x0040);
-      const uint32_t p23 = __byte_perm(__float_as_uint(y[1].x), __float_as_uint(y[1].y), 0x0040);
-      const uint32_t p45 = __byte_perm(__float_as_uint(y[2].x), __float_as_uint(y[2].y), 0x0040);
-      const uint32_t p67 = __byte_perm(__float_as_uint(y[3].x), __float_as_uint(y[3].y), 0x0040);
-      o.lo = __byte_perm(p01, p23, 0x5410);
-      o.hi = __byte_perm(p45, p67, 0x5410);
-    } else {
-      uint32_t e[4];
 #pragma unroll
-      for (int i = 0; i < 4; ++i) {
-        const float2 f = fadd2_rn(y[i], make_float2(-kMagic, -kMagic));   // rint(t), +0 for 0
-        e[i] = e4m3x2(f.x, f.y);
+      for (int j = 0; j < 4; ++j) {
+        uint32_t p[4];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const float2 y = fadd2_rn(fmul2_rn(make_float2(v[8 * j + 2 * i], v[8 * j + 2 * i + 1]), make_float2(rr, rr)),
+                                    make_float2(kMagic, kMagic));
+          acc = fadd2_rn(acc, fadd2_rn(y, make_float2(-kMagic, -kMagic)));
+          // two's-complement byte of rint(t) = low byte of the biased pattern
+          p[i] = __byte_perm(__float_as_uint(y.x), __float_as_uint(y.y), 0x0040);
+        }
+        o.c[j] = make_uint2(__byte_perm(p[0], p[1], 0x5410), __byte_perm(p[2], p[3], 0x5410));
       }
-      o.lo = e[0] | (e[1] << 16);
-      o.hi = e[2] | (e[3] << 16);
+    } else {
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        uint32_t e[4];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const float2 y = fadd2_rn(fmul2_rn(make_float2(v[8 * j + 2 * i], v[8 * j + 2 * i + 1]), make_float2(rr, rr)),
+                                    make_float2(kMagic, kMagic));
+          const float2 f = fadd2_rn(y, make_float2(-kMagic, -kMagic));   // rint(t), +0 for 0
+          acc = fadd2_rn(acc, f);
+          e[i] = e4m3x2(f.x, f.y);
+        }
+        o.c[j] = make_uint2(e[0] | (e[1] << 16), e[2] | (e[3] << 16));
+      }
     }
+    qsf = acc.x + acc.y;                       // integers < 2^13: exact
   } else {
     const int iq = is8 ? 127 : 7;
-    uint32_t bytes[8];
 #pragma unroll
-    for (int j = 0; j < 8; ++j) {
-      const float t = __fmul_rn(v[j], r);
-      int q = __float2int_rn(t);                // cvt.rni.s32.f32: half-even, NaN -> 0, saturating
-      q = min(max(q, -iq), iq);
-      qs += q;
-      bytes[j] = is8 ? ((uint32_t)q & 0xFFu) : e4m3_of_int4(q);
+    for (int j = 0; j < 4; ++j) {
+      uint32_t bytes[8];
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        const float t = __fmul_rn(v[8 * j + i], r);
+        int q = __float2int_rn(t);              // cvt.rni.s32.f32: half-even, NaN -> 0, saturating
+        q = min(max(q, -iq), iq);
+        qsi += q;
+        bytes[i] = is8 ? ((uint32_t)q & 0xFFu) : e4m3_of_int4(q);
+      }
+      o.c[j] = make_uint2(bytes[0] | (bytes[1] << 8) | (bytes[2] << 16) | (bytes[3] << 24),
+                          bytes[4] | (bytes[5] << 8) | (bytes[6] << 16) | (bytes[7] << 24));
     }
-    o.lo = bytes[0] | (bytes[1] << 8) | (bytes[2] << 16) | (bytes[3] << 24);
-    o.hi = bytes[4] | (bytes[5] << 8) | (bytes[6] << 16) | (bytes[7] << 24);
   }
-  qs += __shfl_xor_sync(0xffffffffu, qs, 8);
-  qs += __shfl_xor_sync(0xffffffffu, qs, 4);
-  qs += __shfl_xor_sync(0xffffffffu, qs, 2);
+  int qs = qsi + (int)qsf;
   qs += __shfl_xor_sync(0xffffffffu, qs, 1);
+  qs += __shfl_xor_sync(0xffffffffu, qs, 2);
   o.q = qs;
   return o;
 }
 
-// WPR warps cooperate on one token row; a CTA of 8 warps covers 8/WPR rows.
+// WPR warps cooperate on one token row; a CTA of 8 warps covers 8/WPR rows.  A warp step
+// covers a group of 8 consecutive blocks (1024 channels, 2 KB of input): lane l works on block
+// 8g + l/4 with sub = l%4, loading 4 x 16 B at channel offsets 32 j + 8 sub -- every load
+// instruction reads 64 contiguous bytes of each of the 8 blocks (whole 32-byte sectors) and
+// every code store writes 32 contiguous bytes per block.
 template <bool BF16, int WPR>
 __global__ void __launch_bounds__(256) k_quantize(const uint16_t* __restrict__ x, int64_t M,
                                                   int64_t K, int64_t ldx, int64_t Mp, TagMask tags,
@@ -167,58 +176,61 @@ __global__ void __launch_bounds__(256) k_quantize(const uint16_t* __restrict__ x
                                                   float* __restrict__ corr,
                                                   float* __restrict__ scales) {
   constexpr int ROWS = 8 / WPR;
-  __shared__ float s_part[8][2];
+  __shared__ float s_part[8];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int row_in_cta = warp / WPR, wi = warp % WPR;
   const int64_t m = (int64_t)blockIdx.x * ROWS + row_in_cta;
-  const int half = lane >> 4, sub = lane & 15;
+  const int bl = lane >> 2, sub = lane & 3;
   const int nb = (int)(K / kBlockK);
-  const int npairs = (nb + 1) / 2;
-  float cpart = 0.f;   // sum over this half's INT4 blocks of s * qsum (binary32)
-  if (m < Mp) {
-    const bool live = m < M;
-    const uint16_t* xrow = x + (live ? m : 0) * ldx;
-    uint8_t* crow = codes + (live ? m : 0) * K;
-    constexpr int U = 4;   // block pairs in flight per warp (64 B per lane)
-    for (int p0 = wi; p0 < npairs; p0 += WPR * U) {
-      uint4 raw[U];
+  const int ngroups = (nb + 7) >> 3;
+  float cpart = 0.f;   // sum over this lane's INT4 blocks of s * qsum (binary32, lanes sub == 0)
+  if (m < M) {
+    const uint16_t* xrow = x + m * ldx + sub * 8;
+    uint8_t* crow = codes + m * K + sub * 8;
+    for (int g = wi; g < ngroups; g += WPR) {
+      const int b = g * 8 + bl;
+      const bool bvalid = b < nb;
+      uint4 raw[4];
 #pragma unroll
-      for (int u = 0; u < U; ++u) {
-        const int b = (p0 + u * WPR) * 2 + half;
-        raw[u] = make_uint4(0, 0, 0, 0);
-        if (live && (p0 + u * WPR) < npairs && b < nb)
-          raw[u] = ldg_stream(xrow + (int64_t)b * kBlockK + sub * 8);
+      for (int j = 0; j < 4; ++j)
+        raw[j] = bvalid ? ldg_stream(xrow + b * kBlockK + 32 * j) : make_uint4(0, 0, 0, 0);
+      float v[32];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        float t[8];
+        unpack8<BF16>(raw[j], t);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) v[8 * j + i] = t[i];
       }
+      const bool is8 = bvalid && ((tags.w[b >> 5] >> (b & 31)) & 1u);
+      const LaneOut o = quantize32(v, is8);
+      if (bvalid) {
+        uint8_t* cb = crow + b * kBlockK;
 #pragma unroll
-      for (int u = 0; u < U; ++u) {
-        const int pp = p0 + u * WPR;
-        if (pp >= npairs) break;                 // warp-uniform
-        const int b = pp * 2 + half;
-        const bool bvalid = b < nb;
-        float v[8];
-        unpack8<BF16>(raw[u], v);
-        const bool is8 = bvalid ? tags.get(b) : false;
-        BlockOut o = quantize8(v, is8);
-        if (bvalid) {
-          if (live)
-            *reinterpret_cast<uint2*>(crow + (int64_t)b * kBlockK + sub * 8) = make_uint2(o.lo, o.hi);
-          if (sub == 0) {
-            scales[(int64_t)b * Mp + m] = o.s;
-            qsum[(int64_t)b * Mp + m] = (int16_t)o.q;
-            if (!is8) cpart = __fadd_rn(cpart, __fmul_rn(o.s, (float)o.q));
-          }
+        for (int j = 0; j < 4; ++j) *reinterpret_cast<uint2*>(cb + 32 * j) = o.c[j];
+        if (sub == 0) {
+          scales[(int64_t)b * Mp + m] = o.s;
+          qsum[(int64_t)b * Mp + m] = (int16_t)o.q;
+          if (!is8) cpart = __fadd_rn(cpart, __fmul_rn(o.s, (float)o.q));
         }
       }
     }
+  } else if (m < Mp) {
+    // padding rows: scales and qsum 0
+    for (int b = wi * 32 + lane; b < nb; b += WPR * 32) {
+      scales[(int64_t)b * Mp + m] = 0.f;
+      qsum[(int64_t)b * Mp + m] = 0;
+    }
   }
-  if (sub == 0) s_part[warp][half] = cpart;
+  // fixed-order reduction of the lanes' partial corrections (lanes with sub != 0 hold 0)
+  cpart = __fadd_rn(cpart, __shfl_xor_sync(0xffffffffu, cpart, 4));
+  cpart = __fadd_rn(cpart, __shfl_xor_sync(0xffffffffu, cpart, 8));
+  cpart = __fadd_rn(cpart, __shfl_xor_sync(0xffffffffu, cpart, 16));
+  if (lane == 0) s_part[warp] = cpart;
   __syncthreads();
   if (wi == 0 && lane == 0 && m < Mp) {
     float c = 0.f;
-    for (int i = 0; i < WPR; ++i) {
-      c = __fadd_rn(c, s_part[row_in_cta * WPR + i][0]);
-      c = __fadd_rn(c, s_part[row_in_cta * WPR + i][1]);
-    }
+    for (int i = 0; i < WPR; ++i) c = __fadd_rn(c, s_part[row_in_cta * WPR + i]);
     corr[m] = __fmul_rn(8.f, c);
   }
 }
@@ -234,10 +246,11 @@ cudaError_t launch_q(const void* x, int64_t M, int64_t K, int64_t ldx, const Tag
   float* corr = reinterpret_cast<float*>(base + L.corr_off);
   const int64_t Mp = L.Mp;
   const int64_t nb = L.nb;
-  // enough CTAs for ~16 per SM (memory-level parallelism), warps of a row sharing its pairs
-  const int64_t target = 16 * 148;
+  // enough CTAs for ~8 per SM (memory-level parallelism), warps of a row sharing its groups
+  const int64_t target = 8 * 148;
+  const int64_t ngroups = (nb + 7) / 8;
   int wpr = 1;
-  while (wpr < 8 && ceil_div(Mp, 8 / wpr) < target && (nb + 1) / 2 >= 2 * wpr) wpr *= 2;
+  while (wpr < 8 && ceil_div(Mp, 8 / wpr) < target && ngroups >= 2 * wpr) wpr *= 2;
   const int rows = 8 / wpr;
   const dim3 grid((unsigned)ceil_div(Mp, rows));
   const uint16_t* xp = static_cast<const uint16_t*>(x);

@@ -114,8 +114,23 @@ __device__ __forceinline__ void mbar_wait_addr(uint32_t a, uint32_t parity) {
       "r"(parity), "n"(1000000), "l"((uint64_t)COMET_MBAR_TIMEOUT_NS)
       : "memory");
 }
+#ifndef COMET_HANG_PRINT
+#define COMET_HANG_PRINT 0
+#endif
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+#if COMET_HANG_PRINT
+  // diagnostic build: report the stuck barrier before trapping
+  const uint64_t t0 = globaltimer_ns();
+  while (!mbar_try_wait(smem_u32(bar), parity)) {
+    if (globaltimer_ns() - t0 > 500000000ull) {
+      printf("hang: block %d thread %d bar smem 0x%x parity %u\n", (int)blockIdx.x, (int)threadIdx.x,
+             smem_u32(bar), parity);
+      __trap();
+    }
+  }
+#else
   mbar_wait_addr(smem_u32(bar), parity);
+#endif
 }
 
 // ------------------------------------------------------------------ explicit shared loads
@@ -155,6 +170,15 @@ __device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, u
       "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes"
       " [%0], [%1, {%3, %4}], [%2];" ::"r"(smem_u32(dst)),
       "l"(map), "r"(smem_u32(bar)), "r"(c0), "r"(c1)
+      : "memory");
+}
+// 3D tiled load global -> shared, completion counted on `bar` (bytes).
+__device__ __forceinline__ void tma_load_3d(void* dst, const CUtensorMap* map, uint64_t* bar,
+                                            int32_t c0, int32_t c1, int32_t c2) {
+  asm volatile(
+      "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%3, %4, %5}], [%2];" ::"r"(smem_u32(dst)),
+      "l"(map), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "r"(c2)
       : "memory");
 }
 __device__ __forceinline__ void tma_load_2d_hint(void* dst, const CUtensorMap* map, uint64_t* bar,

@@ -150,7 +150,10 @@ def test_planner_cover_order_and_balance(M, N, K, frac, P, mode, orientation):
     assert abs(float(ms) - info["max_cta_cost"]) < 1e-6
     lb = oplan.lower_bound(info["n_tiles"], tags, P, 1, Fraction(c8).limit_denominator())
     if info["split_mode"] == 1:
-        assert float(ms) <= float(lb) + c8 + 1e-9        # stream-K: within one unit of perfect
+        # stream-K: within one scheduling unit of perfect (the decode kernel schedules 4 K-blocks
+        # per unit at tile_n <= 32)
+        kgran = 4 if (info["orientation"] == 1 and info["tile_n"] <= 32) else 1
+        assert float(ms) <= float(lb) + kgran * c8 + 1e-9
     # every CTA runs its non-owner segments (kb_begin > 0 of a split tile) before any owner item
     d = plan.describe()
     split_tiles = {}

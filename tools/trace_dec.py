@@ -1,0 +1,96 @@
+"""Diagnostic: timeline of the decode GEMM (orientation 1) on LLaMA-3-70B gate/up at small M.
+Needs a COMET_TRACE=1 (or COMET_DIAG=1) build.  Prints per-CTA start/end spread (globaltimer)
+and, for CTA 0, the clock64 timeline of every role:
+  0 producer issued stage s | 1/2 MMA after full / after a_full wait (stage) |
+  3/5 widen group 0 after full wait / after a_full arrive (stage seq) | 4/6 same, group 1 |
+  7/8/9 promotion after s_full / after acc_full / done (K-block) | 10/11/12 epilogue of item i:
+  start / partials ready (owner of a split tile) / done.
+Usage: python tools/trace_dec.py [M] [layer]"""
+import ctypes
+import os
+import sys
+
+import numpy as np
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import paper_conf_asplos_liu0rxpwl0w25_b200 as cb  # noqa: E402
+from paper_conf_asplos_liu0rxpwl0w25_b200 import synth  # noqa: E402
+
+M = int(sys.argv[1]) if len(sys.argv) > 1 else 1
+layer = sys.argv[2] if len(sys.argv) > 2 else "gate_up"
+K, N = {"gate_up": (8192, 28672), "down": (28672, 8192), "qkv": (8192, 10240)}[layer]
+rng = np.random.default_rng(0)
+tags = synth.make_tags(K, 0.05, rng)
+x = torch.randn(M, K, device="cuda", dtype=torch.float16)
+w = torch.randint(-8, 8, (N, K), device="cuda", dtype=torch.int8)
+sw = torch.rand(N, device="cuda", dtype=torch.float32)
+act, sc = cb.quantize_act(x, tags)
+wp = cb.pack_weight(w)
+plan = cb.Plan(M, N, K, tags)
+y = cb.w4ax_gemm(plan, act, sc, wp, sw)
+buf = torch.zeros(32768 + 4 * 1024, dtype=torch.int64, device="cuda")
+flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+L = cb.lib()
+L.comet_debug_set_trace.argtypes = [ctypes.c_void_p]
+L.comet_debug_set_trace(ctypes.c_void_p(buf.data_ptr()))
+for i in range(3):
+    flush.fill_(i)
+    torch.cuda.synchronize()
+    buf.zero_()
+    cb.w4ax_gemm(plan, act, sc, wp, sw, out=y)
+    torch.cuda.synchronize()
+L.comet_debug_set_trace(None)
+b = buf.cpu().numpy()
+info = plan.info()
+print("plan", {k: info[k] for k in ("tile_n", "num_ctas", "split_mode", "n_tiles", "n_items", "n_split_tiles")})
+g = b[32768:32768 + 4 * info["num_ctas"]].reshape(-1, 4)
+t0 = g[:, 0].min()
+print("CTA start  (us) min/med/max", *(np.round(np.percentile(g[:, 0] - t0, [0, 50, 100]) / 1e3, 2)))
+print("CTA setup  (us) min/med/max", *(np.round(np.percentile(g[:, 1] - t0, [0, 50, 100]) / 1e3, 2)))
+print("CTA end    (us) min/med/max", *(np.round(np.percentile(g[:, 2] - t0, [0, 50, 100]) / 1e3, 2)))
+print("slowest CTAs", np.argsort(g[:, 2])[-5:].tolist(), np.round((np.sort(g[:, 2])[-5:] - t0) / 1e3, 2).tolist())
+items = plan.describe()
+for cta in (0, 1):
+    t = b[:32768].reshape(2, 16, 1024)[cta]
+    base = t[0][0]
+    n_st = int((t[0] > 0).sum())
+    n_kb = int((t[9] > 0).sum())
+    print(f"--- CTA {cta}: {n_st} stages, {n_kb} K-blocks promoted, items",
+          [tuple(r[1:]) for r in items if r[0] == cta])
+
+    def rel(e, n):
+        return (t[e][:n] - base).astype(np.int64)
+
+    prod = rel(0, n_st)
+    n_m = (n_st + 1) // 2                      # MMA events: issuer 0 = even stages only
+    mma_full, mma_a = rel(1, n_m), rel(2, n_m)
+    pro_s, pro_acc, pro_done = rel(7, n_kb), rel(8, n_kb), rel(9, n_kb)
+    print("producer issue  (clk) first 12:", prod[:12].tolist())
+    print("MMA(even) after full   first 6:", mma_full[:6].tolist())
+    print("MMA(even) after a_full first 6:", mma_a[:6].tolist())
+    wg = [rel(3, n_st), rel(4, n_st), rel(5, n_st), rel(6, n_st)]
+    wstart = np.where(np.arange(n_st) % 2 == 0, wg[0], wg[1])
+    wdone = np.where(np.arange(n_st) % 2 == 0, wg[2], wg[3])
+    print("widen start            first 12:", wstart[:12].tolist())
+    print("widen done             first 12:", wdone[:12].tolist())
+    print("promo after acc_full   first 12:", pro_acc[:12].tolist())
+    print("promo done             first 12:", pro_done[:12].tolist())
+    if n_st > 8:
+        ev2 = np.arange(2, n_m - 1)
+        print("steady state medians (clk per stage): producer", np.median(np.diff(prod[4:])),
+              "mma (per 2 stages)", np.median(np.diff(mma_a[2:])), "widen", np.median(np.diff(wdone[4:])),
+              "promo per kb", np.median(np.diff(pro_done[4:])))
+        print("latency producer->mma full (even)", np.median(mma_full[ev2] - prod[2 * ev2]),
+              "widen start - producer", np.median(wstart[4:] - prod[4:]),
+              "widen dur", np.median(wdone[4:] - wstart[4:]),
+              "mma a_full wait", np.median(mma_a[2:] - mma_full[2:]))
+    m13, m14, m15 = rel(13, n_m), rel(14, n_m), rel(15, n_m)
+    ev = np.arange(2, n_m - 2)
+    print("MMA per stage medians: a_full->acc_empty(c0)", np.median(m13[ev] - mma_a[ev]),
+          "issue c0 (4 MMAs)", np.median(m14[ev] - m13[ev]), "c1 + commits", np.median(m15[ev] - m14[ev]),
+          "commits -> next full", np.median(mma_full[ev + 1] - m15[ev]))
+    print("MMA a_full / acc0 / c0 issued / done, stages 4..9:", [(int(mma_a[i]), int(m13[i]), int(m14[i]), int(m15[i])) for i in range(2, 7)])
+    ep = [(t[10][i] - base, t[11][i] - base if t[11][i] else -1, t[12][i] - base) for i in range(8) if t[10][i]]
+    print("epilogues (start, partials ready, done):", ep)
+    print("end of last promotion", pro_done[-1] if n_kb else None)
