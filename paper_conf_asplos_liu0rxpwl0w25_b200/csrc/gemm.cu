@@ -45,50 +45,45 @@ namespace {
 #ifndef COMET_DEC_ABLATE
 #define COMET_DEC_ABLATE 0      // timing experiments only (wrong results): bit 0 no MMAs, bit 1 no
 #endif                          // TMEM stores of widened weights, bit 2 no accumulator loads
-#ifndef COMET_DEC_ISSUERS
-#define COMET_DEC_ISSUERS 2     // MMA-issuing threads (warps 1 and 3 alternate stages)
-#endif
 
 constexpr int kWidenWarp0 = 4;
 constexpr int kPromoWarp0 = 12;
 
-// One pipeline stage = KS consecutive K-blocks of one tile (KS = 4 for NT <= 32, else 2):
-//   W   KS/2 boxes of 128 weight rows x 128 B (two K-blocks of packed nibbles per row), SW128
-//   X   one 3D box [KS K-blocks][NT tokens][128 B] of activation codes, SW128 (UMMA B operand)
-//   S   one 2D box [KS][NT] of per-token scales s_a
-// all on one mbarrier.  The stage is released by the MMA commit, the 4 widen warps and the 4
-// promotion warps (which read the scales from it).
-// TMEM columns: [0, NA * 32 KS) widened-weight A buffers (one per widen group), then NACC
+// One pipeline stage = KS consecutive K-blocks of one tile (KS = 4 for NT <= 32, else 2), in
+// two rings with their own barriers so the big weight slot is recycled as soon as it is read:
+//   W ring  KS/2 boxes of 128 weight rows x 128 B (two K-blocks of packed nibbles per row),
+//           SW128; released by the 8 widen warps right after their shared-memory loads.
+//   X ring  one 3D box [KS K-blocks][NT tokens][128 B] of activation codes (SW128, the UMMA B
+//           operand) + one 2D box [KS][NT] of per-token scales; released by the MMA commit and
+//           the 4 promotion warps (which read the scales).
+// Two producer threads (warp 0: W ring, warp 2: X ring).  Every widen warp takes part in every
+// stage: warp 4 + 4h + q widens rows 32q .. 32q+31 of K-blocks [h KS/2, (h+1) KS/2).
+// TMEM columns: [0, 2 * 32 KS) two widened-weight A buffers (alternate stages), then NACC
 // accumulator sets of KS x NT columns (one accumulator per K-block of a stage).
 template <int NT>
 struct Cfg {
   static constexpr int KS = NT <= 32 ? 4 : 2;                  // K-blocks per stage
-  static constexpr int NA = 2;                                 // = widen groups
+  static constexpr int NA = 2;
   static constexpr int A_COLS = 32 * KS;
   static constexpr int ACC_SET = KS * NT;                      // accumulator columns per stage
   static constexpr int NACC_RAW = (512 - NA * A_COLS) / ACC_SET;
-  // Two MMA issuers and two widen groups take alternate stages.  An mbarrier wait is only sound
-  // if the waiter observes every phase of that barrier (a parity wait cannot tell phase k+2 from
-  // phase k), so each alternating role must always land on the same barriers: the stage count
-  // and the accumulator-set count are even (or there is a single issuer).
-  static constexpr int ISSUERS = (COMET_DEC_ISSUERS == 2 && NACC_RAW >= 2) ? 2 : 1;
-  static constexpr int NACC_C = NACC_RAW > 4 ? 4 : NACC_RAW;
-  static constexpr int NACC = ISSUERS == 2 ? (NACC_C & ~1) : NACC_C;
+  static constexpr int NACC = NACC_RAW > 4 ? 4 : NACC_RAW;
   static constexpr uint32_t ACC_COL = NA * A_COLS;
   static constexpr int XKB_BYTES = NT * 128;                   // one K-block of codes
   static constexpr int W_BYTES = KS * kTileW * 64;             // KS K-blocks of packed weights
   static constexpr int S_BYTES = KS * NT * 4;
-  static constexpr int STAGE_RAW = W_BYTES + KS * XKB_BYTES + S_BYTES;
-  static constexpr int STAGE_BYTES = (STAGE_RAW + 1023) / 1024 * 1024;
-  static constexpr int STAGES_RAW = (222 * 1024) / STAGE_BYTES;
-  static constexpr int STAGES = (STAGES_RAW > 8 ? 8 : STAGES_RAW) & ~1;   // even (see ISSUERS)
-  static constexpr int SMEM_DATA = STAGES * STAGE_BYTES;
-  static constexpr int N_BARS = 2 * STAGES + 2 * NA + 2 * NACC;
+  static constexpr int X_STAGE = (KS * XKB_BYTES + S_BYTES + 1023) / 1024 * 1024;
+  static constexpr int SX = 4;                                 // X ring depth
+  static constexpr int SMEM_BUDGET = 224 * 1024;            // 227 KB minus alignment, barriers, tags
+  static constexpr int SW_RAW = (SMEM_BUDGET - SX * X_STAGE) / W_BYTES;
+  static constexpr int SW = SW_RAW > 8 ? 8 : SW_RAW;           // W ring depth
+  static constexpr int SMEM_DATA = SW * W_BYTES + SX * X_STAGE;
+  static constexpr int N_BARS = 2 * SW + 2 * SX + 2 * NA + 2 * NACC;
   static constexpr int SMEM_BYTES = 1024 + SMEM_DATA + N_BARS * 8 + 16 + kMaxBlocks;
   static constexpr int CH = NT < 32 ? NT : 32;                 // promotion column chunk
   static_assert(NT % 16 == 0 && NT <= 128, "decode tile");
   static_assert(NACC >= 1 && NACC * ACC_SET + NA * A_COLS <= 512, "TMEM budget");
-  static_assert(STAGES >= 2 && (ISSUERS == 1 || NACC % 2 == 0), "alternating roles");
+  static_assert(SW >= 2 && SX >= 2, "ring depths");
   static_assert(SMEM_BYTES <= 227 * 1024, "shared memory budget");
 };
 
@@ -101,21 +96,24 @@ __device__ __forceinline__ void tmem_ld_cols(uint32_t taddr, uint32_t* r) {
 template <int NT, int DEBUG>
 __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ GemmParams P) {
   using C = Cfg<NT>;
-  constexpr int S = C::STAGES;
+  constexpr int SW = C::SW;
+  constexpr int SX = C::SX;
   constexpr int NA = C::NA;
   constexpr int NACC = C::NACC;
   constexpr int KS = C::KS;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   // keep the pointer derived from the __shared__ array (shared address space) when aligning
   uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
-  auto sW = [&](int st) { return smem + st * C::STAGE_BYTES; };
-  auto sX = [&](int st) { return smem + st * C::STAGE_BYTES + C::W_BYTES; };
-  auto sS = [&](int st) { return smem + st * C::STAGE_BYTES + C::W_BYTES + KS * C::XKB_BYTES; };
+  auto sW = [&](int st) { return smem + st * C::W_BYTES; };
+  auto sX = [&](int st) { return smem + SW * C::W_BYTES + st * C::X_STAGE; };
+  auto sS = [&](int st) { return smem + SW * C::W_BYTES + st * C::X_STAGE + KS * C::XKB_BYTES; };
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + C::SMEM_DATA);
-  uint64_t* full = bars;                    // [S]    TMA -> (MMA, widen, promotion)
-  uint64_t* empty = bars + S;               // [S]    MMA commit + 4 widen + 4 promotion warps -> TMA
-  uint64_t* a_full = bars + 2 * S;          // [NA]   widen group -> MMA
-  uint64_t* a_empty = a_full + NA;          // [NA]   MMA commit -> widen group
+  uint64_t* full_w = bars;                  // [SW]   TMA -> widen
+  uint64_t* empty_w = full_w + SW;          // [SW]   8 widen warps -> W producer
+  uint64_t* full_x = empty_w + SW;          // [SX]   TMA -> (MMA, promotion)
+  uint64_t* empty_x = full_x + SX;          // [SX]   MMA commit + 4 promotion warps -> X producer
+  uint64_t* a_full = empty_x + SX;          // [NA]   8 widen warps -> MMA
+  uint64_t* a_empty = a_full + NA;          // [NA]   MMA commit -> widen
   uint64_t* acc_full = a_empty + NA;        // [NACC] MMA commit -> promotion
   uint64_t* acc_empty = acc_full + NACC;    // [NACC] promotion -> MMA
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bars + C::N_BARS);
@@ -135,16 +133,20 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
     tma_prefetch(&P.map_x);
     tma_prefetch(&P.map_w);
     tma_prefetch(&P.map_s);
-    for (int i = 0; i < S; ++i) {
-      mbar_init(&full[i], 1);
-      mbar_init(&empty[i], 1 + 4 + 4);
+    for (int i = 0; i < SW; ++i) {
+      mbar_init(&full_w[i], 1);
+      mbar_init(&empty_w[i], 8);
+    }
+    for (int i = 0; i < SX; ++i) {
+      mbar_init(&full_x[i], 1);
+      mbar_init(&empty_x[i], 2 + 4);
     }
     for (int i = 0; i < NA; ++i) {
-      mbar_init(&a_full[i], 4);
-      mbar_init(&a_empty[i], 1);
+      mbar_init(&a_full[i], 8);
+      mbar_init(&a_empty[i], 2);
     }
     for (int i = 0; i < NACC; ++i) {
-      mbar_init(&acc_full[i], 1);
+      mbar_init(&acc_full[i], 2);
       mbar_init(&acc_empty[i], 4);
     }
     fence_mbar_init();
@@ -164,65 +166,76 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
   if (warp < kWidenWarp0) {
     setmaxnreg_dec<40>();
     if (warp == 0 && lane == 0) {
-      // ------------------------------------------------------------------ TMA producer
-      int stage = 0;
+      // ------------------------------------------------------------------ W producer
+      int st = 0;
       uint32_t ph = 0;
       for (int it = it_begin; it < it_end; ++it) {
         const WorkItem w = load_item(P, it, debug);
-        const int n_tile = w.tile / P.n_m_tiles, m_tile = w.tile % P.n_m_tiles;
-        const int m0 = m_tile * NT, n0 = n_tile * kTileW;
+        const int n0 = (w.tile / P.n_m_tiles) * kTileW;
         for (int kb = w.kb_begin; kb < w.kb_end; kb += KS) {
           const int npair = (min(KS, w.kb_end - kb) + 1) >> 1;
-          mbar_wait(&empty[stage], ph ^ 1);
-          mbar_arrive_expect_tx(&full[stage], npair * 2 * kTileW * 64 + KS * C::XKB_BYTES + C::S_BYTES);
+          mbar_wait(&empty_w[st], ph ^ 1);
+          mbar_arrive_expect_tx(&full_w[st], npair * 2 * kTileW * 64);
           for (int p = 0; p < npair; ++p)
-            tma_load_2d(sW(stage) + p * 2 * kTileW * 64, &P.map_w, &full[stage], (kb + 2 * p) * 64, n0);
-          tma_load_3d(sX(stage), &P.map_x, &full[stage], 0, m0, kb);
-          tma_load_2d(sS(stage), &P.map_s, &full[stage], m0, kb);
+            tma_load_2d(sW(st) + p * 2 * kTileW * 64, &P.map_w, &full_w[st], (kb + 2 * p) * 64, n0);
           trace_ev(P, 0, tr++);
-          if (++stage == S) { stage = 0; ph ^= 1; }
+          if (++st == SW) { st = 0; ph ^= 1; }
         }
       }
-    } else if ((warp == 1 || (C::ISSUERS == 2 && warp == 3)) && lane == 0) {
-      // ------------------------------------------------------------------ MMA issuer(s)
-      // With two issuers, warp 1 takes the even stages and warp 3 the odd ones; tcgen05.commit
-      // tracks the issuing thread's own MMAs, so each commits exactly the stages it issued.
+    } else if (warp == 2 && lane == 0) {
+      // ------------------------------------------------------------------ X producer
+      int st = 0;
+      uint32_t ph = 0;
+      for (int it = it_begin; it < it_end; ++it) {
+        const WorkItem w = load_item(P, it, debug);
+        const int m0 = (w.tile % P.n_m_tiles) * NT;
+        for (int kb = w.kb_begin; kb < w.kb_end; kb += KS) {
+          mbar_wait(&empty_x[st], ph ^ 1);
+          mbar_arrive_expect_tx(&full_x[st], KS * C::XKB_BYTES + C::S_BYTES);
+          tma_load_3d(sX(st), &P.map_x, &full_x[st], 0, m0, kb);
+          tma_load_2d(sS(st), &P.map_s, &full_x[st], m0, kb);
+          if (++st == SX) { st = 0; ph ^= 1; }
+        }
+      }
+    } else if ((warp == 1 || warp == 3) && lane == 0) {
+      // ------------------------------------------------------------------ MMA issuers
+      // Two issuing threads share every stage: warp 1 issues the stage's even K-blocks, warp 3
+      // the odd ones (each K-block has its own accumulator).  tcgen05.commit tracks the
+      // issuing thread's own MMAs, so both commit each stage's barriers (counts 2).
       const int par = warp == 1 ? 0 : 1;
       const uint32_t id_f8 = idesc_f8f6f4_e4m3(128, NT);
       const uint32_t id_i8 = idesc_i8(128, NT);
-      int stage = 0, ab = 0, accs = 0, seq = 0;
-      uint32_t ph = 0, aph = 0, accph = 0;
+      int sx = 0, ab = 0, accs = 0;
+      uint32_t xph = 0, aph = 0, accph = 0;
       for (int it = it_begin; it < it_end; ++it) {
         const WorkItem w = load_item(P, it, debug);
-        for (int kb = w.kb_begin; kb < w.kb_end; kb += KS, ++seq) {
-          if (C::ISSUERS == 1 || (seq & 1) == par) {
-            const int nk = min(KS, w.kb_end - kb);
-            mbar_wait(&full[stage], ph);
-            mbar_wait(&a_full[ab], aph);
-            mbar_wait(&acc_empty[accs], accph ^ 1);
-            if (par == 0) trace_ev(P, 1, tr++);
-            tc_fence_after();
-            const uint32_t d0 = tbase + C::ACC_COL + accs * C::ACC_SET;
-            const uint32_t a0 = tbase + ab * C::A_COLS;
-            const uint64_t b0 = sdesc_kmajor_sw128(smem_u32(sX(stage)));
-            for (int c = 0; c < nk; ++c) {
-              const uint32_t d = d0 + c * NT, a = a0 + c * 32;
-              const uint64_t bd = b0 + (uint64_t)((c * C::XKB_BYTES) >> 4);
-              if (COMET_DEC_ABLATE & 1) {
-              } else if (lds_u8(s_tags_a + kb + c)) {
+        for (int kb = w.kb_begin; kb < w.kb_end; kb += KS) {
+          const int nk = min(KS, w.kb_end - kb);
+          mbar_wait(&full_x[sx], xph);
+          mbar_wait(&a_full[ab], aph);
+          mbar_wait(&acc_empty[accs], accph ^ 1);
+          if (par == 0) trace_ev(P, 1, tr);
+          tc_fence_after();
+          const uint32_t d0 = tbase + C::ACC_COL + accs * C::ACC_SET;
+          const uint32_t a0 = tbase + ab * C::A_COLS;
+          const uint64_t b0 = sdesc_kmajor_sw128(smem_u32(sX(sx)));
+          for (int c = par; c < nk; c += 2) {
+            const uint32_t d = d0 + c * NT, a = a0 + c * 32;
+            const uint64_t bd = b0 + (uint64_t)((c * C::XKB_BYTES) >> 4);
+            if (COMET_DEC_ABLATE & 1) {
+            } else if (lds_u8(s_tags_a + kb + c)) {
 #pragma unroll
-                for (int k = 0; k < 4; ++k) mma_i8_ts(d, a + 8 * k, bd + 2 * k, id_i8, k);
-              } else {
+              for (int k = 0; k < 4; ++k) mma_i8_ts(d, a + 8 * k, bd + 2 * k, id_i8, k);
+            } else {
 #pragma unroll
-                for (int k = 0; k < 4; ++k) mma_f8_ts(d, a + 8 * k, bd + 2 * k, id_f8, k);
-              }
+              for (int k = 0; k < 4; ++k) mma_f8_ts(d, a + 8 * k, bd + 2 * k, id_f8, k);
             }
-            tc_commit(&acc_full[accs]);
-            tc_commit(&empty[stage]);
-            tc_commit(&a_empty[ab]);
-            if (par == 0) trace_ev(P, 2, tr - 1);
           }
-          if (++stage == S) { stage = 0; ph ^= 1; }
+          tc_commit(&acc_full[accs]);
+          tc_commit(&empty_x[sx]);
+          tc_commit(&a_empty[ab]);
+          if (par == 0) trace_ev(P, 2, tr++);
+          if (++sx == SX) { sx = 0; xph ^= 1; }
           if (++ab == NA) { ab = 0; aph ^= 1; }
           if (++accs == NACC) { accs = 0; accph ^= 1; }
         }
@@ -231,75 +244,71 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
   } else if (warp < kPromoWarp0) {
     setmaxnreg_dec<112>();
     // -------------------------------------------------------------------- widen (W -> TMEM A)
-    const int grp = (warp - kWidenWarp0) >> 2;    // this group takes stages with seq % 2 == grp
+    constexpr int KH = KS / 2;                    // K-blocks per widen warp and stage
+    const int half = (warp - kWidenWarp0) >> 2;   // K-blocks [half KH, (half+1) KH) of a stage
     const int q = warp & 3;
     const int r = q * 32 + lane;                  // TMEM lane = weight row within the tile
     const uint32_t lane_addr = (uint32_t)(q * 32) << 16;
     const int sw = r & 7;                         // TMA 128-byte swizzle: chunk ^= row bits [0:2]
-    int stage = 0, seq = 0;
+    int st = 0, ab = 0;
     uint32_t ph = 0, aph = 0;
+    int seq = 0;
     for (int it = it_begin; it < it_end; ++it) {
       const WorkItem w = load_item(P, it, debug);
       for (int kb = w.kb_begin; kb < w.kb_end; kb += KS, ++seq) {
-        if ((seq & 1) == grp) {
-          const int nk = min(KS, w.kb_end - kb);
-          mbar_wait(&full[stage], ph);
-          if (lane == 0 && q == 0) trace_ev(P, 3 + grp, seq);
-          mbar_wait(&a_empty[grp], aph ^ 1);
-          tc_fence_after();
-          const uint32_t wbase = smem_u32(sW(stage)) + r * 128;
+        const int nk = min(KS, w.kb_end - kb);
+        mbar_wait(&full_w[st], ph);
+        if (lane == 0 && q == 0) trace_ev(P, 3 + half, seq);
+        // this warp's K-blocks of the stage: 4 x 16 B per K-block (row r, 128B-swizzled chunks)
+        uint4 cc[4 * KH];
 #pragma unroll
-          for (int p = 0; p < KS / 2; ++p) {
-            if (2 * p < nk) {
-              uint4 c[8];
+        for (int i = 0; i < KH; ++i) {
+          const int cb = half * KH + i;
+          const uint32_t row = smem_u32(sW(st)) + (cb >> 1) * 2 * kTileW * 64 + r * 128;
 #pragma unroll
-              for (int j = 0; j < 8; ++j) c[j] = lds128(wbase + p * 2 * kTileW * 64 + ((j ^ sw) << 4));
+          for (int j = 0; j < 4; ++j)
+            cc[4 * i + j] = cb < nk ? lds128(row + ((((cb & 1) * 4 + j) ^ sw) << 4)) : make_uint4(0, 0, 0, 0);
+        }
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&empty_w[st]);
+        mbar_wait(&a_empty[ab], aph ^ 1);
+        tc_fence_after();
 #pragma unroll
-              for (int h = 0; h < 2; ++h) {
-                if (2 * p + h < nk) {
-                  const bool is8 = lds_u8(s_tags_a + kb + 2 * p + h) != 0;
-                  uint32_t o[32];
+        for (int i = 0; i < KH; ++i) {
+          const int cb = half * KH + i;
+          if (cb < nk) {
+            const bool is8 = lds_u8(s_tags_a + kb + cb) != 0;
+            uint32_t o[32];
 #pragma unroll
-                  for (int j = 0; j < 4; ++j) {
-                    const uint32_t pw[4] = {c[4 * h + j].x, c[4 * h + j].y, c[4 * h + j].z, c[4 * h + j].w};
+            for (int j = 0; j < 4; ++j) {
+              const uint32_t pw[4] = {cc[4 * i + j].x, cc[4 * i + j].y, cc[4 * i + j].z, cc[4 * i + j].w};
 #pragma unroll
-                    for (int i = 0; i < 4; ++i) {
-                      const uint32_t pv = pw[i];
-                      const int g = 2 * (j * 4 + i);
-                      if (is8) {
-                        o[g] = ((pv << 4) & 0xF0F0F0F0u) ^ 0x80808080u;
-                        o[g + 1] = (pv & 0xF0F0F0F0u) ^ 0x80808080u;
-                      } else {
-                        o[g] = pv & 0x0F0F0F0Fu;
-                        o[g + 1] = (pv >> 4) & 0x0F0F0F0Fu;
-                      }
-                    }
-                  }
-                  if (!(COMET_DEC_ABLATE & 2)) tmem_st32(tbase + grp * C::A_COLS + (2 * p + h) * 32 + lane_addr, o);
+              for (int e = 0; e < 4; ++e) {
+                const uint32_t pv = pw[e];
+                const int g = 2 * (j * 4 + e);
+                if (is8) {
+                  o[g] = ((pv << 4) & 0xF0F0F0F0u) ^ 0x80808080u;
+                  o[g + 1] = (pv & 0xF0F0F0F0u) ^ 0x80808080u;
+                } else {
+                  o[g] = pv & 0x0F0F0F0Fu;
+                  o[g + 1] = (pv >> 4) & 0x0F0F0F0Fu;
                 }
               }
             }
+            if (!(COMET_DEC_ABLATE & 2)) tmem_st32(tbase + ab * C::A_COLS + cb * 32 + lane_addr, o);
           }
-          __syncwarp();
-          if (lane == 0) mbar_arrive(&empty[stage]);
-          if (!(COMET_DEC_ABLATE & 2)) tmem_wait_st();
-          tc_fence_before();
-          __syncwarp();
-          if (lane == 0) mbar_arrive(&a_full[grp]);
-          if (lane == 0 && q == 0) trace_ev(P, 5 + grp, seq);
-#if COMET_HANG_PRINT
-          if (blockIdx.x == 0 && lane == 0) printf("widen warp %d seq %d done\n", warp, seq);
-#endif
-          aph ^= 1;
         }
-        if (++stage == S) { stage = 0; ph ^= 1; }
+        if (!(COMET_DEC_ABLATE & 2)) tmem_wait_st();
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&a_full[ab]);
+        if (lane == 0 && q == 0) trace_ev(P, 5 + half, seq);
+        if (++st == SW) { st = 0; ph ^= 1; }
+        if (++ab == NA) { ab = 0; aph ^= 1; }
       }
     }
   } else {
     setmaxnreg_inc<208>();
-#if COMET_HANG_PRINT
-    if (blockIdx.x == 0 && (threadIdx.x & 31) == 0) printf("promo warp %d started\n", warp);
-#endif
     // -------------------------------------------------------------------- promotion + epilogue
     // TMEM accumulator: lane = weight row (n), column = token (m); 32x32b loads give thread t of
     // warp quarter q the row 32q + t and every token column of the tile.
@@ -308,8 +317,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
     const int row = q * 32 + lane;
     const uint32_t lane_addr = (uint32_t)(q * 32) << 16;
     const int ptid = threadIdx.x - kPromoWarp0 * 32;
-    int stage = 0, accs = 0;
-    uint32_t ph = 0, accph = 0;
+    int sx = 0, accs = 0;
+    uint32_t xph = 0, accph = 0;
     for (int it = it_begin; it < it_end; ++it) {
       const WorkItem w = load_item(P, it, debug);
       const int n_tile = w.tile / P.n_m_tiles, m_tile = w.tile % P.n_m_tiles;
@@ -317,21 +326,32 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
       const bool owner = (w.flags & 2) != 0;
       const bool split = (w.flags & 1) != 0;
       const int n = n0 + row;
+      // epilogue operands loaded now (their latency overlaps the K loop): s_w[n] and, for the
+      // owner, corr[m] (the offset-binary weight correction, applied once at the end)
+      const float swv = n < P.N ? __ldg(P.w_scales + n) * 512.f : 0.f;
+      constexpr bool kEarlyCorr = NT <= 32;        // registers: NT > 32 loads corr at the end
+      float cr[kEarlyCorr ? NT : 1];
+      if constexpr (kEarlyCorr) {
+#pragma unroll
+        for (int j = 0; j < NT; ++j) {
+          const int64_t m = m0 + j;
+          cr[j] = (owner && m < P.Mp) ? __ldg(P.corr + m) * 0.001953125f : 0.f;   // 2^-9
+        }
+      }
       float acc[NT];
       int32_t dacc[DEBUG ? NT : 1];
 #pragma unroll
       for (int j = 0; j < NT; ++j) {
-        const int64_t m = m0 + j;
-        acc[j] = (owner && m < P.Mp) ? -__ldg(P.corr + m) * 0.001953125f : 0.f;   // 2^-9
+        acc[j] = 0.f;
         if (DEBUG) dacc[j] = 0;
       }
       for (int kb0 = w.kb_begin; kb0 < w.kb_end; kb0 += KS) {
         const int nk = min(KS, w.kb_end - kb0);
-        mbar_wait(&full[stage], ph);
+        mbar_wait(&full_x[sx], xph);
         mbar_wait(&acc_full[accs], accph);
         if (ptid == 0) trace_ev(P, 7, tr);
         tc_fence_after();
-        const uint32_t sbase = smem_u32(sS(stage));
+        const uint32_t sbase = smem_u32(sS(sx));
         for (int c = 0; c < nk; ++c) {
           const int kb = kb0 + c;
           const bool is8 = lds_u8(s_tags_a + kb) != 0;
@@ -393,13 +413,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
         __syncwarp();
         if (lane == 0) {
           mbar_arrive(&acc_empty[accs]);
-          mbar_arrive(&empty[stage]);
+          mbar_arrive(&empty_x[sx]);
         }
         if (ptid == 0) trace_ev(P, 8, tr++);
-#if COMET_HANG_PRINT
-        if (blockIdx.x == 0 && lane == 0) printf("promo warp %d kb0 %d done\n", warp, kb0);
-#endif
-        if (++stage == S) { stage = 0; ph ^= 1; }
+        if (++sx == SX) { sx = 0; xph ^= 1; }
         if (++accs == NACC) { accs = 0; accph ^= 1; }
       }
       // ---------------------------------------------------------------- epilogue
@@ -413,9 +430,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
               P.ws_part + ((int64_t)w.fix * (P.max_seg - 1) + (seg - 1)) * part_tile);
 #pragma unroll
           for (int j = 0; j < NT; j += 4) dst[(j / 4) * 128 + ptid] = make_float4(acc[j], acc[j + 1], acc[j + 2], acc[j + 3]);
-          __threadfence();
+          // the 128 threads' partial stores, ordered by the CTA barrier, are published by one
+          // thread's gpu-scope release (cumulative)
           named_bar_sync(1, 128);
-          if (ptid == 0) st_release_gpu(P.ws_flags + (int64_t)w.fix * P.max_seg + seg, P.epoch);
+          if (ptid == 0) {
+            fence_acq_rel_gpu();
+            st_release_gpu(P.ws_flags + (int64_t)w.fix * P.max_seg + seg, P.epoch);
+          }
           if (ptid == 0) trace_ev(P, 12, it - it_begin);
           continue;
         }
@@ -445,12 +466,14 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
         }
       }
       if (n < P.N) {
-        const float swv = __ldg(P.w_scales + n) * 512.f;
 #pragma unroll
         for (int j = 0; j < NT; ++j) {
           const int64_t m = m0 + j;
           if (m < P.M) {
-            const float yv = acc[j] * swv;
+            float c0;
+            if constexpr (kEarlyCorr) c0 = cr[j];
+            else c0 = owner ? __ldg(P.corr + m) * 0.001953125f : 0.f;
+            const float yv = (acc[j] - c0) * swv;
             const int64_t off = m * P.ldy + n;
             if (P.ydt == COMET_F16) reinterpret_cast<__half*>(P.y)[off] = __float2half_rn(yv);
             else if (P.ydt == COMET_BF16) reinterpret_cast<__nv_bfloat16*>(P.y)[off] = __float2bfloat16_rn(yv);

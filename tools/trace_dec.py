@@ -55,7 +55,7 @@ for cta in (0, 1):
     t = b[:32768].reshape(2, 16, 1024)[cta]
     base = t[0][0]
     n_st = int((t[0] > 0).sum())
-    n_kb = int((t[9] > 0).sum())
+    n_kb = int((t[8] > 0).sum())
     print(f"--- CTA {cta}: {n_st} stages, {n_kb} K-blocks promoted, items",
           [tuple(r[1:]) for r in items if r[0] == cta])
 
@@ -64,33 +64,27 @@ for cta in (0, 1):
 
     prod = rel(0, n_st)
     n_m = (n_st + 1) // 2                      # MMA events: issuer 0 = even stages only
-    mma_full, mma_a = rel(1, n_m), rel(2, n_m)
-    pro_s, pro_acc, pro_done = rel(7, n_kb), rel(8, n_kb), rel(9, n_kb)
-    print("producer issue  (clk) first 12:", prod[:12].tolist())
-    print("MMA(even) after full   first 6:", mma_full[:6].tolist())
-    print("MMA(even) after a_full first 6:", mma_a[:6].tolist())
+    m_go, m_done = rel(1, n_m), rel(2, n_m)
     wg = [rel(3, n_st), rel(4, n_st), rel(5, n_st), rel(6, n_st)]
-    wstart = np.where(np.arange(n_st) % 2 == 0, wg[0], wg[1])
-    wdone = np.where(np.arange(n_st) % 2 == 0, wg[2], wg[3])
-    print("widen start            first 12:", wstart[:12].tolist())
-    print("widen done             first 12:", wdone[:12].tolist())
-    print("promo after acc_full   first 12:", pro_acc[:12].tolist())
-    print("promo done             first 12:", pro_done[:12].tolist())
+    idx = np.arange(n_st)
+    wstart = np.minimum(wg[0], wg[1])          # v4: both widen halves take every stage
+    wdone = np.maximum(wg[2], wg[3])
+    p_go, p_done = rel(7, n_st), rel(8, n_st)
+    print("producer issue   first 10:", prod[:10].tolist())
+    print("widen start      first 10:", wstart[:10].tolist())
+    print("widen done       first 10:", wdone[:10].tolist())
+    print("MMA(even) go     first 5 :", m_go[:5].tolist())
+    print("MMA(even) done   first 5 :", m_done[:5].tolist())
+    print("promo go         first 10:", p_go[:10].tolist())
+    print("promo done       first 10:", p_done[:10].tolist())
     if n_st > 8:
-        ev2 = np.arange(2, n_m - 1)
-        print("steady state medians (clk per stage): producer", np.median(np.diff(prod[4:])),
-              "mma (per 2 stages)", np.median(np.diff(mma_a[2:])), "widen", np.median(np.diff(wdone[4:])),
-              "promo per kb", np.median(np.diff(pro_done[4:])))
-        print("latency producer->mma full (even)", np.median(mma_full[ev2] - prod[2 * ev2]),
-              "widen start - producer", np.median(wstart[4:] - prod[4:]),
-              "widen dur", np.median(wdone[4:] - wstart[4:]),
-              "mma a_full wait", np.median(mma_a[2:] - mma_full[2:]))
-    m13, m14, m15 = rel(13, n_m), rel(14, n_m), rel(15, n_m)
-    ev = np.arange(2, n_m - 2)
-    print("MMA per stage medians: a_full->acc_empty(c0)", np.median(m13[ev] - mma_a[ev]),
-          "issue c0 (4 MMAs)", np.median(m14[ev] - m13[ev]), "c1 + commits", np.median(m15[ev] - m14[ev]),
-          "commits -> next full", np.median(mma_full[ev + 1] - m15[ev]))
-    print("MMA a_full / acc0 / c0 issued / done, stages 4..9:", [(int(mma_a[i]), int(m13[i]), int(m14[i]), int(m15[i])) for i in range(2, 7)])
+        e = np.arange(3, n_st - 1)
+        em = np.arange(2, n_m - 1)
+        print("per-stage period medians: producer", np.median(np.diff(prod[3:])), "widen", np.median(np.diff(wdone[3:])),
+              "promo", np.median(np.diff(p_done[3:])), "MMA (2 stages)", np.median(np.diff(m_done[2:])))
+        print("latencies: producer->widen start", np.median(wstart[e] - prod[e]), "widen dur", np.median(wdone[e] - wstart[e]),
+              "widen done->MMA go", np.median(m_go[em] - wdone[2 * em]), "MMA issue dur", np.median(m_done[em] - m_go[em]),
+              "MMA done->promo go", np.median(p_go[2 * em] - m_done[em]), "promo dur", np.median(p_done[e] - p_go[e]))
     ep = [(t[10][i] - base, t[11][i] - base if t[11][i] else -1, t[12][i] - base) for i in range(8) if t[10][i]]
     print("epilogues (start, partials ready, done):", ep)
-    print("end of last promotion", pro_done[-1] if n_kb else None)
+    print("end of last promotion", p_done[-1] if n_st else None)
