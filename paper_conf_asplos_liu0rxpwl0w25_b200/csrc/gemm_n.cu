@@ -28,6 +28,12 @@
 #ifndef COMET_ISSUERS
 #define COMET_ISSUERS 2   // MMA issuing threads (K-blocks alternate between them)
 #endif
+#ifndef COMET_PRODUCERS
+#define COMET_PRODUCERS 1   // TMA-issuing warps (2: K-blocks alternate between them)
+#endif
+#ifndef COMET_PROMO_SB
+#define COMET_PROMO_SB 0
+#endif
 #ifndef COMET_NSUB
 #define COMET_NSUB 1   // 2: split each K-block's MMA into two sub-MMAs (experimental, slower)
 #endif
@@ -72,8 +78,12 @@ struct CfgN {
   static constexpr int NEED = LOADALL ? ACC_REGS + COLS + 24 : ACC_REGS + 2 * 16 + 24;
   static constexpr int REG_LOW = promo_regs(40) >= NEED ? 40 : 32;
   static constexpr int REG_PROMO = promo_regs(REG_LOW);
+  // SB: single-buffered 32-column batches (fewer, larger TMEM loads in flight) when the
+  // double-buffered 32-column form does not fit (variant experiments: COMET_PROMO_SB)
+  static constexpr bool SB = !LOADALL && COMET_PROMO_SB && REG_PROMO < ACC_REGS + 2 * 32 + 24 &&
+                             REG_PROMO >= ACC_REGS + 32 + 24 && COLS % 32 == 0;
   static constexpr int PB = LOADALL ? COLS
-                          : ((REG_PROMO >= ACC_REGS + 2 * 32 + 24 && COLS % 32 == 0) ? 32 : 16);
+                          : ((SB || (REG_PROMO >= ACC_REGS + 2 * 32 + 24 && COLS % 32 == 0)) ? 32 : 16);
   static constexpr int NACC_TMEM = 512 / BN >= 4 ? 4 : 512 / BN;   // accumulators TMEM holds
   // NSUB = 2: each K-block is issued as two N = BN/2 sub-MMAs, one per promotion warpgroup, each
   // with its own ready / full barriers and issuing thread, so promotion of one half overlaps the
@@ -89,6 +99,7 @@ struct CfgN {
   // lands on the mma_ready barrier of slot (kb + NACC) % S)
   static constexpr int NACC = NACC_TMEM < S ? NACC_TMEM : S - 1;
   static constexpr int SS = S + NACC;
+  static constexpr int PRODUCERS = (COMET_PRODUCERS == 2 && S % 2 == 0 && SS % 2 == 0) ? 2 : 1;
   // [slots][output staging][scale ring SS x BM][w_scales 2 x BN][barriers][tmem][tags]
   static constexpr int SMEM_DATA = S * SLOT_BYTES + STAGE_BYTES + SS * BM * 4 + 2 * BN * 4;
   static constexpr int N_BARS = 2 * S + NSUB * S + NSUB * NACC;
@@ -184,17 +195,23 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
 
   if (warp < 4) {
     setmaxnreg_dec<C::REG_LOW>();
-    if (warp == 0 && lane == 0) {
-      // ------------------------------------------------------------------ TMA producer
-      int s = 0, sc = 0, tr = 0;
-      uint32_t ph = 0;
+    if ((warp == 0 || (C::PRODUCERS == 2 && warp == 2)) && lane == 0) {
+      // ------------------------------------------------------------------ TMA producer(s)
+      // TMA loads issued by one warp complete one after another (~1000 clk each under load,
+      // profiles/r01/probe_stream.txt), so two warps (0 and 2) issue alternate K-blocks.  Each
+      // producer only reuses its own slots (S even), so it observes every phase it waits on.
+      const int par = warp == 0 ? 0 : 1;
+      int j = 0, tr = 0;
       for (int it = it_begin; it < it_end; ++it) {
         const WorkItem w = load_item(P, it, debug);
         const int n_tile = w.tile / P.n_m_tiles, m_tile = w.tile % P.n_m_tiles;
         const int m0 = m_tile * (BM * CG) + BM * rank, n0 = n_tile * BN + C::WROWS * rank;
         const uint32_t sbytes = m0 < P.Mp ? (uint32_t)(min((int64_t)BM, P.Mp - m0) * 4) : 0u;
-        for (int kb = w.kb_begin; kb < w.kb_end; ++kb) {
-          trace_ev(P, 14, tr);
+        for (int kb = w.kb_begin; kb < w.kb_end; ++kb, ++j) {
+          if (C::PRODUCERS == 2 && (j & 1) != par) continue;
+          const int s = j % S, sc = j % SS;
+          const uint32_t ph = (uint32_t)(j / S) & 1u;
+          if (par == 0) trace_ev(P, 14, tr);
           mbar_wait(&slot_free[s], ph ^ 1);
           if (diag_ablate(P) & 32) {                       // diagnostic: no global loads
             mbar_arrive(&full[s]);
@@ -204,9 +221,7 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
             tma_load_2d(sWp(s), &P.map_w, &full[s], kb * 64, n0);
             if (sbytes) bulk_load(sS + sc * BM, P.scales + (int64_t)kb * P.Mp + m0, sbytes, &full[s]);
           }
-          trace_ev(P, 0, tr++);
-          if (++s == S) { s = 0; ph ^= 1; }
-          if (++sc == SS) sc = 0;
+          if (par == 0) trace_ev(P, 0, tr++);
         }
       }
     } else if ((warp == 1 || (COMET_ISSUERS == 2 && warp == 3)) && lane == 0 && rank == 0) {
@@ -406,6 +421,41 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
         // folded in; the accumulator is released once the last load has landed.
         constexpr int PB = C::PB;                         // columns per TMEM load batch
         constexpr int NB_ = COLS / PB;
+        if constexpr (C::SB) {
+          // single-buffered batches: load, wait, fold; release after the last load landed
+          float s;
+          asm volatile("ld.shared.f32 %0, [%1];" : "=f"(s) : "r"(s_scale_r + 4u * BM * sc));
+          if (is8) s *= 1.220703125e-04f;
+          const float2 s2 = make_float2(s, s);
+#pragma unroll
+          for (int b = 0; b < NB_; ++b) {
+            uint32_t v[PB];
+            tmem_ld_32x32b<PB>(taddr + b * PB, v);
+            tmem_wait_ld();
+            if (b + 1 == NB_) {
+              tc_fence_before();
+              __syncwarp();
+              if (lane == 0) mbar_arrive_cluster(ready_rel + rs * 8);
+            }
+            if (is8) {
+#pragma unroll
+              for (int c = 0; c < PB; ++c) v[c] = __float_as_uint(__int2float_rn((int)v[c]));
+            }
+#pragma unroll
+            for (int c = 0; c < PB; c += 2) {
+              const int a = b * PB + c;
+              float2 y = ffma2(make_float2(__uint_as_float(v[c]), __uint_as_float(v[c + 1])), s2,
+                               make_float2(acc[a], acc[a + 1]));
+              acc[a] = y.x;
+              acc[a + 1] = y.y;
+            }
+          }
+          ++tr;
+          if (++accb == NACC) { accb = 0; accph ^= 1; }
+          if (++sc == SS) sc = 0;
+          if (++rs == S) rs = 0;
+          continue;
+        }
         uint32_t vb[NB_ > 1 ? 2 : 1][PB];
         tmem_ld_32x32b<PB>(taddr, vb[0]);
         if (threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 8, tr);

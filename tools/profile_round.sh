@@ -9,3 +9,7 @@ SHORT="python bench.py --steps 2 --warmup 3 --e2e-steps 0 --cpu-budget 0 --decod
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 200 --csv --log-file gpurun_out/launches.csv $SHORT > /dev/null 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_w4ax -s 3 -c 3 -f -o gpurun_out/prof_gemm $SHORT > gpurun_out/prof_gemm.log 2>&1; tail -2 gpurun_out/prof_gemm.log
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:k_quantize -s 6 -c 3 -f -o gpurun_out/prof_quant $SHORT > gpurun_out/prof_quant.log 2>&1; tail -2 gpurun_out/prof_quant.log
+# decode GEMM (LLaMA-3-70B gate/up, M=1): one ncu --set full capture
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:^k_w4ax$ -s 2 -c 1 -f -o gpurun_out/prof_dec python tools/decode_time.py --Ms 1 --layers gate_up --iters 2 > gpurun_out/prof_dec.log 2>&1; tail -2 gpurun_out/prof_dec.log
+# TMA streaming probe (HBM and L2-resident, 1..4 issuing warps)
+timeout 300 ./tools/probe/probe_stream 1 > gpurun_out/probe_stream.txt 2>&1
