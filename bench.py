@@ -366,8 +366,12 @@ def run_comet(args, rank, world, local_rank):
                 outs[L["name"]] = torch.empty((M_TOKENS, L["N"]), dtype=torch.float16).pin_memory()
 
             def e2e_step():
+                # one step = the three layers through the public host-buffer call; the async
+                # form lets layer i+1's uploads overlap layer i's downloads (PCIe full duplex)
                 for L in layers:
-                    cb.w4ax_linear_host(L["plan"], L["x_host"], L["wp"], L["sw"], outs[L["name"]], scr[L["name"]])
+                    cb.w4ax_linear_host(L["plan"], L["x_host"], L["wp"], L["sw"], outs[L["name"]], scr[L["name"]],
+                                        blocking=False)
+                torch.cuda.synchronize()
         else:
             outs = {L["name"]: torch.empty(L["y"].shape, dtype=L["y"].dtype).pin_memory() for L in layers}
 
@@ -397,7 +401,7 @@ def run_comet(args, rank, world, local_rank):
             e_ms = t.item()
         e2e = {"value": total_ops() / (e_ms * 1e-3) / 1e12, "unit": "TOPS", "h2d_bytes_per_step": h2d,
                "d2h_bytes_per_step": d2h, "ms_per_step": e_ms,
-               "path": "comet_w4ax_linear_host (C ABI, pinned host buffers)" if world == 1 else
+               "path": "comet_w4ax_linear_host_async x3 + sync (C ABI, pinned host buffers, 1024-row chunk pipeline)" if world == 1 else
                        "public API: H2D copy + quantize_act + w4ax_gemm (+ NCCL all_reduce) + D2H copy"}
 
     cpu = cpu_baseline_sample(args.cpu_budget) if (rank == 0 and world == 1 and args.cpu_budget > 0) else None

@@ -214,15 +214,34 @@ comet_status_t comet_w4ax_gemm(comet_plan_t plan, const void* act_packed, const 
 
 /*
  * Convenience: the whole hot path for one linear layer with HOST buffers (used for the
- * end-to-end measurement).  Copies x_host (pinned recommended) to the device, quantises,
- * runs the GEMM and copies y back to y_host, all on `stream`, then synchronises the stream.
- * Device scratch (x, act, scales, y) is taken from `scratch` (comet_linear_scratch_bytes).
+ * end-to-end measurement).  Copies x_host [M][K] (F16/BF16, pinned host memory for overlap) to
+ * the device, quantises, runs the GEMM and copies y [M][N] back to y_host.
+ *   M < 2048: all on `stream`, in order.
+ *   M >= 2048: pipelined over chunks of 1024 token rows -- chunk c's H2D copy (an internal copy
+ *   stream), its quantise + GEMM (on `stream`, with an internal sub-plan of the same scheduler
+ *   configuration) and its D2H copy (a second internal copy stream) overlap the neighbouring
+ *   chunks' transfers and compute.  The uploads start at once (ordered only after the previous
+ *   call with this plan has finished reading its scratch); quantise + GEMM follow the work
+ *   already queued on `stream`; the downloads run on the internal stream.
+ * comet_w4ax_linear_host returns when y_host is complete.  The _async form returns at once:
+ * x_host and y_host must stay valid, and y_host is complete after comet_linear_host_wait(plan)
+ * (or a device synchronize); for M < 2048 completion of `stream` suffices.  Device scratch (x,
+ * act, scales, y, the sub-plans' fix-up workspace) comes from `scratch` (256-byte aligned, at
+ * least comet_linear_scratch_bytes(plan, xdt, ydt) bytes; that call also builds the sub-plans)
+ * and must not be used by anything else while calls are in flight.  `workspace` is the plan's
+ * own fix-up workspace (used when M < 2048).  Not thread-safe per plan.
  */
 size_t comet_linear_scratch_bytes(comet_plan_t plan, comet_dtype_t xdt, comet_dtype_t ydt);
 comet_status_t comet_w4ax_linear_host(comet_plan_t plan, const void* x_host, comet_dtype_t xdt,
                                       const void* w_packed, const float* w_scales, void* y_host,
                                       comet_dtype_t ydt, void* scratch, size_t scratch_bytes,
                                       void* workspace, size_t ws_bytes, void* stream);
+comet_status_t comet_w4ax_linear_host_async(comet_plan_t plan, const void* x_host, comet_dtype_t xdt,
+                                            const void* w_packed, const float* w_scales, void* y_host,
+                                            comet_dtype_t ydt, void* scratch, size_t scratch_bytes,
+                                            void* workspace, size_t ws_bytes, void* stream);
+/* Block until the downloads of the last comet_w4ax_linear_host(_async) call with `plan` are done. */
+comet_status_t comet_linear_host_wait(comet_plan_t plan);
 
 const char* comet_status_string(comet_status_t s);
 const char* comet_last_error(void);

@@ -89,6 +89,8 @@ def lib():
         "comet_w4ax_gemm": (I32, [P, P, P, P, P, P, I32, I64, P, P, P, SZ, P]),
         "comet_linear_scratch_bytes": (SZ, [P, I32, I32]),
         "comet_w4ax_linear_host": (I32, [P, P, I32, P, P, P, I32, P, SZ, P, SZ, P]),
+        "comet_w4ax_linear_host_async": (I32, [P, P, I32, P, P, P, I32, P, SZ, P, SZ, P]),
+        "comet_linear_host_wait": (I32, [P]),
         "comet_status_string": (ctypes.c_char_p, [I32]),
         "comet_last_error": (ctypes.c_char_p, []),
         "comet_version": (ctypes.c_char_p, []),
@@ -268,13 +270,21 @@ def linear_scratch_bytes(plan: Plan, xdt: int, ydt: int) -> int:
     return int(lib().comet_linear_scratch_bytes(plan.handle, xdt, ydt))
 
 
-def w4ax_linear_host(plan: Plan, x_host, w_packed, w_scales, y_host, scratch, *, stream=None):
-    """comet_w4ax_linear_host: host (pinned) x in, host y out; H2D, quantise, GEMM, D2H."""
+def w4ax_linear_host(plan: Plan, x_host, w_packed, w_scales, y_host, scratch, *, stream=None,
+                     blocking: bool = True):
+    """comet_w4ax_linear_host(_async): host (pinned) x in, host y out; H2D, quantise, GEMM, D2H
+    (chunk-pipelined over three streams for M >= 2048).  blocking=False returns at once: y_host
+    is complete after linear_host_wait(plan) (or a device synchronize)."""
     ws = plan.workspace(w_packed.device)
-    _check(lib().comet_w4ax_linear_host(plan.handle, ctypes.c_void_p(x_host.data_ptr()), _dt(x_host.dtype),
-                                        ctypes.c_void_p(w_packed.data_ptr()),
-                                        ctypes.c_void_p(w_scales.data_ptr()),
-                                        ctypes.c_void_p(y_host.data_ptr()), _dt(y_host.dtype),
-                                        ctypes.c_void_p(scratch.data_ptr()), scratch.numel(),
-                                        ctypes.c_void_p(ws.data_ptr()), ws.numel(), _stream(stream)))
+    fn = lib().comet_w4ax_linear_host if blocking else lib().comet_w4ax_linear_host_async
+    _check(fn(plan.handle, ctypes.c_void_p(x_host.data_ptr()), _dt(x_host.dtype),
+              ctypes.c_void_p(w_packed.data_ptr()), ctypes.c_void_p(w_scales.data_ptr()),
+              ctypes.c_void_p(y_host.data_ptr()), _dt(y_host.dtype),
+              ctypes.c_void_p(scratch.data_ptr()), scratch.numel(),
+              ctypes.c_void_p(ws.data_ptr()), ws.numel(), _stream(stream)))
     return y_host
+
+
+def linear_host_wait(plan: Plan):
+    """comet_linear_host_wait: block until the plan's last host-buffer call has landed in y_host."""
+    _check(lib().comet_linear_host_wait(plan.handle))

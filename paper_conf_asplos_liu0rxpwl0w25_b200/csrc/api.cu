@@ -8,6 +8,17 @@
 
 struct comet_plan_s {
   comet::Plan p;
+  comet_sched_config cfg{};          // as resolved at create time (sub-plans reuse it)
+  // comet_w4ax_linear_host pipeline: token chunks of kLinChunk rows, each with its own H2D copy,
+  // quantise + GEMM and D2H copy on three streams, so the PCIe transfers of neighbouring chunks
+  // overlap each other (full duplex) and the compute.  Created on first use.
+  comet_plan_s* chunk = nullptr;     // sub-plan, M = kLinChunk
+  comet_plan_s* tail = nullptr;      // sub-plan, M = M % kLinChunk (when nonzero)
+  cudaStream_t s_h2d = nullptr, s_d2h = nullptr;
+  std::vector<cudaEvent_t> ev;       // [3 per chunk]: H2D done, compute done, D2H done; + 2:
+                                     // last quantise of the previous call, its last D2H
+  bool prev_call = false;            // the two events above were recorded
+  void* ws_zeroed = nullptr;         // scratch address whose fix-up workspace was last zeroed
 };
 
 namespace comet {
@@ -220,12 +231,18 @@ comet_status_t comet_plan_create(int64_t M, int64_t N, int64_t K, const uint8_t*
     }
   }
   if (workspace_bytes) *workspace_bytes = p.ws_bytes;
+  h->cfg = cfg;
   *out = h;
   return COMET_OK;
 }
 
 comet_status_t comet_plan_destroy(comet_plan_t plan) {
   if (!plan) return COMET_OK;
+  if (plan->chunk) comet_plan_destroy(plan->chunk);
+  if (plan->tail) comet_plan_destroy(plan->tail);
+  for (cudaEvent_t e : plan->ev) cudaEventDestroy(e);
+  if (plan->s_h2d) cudaStreamDestroy(plan->s_h2d);
+  if (plan->s_d2h) cudaStreamDestroy(plan->s_d2h);
   if (plan->p.d_cta_begin) cudaFree(plan->p.d_cta_begin);
   if (plan->p.d_items) cudaFree(plan->p.d_items);
   delete plan;
@@ -293,57 +310,195 @@ comet_status_t comet_w4ax_gemm(comet_plan_t plan, const void* act_packed, const 
   return st;
 }
 
-static size_t scratch_layout(const Plan& p, comet_dtype_t xdt, comet_dtype_t ydt, size_t* x_off,
-                             size_t* act_off, size_t* sc_off, size_t* y_off) {
+// Pipelined host path: chunks of kLinChunk token rows once M >= 2 kLinChunk.
+static constexpr int64_t kLinChunk = 1024;
+
+static int64_t lin_chunks(const Plan& p) { return p.M >= 2 * kLinChunk ? ceil_div(p.M, kLinChunk) : 1; }
+
+// Sub-plans of the pipelined path (device plans, same scheduler configuration as the parent).
+static comet_status_t ensure_subplans(comet_plan_t plan) {
+  const Plan& p = plan->p;
+  if (lin_chunks(p) == 1 || plan->chunk) return COMET_OK;
+  comet_sched_config cfg = plan->cfg;
+  cfg.device_plan = 1;
+  comet_status_t st = comet_plan_create(kLinChunk, p.N, p.K, p.tags.data(), &cfg, &plan->chunk, nullptr);
+  if (st != COMET_OK) return st;
+  const int64_t rem = p.M % kLinChunk;
+  if (rem) {
+    st = comet_plan_create(rem, p.N, p.K, p.tags.data(), &cfg, &plan->tail, nullptr);
+    if (st != COMET_OK) return st;
+  }
+  return COMET_OK;
+}
+
+struct LinLayout {
+  size_t x_off, act_off, sc_off, y_off, ws_chunk_off, ws_tail_off, total;
+};
+
+// scratch: [x: M x K (16-bit)] [act packed: one chunk] [scales: one chunk] [y: M x N]
+//          [fix-up workspace of the chunk plan] [... of the tail plan]
+static LinLayout lin_layout(comet_plan_t plan, comet_dtype_t ydt) {
+  const Plan& p = plan->p;
+  const int64_t mc = lin_chunks(p) == 1 ? p.M : kLinChunk;
   comet_act_layout_t L;
-  act_layout(p.M, p.K, &L);
+  act_layout(mc, p.K, &L);
+  LinLayout o;
   size_t off = 0;
-  *x_off = off;
+  o.x_off = off;
   off += (size_t)round_up(p.M * p.K * 2, 256);
-  *act_off = off;
+  o.act_off = off;
   off += L.total_bytes;
-  *sc_off = off;
+  o.sc_off = off;
   off += (size_t)round_up((int64_t)(L.nb * L.Mp * 4), 256);
-  *y_off = off;
+  o.y_off = off;
   off += (size_t)round_up(p.M * p.N * (ydt == COMET_F32 ? 4 : 2), 256);
-  (void)xdt;
-  return off;
+  o.ws_chunk_off = off;
+  if (plan->chunk) off += (size_t)round_up((int64_t)plan->chunk->p.ws_bytes, 256);
+  o.ws_tail_off = off;
+  if (plan->tail) off += (size_t)round_up((int64_t)plan->tail->p.ws_bytes, 256);
+  o.total = off;
+  return o;
 }
 
 size_t comet_linear_scratch_bytes(comet_plan_t plan, comet_dtype_t xdt, comet_dtype_t ydt) {
+  (void)xdt;
   if (!plan) return 0;
-  size_t a, b, c, d;
-  return scratch_layout(plan->p, xdt, ydt, &a, &b, &c, &d);
+  if (ensure_subplans(plan) != COMET_OK) return 0;
+  return lin_layout(plan, ydt).total;
+}
+
+static comet_status_t linear_host(comet_plan_t plan, const void* x_host, comet_dtype_t xdt,
+                                  const void* w_packed, const float* w_scales, void* y_host,
+                                  comet_dtype_t ydt, void* scratch, size_t scratch_bytes,
+                                  void* workspace, size_t ws_bytes, void* stream, bool blocking) {
+  if (!plan || !x_host || !y_host || !scratch) return fail(COMET_ERR_INVALID_ARG, "NULL pointer argument");
+  if (xdt != COMET_F16 && xdt != COMET_BF16) return fail(COMET_ERR_INVALID_ARG, "xdt must be F16 or BF16");
+  Plan& p = plan->p;
+  comet_status_t st = ensure_subplans(plan);
+  if (st != COMET_OK) return st;
+  const LinLayout lay = lin_layout(plan, ydt);
+  if (scratch_bytes < lay.total) return fail(COMET_ERR_WORKSPACE_TOO_SMALL, "scratch smaller than comet_linear_scratch_bytes");
+  if ((reinterpret_cast<uintptr_t>(scratch) & 255u) != 0) return fail(COMET_ERR_MISALIGNED, "scratch must be 256-byte aligned");
+  uint8_t* s = static_cast<uint8_t*>(scratch);
+  cudaStream_t cs = static_cast<cudaStream_t>(stream);
+  const size_t esz = ydt == COMET_F32 ? 4 : 2;
+  const int64_t nch = lin_chunks(p);
+  cudaError_t e;
+  if (nch == 1) {
+    // one chunk: H2D, quantise, GEMM, D2H in order on `stream`
+    e = cudaMemcpyAsync(s + lay.x_off, x_host, (size_t)(p.M * p.K * 2), cudaMemcpyHostToDevice, cs);
+    if (e != cudaSuccess) return cuda_status(e, "H2D copy");
+    st = comet_quantize_act(s + lay.x_off, xdt, p.M, p.K, p.K, p.tags.data(), nullptr, s + lay.act_off,
+                            reinterpret_cast<float*>(s + lay.sc_off), stream);
+    if (st != COMET_OK) return st;
+    const int l1 = g_launches;
+    st = comet_w4ax_gemm(plan, s + lay.act_off, reinterpret_cast<float*>(s + lay.sc_off), w_packed, w_scales,
+                         s + lay.y_off, ydt, p.N, nullptr, nullptr, workspace, ws_bytes, stream);
+    if (st != COMET_OK) return st;
+    const int l2 = g_launches;
+    e = cudaMemcpyAsync(y_host, s + lay.y_off, (size_t)(p.M * p.N) * esz, cudaMemcpyDeviceToHost, cs);
+    if (e != cudaSuccess) return cuda_status(e, "D2H copy");
+    if (blocking) {
+      e = cudaStreamSynchronize(cs);
+      if (e != cudaSuccess) return cuda_status(e, "stream synchronize");
+    }
+    g_launches = l1 + l2;
+    return COMET_OK;
+  }
+  // pipelined.  Dependencies: chunk c's quantise + GEMM (on `stream`, so after the caller's prior
+  // work) wait for its H2D; its D2H waits for its GEMM.  Across calls with this plan: the H2D
+  // copies wait for the previous call's last quantise (the last reader of the scratch x region)
+  // and the first GEMM waits for the previous call's last D2H (the last reader of scratch y).
+  // Nothing else orders the copy streams, so one call's uploads overlap the previous call's
+  // downloads and compute.
+  if (!plan->s_h2d) {
+    e = cudaStreamCreateWithFlags(&plan->s_h2d, cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&plan->s_d2h, cudaStreamNonBlocking);
+    if (e != cudaSuccess) return cuda_status(e, "copy stream create");
+  }
+  while ((int64_t)plan->ev.size() < 3 * nch + 2) {
+    cudaEvent_t ev;
+    e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming);
+    if (e != cudaSuccess) return cuda_status(e, "event create");
+    plan->ev.push_back(ev);
+  }
+  cudaEvent_t ev_quant_last = plan->ev[3 * nch], ev_d2h_last = plan->ev[3 * nch + 1];
+  // zero the sub-plans' stream-K flag workspace the first time this scratch is used (flags are
+  // compared with per-plan epochs that start at 1)
+  if (plan->ws_zeroed != scratch) {
+    e = cudaMemsetAsync(s + lay.ws_chunk_off, 0, lay.total - lay.ws_chunk_off, cs);
+    if (e != cudaSuccess) return cuda_status(e, "workspace clear");
+    plan->ws_zeroed = scratch;
+  }
+  if (plan->prev_call) {
+    e = cudaStreamWaitEvent(plan->s_h2d, ev_quant_last, 0);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(cs, ev_d2h_last, 0);
+    if (e != cudaSuccess) return cuda_status(e, "stream ordering");
+  }
+  int launches = 0;
+  for (int64_t c = 0; c < nch; ++c) {
+    const int64_t m0 = c * kLinChunk, rows = std::min<int64_t>(kLinChunk, p.M - m0);
+    comet_plan_t sub = rows == kLinChunk ? plan->chunk : plan->tail;
+    uint8_t* ws = s + (rows == kLinChunk ? lay.ws_chunk_off : lay.ws_tail_off);
+    cudaEvent_t e_h2d = plan->ev[3 * c], e_comp = plan->ev[3 * c + 1];
+    e = cudaMemcpyAsync(s + lay.x_off + (size_t)(m0 * p.K * 2), static_cast<const uint8_t*>(x_host) + (size_t)(m0 * p.K * 2),
+                        (size_t)(rows * p.K * 2), cudaMemcpyHostToDevice, plan->s_h2d);
+    if (e == cudaSuccess) e = cudaEventRecord(e_h2d, plan->s_h2d);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(cs, e_h2d, 0);
+    if (e != cudaSuccess) return cuda_status(e, "H2D copy");
+    st = comet_quantize_act(s + lay.x_off + (size_t)(m0 * p.K * 2), xdt, rows, p.K, p.K, p.tags.data(), nullptr,
+                            s + lay.act_off, reinterpret_cast<float*>(s + lay.sc_off), stream);
+    if (st != COMET_OK) return st;
+    launches += g_launches;
+    if (c == nch - 1) {
+      e = cudaEventRecord(ev_quant_last, cs);
+      if (e != cudaSuccess) return cuda_status(e, "event record");
+    }
+    st = comet_w4ax_gemm(sub, s + lay.act_off, reinterpret_cast<float*>(s + lay.sc_off), w_packed, w_scales,
+                         s + lay.y_off + (size_t)(m0 * p.N) * esz, ydt, p.N, nullptr, nullptr, ws,
+                         sub->p.ws_bytes, stream);
+    if (st != COMET_OK) return st;
+    launches += g_launches;
+    e = cudaEventRecord(e_comp, cs);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(plan->s_d2h, e_comp, 0);
+    if (e == cudaSuccess)
+      e = cudaMemcpyAsync(static_cast<uint8_t*>(y_host) + (size_t)(m0 * p.N) * esz, s + lay.y_off + (size_t)(m0 * p.N) * esz,
+                          (size_t)(rows * p.N) * esz, cudaMemcpyDeviceToHost, plan->s_d2h);
+    if (e != cudaSuccess) return cuda_status(e, "D2H copy");
+  }
+  e = cudaEventRecord(ev_d2h_last, plan->s_d2h);
+  if (e != cudaSuccess) return cuda_status(e, "event record");
+  plan->prev_call = true;
+  if (blocking) {
+    e = cudaEventSynchronize(ev_d2h_last);
+    if (e != cudaSuccess) return cuda_status(e, "D2H synchronize");
+  }
+  g_launches = launches;
+  return COMET_OK;
+}
+
+comet_status_t comet_linear_host_wait(comet_plan_t plan) {
+  if (!plan) return fail(COMET_ERR_INVALID_ARG, "NULL plan");
+  if (lin_chunks(plan->p) == 1 || !plan->prev_call) return COMET_OK;
+  cudaError_t e = cudaEventSynchronize(plan->ev[3 * lin_chunks(plan->p) + 1]);
+  if (e != cudaSuccess) return cuda_status(e, "D2H synchronize");
+  return COMET_OK;
 }
 
 comet_status_t comet_w4ax_linear_host(comet_plan_t plan, const void* x_host, comet_dtype_t xdt,
                                       const void* w_packed, const float* w_scales, void* y_host,
                                       comet_dtype_t ydt, void* scratch, size_t scratch_bytes,
                                       void* workspace, size_t ws_bytes, void* stream) {
-  if (!plan || !x_host || !y_host || !scratch) return fail(COMET_ERR_INVALID_ARG, "NULL pointer argument");
-  Plan& p = plan->p;
-  size_t xo, ao, so, yo;
-  size_t need = scratch_layout(p, xdt, ydt, &xo, &ao, &so, &yo);
-  if (scratch_bytes < need) return fail(COMET_ERR_WORKSPACE_TOO_SMALL, "scratch smaller than comet_linear_scratch_bytes");
-  if ((reinterpret_cast<uintptr_t>(scratch) & 255u) != 0) return fail(COMET_ERR_MISALIGNED, "scratch must be 256-byte aligned");
-  uint8_t* s = static_cast<uint8_t*>(scratch);
-  cudaStream_t st_ = static_cast<cudaStream_t>(stream);
-  cudaError_t e = cudaMemcpyAsync(s + xo, x_host, (size_t)(p.M * p.K * 2), cudaMemcpyHostToDevice, st_);
-  if (e != cudaSuccess) return cuda_status(e, "H2D copy");
-  comet_status_t st = comet_quantize_act(s + xo, xdt, p.M, p.K, p.K, p.tags.data(), nullptr, s + ao,
-                                         reinterpret_cast<float*>(s + so), stream);
-  if (st != COMET_OK) return st;
-  int l1 = g_launches;
-  st = comet_w4ax_gemm(plan, s + ao, reinterpret_cast<float*>(s + so), w_packed, w_scales, s + yo, ydt,
-                       p.N, nullptr, nullptr, workspace, ws_bytes, stream);
-  if (st != COMET_OK) return st;
-  int l2 = g_launches;
-  e = cudaMemcpyAsync(y_host, s + yo, (size_t)(p.M * p.N * (ydt == COMET_F32 ? 4 : 2)), cudaMemcpyDeviceToHost, st_);
-  if (e != cudaSuccess) return cuda_status(e, "D2H copy");
-  e = cudaStreamSynchronize(st_);
-  if (e != cudaSuccess) return cuda_status(e, "stream synchronize");
-  g_launches = l1 + l2;
-  return COMET_OK;
+  return linear_host(plan, x_host, xdt, w_packed, w_scales, y_host, ydt, scratch, scratch_bytes, workspace,
+                     ws_bytes, stream, true);
+}
+
+comet_status_t comet_w4ax_linear_host_async(comet_plan_t plan, const void* x_host, comet_dtype_t xdt,
+                                            const void* w_packed, const float* w_scales, void* y_host,
+                                            comet_dtype_t ydt, void* scratch, size_t scratch_bytes,
+                                            void* workspace, size_t ws_bytes, void* stream) {
+  return linear_host(plan, x_host, xdt, w_packed, w_scales, y_host, ydt, scratch, scratch_bytes, workspace,
+                     ws_bytes, stream, false);
 }
 
 }  // extern "C"

@@ -237,6 +237,9 @@ FULL = [
     ("l3_70b_qkv_m4096", 4096, 8192, 10240, 0.05),
     ("l3_70b_gateup_tp8_m32", 32, 8192, 3584, 0.05),
     ("l3_70b_down_tp8_m1", 1, 3584, 8192, 0.05),
+    ("l3_70b_gateup_m1", 1, 8192, 28672, 0.05),      # config 5 (decode sweep of bench.py)
+    ("l3_70b_down_m8", 8, 28672, 8192, 0.05),
+    ("l3_70b_qkv_m32", 32, 8192, 10240, 0.05),
 ]
 
 
@@ -248,3 +251,27 @@ def test_gemm_full_size(name, M, K, N, frac):
     rows = synth.sample_rows(M, 8, p.x)
     yref, acc_sum, codes, scales = oracle.w4ax_rows(p.x, p.tags, p.w, p.s_w, rows)
     _close(y[torch.from_numpy(rows).to(DEV)], yref, torch.float16)
+
+
+# ------------------------------------------------------------------------------- host-buffer path
+
+@pytest.mark.parametrize("M,blocking", [(300, True), (2500, True), (2500, False), (4096, False)])
+def test_linear_host_pipeline(M, blocking):
+    """comet_w4ax_linear_host(_async): pinned host x in, host y out.  M >= 2048 runs the
+    1024-row chunk pipeline (three streams, sub-plans, ragged last chunk at 2500)."""
+    K, N = 1024, 384
+    p = synth.make_problem(M, K, N, frac=0.25, seed=M + 7)
+    wp = cb.pack_weight(torch.from_numpy(p.w).to(DEV))
+    sw = torch.from_numpy(p.s_w).to(DEV)
+    plan = cb.Plan(M, N, K, p.tags)
+    x_host = torch.from_numpy(p.x).pin_memory()
+    y_host = torch.full((M, N), float("nan"), dtype=torch.float16).pin_memory()
+    scratch = torch.empty(cb.linear_scratch_bytes(plan, cb.COMET_F16, cb.COMET_F16), dtype=torch.uint8, device=DEV)
+    for _ in range(2):          # second call reuses the scratch (stream-K flags, epochs)
+        y_host.fill_(float("nan"))
+        cb.w4ax_linear_host(plan, x_host, wp, sw, y_host, scratch, blocking=blocking)
+        if not blocking:
+            cb.linear_host_wait(plan)
+            torch.cuda.synchronize()
+        yref, _, _, _ = oracle.w4ax(p.x, p.tags, p.w, p.s_w)
+        _close(y_host, yref, torch.float16)
