@@ -32,7 +32,10 @@
 #define COMET_PRODUCERS 1   // TMA-issuing warps (2: K-blocks alternate between them)
 #endif
 #ifndef COMET_PROMO_SB
-#define COMET_PROMO_SB 0
+#define COMET_PROMO_SB 1    // single-buffered 32-column promotion batches when they fit
+#endif
+#ifndef COMET_WIDEN40
+#define COMET_WIDEN40 1     // widen warpgroups at 40 registers when promotion still fits
 #endif
 #ifndef COMET_NSUB
 #define COMET_NSUB 1   // 2: split each K-block's MMA into two sub-MMAs (experimental, slower)
@@ -77,7 +80,13 @@ struct CfgN {
   static constexpr bool LOADALL = COLS <= 120 && promo_regs(32) >= ACC_REGS + COLS + 24;
   static constexpr int NEED = LOADALL ? ACC_REGS + COLS + 24 : ACC_REGS + 2 * 16 + 24;
   static constexpr int REG_LOW = promo_regs(40) >= NEED ? 40 : 32;
-  static constexpr int REG_PROMO = promo_regs(REG_LOW);
+  // the widen warpgroups keep 40 registers (their loop state spills at 32) whenever the
+  // producer/MMA warpgroup at 32 still leaves promotion its working set
+  static constexpr int promo_regs2(int low0, int loww) {
+    return ((REG_POOL - low0 - loww * NWG) / NPW / 8) * 8 > 248 ? 248 : ((REG_POOL - low0 - loww * NWG) / NPW / 8) * 8;
+  }
+  static constexpr int REG_WIDEN = (REG_LOW == 32 && COMET_WIDEN40 && promo_regs2(32, 40) >= NEED) ? 40 : REG_LOW;
+  static constexpr int REG_PROMO = promo_regs2(REG_LOW, REG_WIDEN);
   // SB: single-buffered 32-column batches (fewer, larger TMEM loads in flight) when the
   // double-buffered 32-column form does not fit (variant experiments: COMET_PROMO_SB)
   static constexpr bool SB = !LOADALL && COMET_PROMO_SB && REG_PROMO < ACC_REGS + 2 * 32 + 24 &&
@@ -277,7 +286,7 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
       }
     }
   } else if (warp < kPromoWarp0) {
-    setmaxnreg_dec<C::REG_LOW>();
+    setmaxnreg_dec<C::REG_WIDEN>();
     // -------------------------------------------------------------------- widen (W -> smem B)
     // The NWG widen warpgroups take K-blocks in turn; thread t of a group converts weight rows
     // t, t + 128, ... of its K-blocks.  INT4 block: byte = u (E4M3 u * 2^-9); INT8 block:
