@@ -418,6 +418,7 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
           tc_fence_before();
           __syncwarp();
           if (lane == 0) mbar_arrive_cluster(ready_rel + rs * 8);
+          if (threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 7, tr);
           ++tr;
           if (++accb == NACC) { accb = 0; accph ^= 1; }
           if (++sc == SS) sc = 0;
@@ -441,10 +442,12 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
             uint32_t v[PB];
             tmem_ld_32x32b<PB>(taddr + b * PB, v);
             tmem_wait_ld();
+            if (b == 0 && threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 9, tr);
             if (b + 1 == NB_) {
               tc_fence_before();
               __syncwarp();
               if (lane == 0) mbar_arrive_cluster(ready_rel + rs * 8);
+              if (threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 10, tr);
             }
             if (is8) {
 #pragma unroll
@@ -459,6 +462,7 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
               acc[a + 1] = y.y;
             }
           }
+          if (threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 7, tr);
           ++tr;
           if (++accb == NACC) { accb = 0; accph ^= 1; }
           if (++sc == SS) sc = 0;
