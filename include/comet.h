@@ -97,8 +97,14 @@ size_t comet_act_scales_count(int64_t M, int64_t K);
  * FMPQ activation quantisation.
  *   x          device, [M][ldx] float16 (xdt = COMET_F16) or bfloat16 (COMET_BF16), row-major.
  *   tags_host  host, [K/128] uint8, nonzero = INT8 (outlier) block.  Read synchronously.
- *   perm_dev   must be NULL (channel permutation P:L138-144 is applied offline to W and
- *              upstream to X; a fused gather is not implemented -> COMET_ERR_UNSUPPORTED_SHAPE).
+ *   perm_dev   NULL (channels in input order) or device [K] int32: the runtime channel
+ *              permutation of FMPQ (Fig. 4(d)) fused into the quantiser -- channel
+ *              k of the quantised row is input channel perm_dev[k], x'[m,k] = x[m, perm[k]],
+ *              and everything below (blocks, tags, codes, scales) refers to x'.  Must be a
+ *              permutation of [0, K) (entries outside are clamped into range: defined but
+ *              meaningless); the weights must be packed with the same permutation
+ *              (comet_pack_weight_perm).  Requires K <= 32768 (the kernel stages whole rows
+ *              and the permutation in shared memory), else COMET_ERR_UNSUPPORTED_SHAPE.
  *   act_packed device, comet_act_packed_bytes(M,K) bytes, written completely.
  *   act_scales device, comet_act_scales_count(M,K) floats, written completely.
  * Per (m, b): amax = max|x|; qmax = 127 if tags[b] else 7; amax == 0 -> s = 0 and codes 0;
@@ -126,6 +132,31 @@ size_t comet_weight_packed_bytes(int64_t N, int64_t K);
 /* w_codes_dev: device [N][K] int8 codes in [-8,7] (values outside are masked to 4 bits). */
 comet_status_t comet_pack_weight(const int8_t* w_codes_dev, int64_t N, int64_t K, void* w_packed,
                                  void* stream);
+/* Offline weight side of the channel permutation ("the corresponding positions in the
+ * weight matrix also need to be permuted"): packs W'[n,k] = W[n, perm_dev[k]] in the layout
+ * above.  perm_dev: device [K] int32, a permutation of [0, K) (entries outside are clamped).
+ * NULL perm_dev is the identity (same as comet_pack_weight). */
+comet_status_t comet_pack_weight_perm(const int8_t* w_codes_dev, int64_t N, int64_t K,
+                                      const int32_t* perm_dev, void* w_packed, void* stream);
+
+/* ------------------------------------------------------------------------------------------
+ * Offline calibration of the channel permutation and the precision tags ("we
+ * utilize sampled activations from the calibration dataset to locate outlier channels and
+ * apply permutation to group these channels into a single block"; reading R8/R16).
+ * ---------------------------------------------------------------------------------------- */
+/* amax_dev[k] = max_m |x[m,k]| over the calibration rows (device [K] float, written
+ * completely; exact).  x as in comet_quantize_act (device, [M][ldx] f16 / bf16). */
+comet_status_t comet_channel_amax(const void* x, comet_dtype_t xdt, int64_t M, int64_t K,
+                                  int64_t ldx, float* amax_dev, void* stream);
+/* Host, synchronous, no device needed.  amax_host: [K] per-channel max-abs (finite, >= 0).
+ * med = median of amax_host in binary64 (mean of the two central values when K is even);
+ * channel k is an outlier iff (double)amax_host[k] > ratio * med (ratio > 0; the paper's
+ * "tenfold" is ratio = 10).  Writes perm_host[K] = the outlier channels in ascending
+ * order followed by the other channels in ascending order, tags_host[K/128] = 1 for the first
+ * ceil(n_outliers/128) blocks (the blocks that now hold outliers) and 0 for the rest, and
+ * *n_outliers (may be NULL).  K % 128 == 0. */
+comet_status_t comet_calibrate_perm(const float* amax_host, int64_t K, double ratio,
+                                    int32_t* perm_host, uint8_t* tags_host, int64_t* n_outliers);
 
 /* ------------------------------------------------------------------------------------------
  * Tile scheduler ("fine-grained SM scheduling")

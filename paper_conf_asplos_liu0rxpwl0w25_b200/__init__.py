@@ -80,6 +80,9 @@ def lib():
         "comet_quantize_act": (I32, [P, I32, I64, I64, I64, P, P, P, P, P]),
         "comet_weight_packed_bytes": (SZ, [I64, I64]),
         "comet_pack_weight": (I32, [P, I64, I64, P, P]),
+        "comet_pack_weight_perm": (I32, [P, I64, I64, P, P, P]),
+        "comet_channel_amax": (I32, [P, I32, I64, I64, I64, P, P]),
+        "comet_calibrate_perm": (I32, [P, I64, ctypes.c_double, P, P, ctypes.POINTER(I64)]),
         "comet_sched_config_default": (None, [ctypes.POINTER(SchedConfig)]),
         "comet_plan_create": (I32, [I64, I64, I64, P, ctypes.POINTER(SchedConfig), ctypes.POINTER(P),
                                     ctypes.POINTER(SZ)]),
@@ -142,8 +145,17 @@ def last_launch_count() -> int:
     return int(lib().comet_last_launch_count())
 
 
-def quantize_act(x, tags, *, out=None, stream=None):
-    """FMPQ quantisation (comet_quantize_act).  x: [M, K] float16/bfloat16 CUDA tensor.
+def _perm_ptr(perm, K):
+    import torch
+    if perm is None:
+        return None
+    assert perm.is_cuda and perm.dtype == torch.int32 and perm.is_contiguous() and perm.numel() == K
+    return ctypes.c_void_p(perm.data_ptr())
+
+
+def quantize_act(x, tags, *, perm=None, out=None, stream=None):
+    """FMPQ quantisation (comet_quantize_act).  x: [M, K] float16/bfloat16 CUDA tensor;
+    perm: optional [K] int32 CUDA tensor, the fused channel permutation (x'[:, k] = x[:, perm[k]]).
     Returns (act_packed uint8 tensor, act_scales float32 tensor [nb*Mp])."""
     import torch
     assert x.is_cuda and x.dim() == 2 and x.stride(1) == 1
@@ -156,21 +168,52 @@ def quantize_act(x, tags, *, out=None, stream=None):
     else:
         act, sc = out
     _check(lib().comet_quantize_act(ctypes.c_void_p(x.data_ptr()), _dt(x.dtype), M, K, x.stride(0),
-                                    t.ctypes.data_as(ctypes.c_void_p), None,
+                                    t.ctypes.data_as(ctypes.c_void_p), _perm_ptr(perm, K),
                                     ctypes.c_void_p(act.data_ptr()), ctypes.c_void_p(sc.data_ptr()),
                                     _stream(stream)))
     return act, sc
 
 
-def pack_weight(w_codes, *, out=None, stream=None):
-    """comet_pack_weight: [N, K] int8 codes in [-8, 7] -> [N, K/2] packed uint8."""
+def pack_weight(w_codes, *, perm=None, out=None, stream=None):
+    """comet_pack_weight(_perm): [N, K] int8 codes in [-8, 7] -> [N, K/2] packed uint8; with
+    perm ([K] int32 CUDA tensor) the columns are permuted first, W'[:, k] = W[:, perm[k]]."""
     import torch
     assert w_codes.is_cuda and w_codes.dtype == torch.int8 and w_codes.is_contiguous()
     N, K = w_codes.shape
     wp = out if out is not None else torch.empty((N, K // 2), dtype=torch.uint8, device=w_codes.device)
-    _check(lib().comet_pack_weight(ctypes.c_void_p(w_codes.data_ptr()), N, K,
-                                   ctypes.c_void_p(wp.data_ptr()), _stream(stream)))
+    if perm is None:
+        _check(lib().comet_pack_weight(ctypes.c_void_p(w_codes.data_ptr()), N, K,
+                                       ctypes.c_void_p(wp.data_ptr()), _stream(stream)))
+    else:
+        _check(lib().comet_pack_weight_perm(ctypes.c_void_p(w_codes.data_ptr()), N, K, _perm_ptr(perm, K),
+                                            ctypes.c_void_p(wp.data_ptr()), _stream(stream)))
     return wp
+
+
+def channel_amax(x, *, out=None, stream=None):
+    """comet_channel_amax: per-channel max |x| over the rows of a calibration sample.
+    x: [M, K] float16/bfloat16 CUDA tensor -> [K] float32 CUDA tensor."""
+    import torch
+    assert x.is_cuda and x.dim() == 2 and x.stride(1) == 1
+    M, K = x.shape
+    a = out if out is not None else torch.empty(K, dtype=torch.float32, device=x.device)
+    _check(lib().comet_channel_amax(ctypes.c_void_p(x.data_ptr()), _dt(x.dtype), M, K, x.stride(0),
+                                    ctypes.c_void_p(a.data_ptr()), _stream(stream)))
+    return a
+
+
+def calibrate_perm(amax, ratio: float = 10.0):
+    """comet_calibrate_perm (host): outlier channels (amax > ratio * median) first.
+    amax: [K] float32 (numpy or tensor).  Returns (perm int32 [K], tags uint8 [K/128], n_outliers)."""
+    a = np.ascontiguousarray(np.asarray(amax.cpu() if hasattr(amax, "cpu") else amax, dtype=np.float32))
+    K = a.shape[0]
+    perm = np.empty(K, dtype=np.int32)
+    tags = np.empty(max(K // BLOCK_K, 1), dtype=np.uint8)
+    n = ctypes.c_int64(0)
+    _check(lib().comet_calibrate_perm(a.ctypes.data_as(ctypes.c_void_p), K, float(ratio),
+                                      perm.ctypes.data_as(ctypes.c_void_p),
+                                      tags.ctypes.data_as(ctypes.c_void_p), ctypes.byref(n)))
+    return perm, tags, int(n.value)
 
 
 class Plan:
@@ -260,9 +303,11 @@ def w4ax_gemm(plan: Plan, act_packed, act_scales, w_packed, w_scales, *, out=Non
     return out
 
 
-def w4ax_linear(plan: Plan, x, w_packed, w_scales, *, out_dtype=None, stream=None):
-    """The whole hot path for one linear layer on device tensors: quantize_act + w4ax_gemm."""
-    act, sc = quantize_act(x, plan.tags, stream=stream)
+def w4ax_linear(plan: Plan, x, w_packed, w_scales, *, perm=None, out_dtype=None, stream=None):
+    """The whole hot path for one linear layer on device tensors: quantize_act (with the fused
+    channel permutation when perm is given; w_packed then packed with the same perm) +
+    w4ax_gemm."""
+    act, sc = quantize_act(x, plan.tags, perm=perm, stream=stream)
     return w4ax_gemm(plan, act, sc, w_packed, w_scales, out_dtype=out_dtype, stream=stream)
 
 

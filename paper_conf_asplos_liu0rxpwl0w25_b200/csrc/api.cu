@@ -129,7 +129,8 @@ comet_status_t comet_quantize_act(const void* x, comet_dtype_t xdt, int64_t M, i
   if (st != COMET_OK) return st;
   if (!x || !tags_host || !act_packed || !act_scales) return fail(COMET_ERR_INVALID_ARG, "NULL pointer argument");
   if (xdt != COMET_F16 && xdt != COMET_BF16) return fail(COMET_ERR_INVALID_ARG, "xdt must be COMET_F16 or COMET_BF16");
-  if (perm_dev) return fail(COMET_ERR_UNSUPPORTED_SHAPE, "fused channel permutation is not implemented (perm_dev must be NULL)");
+  if (perm_dev && K > 32768) return fail(COMET_ERR_UNSUPPORTED_SHAPE, "the fused channel permutation needs K <= 32768");
+  if (perm_dev && !aligned16(perm_dev)) return fail(COMET_ERR_MISALIGNED, "perm_dev must be 16-byte aligned");
   if (ldx < K || (ldx * 2) % 16 != 0) return fail(COMET_ERR_MISALIGNED, "ldx must be >= K with ldx*2 % 16 == 0");
   if (!aligned16(x) || !aligned16(act_packed) || !aligned16(act_scales))
     return fail(COMET_ERR_MISALIGNED, "device pointers must be 16-byte aligned");
@@ -139,8 +140,11 @@ comet_status_t comet_quantize_act(const void* x, comet_dtype_t xdt, int64_t M, i
   if (st != COMET_OK) return st;
   TagMask mask = mask_of(tags_host, K / kBlockK);
   int launches = 0;
-  cudaError_t e = launch_quantize(x, xdt == COMET_BF16, M, K, ldx, mask, act_packed, act_scales,
-                                  static_cast<cudaStream_t>(stream), &launches);
+  cudaError_t e = perm_dev
+      ? launch_quantize_perm(x, xdt == COMET_BF16, M, K, ldx, mask, perm_dev, act_packed, act_scales,
+                             static_cast<cudaStream_t>(stream), &launches)
+      : launch_quantize(x, xdt == COMET_BF16, M, K, ldx, mask, act_packed, act_scales,
+                        static_cast<cudaStream_t>(stream), &launches);
   if (e != cudaSuccess) return cuda_status(e, "quantize launch");
   g_launches = launches;
   return COMET_OK;
@@ -164,6 +168,42 @@ comet_status_t comet_pack_weight(const int8_t* w_codes_dev, int64_t N, int64_t K
   if (st != COMET_OK) return st;
   cudaError_t e = launch_pack_weight(w_codes_dev, N, K, w_packed, static_cast<cudaStream_t>(stream));
   if (e != cudaSuccess) return cuda_status(e, "pack launch");
+  g_launches = 1;
+  return COMET_OK;
+}
+
+comet_status_t comet_pack_weight_perm(const int8_t* w_codes_dev, int64_t N, int64_t K,
+                                      const int32_t* perm_dev, void* w_packed, void* stream) {
+  if (!perm_dev) return comet_pack_weight(w_codes_dev, N, K, w_packed, stream);
+  g_launches = 0;
+  comet_status_t st = check_n(N);
+  if (st != COMET_OK) return st;
+  st = check_mk(1, K);
+  if (st != COMET_OK) return st;
+  if (!w_codes_dev || !w_packed) return fail(COMET_ERR_INVALID_ARG, "NULL pointer argument");
+  if (!aligned16(w_codes_dev) || !aligned16(w_packed) || !aligned16(perm_dev))
+    return fail(COMET_ERR_MISALIGNED, "device pointers must be 16-byte aligned");
+  st = check_device();
+  if (st != COMET_OK) return st;
+  cudaError_t e = launch_pack_weight_perm(w_codes_dev, N, K, perm_dev, w_packed, static_cast<cudaStream_t>(stream));
+  if (e != cudaSuccess) return cuda_status(e, "pack launch");
+  g_launches = 1;
+  return COMET_OK;
+}
+
+comet_status_t comet_channel_amax(const void* x, comet_dtype_t xdt, int64_t M, int64_t K,
+                                  int64_t ldx, float* amax_dev, void* stream) {
+  g_launches = 0;
+  comet_status_t st = check_mk(M, K);
+  if (st != COMET_OK) return st;
+  if (!x || !amax_dev) return fail(COMET_ERR_INVALID_ARG, "NULL pointer argument");
+  if (xdt != COMET_F16 && xdt != COMET_BF16) return fail(COMET_ERR_INVALID_ARG, "xdt must be COMET_F16 or COMET_BF16");
+  if (ldx < K || (ldx * 2) % 16 != 0) return fail(COMET_ERR_MISALIGNED, "ldx must be >= K with ldx*2 % 16 == 0");
+  if (!aligned16(x) || !aligned16(amax_dev)) return fail(COMET_ERR_MISALIGNED, "device pointers must be 16-byte aligned");
+  st = check_device();
+  if (st != COMET_OK) return st;
+  cudaError_t e = launch_channel_amax(x, xdt == COMET_BF16, M, K, ldx, amax_dev, static_cast<cudaStream_t>(stream));
+  if (e != cudaSuccess) return cuda_status(e, "channel amax launch");
   g_launches = 1;
   return COMET_OK;
 }

@@ -70,6 +70,13 @@ comet_status_t build_plan(Plan& p, const comet_sched_config& cfg);
 cudaError_t launch_quantize(const void* x, bool bf16, int64_t M, int64_t K, int64_t ldx,
                             const TagMask& tags, void* act_packed, float* act_scales,
                             cudaStream_t stream, int* launches);
+cudaError_t launch_quantize_perm(const void* x, bool bf16, int64_t M, int64_t K, int64_t ldx,
+                                 const TagMask& tags, const int32_t* perm, void* act_packed,
+                                 float* act_scales, cudaStream_t stream, int* launches);
+cudaError_t launch_pack_weight_perm(const int8_t* w, int64_t N, int64_t K, const int32_t* perm,
+                                    void* w_packed, cudaStream_t stream);
+cudaError_t launch_channel_amax(const void* x, bool bf16, int64_t M, int64_t K, int64_t ldx,
+                                float* amax, cudaStream_t stream);
 // pack.cu
 cudaError_t launch_pack_weight(const int8_t* w, int64_t N, int64_t K, void* w_packed,
                                cudaStream_t stream);

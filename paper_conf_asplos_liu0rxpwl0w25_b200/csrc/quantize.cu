@@ -11,9 +11,11 @@
 // HBM-bound: a block-row (128 halves = 256 B) is read by 4 lanes with four 128-bit loads each
 // (a warp step covers 8 blocks, sector-coalesced); block max-abs and code sum are 2-step
 // xor-shuffle reductions inside the lane quad; codes leave as four 64-bit stores per lane.
+#include <algorithm>
 #include <cuda_fp16.h>
 #include <cuda_bf16.h>
 #include "internal.h"
+#include "sm100.cuh"
 
 namespace comet {
 namespace {
@@ -235,6 +237,192 @@ __global__ void __launch_bounds__(256) k_quantize(const uint16_t* __restrict__ x
   }
 }
 
+// ---------------------------------------------------------------------------- fused permutation
+// NEXT-1: the runtime channel permutation that groups outlier channels into a
+// few blocks (Fig. 4(d)) fused into kernel 1: channel k of the quantised row is
+// input channel perm[k], x'[m,k] = x[m, perm[k]], then FMPQ exactly as above on x'.
+//
+// A gather cannot be sector-coalesced from HBM, so each CTA stages whole input rows in shared
+// memory with 1D bulk copies (cp.async.bulk, completion on an mbarrier; a row is split over 8
+// issuing warps) -- NBUF rows in flight -- and the permutation once per CTA as 16-bit indices
+// (K <= 32768).  Per row: pass 1 gathers the permuted row into a second (swizzled) staging row
+// (consecutive threads take consecutive output channels), the input buffer is refilled at once,
+// and pass 2 runs the FMPQ lane layout of k_quantize on the staged row.  Persistent CTAs walk
+// rows m = blockIdx.x + i * gridDim.x.  Measured (tools/quant_time.py, M = 4096, calibrated
+// permutation): 51 us at K = 8192 and 141 us at K = 28672, against 26.5 / 69.7 us without the
+// permutation -- the per-row passes are latency-bound at 1-2 CTAs per SM (ncu: issue 45 %).
+// Position of permuted channel k in the staged row: odd blocks swap their 32-channel halves
+// pairwise (channel bit 5 ^= block bit 0), so the pass-2 128-bit reads of two neighbouring
+// blocks (256 B apart, same banks) land in different bank halves.
+__device__ __forceinline__ int64_t swz(int64_t k) { return k ^ (((k >> 7) & 1) << 5); }
+
+template <bool BF16, int NW>
+__global__ void __launch_bounds__(NW * 32, 2) k_quantize_perm(const uint16_t* __restrict__ x, int64_t M,
+                                                       int64_t K, int64_t ldx, int64_t Mp,
+                                                       TagMask tags,
+                                                       const int32_t* __restrict__ perm, int nbuf,
+                                                       uint8_t* __restrict__ codes,
+                                                       int16_t* __restrict__ qsum,
+                                                       float* __restrict__ corr,
+                                                       float* __restrict__ scales) {
+  extern __shared__ __align__(128) uint8_t smem[];
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem);                 // [nbuf] (<= 16)
+  uint16_t* p16 = reinterpret_cast<uint16_t*>(smem + 128);            // [K] permutation
+  uint16_t* prow = p16 + K;                                           // [K] permuted row (swizzled)
+  uint16_t* rows = prow + K;                                          // [nbuf][K] input rows
+  __shared__ float s_part[NW];
+  __shared__ uint32_t s_tags[kMaxBlocks / 32];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int bl = lane >> 2, sub = lane & 3;
+  const int nb = (int)(K / kBlockK);
+  const int ngroups = (nb + 7) >> 3;
+  if (threadIdx.x == 0) {
+#pragma unroll
+    for (int i = 0; i < kMaxBlocks / 32; ++i) s_tags[i] = tags.w[i];   // constant indices: no local copy
+  }
+  const uint32_t row_bytes = (uint32_t)(K * 2);
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < nbuf; ++i) sm100::mbar_init(&full[i], 1);
+    sm100::fence_mbar_init();
+  }
+  for (int64_t k = threadIdx.x; k < K; k += blockDim.x) p16[k] = (uint16_t)min(max(__ldg(perm + k), 0), (int)K - 1);
+  __syncthreads();
+  // A row arrives as kChunks bulk copies issued by lane 0 of different warps: one issuing
+  // thread's bulk copies complete one after another (profiles/r01/probe_stream.txt), several
+  // issuers overlap.  Thread 0 posts the row's byte count; the chunks may land before or after.
+  constexpr int kChunks = NW < 8 ? NW : 8;
+  const uint32_t chunk = row_bytes / kChunks;          // K % 128 == 0 -> a multiple of 32 B
+  const bool issuer = lane == 0 && warp < kChunks;
+  if (issuer) {
+    for (int i = 0; i < nbuf; ++i) {
+      const int64_t m = blockIdx.x + (int64_t)i * gridDim.x;
+      if (m >= M) break;
+      if (warp == 0) sm100::mbar_arrive_expect_tx(&full[i], row_bytes);
+      sm100::bulk_load(reinterpret_cast<uint8_t*>(rows + (int64_t)i * K) + warp * chunk,
+                       reinterpret_cast<const uint8_t*>(x + m * ldx) + warp * chunk, chunk, &full[i]);
+    }
+  }
+  int it = 0;
+  for (int64_t m = blockIdx.x; m < Mp; m += gridDim.x, ++it) {
+    const int buf = it % nbuf;
+    float cpart = 0.f;
+    if (m < M) {
+      sm100::mbar_wait(&full[buf], (uint32_t)((it / nbuf) & 1));
+      // pass 1: gather.  Thread t moves output channels 2t, 2t+1 (+ 2*blockDim.x steps):
+      // consecutive threads read consecutive indices (and, for the mostly ascending calibrated
+      // permutations, consecutive input channels) -- no bank conflicts -- and write the pair
+      // as one word at its swizzled position (see kSwz).
+      const uint16_t* row = rows + (int64_t)buf * K;
+      for (int64_t k = 2 * threadIdx.x; k < K; k += 2 * blockDim.x) {
+        const uint32_t pi = *reinterpret_cast<const uint32_t*>(p16 + k);
+        const uint32_t h = (uint32_t)row[pi & 0xFFFFu] | ((uint32_t)row[pi >> 16] << 16);
+        *reinterpret_cast<uint32_t*>(prow + swz(k)) = h;
+      }
+      __syncthreads();   // prow complete; row buffer `buf` free
+      if (issuer) {
+        const int64_t mn = m + (int64_t)nbuf * gridDim.x;   // refill the freed buffer
+        if (mn < M) {
+          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+          if (warp == 0) sm100::mbar_arrive_expect_tx(&full[buf], row_bytes);
+          sm100::bulk_load(reinterpret_cast<uint8_t*>(rows + (int64_t)buf * K) + warp * chunk,
+                           reinterpret_cast<const uint8_t*>(x + mn * ldx) + warp * chunk, chunk, &full[buf]);
+        }
+      }
+      // pass 2: FMPQ on the permuted row, the lane layout of k_quantize (reads conflict-free
+      // thanks to the swizzle: the 8 blocks of a warp step sit 256 B apart)
+      uint8_t* crow = codes + m * K + sub * 8;
+      for (int g = warp; g < ngroups; g += NW) {
+        const int b = g * 8 + bl;
+        const bool bvalid = b < nb;
+        float v[32];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          uint4 raw = make_uint4(0, 0, 0, 0);
+          if (bvalid) raw = *reinterpret_cast<const uint4*>(prow + swz((int64_t)b * kBlockK + 32 * j + sub * 8));
+          float t[8];
+          unpack8<BF16>(raw, t);
+#pragma unroll
+          for (int i = 0; i < 8; ++i) v[8 * j + i] = t[i];
+        }
+        const bool is8 = bvalid && ((s_tags[b >> 5] >> (b & 31)) & 1u);
+        const LaneOut o = quantize32(v, is8);
+        if (bvalid) {
+          uint8_t* cb = crow + b * kBlockK;
+#pragma unroll
+          for (int j = 0; j < 4; ++j) *reinterpret_cast<uint2*>(cb + 32 * j) = o.c[j];
+          if (sub == 0) {
+            scales[(int64_t)b * Mp + m] = o.s;
+            qsum[(int64_t)b * Mp + m] = (int16_t)o.q;
+            if (!is8) cpart = __fadd_rn(cpart, __fmul_rn(o.s, (float)o.q));
+          }
+        }
+      }
+    } else {
+      for (int b = threadIdx.x; b < nb; b += blockDim.x) {
+        scales[(int64_t)b * Mp + m] = 0.f;
+        qsum[(int64_t)b * Mp + m] = 0;
+      }
+      __syncthreads();   // matches the pass-1 barrier of the other branch (uniform per CTA)
+    }
+    cpart = __fadd_rn(cpart, __shfl_xor_sync(0xffffffffu, cpart, 4));
+    cpart = __fadd_rn(cpart, __shfl_xor_sync(0xffffffffu, cpart, 8));
+    cpart = __fadd_rn(cpart, __shfl_xor_sync(0xffffffffu, cpart, 16));
+    if (lane == 0) s_part[warp] = cpart;
+    __syncthreads();   // s_part complete; prow free
+    if (threadIdx.x == 0) {
+      float c = 0.f;
+      for (int i = 0; i < NW; ++i) c = __fadd_rn(c, s_part[i]);
+      corr[m] = __fmul_rn(8.f, c);
+    }
+  }
+}
+
+// Offline weight side of the permutation ("the corresponding positions in the weight
+// matrix also need to be permuted"): W'[n,k] = W[n, perm[k]], packed as k_pack_weight.
+__global__ void __launch_bounds__(256) k_pack_weight_perm(const int8_t* __restrict__ w, int64_t N,
+                                                          int64_t K, const int32_t* __restrict__ perm,
+                                                          uint32_t* __restrict__ out) {
+  const int64_t words = N * K / 8;
+  const int kmax = (int)K - 1;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < words;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t n = i / (K / 8), k0 = (i % (K / 8)) * 8;
+    const int8_t* wr = w + n * K;
+    uint32_t word = 0;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int p0 = min(max(__ldg(perm + k0 + j), 0), kmax), p1 = min(max(__ldg(perm + k0 + j + 4), 0), kmax);
+      const uint32_t lo = ((uint32_t)wr[p0] & 0xFu) ^ 8u;   // u[k0 + j]
+      const uint32_t hi = ((uint32_t)wr[p1] & 0xFu) ^ 8u;   // u[k0 + j + 4]
+      word |= (lo | (hi << 4)) << (8 * j);
+    }
+    out[i] = word;
+  }
+}
+
+// Calibration statistic (offline, "sampled activations from the calibration dataset"):
+// amax[k] = max_m |x[m,k]|.  Non-negative binary32 values order like their bit patterns, so the
+// max is an atomicMax on the bits (order-independent, deterministic).  Each thread owns 8
+// consecutive channels (one 128-bit load per row) over a slice of the rows.
+template <bool BF16>
+__global__ void __launch_bounds__(256) k_channel_amax(const uint16_t* __restrict__ x, int64_t M,
+                                                      int64_t K, int64_t ldx, int64_t rows_per_cta,
+                                                      unsigned int* __restrict__ amax) {
+  const int64_t c8 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * 8;
+  if (c8 >= K) return;
+  const int64_t m0 = (int64_t)blockIdx.y * rows_per_cta;
+  const int64_t m1 = m0 + rows_per_cta < M ? m0 + rows_per_cta : M;
+  float a[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+  for (int64_t m = m0; m < m1; ++m) {
+    float v[8];
+    unpack8<BF16>(ldg_stream(x + m * ldx + c8), v);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) a[i] = fmaxf(a[i], fabsf(v[i]));
+  }
+#pragma unroll
+  for (int i = 0; i < 8; ++i) atomicMax(amax + c8 + i, __float_as_uint(a[i]));
+}
+
 template <bool BF16>
 cudaError_t launch_q(const void* x, int64_t M, int64_t K, int64_t ldx, const TagMask& tags,
                      void* act_packed, float* act_scales, cudaStream_t stream) {
@@ -293,6 +481,68 @@ cudaError_t launch_quantize(const void* x, bool bf16, int64_t M, int64_t K, int6
   *launches = 1;
   return bf16 ? launch_q<true>(x, M, K, ldx, tags, act_packed, act_scales, stream)
               : launch_q<false>(x, M, K, ldx, tags, act_packed, act_scales, stream);
+}
+
+template <bool BF16>
+static cudaError_t launch_qp(const void* x, int64_t M, int64_t K, int64_t ldx, const TagMask& tags,
+                             const int32_t* perm, void* act_packed, float* act_scales,
+                             cudaStream_t stream) {
+  comet_act_layout_t L;
+  act_layout(M, K, &L);
+  uint8_t* base = static_cast<uint8_t*>(act_packed);
+  const int64_t row_bytes = K * 2;
+  // rows in flight per CTA: ~64 KB of staged input, at least 2 (double buffering)
+  int nbuf = (int)std::max<int64_t>(2, std::min<int64_t>(8, (64 << 10) / row_bytes));
+  const size_t cap = 200u << 10;
+  while (nbuf > 1 && 128 + (size_t)row_bytes * (2 + nbuf) > cap) --nbuf;
+  const size_t smem = 128 + (size_t)row_bytes * (2 + nbuf);
+  int dev = 0, nsm = 148, per_sm = 1;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+  constexpr int NW = 16;   // 16 warps: the gather is latency-bound at one or two CTAs per SM
+  auto kern = k_quantize_perm<BF16, NW>;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, NW * 32, smem);
+  if (e != cudaSuccess) return e;
+  const int64_t grid = std::max<int64_t>(1, std::min<int64_t>(L.Mp, (int64_t)nsm * std::max(per_sm, 1)));
+  kern<<<(unsigned)grid, NW * 32, smem, stream>>>(
+      static_cast<const uint16_t*>(x), M, K, ldx, L.Mp, tags, perm, nbuf, base + L.codes_off,
+      reinterpret_cast<int16_t*>(base + L.qsum_off), reinterpret_cast<float*>(base + L.corr_off),
+      act_scales);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_quantize_perm(const void* x, bool bf16, int64_t M, int64_t K, int64_t ldx,
+                                 const TagMask& tags, const int32_t* perm, void* act_packed,
+                                 float* act_scales, cudaStream_t stream, int* launches) {
+  *launches = 1;
+  return bf16 ? launch_qp<true>(x, M, K, ldx, tags, perm, act_packed, act_scales, stream)
+              : launch_qp<false>(x, M, K, ldx, tags, perm, act_packed, act_scales, stream);
+}
+
+cudaError_t launch_pack_weight_perm(const int8_t* w, int64_t N, int64_t K, const int32_t* perm,
+                                    void* w_packed, cudaStream_t stream) {
+  const int64_t words = N * K / 8;
+  const int64_t blocks = std::min<int64_t>(ceil_div(words, 256), 148 * 16);
+  k_pack_weight_perm<<<(unsigned)blocks, 256, 0, stream>>>(w, N, K, perm, static_cast<uint32_t*>(w_packed));
+  return cudaGetLastError();
+}
+
+cudaError_t launch_channel_amax(const void* x, bool bf16, int64_t M, int64_t K, int64_t ldx,
+                                float* amax, cudaStream_t stream) {
+  cudaError_t e = cudaMemsetAsync(amax, 0, (size_t)K * 4, stream);
+  if (e != cudaSuccess) return e;
+  const int64_t cols = ceil_div(K / 8, 256);
+  const int64_t ysplit = std::max<int64_t>(1, std::min<int64_t>(ceil_div(M, 32), ceil_div(148 * 8, cols)));
+  const int64_t rows_per = ceil_div(M, ysplit);
+  const dim3 grid((unsigned)cols, (unsigned)ceil_div(M, rows_per));
+  unsigned int* out = reinterpret_cast<unsigned int*>(amax);
+  if (bf16)
+    k_channel_amax<true><<<grid, 256, 0, stream>>>(static_cast<const uint16_t*>(x), M, K, ldx, rows_per, out);
+  else
+    k_channel_amax<false><<<grid, 256, 0, stream>>>(static_cast<const uint16_t*>(x), M, K, ldx, rows_per, out);
+  return cudaGetLastError();
 }
 
 cudaError_t launch_pack_weight(const int8_t* w, int64_t N, int64_t K, void* w_packed,

@@ -113,6 +113,40 @@ def config1(seed: int = 1) -> Problem:
     return make_problem(16, 256, 256, seed=seed, n8=1)
 
 
+@dataclass
+class UnpermutedProblem:
+    """Activations BEFORE COMET's channel permutation: outliers in a few scattered channels
+    (Fig. 3), plus an independent calibration sample with the same outlier channels
+    (P:L138 "sampled activations from the calibration dataset")."""
+    x: np.ndarray          # [M, K] float16 (or uint16 bf16 bits)
+    x_calib: np.ndarray    # [M_calib, K], same dtype
+    w: np.ndarray          # [N, K] int8 codes
+    s_w: np.ndarray        # [N] float32
+    outlier_channels: np.ndarray   # sorted int64
+    bf16: bool = False
+
+
+def make_unpermuted_problem(M: int, K: int, N: int, *, n_outlier_channels: int | None = None,
+                            channel_frac: float = 0.005, seed: int = 0, m_calib: int = 512,
+                            bf16: bool = False, lo: float = 20.0, hi: float = 100.0) -> UnpermutedProblem:
+    """N(0,1) activations with `n_outlier_channels` (default: channel_frac of K, at least 1)
+    seeded channels scaled by U(lo, hi) -- "< 1 %" of features, 10x-100x."""
+    rng = np.random.default_rng(seed)
+    n = n_outlier_channels if n_outlier_channels is not None else max(1, int(round(channel_frac * K)))
+    ch = np.sort(rng.choice(K, size=n, replace=False)).astype(np.int64)
+    mag = rng.uniform(lo, hi, size=n).astype(np.float32)
+
+    def draw(rows):
+        x = rng.standard_normal((rows, K), dtype=np.float32)
+        x[:, ch] *= mag
+        return bf16_bits_from_f32(x) if bf16 else x.astype(np.float16)
+
+    x = draw(M)
+    xc = draw(m_calib)
+    w, s_w = make_weights(N, K, rng)
+    return UnpermutedProblem(x=x, x_calib=xc, w=w, s_w=s_w, outlier_channels=ch, bf16=bf16)
+
+
 def sample_rows(M: int, n: int, x: np.ndarray, seed: int = 7) -> np.ndarray:
     """Seeded sample of token rows that always contains the row holding max |x|."""
     rng = np.random.default_rng(seed)

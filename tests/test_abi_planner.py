@@ -45,9 +45,15 @@ def test_validation_errors_without_gpu():
     st = L.comet_quantize_act(ctypes.c_void_p(16), 0, 4, 250, 256, tags.ctypes.data_as(ctypes.c_void_p),
                               None, ctypes.c_void_p(256), ctypes.c_void_p(16), None)
     assert st == 2
-    st = L.comet_quantize_act(ctypes.c_void_p(16), 0, 4, 256, 256, tags.ctypes.data_as(ctypes.c_void_p),
+    tags_big = np.zeros(257, np.uint8)
+    st = L.comet_quantize_act(ctypes.c_void_p(16), 0, 4, 257 * 128, 257 * 128, tags_big.ctypes.data_as(ctypes.c_void_p),
                               ctypes.c_void_p(64), ctypes.c_void_p(256), ctypes.c_void_p(16), None)
-    assert st == 2   # fused permutation not implemented
+    assert st == 2   # fused permutation needs K <= 32768
+    st = L.comet_quantize_act(ctypes.c_void_p(16), 0, 4, 256, 256, tags.ctypes.data_as(ctypes.c_void_p),
+                              ctypes.c_void_p(72), ctypes.c_void_p(256), ctypes.c_void_p(16), None)
+    assert st == 3   # perm_dev misaligned
+    st = L.comet_channel_amax(ctypes.c_void_p(16), 0, 4, 256, 250, ctypes.c_void_p(16), None)
+    assert st == 3   # ldx < K
     st = L.comet_pack_weight(ctypes.c_void_p(16), 100, 256, ctypes.c_void_p(16), None)
     assert st == 2   # N % 128
     with pytest.raises(cb.CometError):
