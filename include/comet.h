@@ -159,6 +159,28 @@ comet_status_t comet_calibrate_perm(const float* amax_host, int64_t K, double ra
                                     int32_t* perm_host, uint8_t* tags_host, int64_t* n_outliers);
 
 /* ------------------------------------------------------------------------------------------
+ * KV4: INT4 KV-cache quantisation (the "KV4" of W4A4KV4; "a channel-wise 4-bit
+ * quantization strategy for the KV cache", "channel-wise asymmetric INT4 group
+ * quantization"; reading R17).  A K or V cache tensor kv[T][C] (T tokens, C = KV heads x
+ * head_dim channels) is quantised per (group g of `group` consecutive tokens, channel c):
+ *   mn = min x, mx = max x over the group's tokens; d = mx - mn (binary32);
+ *   s = d / 15, r = 15 / d (correctly rounded; d == 0 -> s = r = 0);
+ *   q = clamp(rint_half_even((x - mn) * r), 0, 15)     (binary32, never contracted)
+ *   dequantised x_hat = mn + q * s (two binary32 roundings), rounded to f16/bf16.
+ * Layouts (device, caller-owned):
+ *   kv4_codes  [T][C/2] uint8: byte (t, j) = q[t][2j] | q[t][2j+1] << 4
+ *   kv4_scales [ceil(T/group)][C] float = s;   kv4_mins [ceil(T/group)][C] float = mn
+ * Constraints: T >= 1, C % 64 == 0, group in {32, 64, 128, 256}; ld (elements) >= C with
+ * ld*2 % 16 == 0; pointers 16-byte aligned; inputs finite.  Bit-exact with the CPU oracle.
+ * ---------------------------------------------------------------------------------------- */
+comet_status_t comet_kv4_quantize(const void* kv, comet_dtype_t dt, int64_t T, int64_t C,
+                                  int64_t ld, int group, uint8_t* kv4_codes, float* kv4_scales,
+                                  float* kv4_mins, void* stream);
+comet_status_t comet_kv4_dequantize(const uint8_t* kv4_codes, const float* kv4_scales,
+                                    const float* kv4_mins, int64_t T, int64_t C, int group,
+                                    void* out, comet_dtype_t odt, int64_t ldo, void* stream);
+
+/* ------------------------------------------------------------------------------------------
  * Tile scheduler ("fine-grained SM scheduling")
  * ---------------------------------------------------------------------------------------- */
 typedef struct comet_plan_s* comet_plan_t;   /* opaque, library-owned, immutable after create */

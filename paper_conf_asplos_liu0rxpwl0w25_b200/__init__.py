@@ -83,6 +83,8 @@ def lib():
         "comet_pack_weight_perm": (I32, [P, I64, I64, P, P, P]),
         "comet_channel_amax": (I32, [P, I32, I64, I64, I64, P, P]),
         "comet_calibrate_perm": (I32, [P, I64, ctypes.c_double, P, P, ctypes.POINTER(I64)]),
+        "comet_kv4_quantize": (I32, [P, I32, I64, I64, I64, I32, P, P, P, P]),
+        "comet_kv4_dequantize": (I32, [P, P, P, I64, I64, I32, P, I32, I64, P]),
         "comet_sched_config_default": (None, [ctypes.POINTER(SchedConfig)]),
         "comet_plan_create": (I32, [I64, I64, I64, P, ctypes.POINTER(SchedConfig), ctypes.POINTER(P),
                                     ctypes.POINTER(SZ)]),
@@ -214,6 +216,37 @@ def calibrate_perm(amax, ratio: float = 10.0):
                                       perm.ctypes.data_as(ctypes.c_void_p),
                                       tags.ctypes.data_as(ctypes.c_void_p), ctypes.byref(n)))
     return perm, tags, int(n.value)
+
+
+def kv4_quantize(kv, group: int = 128, *, out=None, stream=None):
+    """comet_kv4_quantize: [T, C] float16/bfloat16 CUDA tensor -> (codes uint8 [T, C/2],
+    scales float32 [ceil(T/group), C], mins float32 [ceil(T/group), C])."""
+    import torch
+    assert kv.is_cuda and kv.dim() == 2 and kv.stride(1) == 1
+    T, C = kv.shape
+    ng = (T + group - 1) // group
+    if out is None:
+        out = (torch.empty((T, C // 2), dtype=torch.uint8, device=kv.device),
+               torch.empty((ng, C), dtype=torch.float32, device=kv.device),
+               torch.empty((ng, C), dtype=torch.float32, device=kv.device))
+    codes, scales, mins = out
+    _check(lib().comet_kv4_quantize(ctypes.c_void_p(kv.data_ptr()), _dt(kv.dtype), T, C, kv.stride(0), group,
+                                    ctypes.c_void_p(codes.data_ptr()), ctypes.c_void_p(scales.data_ptr()),
+                                    ctypes.c_void_p(mins.data_ptr()), _stream(stream)))
+    return codes, scales, mins
+
+
+def kv4_dequantize(codes, scales, mins, group: int = 128, *, out=None, out_dtype=None, stream=None):
+    """comet_kv4_dequantize: -> [T, C] float16 (default) / bfloat16 CUDA tensor."""
+    import torch
+    T, C = codes.shape[0], codes.shape[1] * 2
+    if out is None:
+        out = torch.empty((T, C), dtype=out_dtype or torch.float16, device=codes.device)
+    _check(lib().comet_kv4_dequantize(ctypes.c_void_p(codes.data_ptr()), ctypes.c_void_p(scales.data_ptr()),
+                                      ctypes.c_void_p(mins.data_ptr()), T, C, group,
+                                      ctypes.c_void_p(out.data_ptr()), _dt(out.dtype), out.stride(0),
+                                      _stream(stream)))
+    return out
 
 
 class Plan:

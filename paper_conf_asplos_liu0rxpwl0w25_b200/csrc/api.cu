@@ -208,6 +208,55 @@ comet_status_t comet_channel_amax(const void* x, comet_dtype_t xdt, int64_t M, i
   return COMET_OK;
 }
 
+static comet_status_t check_kv4(int64_t T, int64_t C, int group) {
+  if (T < 1 || T > INT32_MAX) return fail(COMET_ERR_UNSUPPORTED_SHAPE, "T must be in [1, 2^31-1]");
+  if (C < 64 || C % 64 != 0 || C > (int64_t)1 << 20) return fail(COMET_ERR_UNSUPPORTED_SHAPE, "C must be a positive multiple of 64");
+  if (group != 32 && group != 64 && group != 128 && group != 256)
+    return fail(COMET_ERR_UNSUPPORTED_SHAPE, "group must be 32, 64, 128 or 256");
+  if (ceil_div(T, group) > 65535) return fail(COMET_ERR_UNSUPPORTED_SHAPE, "too many token groups (T / group > 65535)");
+  return COMET_OK;
+}
+
+comet_status_t comet_kv4_quantize(const void* kv, comet_dtype_t dt, int64_t T, int64_t C,
+                                  int64_t ld, int group, uint8_t* kv4_codes, float* kv4_scales,
+                                  float* kv4_mins, void* stream) {
+  g_launches = 0;
+  comet_status_t st = check_kv4(T, C, group);
+  if (st != COMET_OK) return st;
+  if (!kv || !kv4_codes || !kv4_scales || !kv4_mins) return fail(COMET_ERR_INVALID_ARG, "NULL pointer argument");
+  if (dt != COMET_F16 && dt != COMET_BF16) return fail(COMET_ERR_INVALID_ARG, "dt must be COMET_F16 or COMET_BF16");
+  if (ld < C || (ld * 2) % 16 != 0) return fail(COMET_ERR_MISALIGNED, "ld must be >= C with ld*2 % 16 == 0");
+  if (!aligned16(kv) || !aligned16(kv4_codes) || !aligned16(kv4_scales) || !aligned16(kv4_mins))
+    return fail(COMET_ERR_MISALIGNED, "device pointers must be 16-byte aligned");
+  st = check_device();
+  if (st != COMET_OK) return st;
+  cudaError_t e = launch_kv4_quantize(kv, dt == COMET_BF16, T, C, ld, group, kv4_codes, kv4_scales,
+                                      kv4_mins, static_cast<cudaStream_t>(stream));
+  if (e != cudaSuccess) return cuda_status(e, "kv4 quantize launch");
+  g_launches = 1;
+  return COMET_OK;
+}
+
+comet_status_t comet_kv4_dequantize(const uint8_t* kv4_codes, const float* kv4_scales,
+                                    const float* kv4_mins, int64_t T, int64_t C, int group,
+                                    void* out, comet_dtype_t odt, int64_t ldo, void* stream) {
+  g_launches = 0;
+  comet_status_t st = check_kv4(T, C, group);
+  if (st != COMET_OK) return st;
+  if (!kv4_codes || !kv4_scales || !kv4_mins || !out) return fail(COMET_ERR_INVALID_ARG, "NULL pointer argument");
+  if (odt != COMET_F16 && odt != COMET_BF16) return fail(COMET_ERR_INVALID_ARG, "odt must be COMET_F16 or COMET_BF16");
+  if (ldo < C || (ldo * 2) % 16 != 0) return fail(COMET_ERR_MISALIGNED, "ldo must be >= C with ldo*2 % 16 == 0");
+  if (!aligned16(kv4_codes) || !aligned16(kv4_scales) || !aligned16(kv4_mins) || !aligned16(out))
+    return fail(COMET_ERR_MISALIGNED, "device pointers must be 16-byte aligned");
+  st = check_device();
+  if (st != COMET_OK) return st;
+  cudaError_t e = launch_kv4_dequantize(kv4_codes, kv4_scales, kv4_mins, T, C, group, out,
+                                        odt == COMET_BF16, ldo, static_cast<cudaStream_t>(stream));
+  if (e != cudaSuccess) return cuda_status(e, "kv4 dequantize launch");
+  g_launches = 1;
+  return COMET_OK;
+}
+
 void comet_sched_config_default(comet_sched_config* cfg) {
   if (!cfg) return;
   memset(cfg, 0, sizeof(*cfg));

@@ -46,6 +46,9 @@ namespace {
 #define COMET_DEC_ABLATE 0      // timing experiments only (wrong results): bit 0 no MMAs, bit 1 no
 #endif                          // TMEM stores of widened weights, bit 2 no accumulator loads
 
+#ifndef COMET_DEC_NA
+#define COMET_DEC_NA 2
+#endif
 constexpr int kWidenWarp0 = 4;
 constexpr int kPromoWarp0 = 12;
 
@@ -63,7 +66,7 @@ constexpr int kPromoWarp0 = 12;
 template <int NT>
 struct Cfg {
   static constexpr int KS = NT <= 32 ? 4 : 2;                  // K-blocks per stage
-  static constexpr int NA = 2;
+  static constexpr int NA = COMET_DEC_NA;                       // widened-weight A buffers
   static constexpr int A_COLS = 32 * KS;
   static constexpr int ACC_SET = KS * NT;                      // accumulator columns per stage
   static constexpr int NACC_RAW = (512 - NA * A_COLS) / ACC_SET;

@@ -1,5 +1,6 @@
 // internal.h -- declarations shared by the libcomet.so translation units (not part of the ABI).
 #pragma once
+#include <algorithm>
 #include <cstdint>
 #include <cstddef>
 #include <string>
@@ -77,6 +78,12 @@ cudaError_t launch_pack_weight_perm(const int8_t* w, int64_t N, int64_t K, const
                                     void* w_packed, cudaStream_t stream);
 cudaError_t launch_channel_amax(const void* x, bool bf16, int64_t M, int64_t K, int64_t ldx,
                                 float* amax, cudaStream_t stream);
+// kv4.cu (NEXT-4)
+cudaError_t launch_kv4_quantize(const void* x, bool bf16, int64_t T, int64_t C, int64_t ldx, int G,
+                                uint8_t* codes, float* scales, float* mins, cudaStream_t stream);
+cudaError_t launch_kv4_dequantize(const uint8_t* codes, const float* scales, const float* mins,
+                                  int64_t T, int64_t C, int G, void* y, bool bf16, int64_t ldy,
+                                  cudaStream_t stream);
 // pack.cu
 cudaError_t launch_pack_weight(const int8_t* w, int64_t N, int64_t K, void* w_packed,
                                cudaStream_t stream);

@@ -147,6 +147,21 @@ def make_unpermuted_problem(M: int, K: int, N: int, *, n_outlier_channels: int |
     return UnpermutedProblem(x=x, x_calib=xc, w=w, s_w=s_w, outlier_channels=ch, bf16=bf16)
 
 
+def make_kv(T: int, C: int, rng: np.random.Generator, *, bf16: bool = False,
+            outlier_channels: int = 4, lo: float = 5.0, hi: float = 20.0):
+    """KV-cache tensor [T tokens, C = heads x head_dim channels]: N(0,1) with a per-channel
+    offset U(-1, 1) and `outlier_channels` channels scaled by U(lo, hi) -- K caches carry
+    channel-wise outliers, V caches few.  float16, or uint16 bf16 bit patterns."""
+    x = rng.standard_normal((T, C), dtype=np.float32)
+    x += rng.uniform(-1.0, 1.0, size=C).astype(np.float32)[None, :]
+    if outlier_channels:
+        ch = rng.choice(C, size=outlier_channels, replace=False)
+        x[:, ch] *= rng.uniform(lo, hi, size=outlier_channels).astype(np.float32)
+    if bf16:
+        return bf16_bits_from_f32(x)
+    return x.astype(np.float16)
+
+
 def sample_rows(M: int, n: int, x: np.ndarray, seed: int = 7) -> np.ndarray:
     """Seeded sample of token rows that always contains the row holding max |x|."""
     rng = np.random.default_rng(seed)
