@@ -220,6 +220,61 @@ def decode_sweep(cb, torch, dev, peaks, Ms=(1, 4, 8, 32), iters=20):
             "layers": out}
 
 
+def next_rows(cb, torch, dev, peaks, iters=20):
+    """SURVEY §8(f) rows built beyond the hot path, timed live (L2 left clean before every
+    launch, CUDA events, median): NEXT-1 fused channel permutation in kernel 1 (LLaMA-3-70B
+    layer inputs at M = 4096, permutation calibrated on a separate sample) against the
+    identity kernel, and NEXT-4 KV4 quantise / dequantise of a LLaMA-3-70B KV cache
+    (8 KV heads x 128 = 1024 channels, 32768 tokens, group 128).  GB/s = algorithmic bytes."""
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    flush_rd = torch.ones(64 << 20, dtype=torch.float32, device=dev)
+    hbm = peaks["hbm_gbs"]
+
+    def t(fn):
+        fn()
+        torch.cuda.synchronize()
+        ws = []
+        for i in range(iters + 3):
+            flush.fill_(i & 0xFF)
+            flush_rd.sum()
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record()
+            fn()
+            b.record()
+            ws.append((a, b))
+        torch.cuda.synchronize()
+        return statistics.median(a.elapsed_time(b) for a, b in ws[3:]) * 1e3
+
+    out = {}
+    for name, K in (("gate_up_qkv_input", 8192), ("down_input", 28672)):
+        up = synth.make_unpermuted_problem(M_TOKENS, K, 128, seed=11, m_calib=256)
+        perm, tags, n_out = cb.calibrate_perm(cb.channel_amax(torch.from_numpy(up.x_calib).to(dev)))
+        x = torch.from_numpy(up.x).to(dev)
+        pd = torch.from_numpy(perm).to(dev)
+        act, sc = cb.quantize_act(x, tags, perm=pd)
+        nbytes = M_TOKENS * K * 2 + M_TOKENS * K + (K // 128) * M_TOKENS * 6
+        us_p = t(lambda: cb.quantize_act(x, tags, perm=pd, out=(act, sc)))
+        us_i = t(lambda: cb.quantize_act(x, tags, out=(act, sc)))
+        out[f"perm_quantize_{name}_K{K}"] = {"us": round(us_p, 2), "GB/s": round(nbytes / us_p / 1e3, 1),
+                                              "frac_hbm": round(nbytes / us_p / 1e3 / hbm, 3),
+                                              "identity_us": round(us_i, 2), "outlier_channels": n_out,
+                                              "int8_blocks": int(tags.sum())}
+        del up, x, act, sc
+    T, C, G = 32768, 1024, 128
+    kv = torch.from_numpy(synth.make_kv(T, C, np.random.default_rng(0))).to(dev)
+    codes, scales, mins = cb.kv4_quantize(kv, G)
+    y = cb.kv4_dequantize(codes, scales, mins, G)
+    nbytes = T * C * 2 + T * C // 2 + (T // G) * C * 8
+    for nm, fn in (("kv4_quantize", lambda: cb.kv4_quantize(kv, G, out=(codes, scales, mins))),
+                   ("kv4_dequantize", lambda: cb.kv4_dequantize(codes, scales, mins, G, out=y))):
+        us = t(fn)
+        out[f"{nm}_T{T}_C{C}"] = {"us": round(us, 2), "GB/s": round(nbytes / us / 1e3, 1),
+                                  "frac_hbm": round(nbytes / us / 1e3 / hbm, 3)}
+    del flush, flush_rd
+    return {"unit": "GB/s", "peak_gbs": hbm, "l2": "256 MiB write + 256 MiB read before every launch",
+            "rows": out}
+
+
 def shard(K, N, kind, tags, rank, world):
     """Tensor-parallel shard of one layer: returns (k0, k1, n0, n1)."""
     if world == 1:
@@ -406,6 +461,7 @@ def run_comet(args, rank, world, local_rank):
 
     cpu = cpu_baseline_sample(args.cpu_budget) if (rank == 0 and world == 1 and args.cpu_budget > 0) else None
     decode = decode_sweep(cb, torch, dev, peaks) if (rank == 0 and world == 1 and args.decode) else None
+    nxt = next_rows(cb, torch, dev, peaks) if (rank == 0 and world == 1 and args.decode) else None
 
     if rank == 0:
         line = {
@@ -425,6 +481,7 @@ def run_comet(args, rank, world, local_rank):
             "gpu_launches": 2 * len(layers) * args.steps,
             "clocks": clocks,
             "decode": decode,
+            "next_rows": nxt,
         }
         if world > 1:
             line["allreduce_ms_per_step"] = ar_ms / args.steps
