@@ -49,6 +49,9 @@ namespace {
 #ifndef COMET_DEC_NA
 #define COMET_DEC_NA 2
 #endif
+#ifndef COMET_DEC_UNIFORM_MMA
+#define COMET_DEC_UNIFORM_MMA 1
+#endif
 constexpr int kWidenWarp0 = 4;
 constexpr int kPromoWarp0 = 12;
 
@@ -200,11 +203,71 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
           if (++st == SX) { st = 0; ph ^= 1; }
         }
       }
-    } else if ((warp == 1 || warp == 3) && lane == 0) {
+    } else if (warp == 1 || warp == 3) {
       // ------------------------------------------------------------------ MMA issuers
-      // Two issuing threads share every stage: warp 1 issues the stage's even K-blocks, warp 3
+      // Two issuing warps share every stage: warp 1 issues the stage's even K-blocks, warp 3
       // the odd ones (each K-block has its own accumulator).  tcgen05.commit tracks the
       // issuing thread's own MMAs, so both commit each stage's barriers (counts 2).
+      // The whole warp runs the loop and every operand is made warp-uniform (shuffle from lane
+      // 0), so the compiler keeps the MMA operands in uniform registers; one elected lane
+      // issues.  (With a lane-0-only loop every tcgen05.mma went through an R2UR waterfall.)
+#if COMET_DEC_UNIFORM_MMA
+      const int par = warp == 1 ? 0 : 1;
+      const uint32_t id_f8 = idesc_f8f6f4_e4m3(128, NT);
+      const uint32_t id_i8 = idesc_i8(128, NT);
+      const uint32_t tb = __shfl_sync(0xffffffffu, tbase, 0);
+      const uint32_t sx0 = __shfl_sync(0xffffffffu, smem_u32(sX(0)), 0);
+      int sx = 0, ab = 0, accs = 0;
+      uint32_t xph = 0, aph = 0, accph = 0;
+      for (int it = it_begin; it < it_end; ++it) {
+        const WorkItem w = load_item(P, it, debug);
+        const int kb_begin = __shfl_sync(0xffffffffu, w.kb_begin, 0);
+        const int kb_end = __shfl_sync(0xffffffffu, w.kb_end, 0);
+        for (int kb = kb_begin; kb < kb_end; kb += KS) {
+          const int nk = min(KS, kb_end - kb);
+          mbar_wait(&full_x[sx], xph);
+          mbar_wait(&a_full[ab], aph);
+          mbar_wait(&acc_empty[accs], accph ^ 1);
+          if (par == 0 && lane == 0) trace_ev(P, 1, tr);
+          tc_fence_after();
+          const uint32_t d0 = tb + C::ACC_COL + accs * C::ACC_SET;
+          const uint32_t a0 = tb + ab * C::A_COLS;
+          const uint64_t b0 = sdesc_kmajor_sw128(sx0 + sx * C::X_STAGE);
+          const uint32_t tagw = __shfl_sync(0xffffffffu, lane < KS ? lds_u8(s_tags_a + kb + lane) : 0u, 0) |
+                                (__shfl_sync(0xffffffffu, lane < KS ? lds_u8(s_tags_a + kb + lane) : 0u, 1) << 1) |
+                                (__shfl_sync(0xffffffffu, lane < KS ? lds_u8(s_tags_a + kb + lane) : 0u, 2) << 2) |
+                                (__shfl_sync(0xffffffffu, lane < KS ? lds_u8(s_tags_a + kb + lane) : 0u, 3) << 3);
+          for (int c = par; c < nk; c += 2) {
+            const uint32_t d = d0 + c * NT, a = a0 + c * 32;
+            const uint64_t bd = b0 + (uint64_t)((c * C::XKB_BYTES) >> 4);
+            if (COMET_DEC_ABLATE & 1) {
+            } else if ((tagw >> c) & 1u) {
+              if (elect_one()) {
+#pragma unroll
+                for (int k = 0; k < 4; ++k) mma_i8_ts(d, a + 8 * k, bd + 2 * k, id_i8, k);
+              }
+            } else {
+              if (elect_one()) {
+#pragma unroll
+                for (int k = 0; k < 4; ++k) mma_f8_ts(d, a + 8 * k, bd + 2 * k, id_f8, k);
+              }
+            }
+            __syncwarp();
+          }
+          if (elect_one()) {
+            tc_commit(&acc_full[accs]);
+            tc_commit(&empty_x[sx]);
+            tc_commit(&a_empty[ab]);
+          }
+          __syncwarp();
+          if (par == 0 && lane == 0) trace_ev(P, 2, tr++);
+          if (++sx == SX) { sx = 0; xph ^= 1; }
+          if (++ab == NA) { ab = 0; aph ^= 1; }
+          if (++accs == NACC) { accs = 0; accph ^= 1; }
+        }
+      }
+#else
+      if (lane == 0) {
       const int par = warp == 1 ? 0 : 1;
       const uint32_t id_f8 = idesc_f8f6f4_e4m3(128, NT);
       const uint32_t id_i8 = idesc_i8(128, NT);
@@ -243,6 +306,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
           if (++accs == NACC) { accs = 0; accph ^= 1; }
         }
       }
+      }
+#endif
     }
   } else if (warp < kPromoWarp0) {
     setmaxnreg_dec<112>();

@@ -28,6 +28,9 @@
 #ifndef COMET_ISSUERS
 #define COMET_ISSUERS 2   // MMA issuing threads (K-blocks alternate between them)
 #endif
+#ifndef COMET_N_UNIFORM_MMA
+#define COMET_N_UNIFORM_MMA 1   // MMA issue loop on the whole warp with uniform operands
+#endif
 #ifndef COMET_PRODUCERS
 #define COMET_PRODUCERS 1   // TMA-issuing warps (2: K-blocks alternate between them)
 #endif
@@ -233,7 +236,67 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
           if (par == 0) trace_ev(P, 0, tr++);
         }
       }
-    } else if ((warp == 1 || (COMET_ISSUERS == 2 && warp == 3)) && lane == 0 && rank == 0) {
+    } else if ((warp == 1 || (COMET_ISSUERS == 2 && warp == 3)) && rank == 0 && COMET_N_UNIFORM_MMA) {
+      // ------------------------------------------------------------------ MMA issuers
+      // Same schedule as below, but the whole warp runs the loop with warp-uniform operands
+      // (shuffled from lane 0) so the MMA operands stay in uniform registers and one elected
+      // lane issues the four MMAs back to back (no per-MMA R2UR waterfall).
+      const int parity = warp == 1 ? 0 : 1;
+      const int h = NSUB == 2 ? parity : 0;
+      constexpr int NMMA = BN / NSUB;
+      const uint32_t id_f8 = idesc_f8f6f4_e4m3(BM * CG, NMMA);
+      const uint32_t id_i8 = idesc_i8(BM * CG, NMMA);
+      const uint32_t tb = __shfl_sync(0xffffffffu, tbase, 0);
+      const uint32_t sx0 = __shfl_sync(0xffffffffu, smem_u32(sX(0)), 0);
+      int j = 0, tr = 0;
+      for (int it = it_begin; it < it_end; ++it) {
+        const WorkItem w = load_item(P, it, debug);
+        const int kb_begin = __shfl_sync(0xffffffffu, w.kb_begin, 0);
+        const int kb_end = __shfl_sync(0xffffffffu, w.kb_end, 0);
+        for (int kb = kb_begin; kb < kb_end; ++kb, ++j) {
+          if (NSUB == 1 && COMET_ISSUERS == 2 && (j & 1) != parity) continue;
+          const int s = j % S, accb = j % NACC;
+          const uint32_t ph = (uint32_t)(j / S) & 1u;
+          mbar_wait(&mma_ready[h * S + s], ph);
+          tc_fence_after();
+          const uint32_t d = tb + accb * BN + h * NMMA;
+          const uint32_t sa = sx0 + s * C::SLOT_BYTES;
+          const uint32_t sbv = sa + C::X_BYTES + h * (C::WROWS / NSUB) * 128;
+          const bool is8 = __shfl_sync(0xffffffffu, lds_u8(s_tags_a + kb), 0) != 0;
+          if (diag_ablate(P) & 8) {
+            // diagnostic: no MMA
+          } else if (is8) {
+            if (elect_one()) {
+#pragma unroll
+              for (int k = 0; k < 4; ++k) {
+                const uint64_t ad = sdesc_kmajor_sw128(sa + 32 * k), bd = sdesc_kmajor_sw128(sbv + 32 * k);
+                if (CG == 2) mma_i8_ss_cg2(d, ad, bd, id_i8, k); else mma_i8_ss(d, ad, bd, id_i8, k);
+              }
+            }
+          } else {
+            if (elect_one()) {
+#pragma unroll
+              for (int k = 0; k < 4; ++k) {
+                const uint64_t ad = sdesc_kmajor_sw128(sa + 32 * k), bd = sdesc_kmajor_sw128(sbv + 32 * k);
+                if (CG == 2) mma_f8_ss_cg2(d, ad, bd, id_f8, k); else mma_f8_ss(d, ad, bd, id_f8, k);
+              }
+            }
+          }
+          __syncwarp();
+          if (elect_one()) {
+            if (CG == 2) {
+              tc_commit_mc(&acc_full[h * NACC + accb], 3);
+              tc_commit_mc(&slot_free[s], 3);
+            } else {
+              tc_commit(&acc_full[h * NACC + accb]);
+              tc_commit(&slot_free[s]);
+            }
+          }
+          __syncwarp();
+          ++tr;
+        }
+      }
+    } else if ((warp == 1 || (COMET_ISSUERS == 2 && warp == 3)) && lane == 0 && rank == 0 && !COMET_N_UNIFORM_MMA) {
       // ------------------------------------------------------------------ MMA issuers
       // Two issuing threads: warp 1 takes the even K-blocks of the CTA's sequence, warp 3 the
       // odd ones (different accumulators and slots), so one thread's barrier wait and commits
