@@ -339,7 +339,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
         }
         __syncwarp();
         if (lane == 0) mbar_arrive(&empty_w[st]);
+        if (lane == 0 && q == 0 && half == 0) trace_ev(P, 13, seq);
         mbar_wait(&a_empty[ab], aph ^ 1);
+        if (lane == 0 && q == 0 && half == 0) trace_ev(P, 14, seq);
         tc_fence_after();
 #pragma unroll
         for (int i = 0; i < KH; ++i) {
@@ -367,6 +369,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
           }
         }
         if (!(COMET_DEC_ABLATE & 2)) tmem_wait_st();
+        if (lane == 0 && q == 0 && half == 0) trace_ev(P, 15, seq);
         tc_fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(&a_full[ab]);

@@ -11,5 +11,6 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_w4
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:k_quantize -s 6 -c 3 -f -o gpurun_out/prof_quant $SHORT > gpurun_out/prof_quant.log 2>&1; tail -2 gpurun_out/prof_quant.log
 # decode GEMM (LLaMA-3-70B gate/up, M=1): one ncu --set full capture
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:^k_w4ax$ -s 2 -c 1 -f -o gpurun_out/prof_dec python tools/decode_time.py --Ms 1 --layers gate_up --iters 2 > gpurun_out/prof_dec.log 2>&1; tail -2 gpurun_out/prof_dec.log
-# TMA streaming probe (HBM and L2-resident, 1..4 issuing warps)
-timeout 300 ./tools/probe/probe_stream 1 > gpurun_out/probe_stream.txt 2>&1
+# NEXT rows: fused-permutation quantise (K = 8192, M = 4096) and the two KV4 kernels
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:k_quantize_perm -s 1 -c 1 -f -o gpurun_out/prof_perm python tools/perm_prof.py 8192 > gpurun_out/prof_perm.log 2>&1; tail -1 gpurun_out/prof_perm.log
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:k_kv4 -s 2 -c 2 -f -o gpurun_out/prof_kv4 python tools/kv4_prof.py > gpurun_out/prof_kv4.log 2>&1; tail -1 gpurun_out/prof_kv4.log
