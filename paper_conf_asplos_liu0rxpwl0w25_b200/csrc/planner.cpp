@@ -127,11 +127,40 @@ comet_status_t build_plan(Plan& p, const comet_sched_config& cfg) {
     else r.push_back({tile, kb, kb + 1});
     load[cta] += ucost[kb];
   };
+  // Tile order for the whole-tile assignments (prefill orientations).  A wave of P concurrent
+  // tiles streams its operands along K once; what a wave touches is (#token tiles) x (token
+  // tile's codes, M_t x K bytes) + (#weight tiles) x (weight tile, tile_w x K/2 bytes).  When
+  // the whole activation matrix fits in L2 (<= 48 MB: every LLaMA layer with K <= 8192 at
+  // M = 4096) the natural order -- token tiles fastest, so each wave covers all of them and
+  // few weight tiles -- reads everything once.  Otherwise (LLaMA-3-70B down, K = 28672:
+  // 117 MB of codes, read 3.5x per launch in the natural order) the tiles are visited in
+  // groups of GN weight tiles with every token tile against each group, GN chosen so a wave
+  // is a balanced block: GN = sqrt(P * token-tile bytes / weight-tile bytes).  Decode
+  // (orientation 1) keeps the natural order.
+  std::vector<int64_t> order((size_t)T);
+  {
+    int64_t gn = p.n_n_tiles;
+    const double act_bytes = (double)p.M * (double)p.K;
+    if (p.orientation >= 2 && act_bytes > 48.0 * (1 << 20)) {
+      const double abytes = (double)p.tile_n * (double)p.K;           // codes per token tile
+      const double wbytes = (double)p.tile_w * (double)p.K / 2.0;     // packed weights per tile
+      gn = std::max<int64_t>(1, std::min<int64_t>(p.n_n_tiles, (int64_t)std::llround(std::sqrt((double)P * abytes / wbytes))));
+    }
+    if (gn >= p.n_n_tiles) {
+      for (int64_t t = 0; t < T; ++t) order[(size_t)t] = t;         // natural: token tiles fastest
+    } else {
+      int64_t i = 0;
+      for (int64_t g0 = 0; g0 < p.n_n_tiles; g0 += gn)
+        for (int64_t m = 0; m < p.n_m_tiles; ++m)
+          for (int64_t n = g0; n < std::min(p.n_n_tiles, g0 + gn); ++n) order[(size_t)i++] = n * p.n_m_tiles + m;
+    }
+  }
   if (mode == 0) {
     using E = std::pair<double, int>;
     std::priority_queue<E, std::vector<E>, std::greater<E>> pq;
     for (int c = 0; c < P; ++c) pq.push({0.0, c});
-    for (int64_t t = 0; t < T; ++t) {
+    for (int64_t ti = 0; ti < T; ++ti) {
+      const int64_t t = order[(size_t)ti];
       auto [l, c] = pq.top();
       pq.pop();
       runs[c].push_back({t, 0, nb});
@@ -171,9 +200,9 @@ comet_status_t build_plan(Plan& p, const comet_sched_config& cfg) {
   } else {
     const int64_t full_waves = std::max<int64_t>(0, T / P - 1);
     const int64_t t_dp = full_waves * P;
-    for (int64_t t = 0; t < t_dp; ++t) {
-      runs[t % P].push_back({t, 0, nb});
-      load[t % P] += tile_cost;
+    for (int64_t ti = 0; ti < t_dp; ++ti) {
+      runs[ti % P].push_back({order[(size_t)ti], 0, nb});
+      load[ti % P] += tile_cost;
     }
     const int64_t t_sk = T - t_dp;
     if (t_sk > 0) {
@@ -182,7 +211,7 @@ comet_status_t build_plan(Plan& p, const comet_sched_config& cfg) {
         for (int kb = 0; kb < nb; ++kb) seq[i * nb + kb] = ucost[kb];
       std::vector<int64_t> cut = best_contiguous_cuts(seq, P);
       for (int c = 0; c < P; ++c)
-        for (int64_t u = cut[c]; u < cut[c + 1]; ++u) add_unit(c, t_dp + u / nb, (int)(u % nb));
+        for (int64_t u = cut[c]; u < cut[c + 1]; ++u) add_unit(c, order[(size_t)(t_dp + u / nb)], (int)(u % nb));
     }
   }
 
