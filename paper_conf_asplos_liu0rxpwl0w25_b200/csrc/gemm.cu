@@ -49,6 +49,9 @@ namespace {
 #ifndef COMET_DEC_NA
 #define COMET_DEC_NA 2
 #endif
+#ifndef COMET_DEC_ST64
+#define COMET_DEC_ST64 0    // 1: one 64-column TMEM store per widen warp and stage (KS = 4)
+#endif
 #ifndef COMET_DEC_UNIFORM_MMA
 #define COMET_DEC_UNIFORM_MMA 1
 #endif
@@ -343,6 +346,33 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
         mbar_wait(&a_empty[ab], aph ^ 1);
         if (lane == 0 && q == 0 && half == 0) trace_ev(P, 14, seq);
         tc_fence_after();
+#if COMET_DEC_ST64
+        if (KH == 2 && half * KH + 1 < nk) {
+          // both K-blocks of this warp in one 64-column TMEM store
+          uint32_t o[64];
+#pragma unroll
+          for (int i = 0; i < 2; ++i) {
+            const bool is8 = lds_u8(s_tags_a + kb + half * KH + i) != 0;
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+              const uint32_t pw[4] = {cc[4 * i + j].x, cc[4 * i + j].y, cc[4 * i + j].z, cc[4 * i + j].w};
+#pragma unroll
+              for (int e = 0; e < 4; ++e) {
+                const uint32_t pv = pw[e];
+                const int g = 32 * i + 2 * (j * 4 + e);
+                if (is8) {
+                  o[g] = ((pv << 4) & 0xF0F0F0F0u) ^ 0x80808080u;
+                  o[g + 1] = (pv & 0xF0F0F0F0u) ^ 0x80808080u;
+                } else {
+                  o[g] = pv & 0x0F0F0F0Fu;
+                  o[g + 1] = (pv >> 4) & 0x0F0F0F0Fu;
+                }
+              }
+            }
+          }
+          if (!(COMET_DEC_ABLATE & 2)) tmem_st64(tbase + ab * C::A_COLS + half * KH * 32 + lane_addr, o);
+        } else
+#endif
 #pragma unroll
         for (int i = 0; i < KH; ++i) {
           const int cb = half * KH + i;

@@ -81,20 +81,28 @@ struct CfgN {
   // LOADALL: every column of the K-block is loaded with one wait, the accumulator released at
   // once, and the FFMA2 folding done afterwards; else 16/32-column batches double-buffered.
   static constexpr bool LOADALL = COLS <= 120 && promo_regs(32) >= ACC_REGS + COLS + 24;
-  static constexpr int NEED = LOADALL ? ACC_REGS + COLS + 24 : ACC_REGS + 2 * 16 + 24;
-  static constexpr int REG_LOW = promo_regs(40) >= NEED ? 40 : 32;
+  static constexpr int NEED_STD = LOADALL ? ACC_REGS + COLS + 24 : ACC_REGS + 2 * 16 + 24;
+  // TIGHT: four promotion warpgroups (16 warps read TMEM: ~360 B/clk/SM against ~215 with 8,
+  // profiles/r01/probe_b200.json) leave each promotion thread ~104 registers: the producer /
+  // MMA warpgroup drops to 24, promotion folds single-buffered 16-column batches.
+  static constexpr int promo_regs3(int low0, int loww) {
+    return ((REG_POOL - low0 - loww * NWG) / NPW / 8) * 8 > 248 ? 248 : ((REG_POOL - low0 - loww * NWG) / NPW / 8) * 8;
+  }
+  static constexpr bool TIGHT = !LOADALL && promo_regs3(32, 32) < NEED_STD;
+  static constexpr int NEED = TIGHT ? ACC_REGS + 16 + 24 : NEED_STD;
+  static constexpr int REG_LOW = TIGHT ? 24 : (promo_regs(40) >= NEED ? 40 : 32);
   // the widen warpgroups keep 40 registers (their loop state spills at 32) whenever the
   // producer/MMA warpgroup at 32 still leaves promotion its working set
   static constexpr int promo_regs2(int low0, int loww) {
     return ((REG_POOL - low0 - loww * NWG) / NPW / 8) * 8 > 248 ? 248 : ((REG_POOL - low0 - loww * NWG) / NPW / 8) * 8;
   }
-  static constexpr int REG_WIDEN = (REG_LOW == 32 && COMET_WIDEN40 && promo_regs2(32, 40) >= NEED) ? 40 : REG_LOW;
+  static constexpr int REG_WIDEN = TIGHT ? 40 : ((REG_LOW == 32 && COMET_WIDEN40 && promo_regs2(32, 40) >= NEED) ? 40 : REG_LOW);
   static constexpr int REG_PROMO = promo_regs2(REG_LOW, REG_WIDEN);
   // SB: single-buffered 32-column batches (fewer, larger TMEM loads in flight) when the
   // double-buffered 32-column form does not fit (variant experiments: COMET_PROMO_SB)
-  static constexpr bool SB = !LOADALL && COMET_PROMO_SB && REG_PROMO < ACC_REGS + 2 * 32 + 24 &&
-                             REG_PROMO >= ACC_REGS + 32 + 24 && COLS % 32 == 0;
-  static constexpr int PB = LOADALL ? COLS
+  static constexpr bool SB = TIGHT || (!LOADALL && COMET_PROMO_SB && REG_PROMO < ACC_REGS + 2 * 32 + 24 &&
+                             REG_PROMO >= ACC_REGS + 32 + 24 && COLS % 32 == 0);
+  static constexpr int PB = TIGHT ? 16 : LOADALL ? COLS
                           : ((SB || (REG_PROMO >= ACC_REGS + 2 * 32 + 24 && COLS % 32 == 0)) ? 32 : 16);
   static constexpr int NACC_TMEM = 512 / BN >= 4 ? 4 : 512 / BN;   // accumulators TMEM holds
   // NSUB = 2: each K-block is issued as two N = BN/2 sub-MMAs, one per promotion warpgroup, each
@@ -257,7 +265,9 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
           if (NSUB == 1 && COMET_ISSUERS == 2 && (j & 1) != parity) continue;
           const int s = j % S, accb = j % NACC;
           const uint32_t ph = (uint32_t)(j / S) & 1u;
+          if (lane == 0) trace_ev(P, parity ? 13 : 1, tr);
           mbar_wait(&mma_ready[h * S + s], ph);
+          if (lane == 0) trace_ev(P, parity ? 11 : 3, tr);
           tc_fence_after();
           const uint32_t d = tb + accb * BN + h * NMMA;
           const uint32_t sa = sx0 + s * C::SLOT_BYTES;
