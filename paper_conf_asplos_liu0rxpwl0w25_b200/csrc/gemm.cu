@@ -52,6 +52,9 @@ namespace {
 #ifndef COMET_DEC_ST64
 #define COMET_DEC_ST64 0    // 1: one 64-column TMEM store per widen warp and stage (KS = 4)
 #endif
+#ifndef COMET_DEC_PDL
+#define COMET_DEC_PDL 1     // launch as a programmatic dependent of kernel 1 (weights stream early)
+#endif
 #ifndef COMET_DEC_UNIFORM_MMA
 #define COMET_DEC_UNIFORM_MMA 1
 #endif
@@ -171,6 +174,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
   const uint32_t tbase = *tmem_holder;
   if (tracing && threadIdx.x == 0) P.trace[32768 + blockIdx.x * 4 + 1] = globaltimer_ns();
   int tr = 0;   // trace index (per role)
+  // Programmatic dependent launch: the kernel may start while the previous kernel of the stream
+  // (kernel 1, quantising this layer's activations) is still running.  Only the weight
+  // producer -- it reads the packed weights and the plan, which no predecessor writes -- runs
+  // ahead and fills the weight ring; every other thread first waits for the predecessor grid
+  // to complete and its memory to be visible (a no-op without a programmatic predecessor).
+  if (!(warp == 0 && lane == 0)) asm volatile("griddepcontrol.wait;" ::: "memory");
 
   if (warp < kWidenWarp0) {
     setmaxnreg_dec<40>();
@@ -602,8 +611,17 @@ cudaError_t launch_nt(const GemmParams& prm, int grid, cudaStream_t stream) {
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
-  k_w4ax<NT, DEBUG><<<grid, kThreads, C::SMEM_BYTES, stream>>>(prm);
-  return cudaGetLastError();
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)grid);
+  cfg.blockDim = dim3(kThreads);
+  cfg.dynamicSmemBytes = C::SMEM_BYTES;
+  cfg.stream = stream;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = COMET_DEC_PDL;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, k_w4ax<NT, DEBUG>, prm);
 }
 
 PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {

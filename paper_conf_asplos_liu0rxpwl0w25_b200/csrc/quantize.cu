@@ -179,6 +179,9 @@ __global__ void __launch_bounds__(256) k_quantize(const uint16_t* __restrict__ x
                                                   float* __restrict__ scales) {
   constexpr int ROWS = 8 / WPR;
   __shared__ float s_part[8];
+  // let a programmatic dependent (the decode GEMM) launch now: it streams weights while this
+  // grid runs and waits for our completion before touching the activations
+  asm volatile("griddepcontrol.launch_dependents;");
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int row_in_cta = warp / WPR, wi = warp % WPR;
   const int64_t m = (int64_t)blockIdx.x * ROWS + row_in_cta;
@@ -266,6 +269,7 @@ __global__ void __launch_bounds__(NW * 32, 2) k_quantize_perm(const uint16_t* __
                                                        float* __restrict__ corr,
                                                        float* __restrict__ scales) {
   extern __shared__ __align__(128) uint8_t smem[];
+  asm volatile("griddepcontrol.launch_dependents;");                  // see k_quantize
   uint64_t* full = reinterpret_cast<uint64_t*>(smem);                 // [nbuf] (<= 16)
   uint16_t* p16 = reinterpret_cast<uint16_t*>(smem + 128);            // [K] permutation
   uint16_t* prow = p16 + K;                                           // [K] permuted row (swizzled)
