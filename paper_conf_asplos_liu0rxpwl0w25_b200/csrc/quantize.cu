@@ -427,6 +427,85 @@ __global__ void __launch_bounds__(256) k_channel_amax(const uint16_t* __restrict
   for (int i = 0; i < 8; ++i) atomicMax(amax + c8 + i, __float_as_uint(a[i]));
 }
 
+// Small-M (decode) variant: a row is split over a cluster of S CTAs (S <= 8) so that a single
+// token row of K = 28672 channels is read by 64 warps in one load round instead of by 8 warps
+// in four.  CTA `part` of the cluster takes the row's 8-block groups part*8 + warp, step 8*S;
+// the correction term corr[m] is reduced across the cluster through distributed shared memory
+// in a fixed (rank, warp) order by rank 0 -- deterministic, no atomics.
+template <bool BF16>
+__global__ void __launch_bounds__(256) k_quantize_split(const uint16_t* __restrict__ x, int64_t M,
+                                                        int64_t K, int64_t ldx, int64_t Mp, int S,
+                                                        TagMask tags,
+                                                        uint8_t* __restrict__ codes,
+                                                        int16_t* __restrict__ qsum,
+                                                        float* __restrict__ corr,
+                                                        float* __restrict__ scales) {
+  __shared__ float s_part[8];
+  asm volatile("griddepcontrol.launch_dependents;");                  // see k_quantize
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int part = (int)sm100::cluster_ctarank();
+  const int64_t m = blockIdx.x / S;
+  const int bl = lane >> 2, sub = lane & 3;
+  const int nb = (int)(K / kBlockK);
+  const int ngroups = (nb + 7) >> 3;
+  float cpart = 0.f;
+  if (m < M) {
+    const uint16_t* xrow = x + m * ldx + sub * 8;
+    uint8_t* crow = codes + m * K + sub * 8;
+    for (int g = part * 8 + warp; g < ngroups; g += 8 * S) {
+      const int b = g * 8 + bl;
+      const bool bvalid = b < nb;
+      uint4 raw[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j)
+        raw[j] = bvalid ? ldg_stream(xrow + b * kBlockK + 32 * j) : make_uint4(0, 0, 0, 0);
+      float v[32];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        float t[8];
+        unpack8<BF16>(raw[j], t);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) v[8 * j + i] = t[i];
+      }
+      const bool is8 = bvalid && ((tags.w[b >> 5] >> (b & 31)) & 1u);
+      const LaneOut o = quantize32(v, is8);
+      if (bvalid) {
+        uint8_t* cb = crow + b * kBlockK;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) *reinterpret_cast<uint2*>(cb + 32 * j) = o.c[j];
+        if (sub == 0) {
+          scales[(int64_t)b * Mp + m] = o.s;
+          qsum[(int64_t)b * Mp + m] = (int16_t)o.q;
+          if (!is8) cpart = __fadd_rn(cpart, __fmul_rn(o.s, (float)o.q));
+        }
+      }
+    }
+  } else if (m < Mp) {
+    for (int b = part * 256 + threadIdx.x; b < nb; b += 256 * S) {
+      scales[(int64_t)b * Mp + m] = 0.f;
+      qsum[(int64_t)b * Mp + m] = 0;
+    }
+  }
+  cpart = __fadd_rn(cpart, __shfl_xor_sync(0xffffffffu, cpart, 4));
+  cpart = __fadd_rn(cpart, __shfl_xor_sync(0xffffffffu, cpart, 8));
+  cpart = __fadd_rn(cpart, __shfl_xor_sync(0xffffffffu, cpart, 16));
+  if (lane == 0) s_part[warp] = cpart;
+  sm100::cluster_sync();                    // every CTA's partials written, visible cluster-wide
+  if (part == 0 && threadIdx.x == 0 && m < Mp) {
+    float c = 0.f;
+    for (int r = 0; r < S; ++r) {
+      const uint32_t base = sm100::mapa_shared(sm100::smem_u32(s_part), (uint32_t)r);
+      for (int i = 0; i < 8; ++i) {
+        float v;
+        asm volatile("ld.shared::cluster.f32 %0, [%1];" : "=f"(v) : "r"(base + 4u * i));
+        c = __fadd_rn(c, v);
+      }
+    }
+    corr[m] = __fmul_rn(8.f, c);
+  }
+  sm100::cluster_sync();                    // keep every CTA's shared memory alive until read
+}
+
 template <bool BF16>
 cudaError_t launch_q(const void* x, int64_t M, int64_t K, int64_t ldx, const TagMask& tags,
                      void* act_packed, float* act_scales, cudaStream_t stream) {
@@ -441,6 +520,23 @@ cudaError_t launch_q(const void* x, int64_t M, int64_t K, int64_t ldx, const Tag
   // enough CTAs for ~8 per SM (memory-level parallelism), warps of a row sharing its groups
   const int64_t target = 8 * 148;
   const int64_t ngroups = (nb + 7) / 8;
+  if (M <= 32 && ngroups > 8) {
+    // decode: split every row over a cluster of S CTAs (one 8-block group per warp)
+    const int S = (int)std::min<int64_t>(8, ceil_div(ngroups, 8));
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)(Mp * S));
+    cfg.blockDim = dim3(256);
+    cfg.stream = stream;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = (unsigned)S;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, k_quantize_split<BF16>, static_cast<const uint16_t*>(x), M, K, ldx,
+                              Mp, S, tags, codes, qsum, corr, act_scales);
+  }
   int wpr = 1;
   while (wpr < 8 && ceil_div(Mp, 8 / wpr) < target && ngroups >= 2 * wpr) wpr *= 2;
   const int rows = 8 / wpr;

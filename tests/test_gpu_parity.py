@@ -61,6 +61,7 @@ def _check_quant(p, act, sc, rows=None):
     (16, 256, None, False),            # config 1
     (1, 4096, 0.05, False), (16, 4096, 0.05, False), (256, 11008, 0.05, False),   # config 2
     (33, 1024, 0.5, True), (1000, 512, 0.25, False), (7, 14336, 0.05, True),
+    (1, 28672, 0.05, False), (32, 28672, 0.05, True), (3, 11008, 0.25, False),   # cluster-split rows
 ])
 def test_quantize_parity(M, K, frac, bf16):
     if frac is None:
