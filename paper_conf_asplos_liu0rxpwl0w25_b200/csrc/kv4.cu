@@ -37,6 +37,43 @@ __device__ __forceinline__ void unpack8f(const uint4& raw, float (&v)[8]) {
   }
 }
 
+// Packed binary32 pairs, each one correctly rounded operation (never contracted: an FFMA2 by
+// +-1 is a single rounding of the sum, and ptxas leaves FMUL2 -> FFMA2 chains alone).
+__device__ __forceinline__ float2 ffma2_rn(float2 a, float2 b, float2 c) {
+  float2 d;
+  asm("{\n\t.reg .b64 ra, rb, rc, rd;\n\tmov.b64 ra, {%2, %3};\n\tmov.b64 rb, {%4, %5};\n\t"
+      "mov.b64 rc, {%6, %7};\n\tfma.rn.f32x2 rd, ra, rb, rc;\n\tmov.b64 {%0, %1}, rd;\n\t}\n"
+      : "=f"(d.x), "=f"(d.y) : "f"(a.x), "f"(a.y), "f"(b.x), "f"(b.y), "f"(c.x), "f"(c.y));
+  return d;
+}
+__device__ __forceinline__ float2 fmul2_rn(float2 a, float2 b) {
+  float2 d;
+  asm("{\n\t.reg .b64 ra, rb, rd;\n\tmov.b64 ra, {%2, %3};\n\tmov.b64 rb, {%4, %5};\n\t"
+      "mul.rn.f32x2 rd, ra, rb;\n\tmov.b64 {%0, %1}, rd;\n\t}\n"
+      : "=f"(d.x), "=f"(d.y) : "f"(a.x), "f"(a.y), "f"(b.x), "f"(b.y));
+  return d;
+}
+// min / max of two packed 16-bit pairs (exact in the input format: no conversion needed)
+template <bool BF16>
+__device__ __forceinline__ uint32_t min2(uint32_t a, uint32_t b) {
+  uint32_t d;
+  if (BF16) asm("min.bf16x2 %0, %1, %2;" : "=r"(d) : "r"(a), "r"(b));
+  else asm("min.f16x2 %0, %1, %2;" : "=r"(d) : "r"(a), "r"(b));
+  return d;
+}
+template <bool BF16>
+__device__ __forceinline__ uint32_t max2(uint32_t a, uint32_t b) {
+  uint32_t d;
+  if (BF16) asm("max.bf16x2 %0, %1, %2;" : "=r"(d) : "r"(a), "r"(b));
+  else asm("max.f16x2 %0, %1, %2;" : "=r"(d) : "r"(a), "r"(b));
+  return d;
+}
+template <bool BF16>
+__device__ __forceinline__ float2 to_f2(uint32_t w) {
+  if (BF16) return make_float2(__uint_as_float(w << 16), __uint_as_float(w & 0xFFFF0000u));
+  return __half22float2(*reinterpret_cast<const __half2*>(&w));
+}
+
 template <bool BF16, int RPT>   // RPT = rows per thread = G / 32
 __global__ void __launch_bounds__(256, 4) k_kv4_quantize(const uint16_t* __restrict__ x, int64_t T,
                                                       int64_t C, int64_t ldx, int G,
@@ -57,25 +94,34 @@ __global__ void __launch_bounds__(256, 4) k_kv4_quantize(const uint16_t* __restr
     raw[i] = (t < T && 32 * i + j < G) ? __ldg(reinterpret_cast<const uint4*>(x + t * ldx + c0))
                                        : make_uint4(0, 0, 0, 0);
   }
-  float lo[8], hi[8];
+  // pass 1: min / max on the packed 16-bit pairs (row slot 0 always holds a valid row)
+  uint32_t lo2[4] = {raw[0].x, raw[0].y, raw[0].z, raw[0].w};
+  uint32_t hi2[4] = {raw[0].x, raw[0].y, raw[0].z, raw[0].w};
 #pragma unroll
-  for (int e = 0; e < 8; ++e) { lo[e] = FLT_MAX; hi[e] = -FLT_MAX; }
-#pragma unroll
-  for (int i = 0; i < RPT; ++i) {
+  for (int i = 1; i < RPT; ++i) {
     const int64_t t = t0 + j + 32 * i;
     if (t < T && 32 * i + j < G) {
-      float v[8];
-      unpack8f<BF16>(raw[i], v);
+      const uint32_t w[4] = {raw[i].x, raw[i].y, raw[i].z, raw[i].w};
 #pragma unroll
-      for (int e = 0; e < 8; ++e) { lo[e] = fminf(lo[e], v[e]); hi[e] = fmaxf(hi[e], v[e]); }
+      for (int e = 0; e < 4; ++e) { lo2[e] = min2<BF16>(lo2[e], w[e]); hi2[e] = max2<BF16>(hi2[e], w[e]); }
     }
   }
+  if (t0 + j >= T) {                                   // this slot has no row: neutral values
 #pragma unroll
-  for (int e = 0; e < 8; ++e) {
-    lo[e] = fminf(lo[e], __shfl_xor_sync(0xffffffffu, lo[e], 8));
-    lo[e] = fminf(lo[e], __shfl_xor_sync(0xffffffffu, lo[e], 16));
-    hi[e] = fmaxf(hi[e], __shfl_xor_sync(0xffffffffu, hi[e], 8));
-    hi[e] = fmaxf(hi[e], __shfl_xor_sync(0xffffffffu, hi[e], 16));
+    for (int e = 0; e < 4; ++e) { lo2[e] = BF16 ? 0x7F7F7F7Fu : 0x7BFF7BFFu; hi2[e] = BF16 ? 0xFF7FFF7Fu : 0xFBFFFBFFu; }
+  }
+#pragma unroll
+  for (int e = 0; e < 4; ++e) {
+    lo2[e] = min2<BF16>(lo2[e], __shfl_xor_sync(0xffffffffu, lo2[e], 8));
+    lo2[e] = min2<BF16>(lo2[e], __shfl_xor_sync(0xffffffffu, lo2[e], 16));
+    hi2[e] = max2<BF16>(hi2[e], __shfl_xor_sync(0xffffffffu, hi2[e], 8));
+    hi2[e] = max2<BF16>(hi2[e], __shfl_xor_sync(0xffffffffu, hi2[e], 16));
+  }
+  float lo[8], hi[8];
+#pragma unroll
+  for (int e = 0; e < 4; ++e) {
+    const float2 l = to_f2<BF16>(lo2[e]), h = to_f2<BF16>(hi2[e]);
+    lo[2 * e] = l.x; lo[2 * e + 1] = l.y; hi[2 * e] = h.x; hi[2 * e + 1] = h.y;
   }
   if (lane < 8) {
 #pragma unroll
@@ -108,16 +154,18 @@ __global__ void __launch_bounds__(256, 4) k_kv4_quantize(const uint16_t* __restr
   for (int i = 0; i < RPT; ++i) {
     const int64_t t = t0 + j + 32 * i;
     if (t < T && 32 * i + j < G) {
-      float v[8];
-      unpack8f<BF16>(raw[i], v);
+      const uint32_t w[4] = {raw[i].x, raw[i].y, raw[i].z, raw[i].w};
       uint32_t word = 0;
 #pragma unroll
-      for (int e = 0; e < 8; ++e) {
+      for (int e = 0; e < 4; ++e) {
         // 0 <= (x - mn) * r <= 15 (1 + 2^-23)^2, so rint lands in [0, 15] and the clamp of the
-        // definition never acts; rint (half-even) by the magic constant 1.5 * 2^23
-        const float tq = __fmul_rn(__fsub_rn(v[e], mn[e]), r[e]);
-        const uint32_t q = __float_as_uint(__fadd_rn(tq, 12582912.0f)) & 0xFu;
-        word |= q << (4 * e);                       // byte e/2: even channel low nibble
+        // definition never acts; rint (half-even) by the magic constant 1.5 * 2^23.  Pairs:
+        // RN(x - mn) = fma(mn, -1, x), RN(. * r), RN(. + magic) = fma(., 1, magic).
+        const float2 v = to_f2<BF16>(w[e]);
+        const float2 d = ffma2_rn(make_float2(mn[2 * e], mn[2 * e + 1]), make_float2(-1.f, -1.f), v);
+        const float2 tq = fmul2_rn(d, make_float2(r[2 * e], r[2 * e + 1]));
+        const float2 y = ffma2_rn(tq, make_float2(1.f, 1.f), make_float2(12582912.0f, 12582912.0f));
+        word |= ((__float_as_uint(y.x) & 0xFu) | ((__float_as_uint(y.y) & 0xFu) << 4)) << (8 * e);
       }
       *reinterpret_cast<uint32_t*>(codes + t * (C / 2) + c0 / 2) = word;
     }
