@@ -28,6 +28,15 @@
 #ifndef COMET_ISSUERS
 #define COMET_ISSUERS 2   // MMA issuing threads (K-blocks alternate between them)
 #endif
+#ifndef COMET_EPI_PAIR
+#define COMET_EPI_PAIR 0   // 1: FP16/BF16 epilogue stages two chunks per fence/barrier round
+#endif
+#ifndef COMET_EPI_DIRECT
+#define COMET_EPI_DIRECT 0   // 1: direct 16-byte global stores instead of the TMA-store epilogue
+#endif
+#ifndef COMET_NSTAGE
+#define COMET_NSTAGE 2   // output staging buffers per promotion warpgroup (TMA-store epilogue)
+#endif
 #ifndef COMET_N_UNIFORM_MMA
 #define COMET_N_UNIFORM_MMA 1   // MMA issue loop on the whole warp with uniform operands
 #endif
@@ -112,7 +121,10 @@ struct CfgN {
   // S pipeline slots, each holding one K-block's activation tile, packed and widened weights;
   // the scale ring has S + NACC slots (reuse is implied by the slot-free barrier, see below).
   // output staging for the TMA-store epilogue: per promotion WG two [128 rows][64 B] buffers
-  static constexpr int STAGE_BYTES = NPW * 2 * 8192;
+  // staging buffers per promotion WG: COMET_NSTAGE when the pipeline keeps >= 4 slots, else 2
+  static constexpr int NSTAGE = (COMET_SMEM_BUDGET_KB * 1024 - NPW * COMET_NSTAGE * 8192) / (SLOT_BYTES + BM * 4) >= 4
+                                    ? COMET_NSTAGE : 2;
+  static constexpr int STAGE_BYTES = NPW * NSTAGE * 8192;
   static constexpr int S_RAW = (COMET_SMEM_BUDGET_KB * 1024 - STAGE_BYTES) / (SLOT_BYTES + BM * 4);
   static constexpr int S = S_RAW > 8 ? 8 : S_RAW;
   // accumulators in TMEM; fewer than the slots (the promotion's release of K-block kb + NACC
@@ -380,7 +392,7 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
 #pragma unroll
           for (int i = 0; i < RPT; ++i) {
             const int row = t + 128 * i;
-            if (row < C::WROWS) {
+            if (row < C::WROWS && !(diag_ablate(P) & 64)) {   // 64: diagnostic, no widen loads
               const uint32_t src = smem_u32(sWp(s)) + row * 64;
               const int sw64 = (row >> 1) & 3;            // TMA 64-byte swizzle of the packed row
 #pragma unroll
@@ -464,12 +476,21 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
       // -corr * 2^-9 (offset-binary weight correction, owner segment only); loaded now, used
       // in the epilogue, so the load latency is off the K-loop's critical path
       const float init = (owner && m < P.Mp) ? -__ldg(P.corr + m) * 0.001953125f : 0.f;
+      // this tile's per-output-channel weight scales: loaded into registers now, written to
+      // shared memory after the K-loop (read in the epilogue), so the global-load latency never
+      // stalls the start of the tile's promotion
+      constexpr int NWS = (BN + 128 * C::NPW - 1) / (128 * C::NPW);
+      float wsv[NWS];
       if (!DEBUG) {
-        // this tile's per-output-channel weight scales -> shared memory (read in the epilogue)
-        for (int i = ptid; i < BN; i += 128 * C::NPW) {
-          const int wgi = i / COLS, c = i % COLS;
-          const int64_t n = (int64_t)n0 + col_n(wgi, c);
-          sWs[tp * BN + i] = n < P.N ? __ldg(P.w_scales + n) : 0.f;
+#pragma unroll
+        for (int k = 0; k < NWS; ++k) {
+          const int i = ptid + k * 128 * C::NPW;
+          wsv[k] = 0.f;
+          if (i < BN) {
+            const int wgi = i / COLS, c = i % COLS;
+            const int64_t n = (int64_t)n0 + col_n(wgi, c);
+            if (n < P.N) wsv[k] = __ldg(P.w_scales + n);
+          }
         }
       }
       float acc[COLS];
@@ -600,6 +621,13 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
         if (++sc == SS) sc = 0;
         if (++rs == S) rs = 0;
       }
+      if (!DEBUG) {
+#pragma unroll
+        for (int k = 0; k < NWS; ++k) {
+          const int i = ptid + k * 128 * C::NPW;
+          if (i < BN) sWs[tp * BN + i] = wsv[k] * 512.f;   // s_w * 2^9 (exact scaling)
+        }
+      }
       // ---------------------------------------------------------------- epilogue
       if (split) {
         const int seg = (w.flags >> 8) & 0xFF;
@@ -663,14 +691,55 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
         // WG's COLS columns leave in chunks of 64 bytes per row (32 half / 16 float columns),
         // staged in a double-buffered, 64B-swizzled [128 rows][64 B] shared tile and written by
         // one TMA tensor store each (coalesced; rows >= M and columns >= N are clipped).
+        if (threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 15, 4 * (it - it_begin));
         named_bar_sync(1, 128 * C::NPW);                  // this tile's w_scales are in smem
+        if (threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 15, 4 * (it - it_begin) + 1);
         const float* sw = sWs + tp * BN + wg * COLS;
-        uint8_t* stage = sY + wg * 2 * 8192;
+        if (COMET_EPI_DIRECT && RUNS == 1) {
+          // direct epilogue: each thread stores its row's COLS outputs with 16-byte global
+          // stores (fire and forget: the promotion continues with the next tile at once)
+          if (m < P.M) {
+            const int nb0 = n0 + wg * COLS;
+            if (P.ydt == COMET_F32) {
+              float* yrow = reinterpret_cast<float*>(P.y) + m * P.ldy + nb0;
+#pragma unroll
+              for (int c = 0; c < COLS; c += 4) {
+                if (nb0 + c < P.N) {
+                  const float4 v = make_float4((acc[c] + init) * sw[c], (acc[c + 1] + init) * sw[c + 1],
+                                               (acc[c + 2] + init) * sw[c + 2], (acc[c + 3] + init) * sw[c + 3]);
+                  *reinterpret_cast<float4*>(yrow + c) = v;
+                }
+              }
+            } else {
+              const bool bf = P.ydt == COMET_BF16;
+              uint16_t* yrow = reinterpret_cast<uint16_t*>(P.y) + m * P.ldy + nb0;
+#pragma unroll
+              for (int c = 0; c < COLS; c += 8) {
+                uint32_t pk[4];
+#pragma unroll
+                for (int i = 0; i < 4; ++i) {
+                  const float f0 = (acc[c + 2 * i] + init) * sw[c + 2 * i];
+                  const float f1 = (acc[c + 2 * i + 1] + init) * sw[c + 2 * i + 1];
+                  if (bf) {
+                    __nv_bfloat162 hv = __floats2bfloat162_rn(f0, f1);
+                    pk[i] = *reinterpret_cast<uint32_t*>(&hv);
+                  } else {
+                    __half2 hv = __floats2half2_rn(f0, f1);
+                    pk[i] = *reinterpret_cast<uint32_t*>(&hv);
+                  }
+                }
+                if (nb0 + c < P.N) *reinterpret_cast<uint4*>(yrow + c) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+              }
+            }
+          }
+          continue;
+        }
+        uint8_t* stage = sY + wg * C::NSTAGE * 8192;
         const uint32_t swz = (uint32_t)((r >> 1) & 3);
         const bool leader = (threadIdx.x & 127) == 0;     // thread 0 of the WG (row 0)
         auto stage_and_store = [&](const uint32_t (&pk)[16], int ncol_off, int esz) {
-          // caller: buffer (ych & 1) is free (see the wait below)
-          const uint32_t rowa = smem_u32(stage + (ych & 1) * 8192) + r * 64;
+          // caller: buffer (ych % NSTAGE) is free (see the wait below)
+          const uint32_t rowa = smem_u32(stage + (ych % C::NSTAGE) * 8192) + r * 64;
 #pragma unroll
           for (int k = 0; k < 4; ++k)
             asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(rowa + ((k ^ swz) << 4)),
@@ -678,13 +747,13 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
           fence_proxy_async_smem();
           named_bar_sync(2 + wg, 128);
           if (leader) {
-            tma_store_2d(&P.map_y, stage + (ych & 1) * 8192, (n0 + col_n(wg, ncol_off)) * esz, m0);
+            tma_store_2d(&P.map_y, stage + (ych % C::NSTAGE) * 8192, (n0 + col_n(wg, ncol_off)) * esz, m0);
             bulk_commit_group();
           }
           ++ych;
         };
-        auto wait_buffer = [&]() {                        // the store 2 chunks ago has read its buffer
-          if (leader) bulk_wait_group_read<1>();
+        auto wait_buffer = [&]() {                        // the store NSTAGE chunks ago has read its buffer
+          if (leader) bulk_wait_group_read<C::NSTAGE - 1>();
           named_bar_sync(2 + wg, 128);
         };
         if (P.ydt == COMET_F32) {
@@ -693,9 +762,47 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
             wait_buffer();
             uint32_t pk[16];
 #pragma unroll
-            for (int i = 0; i < 16; ++i) pk[i] = __float_as_uint((acc[q * 16 + i] + init) * sw[q * 16 + i] * 512.f);
+            for (int i = 0; i < 16; ++i) pk[i] = __float_as_uint((acc[q * 16 + i] + init) * sw[q * 16 + i]);
             stage_and_store(pk, q * 16, 4);
           }
+        } else if (COMET_EPI_PAIR && C::NSTAGE == 2 && (COLS / 32) % 2 == 0) {
+          // two 64-byte chunks per round: both staging buffers filled, one proxy fence and one
+          // barrier, two TMA stores
+          const bool bf = P.ydt == COMET_BF16;
+#pragma unroll
+          for (int q = 0; q < COLS / 32; q += 2) {
+            if (leader) bulk_wait_group_read<0>();
+            named_bar_sync(2 + wg, 128);
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+              uint32_t pk[16];
+#pragma unroll
+              for (int i = 0; i < 16; ++i) {
+                const int c = (q + h) * 32 + 2 * i;
+                const float f0 = (acc[c] + init) * sw[c], f1 = (acc[c + 1] + init) * sw[c + 1];
+                if (bf) {
+                  __nv_bfloat162 hv = __floats2bfloat162_rn(f0, f1);
+                  pk[i] = *reinterpret_cast<uint32_t*>(&hv);
+                } else {
+                  __half2 hv = __floats2half2_rn(f0, f1);
+                  pk[i] = *reinterpret_cast<uint32_t*>(&hv);
+                }
+              }
+              const uint32_t rowa = smem_u32(stage + h * 8192) + r * 64;
+#pragma unroll
+              for (int k = 0; k < 4; ++k)
+                asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(rowa + ((k ^ swz) << 4)),
+                             "r"(pk[4 * k]), "r"(pk[4 * k + 1]), "r"(pk[4 * k + 2]), "r"(pk[4 * k + 3]) : "memory");
+            }
+            fence_proxy_async_smem();
+            named_bar_sync(2 + wg, 128);
+            if (leader) {
+              tma_store_2d(&P.map_y, stage, (n0 + col_n(wg, q * 32)) * 2, m0);
+              tma_store_2d(&P.map_y, stage + 8192, (n0 + col_n(wg, (q + 1) * 32)) * 2, m0);
+              bulk_commit_group();
+            }
+          }
+          ych = 0;
         } else {
           const bool bf = P.ydt == COMET_BF16;
 #pragma unroll
@@ -703,20 +810,29 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
             wait_buffer();
             uint32_t pk[16];
 #pragma unroll
-            for (int i = 0; i < 16; ++i) {
+            for (int i = 0; i < 16; i += 2) {
+              // y = (acc + init) s' = acc s' + init s'  (s' = s_w 2^9), as two FFMA2 pairs
               const int c = q * 32 + 2 * i;
-              const float f0 = (acc[c] + init) * sw[c] * 512.f, f1 = (acc[c + 1] + init) * sw[c + 1] * 512.f;
+              const float4 s4 = *reinterpret_cast<const float4*>(sw + c);
+              const float2 y0 = ffma2(make_float2(acc[c], acc[c + 1]), make_float2(s4.x, s4.y),
+                                      make_float2(init * s4.x, init * s4.y));
+              const float2 y1 = ffma2(make_float2(acc[c + 2], acc[c + 3]), make_float2(s4.z, s4.w),
+                                      make_float2(init * s4.z, init * s4.w));
               if (bf) {
-                __nv_bfloat162 hv = __floats2bfloat162_rn(f0, f1);
-                pk[i] = *reinterpret_cast<uint32_t*>(&hv);
+                __nv_bfloat162 h0 = __floats2bfloat162_rn(y0.x, y0.y), h1 = __floats2bfloat162_rn(y1.x, y1.y);
+                pk[i] = *reinterpret_cast<uint32_t*>(&h0);
+                pk[i + 1] = *reinterpret_cast<uint32_t*>(&h1);
               } else {
-                __half2 hv = __floats2half2_rn(f0, f1);
-                pk[i] = *reinterpret_cast<uint32_t*>(&hv);
+                __half2 h0 = __floats2half2_rn(y0.x, y0.y), h1 = __floats2half2_rn(y1.x, y1.y);
+                pk[i] = *reinterpret_cast<uint32_t*>(&h0);
+                pk[i + 1] = *reinterpret_cast<uint32_t*>(&h1);
               }
             }
             stage_and_store(pk, q * 32, 2);
+            if (q == 1 && threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 15, 4 * (it - it_begin) + 2);
           }
         }
+        if (threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 15, 4 * (it - it_begin) + 3);
       }
     }
     if (!DEBUG && (threadIdx.x & 127) == 0) bulk_wait_group<0>();   // all output stores done

@@ -50,3 +50,29 @@ if (t[10] > 0).any():
 print("  promo wake -> done               ", med([t[7][j] - t[6][j] for j in js]))
 print("  promo done(j) -> MMA issue(j+2)  ", med([issue(j + 2) - t[7][j] for j in js]))
 print("  MMA issue(j) -> MMA issue(j+2)   ", med([issue(j + 2) - issue(j) for j in js]))
+# tile boundaries (whole 64-K-block tiles, gate_up): promotion gap done(j) -> next wait(j+1) and
+# the MMA issue spacing across the boundary, against the interior
+nkb = int(sys.argv[3]) if len(sys.argv) > 3 else 64
+bj = [j for j in range(8, min(n_even * 2, 1000) - 2) if (j + 1) % nkb == 0 and t[7][j] > 0 and t[12][j + 1] > 0]
+ij = [j for j in range(8, min(n_even * 2, 1000) - 2) if (j + 1) % nkb != 0 and t[7][j] > 0 and t[12][j + 1] > 0]
+if bj:
+    print(f"  tile boundaries: {len(bj)}")
+    print("  promo done(j) -> next wait, boundary", med([t[12][j + 1] - t[7][j] for j in bj]))
+    print("  promo done(j) -> next wait, interior", med([t[12][j + 1] - t[7][j] for j in ij]))
+    print("  MMA issue(j) -> issue(j+1), boundary", med([issue(j + 1) - issue(j) for j in bj if issue(j + 1) > 0]))
+    print("  MMA issue(j) -> issue(j+1), interior", med([issue(j + 1) - issue(j) for j in ij if issue(j + 1) > 0]))
+    print("  promo wake(j+1) - promo done(j), boundary", med([t[6][j + 1] - t[7][j] for j in bj]))
+# epilogue phases (event 15 at 4 i + {0: before the WG-group barrier, 1: after it, 2: after chunk
+# 1's store, 3: after the last chunk}) against the tile's last promotion done
+if bj:
+    e15 = t[15]
+    rows = []
+    for k, j in enumerate(bj):
+        i = (j + 1) // nkb - 1
+        if e15[4 * i + 3] > 0:
+            rows.append((e15[4 * i] - t[7][j], e15[4 * i + 1] - e15[4 * i], e15[4 * i + 2] - e15[4 * i + 1],
+                         e15[4 * i + 3] - e15[4 * i + 2], t[12][j + 1] - e15[4 * i + 3]))
+    if rows:
+        r = np.array(rows)
+        print("  epilogue: done->start, group barrier, chunks 0-1, chunks 2-3, ->next wait (medians)",
+              np.median(r, axis=0).astype(int).tolist())
