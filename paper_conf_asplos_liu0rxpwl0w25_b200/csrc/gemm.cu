@@ -723,7 +723,8 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
     return fail(COMET_ERR_CUDA, "cuTensorMapEncodeTiled failed for the packed weights");
   if (normal && !dbg) {
     const int esz = ydt == COMET_F32 ? 4 : 2;
-    if (!make_map_2d(&prm.map_y, y, (uint64_t)p.N * esz, (uint64_t)p.M, (uint64_t)ldy * esz, 64, 128,
+    if (!make_map_2d(&prm.map_y, y, (uint64_t)p.N * esz, (uint64_t)p.M, (uint64_t)ldy * esz, 64,
+                     COMET_EPI_WARP ? 32 : 128,
                      CU_TENSOR_MAP_SWIZZLE_64B))
       return fail(COMET_ERR_CUDA, "cuTensorMapEncodeTiled failed for the output");
   }

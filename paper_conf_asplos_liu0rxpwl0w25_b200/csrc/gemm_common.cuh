@@ -17,7 +17,8 @@ constexpr int kThreads = 512;
 struct __align__(64) GemmParams {
   CUtensorMap map_x;
   CUtensorMap map_w;
-  CUtensorMap map_y;         // prefill kernel: Y as bytes [M][N*esz], box 64 B x 128 rows, 64B swizzle
+  CUtensorMap map_y;         // prefill kernel: Y as bytes [M][N*esz], box 64 B x 128 rows (32 rows
+                             // with COMET_EPI_WARP), 64B swizzle
   CUtensorMap map_s;         // decode kernel: act_scales [nb][Mp] f32, box NT x KS
   const float* scales;       // [nb][Mp]
   const float* corr;         // [Mp]
@@ -84,6 +85,9 @@ __device__ __forceinline__ WorkItem load_item(const GemmParams& P, int idx, bool
 #endif
 #ifndef COMET_TRACE
 #define COMET_TRACE 0       // 1: timeline trace only (tools/trace_gemm.py), no ablation hooks
+#endif
+#ifndef COMET_EPI_WARP
+#define COMET_EPI_WARP 1   // prefill epilogue: every warp stores its own 32 rows (no warpgroup barriers)
 #endif
 #ifndef COMET_ABLATE_CT
 #define COMET_ABLATE_CT 0   // compile-time ablation bits (timing experiments only; wrong results)

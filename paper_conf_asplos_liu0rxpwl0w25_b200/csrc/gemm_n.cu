@@ -737,6 +737,8 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
         uint8_t* stage = sY + wg * C::NSTAGE * 8192;
         const uint32_t swz = (uint32_t)((r >> 1) & 3);
         const bool leader = (threadIdx.x & 127) == 0;     // thread 0 of the WG (row 0)
+        // COMET_EPI_WARP: each warp stores its own 32 rows with its own TMA store (box 32 rows),
+        // synchronising only within the warp; otherwise one store per warpgroup chunk.
         auto stage_and_store = [&](const uint32_t (&pk)[16], int ncol_off, int esz) {
           // caller: buffer (ych % NSTAGE) is free (see the wait below)
           const uint32_t rowa = smem_u32(stage + (ych % C::NSTAGE) * 8192) + r * 64;
@@ -745,16 +747,30 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
             asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(rowa + ((k ^ swz) << 4)),
                          "r"(pk[4 * k]), "r"(pk[4 * k + 1]), "r"(pk[4 * k + 2]), "r"(pk[4 * k + 3]) : "memory");
           fence_proxy_async_smem();
-          named_bar_sync(2 + wg, 128);
-          if (leader) {
-            tma_store_2d(&P.map_y, stage + (ych % C::NSTAGE) * 8192, (n0 + col_n(wg, ncol_off)) * esz, m0);
-            bulk_commit_group();
+          if (COMET_EPI_WARP) {
+            __syncwarp();
+            if (lane == 0) {
+              tma_store_2d(&P.map_y, stage + (ych % C::NSTAGE) * 8192 + (warp & 3) * 32 * 64,
+                           (n0 + col_n(wg, ncol_off)) * esz, m0 + (warp & 3) * 32);
+              bulk_commit_group();
+            }
+          } else {
+            named_bar_sync(2 + wg, 128);
+            if (leader) {
+              tma_store_2d(&P.map_y, stage + (ych % C::NSTAGE) * 8192, (n0 + col_n(wg, ncol_off)) * esz, m0);
+              bulk_commit_group();
+            }
           }
           ++ych;
         };
         auto wait_buffer = [&]() {                        // the store NSTAGE chunks ago has read its buffer
-          if (leader) bulk_wait_group_read<C::NSTAGE - 1>();
-          named_bar_sync(2 + wg, 128);
+          if (COMET_EPI_WARP) {
+            if (lane == 0) bulk_wait_group_read<C::NSTAGE - 1>();
+            __syncwarp();
+          } else {
+            if (leader) bulk_wait_group_read<C::NSTAGE - 1>();
+            named_bar_sync(2 + wg, 128);
+          }
         };
         if (P.ydt == COMET_F32) {
 #pragma unroll
@@ -765,7 +781,7 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
             for (int i = 0; i < 16; ++i) pk[i] = __float_as_uint((acc[q * 16 + i] + init) * sw[q * 16 + i]);
             stage_and_store(pk, q * 16, 4);
           }
-        } else if (COMET_EPI_PAIR && C::NSTAGE == 2 && (COLS / 32) % 2 == 0) {
+        } else if (COMET_EPI_PAIR && !COMET_EPI_WARP && C::NSTAGE == 2 && (COLS / 32) % 2 == 0) {
           // two 64-byte chunks per round: both staging buffers filled, one proxy fence and one
           // barrier, two TMA stores
           const bool bf = P.ydt == COMET_BF16;
@@ -835,7 +851,7 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
         if (threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 15, 4 * (it - it_begin) + 3);
       }
     }
-    if (!DEBUG && (threadIdx.x & 127) == 0) bulk_wait_group<0>();   // all output stores done
+    if (!DEBUG && (COMET_EPI_WARP ? lane == 0 : (threadIdx.x & 127) == 0)) bulk_wait_group<0>();   // all output stores done
   }
 
   tc_fence_before();
