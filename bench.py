@@ -242,7 +242,8 @@ def next_rows(cb, torch, dev, peaks, iters=20):
     """SURVEY §8(f) rows built beyond the hot path, timed live (L2 left clean before every
     launch, CUDA events, median): NEXT-1 fused channel permutation in kernel 1 (LLaMA-3-70B
     layer inputs at M = 4096, permutation calibrated on a separate sample) against the
-    identity kernel, and NEXT-4 KV4 quantise / dequantise of a LLaMA-3-70B KV cache
+    identity kernel, NEXT-3 group-wise weight scales on the decode GEMM against per-channel
+    scales, and NEXT-4 KV4 quantise / dequantise of a LLaMA-3-70B KV cache
     (8 KV heads x 128 = 1024 channels, 32768 tokens, group 128).  GB/s = algorithmic bytes."""
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
     flush_rd = torch.ones(64 << 20, dtype=torch.float32, device=dev)
@@ -278,6 +279,29 @@ def next_rows(cb, torch, dev, peaks, iters=20):
                                               "identity_us": round(us_i, 2), "outlier_channels": n_out,
                                               "int8_blocks": int(tags.sum())}
         del up, x, act, sc
+    # NEXT-3: group-wise weight scales on the decode GEMM (LLaMA-3-70B gate/up, M = 1 and 32),
+    # against the per-channel-scale GEMM on the same inputs
+    K, N = 8192, 28672
+    rng = np.random.default_rng(21)
+    tags = synth.make_tags(K, FRAC, rng)
+    w, s_w = synth.make_weights(N, K, rng)
+    wp = cb.pack_weight(torch.from_numpy(w).to(dev))
+    swd = torch.from_numpy(s_w).to(dev)
+    swg = torch.from_numpy(np.repeat(s_w[None, :], K // 128, axis=0)
+                           * rng.uniform(0.5, 1.5, size=(K // 128, N)).astype(np.float32)).to(dev)
+    del w
+    for M in (1, 32):
+        x = torch.from_numpy(synth.make_activations(M, K, tags, rng)).to(dev)
+        plan = cb.Plan(M, N, K, tags)
+        act, sc = cb.quantize_act(x, tags)
+        y = torch.empty((M, N), dtype=torch.float16, device=dev)
+        nbytes = N * K // 2 + swg.numel() * 4 + act.numel() + sc.numel() * 4 + M * N * 2
+        us_g = t(lambda: cb.w4ax_gemm_grouped(plan, act, sc, wp, swg, out=y))
+        us_c = t(lambda: cb.w4ax_gemm(plan, act, sc, wp, swd, out=y))
+        out[f"grouped_scales_gemm_gate_up_M{M}"] = {"us": round(us_g, 2), "GB/s": round(nbytes / us_g / 1e3, 1),
+                                                    "frac_hbm": round(nbytes / us_g / 1e3 / hbm, 3),
+                                                    "per_channel_us": round(us_c, 2)}
+    del wp, swg
     T, C, G = 32768, 1024, 128
     kv = torch.from_numpy(synth.make_kv(T, C, np.random.default_rng(0))).to(dev)
     codes, scales, mins = cb.kv4_quantize(kv, G)

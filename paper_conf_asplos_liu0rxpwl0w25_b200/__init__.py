@@ -92,6 +92,7 @@ def lib():
         "comet_plan_info": (I32, [P, ctypes.POINTER(PlanInfo)]),
         "comet_plan_describe": (I32, [P, P, I64, ctypes.POINTER(I64)]),
         "comet_w4ax_gemm": (I32, [P, P, P, P, P, P, I32, I64, P, P, P, SZ, P]),
+        "comet_w4ax_gemm_grouped": (I32, [P, P, P, P, P, P, I32, I64, P, P, SZ, P]),
         "comet_linear_scratch_bytes": (SZ, [P, I32, I32]),
         "comet_w4ax_linear_host": (I32, [P, P, I32, P, P, P, I32, P, SZ, P, SZ, P]),
         "comet_w4ax_linear_host_async": (I32, [P, P, I32, P, P, P, I32, P, SZ, P, SZ, P]),
@@ -334,6 +335,27 @@ def w4ax_gemm(plan: Plan, act_packed, act_scales, w_packed, w_scales, *, out=Non
     if debug:
         return out, dacc
     return out
+
+
+def w4ax_gemm_grouped(plan: Plan, act_packed, act_scales, w_packed, w_scales_grouped, *, out=None,
+                      out_dtype=None, debug: bool = False, stream=None):
+    """comet_w4ax_gemm_grouped (NEXT-3): group-wise weight scales w_scales_grouped [K/128, N]
+    float32.  The plan must have orientation 1.  Returns y (and the exact int32 accumulators)."""
+    import torch
+    dev = act_packed.device
+    if out is None:
+        out = torch.empty((plan.M, plan.N), dtype=out_dtype or torch.float16, device=dev)
+    dacc = torch.empty((plan.M, plan.N), dtype=torch.int32, device=dev) if debug else None
+    ws = plan.workspace(dev)
+    assert w_scales_grouped.dtype == torch.float32 and w_scales_grouped.is_contiguous()
+    _check(lib().comet_w4ax_gemm_grouped(plan.handle, ctypes.c_void_p(act_packed.data_ptr()),
+                                         ctypes.c_void_p(act_scales.data_ptr()),
+                                         ctypes.c_void_p(w_packed.data_ptr()),
+                                         ctypes.c_void_p(w_scales_grouped.data_ptr()),
+                                         ctypes.c_void_p(out.data_ptr()), _dt(out.dtype), out.stride(0),
+                                         ctypes.c_void_p(dacc.data_ptr()) if dacc is not None else None,
+                                         ctypes.c_void_p(ws.data_ptr()), ws.numel(), _stream(stream)))
+    return (out, dacc) if debug else out
 
 
 def w4ax_linear(plan: Plan, x, w_packed, w_scales, *, perm=None, out_dtype=None, stream=None):

@@ -399,6 +399,32 @@ comet_status_t comet_w4ax_gemm(comet_plan_t plan, const void* act_packed, const 
   return st;
 }
 
+comet_status_t comet_w4ax_gemm_grouped(comet_plan_t plan, const void* act_packed, const float* act_scales,
+                                       const void* w_packed, const float* w_scales_grouped, void* y,
+                                       comet_dtype_t ydt, int64_t ldy, int32_t* debug_acc,
+                                       void* workspace, size_t ws_bytes, void* stream) {
+  g_launches = 0;
+  if (!plan || !act_packed || !act_scales || !w_packed || !w_scales_grouped || !y)
+    return fail(COMET_ERR_INVALID_ARG, "NULL pointer argument");
+  Plan& p = plan->p;
+  if (ydt != COMET_F16 && ydt != COMET_BF16 && ydt != COMET_F32) return fail(COMET_ERR_INVALID_ARG, "bad ydt");
+  const int esz = ydt == COMET_F32 ? 4 : 2;
+  if (ldy < p.N || (ldy * esz) % 16 != 0) return fail(COMET_ERR_MISALIGNED, "ldy must be >= N with ldy*sizeof(y) % 16 == 0");
+  if ((reinterpret_cast<uintptr_t>(act_packed) & 255u) != 0) return fail(COMET_ERR_MISALIGNED, "act_packed must be 256-byte aligned");
+  if (!aligned16(act_scales) || !aligned16(w_packed) || !aligned16(w_scales_grouped) || !aligned16(y) ||
+      (debug_acc && !aligned16(debug_acc)) || (workspace && !aligned16(workspace)))
+    return fail(COMET_ERR_MISALIGNED, "device pointers must be 16-byte aligned");
+  if (p.orientation != 1)
+    return fail(COMET_ERR_UNSUPPORTED_SHAPE, "group-wise weight scales need a plan with orientation 1 (weights on the MMA M side)");
+  comet_status_t st = check_device();
+  if (st != COMET_OK) return st;
+  int launches = 0;
+  st = launch_gemm(p, act_packed, act_scales, w_packed, w_scales_grouped, y, ydt, ldy, debug_acc, nullptr,
+                   workspace, ws_bytes, static_cast<cudaStream_t>(stream), &launches, true);
+  g_launches = launches;
+  return st;
+}
+
 // Pipelined host path: chunks of kLinChunk token rows once M >= 2 kLinChunk.
 static constexpr int64_t kLinChunk = 1024;
 

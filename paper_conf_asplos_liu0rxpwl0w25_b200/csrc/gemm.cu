@@ -72,7 +72,7 @@ constexpr int kPromoWarp0 = 12;
 // stage: warp 4 + 4h + q widens rows 32q .. 32q+31 of K-blocks [h KS/2, (h+1) KS/2).
 // TMEM columns: [0, 2 * 32 KS) two widened-weight A buffers (alternate stages), then NACC
 // accumulator sets of KS x NT columns (one accumulator per K-block of a stage).
-template <int NT>
+template <int NT, bool GS = false>
 struct Cfg {
   static constexpr int KS = NT <= 32 ? 4 : 2;                  // K-blocks per stage
   static constexpr int NA = COMET_DEC_NA;                       // widened-weight A buffers
@@ -84,7 +84,11 @@ struct Cfg {
   static constexpr int XKB_BYTES = NT * 128;                   // one K-block of codes
   static constexpr int W_BYTES = KS * kTileW * 64;             // KS K-blocks of packed weights
   static constexpr int S_BYTES = KS * NT * 4;
-  static constexpr int X_STAGE = (KS * XKB_BYTES + S_BYTES + 1023) / 1024 * 1024;
+  // GS (group-wise weight scales): the X stage also carries the K-blocks' code sums qsum[b][m]
+  // (int16, [KS][NT]) and weight scales s_w[b][n] (f32, [KS][128])
+  static constexpr int Q_BYTES = GS ? KS * NT * 2 : 0;
+  static constexpr int G_BYTES = GS ? KS * kTileW * 4 : 0;
+  static constexpr int X_STAGE = (KS * XKB_BYTES + S_BYTES + Q_BYTES + G_BYTES + 1023) / 1024 * 1024;
   static constexpr int SX = 4;                                 // X ring depth
   static constexpr int SMEM_BUDGET = 224 * 1024;            // 227 KB minus alignment, barriers, tags
   static constexpr int SW_RAW = (SMEM_BUDGET - SX * X_STAGE) / W_BYTES;
@@ -105,9 +109,15 @@ __device__ __forceinline__ void tmem_ld_cols(uint32_t taddr, uint32_t* r) {
   else tmem_ld_32x32b_x16(taddr, r);
 }
 
-template <int NT, int DEBUG>
+// GS (NEXT-3, reading R18): group-wise weight scales s_w[b][n], one per (128-channel block,
+// output channel), given as w_scales [nb][N].  The weight scale no longer factors out of the K
+// loop, so the promotion folds s_a[m,b] * s_w[b,n] per K-block and removes the offset-binary
+// term per block: INT4 block  acc += s_a s_w (2^-9 sum q u - 2^-6 qsum)   (= s_a s_w 2^-9 sum q w)
+//                 INT8 block  acc += s_a s_w 2^-13 (16 sum q w)
+// and the epilogue only scales by 2^9.
+template <int NT, int DEBUG, bool GS>
 __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ GemmParams P) {
-  using C = Cfg<NT>;
+  using C = Cfg<NT, GS>;
   constexpr int SW = C::SW;
   constexpr int SX = C::SX;
   constexpr int NA = C::NA;
@@ -119,6 +129,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
   auto sW = [&](int st) { return smem + st * C::W_BYTES; };
   auto sX = [&](int st) { return smem + SW * C::W_BYTES + st * C::X_STAGE; };
   auto sS = [&](int st) { return smem + SW * C::W_BYTES + st * C::X_STAGE + KS * C::XKB_BYTES; };
+  auto sQ = [&](int st) { return sS(st) + C::S_BYTES; };          // GS only
+  auto sG = [&](int st) { return sS(st) + C::S_BYTES + C::Q_BYTES; };
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + C::SMEM_DATA);
   uint64_t* full_w = bars;                  // [SW]   TMA -> widen
   uint64_t* empty_w = full_w + SW;          // [SW]   8 widen warps -> W producer
@@ -207,11 +219,16 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
       for (int it = it_begin; it < it_end; ++it) {
         const WorkItem w = load_item(P, it, debug);
         const int m0 = (w.tile % P.n_m_tiles) * NT;
+        const int n0 = (w.tile / P.n_m_tiles) * kTileW;
         for (int kb = w.kb_begin; kb < w.kb_end; kb += KS) {
           mbar_wait(&empty_x[st], ph ^ 1);
-          mbar_arrive_expect_tx(&full_x[st], KS * C::XKB_BYTES + C::S_BYTES);
+          mbar_arrive_expect_tx(&full_x[st], KS * C::XKB_BYTES + C::S_BYTES + C::Q_BYTES + C::G_BYTES);
           tma_load_3d(sX(st), &P.map_x, &full_x[st], 0, m0, kb);
           tma_load_2d(sS(st), &P.map_s, &full_x[st], m0, kb);
+          if (GS) {
+            tma_load_2d(sQ(st), &P.map_q, &full_x[st], m0, kb);
+            tma_load_2d(sG(st), &P.map_g, &full_x[st], n0, kb);
+          }
           if (++st == SX) { st = 0; ph ^= 1; }
         }
       }
@@ -438,8 +455,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
       const int n = n0 + row;
       // epilogue operands loaded now (their latency overlaps the K loop): s_w[n] and, for the
       // owner, corr[m] (the offset-binary weight correction, applied once at the end)
-      const float swv = n < P.N ? __ldg(P.w_scales + n) * 512.f : 0.f;
-      constexpr bool kEarlyCorr = NT <= 32;        // registers: NT > 32 loads corr at the end
+      const float swv = GS ? 512.f : (n < P.N ? __ldg(P.w_scales + n) * 512.f : 0.f);
+      constexpr bool kEarlyCorr = NT <= 32 && !GS; // registers: NT > 32 loads corr at the end
       float cr[kEarlyCorr ? NT : 1];
       if constexpr (kEarlyCorr) {
 #pragma unroll
@@ -465,6 +482,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
         for (int c = 0; c < nk; ++c) {
           const int kb = kb0 + c;
           const bool is8 = lds_u8(s_tags_a + kb) != 0;
+          float swb = 1.f;
+          if (GS) asm volatile("ld.shared.f32 %0, [%1];" : "=f"(swb) : "r"(smem_u32(sG(sx)) + 4u * (c * kTileW + row)));
           const uint32_t tcol = tbase + C::ACC_COL + accs * C::ACC_SET + c * NT + lane_addr;
 #pragma unroll
           for (int ch = 0; ch < NT / CH; ++ch) {
@@ -481,13 +500,35 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
               const float4 f = lds128f(sbase + (c * NT + ch * CH + j) * 4);
               sc[j] = f.x; sc[j + 1] = f.y; sc[j + 2] = f.z; sc[j + 3] = f.w;
             }
+            if (GS) {
+              // fold the block's weight scale into the per-token scales
+#pragma unroll
+              for (int j = 0; j < CH; ++j) sc[j] *= swb;
+            }
+            float qc[GS ? CH : 1];                    // INT4 offset term 2^-6 qsum[b][m] (GS)
+            if (GS && !is8) {
+              // code sums of this K-block's tokens from the X stage (broadcast shared loads; the
+              // box covers rows >= Mp with zeros)
+              const uint32_t qa = smem_u32(sQ(sx)) + 2u * (c * NT + ch * CH);
+#pragma unroll
+              for (int j = 0; j < CH; j += 8) {
+                const uint4 q8 = lds128(qa + 2u * j);
+                const uint32_t qw[4] = {q8.x, q8.y, q8.z, q8.w};
+#pragma unroll
+                for (int e = 0; e < 4; ++e) {
+                  qc[j + 2 * e] = (float)(int16_t)(qw[e] & 0xFFFFu) * 0.015625f;
+                  qc[j + 2 * e + 1] = (float)(int16_t)(qw[e] >> 16) * 0.015625f;
+                }
+              }
+            }
             tmem_wait_ld();
             if (!is8) {
 #pragma unroll
               for (int j = 0; j < CH; j += 2) {
                 const int a = ch * CH + j;
-                const float2 y = ffma2(make_float2(__uint_as_float(v[j]), __uint_as_float(v[j + 1])),
-                                       make_float2(sc[j], sc[j + 1]), make_float2(acc[a], acc[a + 1]));
+                float2 vv = make_float2(__uint_as_float(v[j]), __uint_as_float(v[j + 1]));
+                if (GS) vv = make_float2(vv.x - qc[j], vv.y - qc[j + 1]);   // exact: multiples of 2^-9 below 2^14
+                const float2 y = ffma2(vv, make_float2(sc[j], sc[j + 1]), make_float2(acc[a], acc[a + 1]));
                 acc[a] = y.x;
                 acc[a + 1] = y.y;
               }
@@ -581,7 +622,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
           const int64_t m = m0 + j;
           if (m < P.M) {
             float c0;
-            if constexpr (kEarlyCorr) c0 = cr[j];
+            if constexpr (GS) c0 = 0.f;                // the offset term was removed per block
+            else if constexpr (kEarlyCorr) c0 = cr[j];
             else c0 = owner ? __ldg(P.corr + m) * 0.001953125f : 0.f;
             const float yv = (acc[j] - c0) * swv;
             const int64_t off = m * P.ldy + n;
@@ -602,12 +644,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
   if (warp == 2) tmem_dealloc<512>(tbase);
 }
 
-template <int NT, int DEBUG>
+template <int NT, int DEBUG, bool GS = false>
 cudaError_t launch_nt(const GemmParams& prm, int grid, cudaStream_t stream) {
-  using C = Cfg<NT>;
+  using C = Cfg<NT, GS>;
   static bool attr_set = false;
   if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(k_w4ax<NT, DEBUG>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_BYTES);
+    cudaError_t e = cudaFuncSetAttribute(k_w4ax<NT, DEBUG, GS>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_BYTES);
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
@@ -621,7 +663,7 @@ cudaError_t launch_nt(const GemmParams& prm, int grid, cudaStream_t stream) {
   attr[0].val.programmaticStreamSerializationAllowed = COMET_DEC_PDL;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  return cudaLaunchKernelEx(&cfg, k_w4ax<NT, DEBUG>, prm);
+  return cudaLaunchKernelEx(&cfg, k_w4ax<NT, DEBUG, GS>, prm);
 }
 
 PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
@@ -677,8 +719,10 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
                            const void* w_packed, const float* w_scales, void* y,
                            comet_dtype_t ydt, int64_t ldy, int32_t* debug_acc,
                            int32_t* debug_acc_blocks, void* workspace, size_t ws_bytes,
-                           cudaStream_t stream, int* launches) {
+                           cudaStream_t stream, int* launches, bool grouped) {
   using namespace gemm;
+  if (grouped && p.orientation != 1)
+    return fail(COMET_ERR_UNSUPPORTED_SHAPE, "group-wise weight scales need a plan with orientation 1 (weights on the MMA M side)");
   *launches = 0;
   const bool dbg = debug_acc != nullptr || debug_acc_blocks != nullptr;
   const int debug = debug_acc_blocks ? 2 : (dbg ? 1 : 0);
@@ -715,6 +759,19 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
     if (!make_map(&prm.map_s, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, act_scales, sd, ss, sb,
                   CU_TENSOR_MAP_SWIZZLE_NONE))
       return fail(COMET_ERR_CUDA, "cuTensorMapEncodeTiled failed for the activation scales");
+    if (grouped) {
+      // qsum [nb][Mp] int16, box KS x NT; grouped weight scales [nb][N] f32, box KS x 128
+      const uint64_t qs[1] = {(uint64_t)L.Mp * 2};
+      if (!make_map(&prm.map_q, CU_TENSOR_MAP_DATA_TYPE_UINT16, 2, base + L.qsum_off, sd, qs, sb,
+                    CU_TENSOR_MAP_SWIZZLE_NONE))
+        return fail(COMET_ERR_CUDA, "cuTensorMapEncodeTiled failed for the code sums");
+      const uint64_t gd[2] = {(uint64_t)p.N, (uint64_t)p.nb};
+      const uint64_t gs[1] = {(uint64_t)p.N * 4};
+      const uint32_t gb[2] = {(uint32_t)kTileW, ks};
+      if (!make_map(&prm.map_g, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, w_scales, gd, gs, gb,
+                    CU_TENSOR_MAP_SWIZZLE_NONE))
+        return fail(COMET_ERR_CUDA, "cuTensorMapEncodeTiled failed for the group-wise weight scales");
+    }
   }
   // prefill: 64-byte rows (one K-block) with 64B swizzle; decode: 128-byte rows (two K-blocks)
   if (!make_map_2d(&prm.map_w, w_packed, (uint64_t)(p.K / 2), (uint64_t)p.N, (uint64_t)(p.K / 2),
@@ -770,7 +827,16 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
   if (normal) {
     e = launch_gemm_n(prm, grid, tile_w, cg, debug, stream);
   } else if (dbg) {
-    e = debug == 2 ? launch_nt<32, 2>(prm, grid, stream) : launch_nt<32, 1>(prm, grid, stream);
+    if (grouped) e = debug == 2 ? launch_nt<32, 2, true>(prm, grid, stream) : launch_nt<32, 1, true>(prm, grid, stream);
+    else e = debug == 2 ? launch_nt<32, 2>(prm, grid, stream) : launch_nt<32, 1>(prm, grid, stream);
+  } else if (grouped) {
+    switch (tile_m) {
+      case 16: e = launch_nt<16, 0, true>(prm, grid, stream); break;
+      case 32: e = launch_nt<32, 0, true>(prm, grid, stream); break;
+      case 64: e = launch_nt<64, 0, true>(prm, grid, stream); break;
+      case 128: e = launch_nt<128, 0, true>(prm, grid, stream); break;
+      default: return fail(COMET_ERR_UNSUPPORTED_SHAPE, "unsupported tile_n");
+    }
   } else {
     switch (tile_m) {
       case 16: e = launch_nt<16, 0>(prm, grid, stream); break;

@@ -20,6 +20,8 @@ struct __align__(64) GemmParams {
   CUtensorMap map_y;         // prefill kernel: Y as bytes [M][N*esz], box 64 B x 128 rows (32 rows
                              // with COMET_EPI_WARP), 64B swizzle
   CUtensorMap map_s;         // decode kernel: act_scales [nb][Mp] f32, box NT x KS
+  CUtensorMap map_q;         // decode kernel, grouped scales: qsum [nb][Mp] int16, box NT x KS
+  CUtensorMap map_g;         // decode kernel, grouped scales: s_w [nb][N] f32, box 128 x KS
   const float* scales;       // [nb][Mp]
   const float* corr;         // [Mp]
   const int16_t* qsum;       // [nb][Mp]

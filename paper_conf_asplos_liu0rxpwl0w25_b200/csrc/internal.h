@@ -92,7 +92,7 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
                            const void* w_packed, const float* w_scales, void* y,
                            comet_dtype_t ydt, int64_t ldy, int32_t* debug_acc,
                            int32_t* debug_acc_blocks, void* workspace, size_t ws_bytes,
-                           cudaStream_t stream, int* launches);
+                           cudaStream_t stream, int* launches, bool grouped = false);
 // act layout
 void act_layout(int64_t M, int64_t K, comet_act_layout_t* out);
 

@@ -268,3 +268,40 @@ def test_fig8_remap_and_decomposition_bounds():
     assert planner.makespan(segs, tags, g["cost_int4"], g["cost_int8"]) == Fraction(g["expected"]["remapped_best_whole_tile"])
     with pytest.raises(AssertionError):
         planner.check_cover(segs[:3], g["n_output_tiles"], len(tags))
+
+
+# ---------- NEXT-3: group-wise weight scales (oracle/grouped.py, reading R18) ----------------
+
+def test_grouped_equal_block_scales_reduce_to_per_channel():
+    from oracle import grouped
+    p = synth.make_problem(12, 512, 64, frac=0.25, seed=31)
+    y, acc, codes, scales = oracle.w4ax(p.x, p.tags, p.w, p.s_w)
+    s_wg = np.repeat(p.s_w[None, :], 4, axis=0)
+    yg = grouped.dequant_grouped(acc, scales, s_wg)
+    assert np.allclose(yg, y, rtol=1e-12, atol=0)
+
+
+def test_grouped_exact_rational_config1():
+    from oracle import grouped
+    p = synth.config1()
+    rng = np.random.default_rng(4)
+    s_wg = rng.uniform(0.5, 1.5, size=(2, p.N)).astype(np.float32) / 64
+    _, acc, codes, scales = oracle.w4ax(p.x, p.tags, p.w, p.s_w)
+    yg = grouped.dequant_grouped(acc, scales, s_wg)
+    for m in (0, 7, 15):
+        for n in (0, 100, 255):
+            exact = sum(Fraction(float(scales[m, b])) * Fraction(float(s_wg[b, n])) * int(acc[b, m, n]) for b in range(2))
+            assert abs(Fraction(float(yg[m, n])) - exact) <= abs(exact) * Fraction(1, 2 ** 50)
+
+
+def test_grouped_within_quantisation_error_bound():
+    from oracle import grouped
+    p = synth.make_problem(16, 512, 64, frac=0.25, seed=33)
+    rng = np.random.default_rng(5)
+    s_wg = rng.uniform(0.5, 1.5, size=(4, 64)).astype(np.float32) / (8 * np.sqrt(512))
+    _, acc, codes, scales = oracle.w4ax(p.x, p.tags, p.w, p.s_w)
+    y = grouped.dequant_grouped(acc, scales, s_wg)
+    wd = p.w.astype(np.float64) * np.repeat(s_wg.astype(np.float64).T, BLOCK, axis=1)
+    exact = p.x.astype(np.float64) @ wd.T
+    half_step = np.repeat(scales.astype(np.float64), BLOCK, axis=1) / 2 * (1 + 2.0 ** -20)
+    assert np.all(np.abs(y - exact) <= half_step @ np.abs(wd).T + 1e-12)
