@@ -15,6 +15,10 @@ Parity status per function:
   dequant         pinned (closed form I4, exact Fraction check)
   w4ax_rows       pinned (equals the three functions above, which are pinned)
   planner.*       pinned (Fig. 8 worked example)
+  calibrate.*     pinned (NEXT-1: planted outliers, brute-force order, statistics.median, P:L140
+                  equivalence bound, "< 20 %" claim) -- oracle/calibrate.py
+  kv4.*           pinned (NEXT-4: exact-rational brute force, round-trip bound) -- oracle/kv4.py
+  grouped.*       pinned (NEXT-3: per-channel reduction, exact Fraction, error bound) -- oracle/grouped.py
 """
 from __future__ import annotations
 
