@@ -17,6 +17,10 @@
 #include "internal.h"
 #include "sm100.cuh"
 
+#ifndef COMET_PERM_GATHER
+#define COMET_PERM_GATHER 1   // decode-sized M: fused permutation by direct L1-cached gathers
+#endif
+
 namespace comet {
 namespace {
 
@@ -170,13 +174,17 @@ __device__ __forceinline__ LaneOut quantize32(const float (&v)[32], bool is8) {
 // 8g + l/4 with sub = l%4, loading 4 x 16 B at channel offsets 32 j + 8 sub -- every load
 // instruction reads 64 contiguous bytes of each of the 8 blocks (whole 32-byte sectors) and
 // every code store writes 32 contiguous bytes per block.
-template <bool BF16, int WPR>
+// GATHER: the fused channel permutation (NEXT-1) as direct gathers -- channel k of the row is
+// read from x[m, perm[k]] with 16-bit L1-cached loads (the CTA's rows are re-read sector by
+// sector from L1; calibrated permutations are ascending runs, so a warp's gathers coalesce).
+template <bool BF16, int WPR, bool GATHER = false>
 __global__ void __launch_bounds__(256) k_quantize(const uint16_t* __restrict__ x, int64_t M,
                                                   int64_t K, int64_t ldx, int64_t Mp, TagMask tags,
                                                   uint8_t* __restrict__ codes,
                                                   int16_t* __restrict__ qsum,
                                                   float* __restrict__ corr,
-                                                  float* __restrict__ scales) {
+                                                  float* __restrict__ scales,
+                                                  const int32_t* __restrict__ perm = nullptr) {
   constexpr int ROWS = 8 / WPR;
   __shared__ float s_part[8];
   // let a programmatic dependent (the decode GEMM) launch now: it streams weights while this
@@ -196,9 +204,34 @@ __global__ void __launch_bounds__(256) k_quantize(const uint16_t* __restrict__ x
       const int b = g * 8 + bl;
       const bool bvalid = b < nb;
       uint4 raw[4];
+      if (GATHER) {
+        const uint16_t* xr = x + m * ldx;
+        const int kmax = (int)K - 1;
+        int idx[32];
 #pragma unroll
-      for (int j = 0; j < 4; ++j)
-        raw[j] = bvalid ? ldg_stream(xrow + b * kBlockK + 32 * j) : make_uint4(0, 0, 0, 0);
+        for (int j = 0; j < 4; ++j) {
+          const int k0 = b * kBlockK + 32 * j + sub * 8;
+          int4 p0 = make_int4(0, 0, 0, 0), p1 = make_int4(0, 0, 0, 0);
+          if (bvalid) {
+            p0 = __ldg(reinterpret_cast<const int4*>(perm + k0));
+            p1 = __ldg(reinterpret_cast<const int4*>(perm + k0 + 4));
+          }
+          idx[8 * j + 0] = p0.x; idx[8 * j + 1] = p0.y; idx[8 * j + 2] = p0.z; idx[8 * j + 3] = p0.w;
+          idx[8 * j + 4] = p1.x; idx[8 * j + 5] = p1.y; idx[8 * j + 6] = p1.z; idx[8 * j + 7] = p1.w;
+        }
+        uint32_t h[32];
+#pragma unroll
+        for (int i = 0; i < 32; ++i)
+          h[i] = bvalid ? (uint32_t)__ldg(xr + min(max(idx[i], 0), kmax)) : 0u;
+#pragma unroll
+        for (int j = 0; j < 4; ++j)
+          raw[j] = make_uint4(h[8 * j] | (h[8 * j + 1] << 16), h[8 * j + 2] | (h[8 * j + 3] << 16),
+                              h[8 * j + 4] | (h[8 * j + 5] << 16), h[8 * j + 6] | (h[8 * j + 7] << 16));
+      } else {
+#pragma unroll
+        for (int j = 0; j < 4; ++j)
+          raw[j] = bvalid ? ldg_stream(xrow + b * kBlockK + 32 * j) : make_uint4(0, 0, 0, 0);
+      }
       float v[32];
 #pragma unroll
       for (int j = 0; j < 4; ++j) {
@@ -590,6 +623,27 @@ static cudaError_t launch_qp(const void* x, int64_t M, int64_t K, int64_t ldx, c
   comet_act_layout_t L;
   act_layout(M, K, &L);
   uint8_t* base = static_cast<uint8_t*>(act_packed);
+  // M <= 32 (decode): direct gathers (one row per CTA, the row's sectors re-read from L1) beat
+  // the staged rows -- 8.4 vs 10.2 us at M = 1, 16.4 vs 18.4 at M = 32, K = 28672; at prefill
+  // sizes the staged kernel wins on long rows (141 vs 149 us at K = 28672) and on arbitrary
+  // permutations (157 vs 344 us), tools/quant_time.py.
+  if (COMET_PERM_GATHER && M <= 32) {
+    uint8_t* codes = base + L.codes_off;
+    int16_t* qsum = reinterpret_cast<int16_t*>(base + L.qsum_off);
+    float* corr = reinterpret_cast<float*>(base + L.corr_off);
+    const int64_t Mp = L.Mp, nb = L.nb, target = 8 * 148, ngroups = (nb + 7) / 8;
+    int wpr = 1;
+    while (wpr < 8 && ceil_div(Mp, 8 / wpr) < target && ngroups >= 2 * wpr) wpr *= 2;
+    const dim3 grid((unsigned)ceil_div(Mp, 8 / wpr));
+    const uint16_t* xp = static_cast<const uint16_t*>(x);
+    switch (wpr) {
+      case 1: k_quantize<BF16, 1, true><<<grid, 256, 0, stream>>>(xp, M, K, ldx, Mp, tags, codes, qsum, corr, act_scales, perm); break;
+      case 2: k_quantize<BF16, 2, true><<<grid, 256, 0, stream>>>(xp, M, K, ldx, Mp, tags, codes, qsum, corr, act_scales, perm); break;
+      case 4: k_quantize<BF16, 4, true><<<grid, 256, 0, stream>>>(xp, M, K, ldx, Mp, tags, codes, qsum, corr, act_scales, perm); break;
+      default: k_quantize<BF16, 8, true><<<grid, 256, 0, stream>>>(xp, M, K, ldx, Mp, tags, codes, qsum, corr, act_scales, perm); break;
+    }
+    return cudaGetLastError();
+  }
   const int64_t row_bytes = K * 2;
   // rows in flight per CTA: ~64 KB of staged input, at least 2 (double buffering)
   int nbuf = (int)std::max<int64_t>(2, std::min<int64_t>(8, (64 << 10) / row_bytes));
