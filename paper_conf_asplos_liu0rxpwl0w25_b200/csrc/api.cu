@@ -330,8 +330,7 @@ comet_status_t comet_plan_destroy(comet_plan_t plan) {
   if (plan->chunk) comet_plan_destroy(plan->chunk);
   if (plan->tail) comet_plan_destroy(plan->tail);
   for (cudaEvent_t e : plan->ev) cudaEventDestroy(e);
-  if (plan->s_h2d) cudaStreamDestroy(plan->s_h2d);
-  if (plan->s_d2h) cudaStreamDestroy(plan->s_d2h);
+  // s_h2d / s_d2h are the device's shared copy streams (copy_streams), not owned by the plan
   if (plan->p.d_cta_begin) cudaFree(plan->p.d_cta_begin);
   if (plan->p.d_items) cudaFree(plan->p.d_items);
   delete plan;
@@ -482,6 +481,28 @@ size_t comet_linear_scratch_bytes(comet_plan_t plan, comet_dtype_t xdt, comet_dt
   return lin_layout(plan, ydt).total;
 }
 
+// One host-to-device and one device-to-host copy stream per device, shared by every plan's
+// host pipeline: consecutive calls (e.g. a model's layers issued back to back) then upload and
+// download in call order at the full PCIe rate of each direction, instead of splitting it over
+// several concurrent per-plan streams (which delays the first layer's downloads).
+static cudaError_t copy_streams(cudaStream_t* h2d, cudaStream_t* d2h) {
+  static std::mutex mu;
+  static cudaStream_t streams[64][2] = {};
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  if (dev < 0 || dev >= 64) return cudaErrorInvalidDevice;
+  std::lock_guard<std::mutex> lock(mu);
+  if (!streams[dev][0]) {
+    e = cudaStreamCreateWithFlags(&streams[dev][0], cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&streams[dev][1], cudaStreamNonBlocking);
+    if (e != cudaSuccess) return e;
+  }
+  *h2d = streams[dev][0];
+  *d2h = streams[dev][1];
+  return cudaSuccess;
+}
+
 static comet_status_t linear_host(comet_plan_t plan, const void* x_host, comet_dtype_t xdt,
                                   const void* w_packed, const float* w_scales, void* y_host,
                                   comet_dtype_t ydt, void* scratch, size_t scratch_bytes,
@@ -527,8 +548,7 @@ static comet_status_t linear_host(comet_plan_t plan, const void* x_host, comet_d
   // Nothing else orders the copy streams, so one call's uploads overlap the previous call's
   // downloads and compute.
   if (!plan->s_h2d) {
-    e = cudaStreamCreateWithFlags(&plan->s_h2d, cudaStreamNonBlocking);
-    if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&plan->s_d2h, cudaStreamNonBlocking);
+    e = copy_streams(&plan->s_h2d, &plan->s_d2h);
     if (e != cudaSuccess) return cuda_status(e, "copy stream create");
   }
   while ((int64_t)plan->ev.size() < 3 * nch + 2) {
