@@ -52,6 +52,9 @@ namespace {
 #ifndef COMET_DEC_ST64
 #define COMET_DEC_ST64 0    // 1: one 64-column TMEM store per widen warp and stage (KS = 4)
 #endif
+#ifndef COMET_DEC_SX32
+#define COMET_DEC_SX32 4    // X ring depth for NT >= 32 (a shallower X ring leaves room for weights)
+#endif
 #ifndef COMET_DEC_PDL
 #define COMET_DEC_PDL 1     // launch as a programmatic dependent of kernel 1 (weights stream early)
 #endif
@@ -89,7 +92,7 @@ struct Cfg {
   static constexpr int Q_BYTES = GS ? KS * NT * 2 : 0;
   static constexpr int G_BYTES = GS ? KS * kTileW * 4 : 0;
   static constexpr int X_STAGE = (KS * XKB_BYTES + S_BYTES + Q_BYTES + G_BYTES + 1023) / 1024 * 1024;
-  static constexpr int SX = 4;                                 // X ring depth
+  static constexpr int SX = NT >= 32 ? COMET_DEC_SX32 : 4;     // X ring depth
   static constexpr int SMEM_BUDGET = 224 * 1024;            // 227 KB minus alignment, barriers, tags
   static constexpr int SW_RAW = (SMEM_BUDGET - SX * X_STAGE) / W_BYTES;
   static constexpr int SW = SW_RAW > 8 ? 8 : SW_RAW;           // W ring depth
