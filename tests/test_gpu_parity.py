@@ -276,3 +276,20 @@ def test_linear_host_pipeline(M, blocking):
             torch.cuda.synchronize()
         yref, _, _, _ = oracle.w4ax(p.x, p.tags, p.w, p.s_w)
         _close(y_host, yref, torch.float16)
+
+
+def test_gemm_single_cta_tiles_repeated():
+    """Regression: the 192/160-wide single-CTA tiles (S = 3 pipeline slots) once alternated two
+    widen groups and two MMA issuers over an odd slot count, so a role could pass a parity wait
+    one phase early -- an intermittent launch failure (tools/stress_gemm.py).  Repeat them."""
+    for it in range(12):
+        for (M, N, sm, tw) in ((300, 1152, 1, 192), (230, 1280, 0, 160), (129, 384, 1, 192)):
+            p = synth.make_problem(M, 1024, N, frac=0.25, seed=M + N)
+            act, sc = _quant(p)
+            wp = cb.pack_weight(torch.from_numpy(p.w).to(DEV))
+            plan = cb.Plan(M, N, 1024, p.tags, split_mode=sm, num_sms=23, orientation=2, tile_w=tw)
+            y = cb.w4ax_gemm(plan, act, sc, wp, torch.from_numpy(p.s_w).to(DEV), out_dtype=torch.float32)
+            torch.cuda.synchronize()
+            if it == 0:
+                yref, _, _, _ = oracle.w4ax(p.x, p.tags, p.w, p.s_w)
+                _close(y, yref, torch.float32)
