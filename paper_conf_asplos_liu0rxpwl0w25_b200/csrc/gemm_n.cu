@@ -28,12 +28,6 @@
 #ifndef COMET_ISSUERS
 #define COMET_ISSUERS 2   // MMA issuing threads (K-blocks alternate between them)
 #endif
-#ifndef COMET_EPI_PAIR
-#define COMET_EPI_PAIR 0   // 1: FP16/BF16 epilogue stages two chunks per fence/barrier round
-#endif
-#ifndef COMET_EPI_DIRECT
-#define COMET_EPI_DIRECT 0   // 1: direct 16-byte global stores instead of the TMA-store epilogue
-#endif
 #ifndef COMET_NSTAGE
 #define COMET_NSTAGE 2   // output staging buffers per promotion warpgroup (TMA-store epilogue)
 #endif
@@ -704,45 +698,6 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
         named_bar_sync(1, 128 * C::NPW);                  // this tile's w_scales are in smem
         if (threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 15, 4 * (it - it_begin) + 1);
         const float* sw = sWs + tp * BN + wg * COLS;
-        if (COMET_EPI_DIRECT && RUNS == 1) {
-          // direct epilogue: each thread stores its row's COLS outputs with 16-byte global
-          // stores (fire and forget: the promotion continues with the next tile at once)
-          if (m < P.M) {
-            const int nb0 = n0 + wg * COLS;
-            if (P.ydt == COMET_F32) {
-              float* yrow = reinterpret_cast<float*>(P.y) + m * P.ldy + nb0;
-#pragma unroll
-              for (int c = 0; c < COLS; c += 4) {
-                if (nb0 + c < P.N) {
-                  const float4 v = make_float4((acc[c] + init) * sw[c], (acc[c + 1] + init) * sw[c + 1],
-                                               (acc[c + 2] + init) * sw[c + 2], (acc[c + 3] + init) * sw[c + 3]);
-                  *reinterpret_cast<float4*>(yrow + c) = v;
-                }
-              }
-            } else {
-              const bool bf = P.ydt == COMET_BF16;
-              uint16_t* yrow = reinterpret_cast<uint16_t*>(P.y) + m * P.ldy + nb0;
-#pragma unroll
-              for (int c = 0; c < COLS; c += 8) {
-                uint32_t pk[4];
-#pragma unroll
-                for (int i = 0; i < 4; ++i) {
-                  const float f0 = (acc[c + 2 * i] + init) * sw[c + 2 * i];
-                  const float f1 = (acc[c + 2 * i + 1] + init) * sw[c + 2 * i + 1];
-                  if (bf) {
-                    __nv_bfloat162 hv = __floats2bfloat162_rn(f0, f1);
-                    pk[i] = *reinterpret_cast<uint32_t*>(&hv);
-                  } else {
-                    __half2 hv = __floats2half2_rn(f0, f1);
-                    pk[i] = *reinterpret_cast<uint32_t*>(&hv);
-                  }
-                }
-                if (nb0 + c < P.N) *reinterpret_cast<uint4*>(yrow + c) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
-              }
-            }
-          }
-          continue;
-        }
         uint8_t* stage = sY + wg * C::NSTAGE * 8192;
         const uint32_t swz = (uint32_t)((r >> 1) & 3);
         const bool leader = (threadIdx.x & 127) == 0;     // thread 0 of the WG (row 0)
@@ -790,44 +745,6 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
             for (int i = 0; i < 16; ++i) pk[i] = __float_as_uint((acc[q * 16 + i] + init) * sw[q * 16 + i]);
             stage_and_store(pk, q * 16, 4);
           }
-        } else if (COMET_EPI_PAIR && !COMET_EPI_WARP && C::NSTAGE == 2 && (COLS / 32) % 2 == 0) {
-          // two 64-byte chunks per round: both staging buffers filled, one proxy fence and one
-          // barrier, two TMA stores
-          const bool bf = P.ydt == COMET_BF16;
-#pragma unroll
-          for (int q = 0; q < COLS / 32; q += 2) {
-            if (leader) bulk_wait_group_read<0>();
-            named_bar_sync(2 + wg, 128);
-#pragma unroll
-            for (int h = 0; h < 2; ++h) {
-              uint32_t pk[16];
-#pragma unroll
-              for (int i = 0; i < 16; ++i) {
-                const int c = (q + h) * 32 + 2 * i;
-                const float f0 = (acc[c] + init) * sw[c], f1 = (acc[c + 1] + init) * sw[c + 1];
-                if (bf) {
-                  __nv_bfloat162 hv = __floats2bfloat162_rn(f0, f1);
-                  pk[i] = *reinterpret_cast<uint32_t*>(&hv);
-                } else {
-                  __half2 hv = __floats2half2_rn(f0, f1);
-                  pk[i] = *reinterpret_cast<uint32_t*>(&hv);
-                }
-              }
-              const uint32_t rowa = smem_u32(stage + h * 8192) + r * 64;
-#pragma unroll
-              for (int k = 0; k < 4; ++k)
-                asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(rowa + ((k ^ swz) << 4)),
-                             "r"(pk[4 * k]), "r"(pk[4 * k + 1]), "r"(pk[4 * k + 2]), "r"(pk[4 * k + 3]) : "memory");
-            }
-            fence_proxy_async_smem();
-            named_bar_sync(2 + wg, 128);
-            if (leader) {
-              tma_store_2d(&P.map_y, stage, (n0 + col_n(wg, q * 32)) * 2, m0);
-              tma_store_2d(&P.map_y, stage + 8192, (n0 + col_n(wg, (q + 1) * 32)) * 2, m0);
-              bulk_commit_group();
-            }
-          }
-          ych = 0;
         } else {
           const bool bf = P.ydt == COMET_BF16;
 #pragma unroll
