@@ -55,6 +55,9 @@ namespace {
 #ifndef COMET_DEC_SX32
 #define COMET_DEC_SX32 4    // X ring depth for NT >= 32 (a shallower X ring leaves room for weights)
 #endif
+#ifndef COMET_DEC_WIDEN_PF
+#define COMET_DEC_WIDEN_PF 0   // 1: widen warps load stage s+1 weights before storing stage s (measured slower)
+#endif
 #ifndef COMET_DEC_PDL
 #define COMET_DEC_PDL 1     // launch as a programmatic dependent of kernel 1 (weights stream early)
 #endif
@@ -353,6 +356,90 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
     int st = 0, ab = 0;
     uint32_t ph = 0, aph = 0;
     int seq = 0;
+#if COMET_DEC_WIDEN_PF
+    // Software-pipelined: the shared-memory loads of stage s+1's packed weights are issued
+    // before stage s is converted and stored into TMEM, so their latency (~1000 clk when they
+    // queue behind the previous stage's tcgen05.st in the memory pipe) overlaps the stores
+    // instead of preceding them.
+    int it = it_begin;
+    WorkItem w{};
+    int kb = 0;
+    if (it < it_end) { w = load_item(P, it, debug); kb = w.kb_begin; }
+    uint4 cn[4 * KH];
+    int kb_n = 0, nk_n = 0, seq_f = 0;
+    auto fetch = [&]() {
+      nk_n = min(KS, w.kb_end - kb);
+      kb_n = kb;
+      mbar_wait(&full_w[st], ph);
+      if (lane == 0 && q == 0) trace_ev(P, 3 + half, seq_f);
+#pragma unroll
+      for (int i = 0; i < KH; ++i) {
+        const int cb = half * KH + i;
+        const uint32_t row = smem_u32(sW(st)) + (cb >> 1) * 2 * kTileW * 64 + r * 128;
+#pragma unroll
+        for (int j = 0; j < 4; ++j)
+          cn[4 * i + j] = (cb < nk_n && !(COMET_DEC_ABLATE & 8)) ? lds128(row + ((((cb & 1) * 4 + j) ^ sw) << 4))
+                                                                 : make_uint4(r, j, i, 0);
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty_w[st]);
+      if (++st == SW) { st = 0; ph ^= 1; }
+      ++seq_f;
+      kb += KS;                                   // advance to the next stage of the work list
+      if (kb >= w.kb_end) {
+        ++it;
+        if (it < it_end) { w = load_item(P, it, debug); kb = w.kb_begin; }
+      }
+    };
+    bool have = it < it_end;
+    if (have) fetch();
+    while (have) {
+      uint4 cc[4 * KH];
+#pragma unroll
+      for (int i = 0; i < 4 * KH; ++i) cc[i] = cn[i];
+      const int nk = nk_n, kbc = kb_n;
+      const bool have_next = it < it_end;
+      if (have_next) fetch();
+      mbar_wait(&a_empty[ab], aph ^ 1);
+      if (lane == 0 && q == 0 && half == 0) trace_ev(P, 14, seq);
+      tc_fence_after();
+#pragma unroll
+      for (int i = 0; i < KH; ++i) {
+        const int cb = half * KH + i;
+        if (cb < nk) {
+          const bool is8 = lds_u8(s_tags_a + kbc + cb) != 0;
+          uint32_t o[32];
+#pragma unroll
+          for (int j = 0; j < 4; ++j) {
+            const uint32_t pw[4] = {cc[4 * i + j].x, cc[4 * i + j].y, cc[4 * i + j].z, cc[4 * i + j].w};
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+              const uint32_t pv = pw[e];
+              const int g = 2 * (j * 4 + e);
+              if (is8) {
+                o[g] = ((pv << 4) & 0xF0F0F0F0u) ^ 0x80808080u;
+                o[g + 1] = (pv & 0xF0F0F0F0u) ^ 0x80808080u;
+              } else {
+                o[g] = pv & 0x0F0F0F0Fu;
+                o[g + 1] = (pv >> 4) & 0x0F0F0F0Fu;
+              }
+            }
+          }
+          if (!(COMET_DEC_ABLATE & 2)) tmem_st32(tbase + ab * C::A_COLS + cb * 32 + lane_addr, o);
+        }
+      }
+      if (lane == 0 && q == 0 && half == 0) trace_ev(P, 13, seq);   // stores issued
+      if (!(COMET_DEC_ABLATE & 2)) tmem_wait_st();
+      if (lane == 0 && q == 0 && half == 0) trace_ev(P, 15, seq);
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&a_full[ab]);
+      if (lane == 0 && q == 0) trace_ev(P, 5 + half, seq);
+      if (++ab == NA) { ab = 0; aph ^= 1; }
+      ++seq;
+      have = have_next;
+    }
+#else
     for (int it = it_begin; it < it_end; ++it) {
       const WorkItem w = load_item(P, it, debug);
       for (int kb = w.kb_begin; kb < w.kb_end; kb += KS, ++seq) {
@@ -367,11 +454,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
           const uint32_t row = smem_u32(sW(st)) + (cb >> 1) * 2 * kTileW * 64 + r * 128;
 #pragma unroll
           for (int j = 0; j < 4; ++j)
-            cc[4 * i + j] = cb < nk ? lds128(row + ((((cb & 1) * 4 + j) ^ sw) << 4)) : make_uint4(0, 0, 0, 0);
+            cc[4 * i + j] = (cb < nk && !(COMET_DEC_ABLATE & 8)) ? lds128(row + ((((cb & 1) * 4 + j) ^ sw) << 4))
+                                                                 : make_uint4(r, j, i, 0);   // 8: diagnostic, no weight reads
         }
         __syncwarp();
         if (lane == 0) mbar_arrive(&empty_w[st]);
-        if (lane == 0 && q == 0 && half == 0) trace_ev(P, 13, seq);
         mbar_wait(&a_empty[ab], aph ^ 1);
         if (lane == 0 && q == 0 && half == 0) trace_ev(P, 14, seq);
         tc_fence_after();
@@ -427,6 +514,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
             if (!(COMET_DEC_ABLATE & 2)) tmem_st32(tbase + ab * C::A_COLS + cb * 32 + lane_addr, o);
           }
         }
+        if (lane == 0 && q == 0 && half == 0) trace_ev(P, 13, seq);   // stores issued
         if (!(COMET_DEC_ABLATE & 2)) tmem_wait_st();
         if (lane == 0 && q == 0 && half == 0) trace_ev(P, 15, seq);
         tc_fence_before();
@@ -437,6 +525,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
         if (++ab == NA) { ab = 0; aph ^= 1; }
       }
     }
+#endif
   } else {
     setmaxnreg_inc<208>();
     // -------------------------------------------------------------------- promotion + epilogue

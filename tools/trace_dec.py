@@ -87,8 +87,9 @@ for cta in (0, 1):
               "MMA done->promo go", np.median(p_go[2 * em] - m_done[em]), "promo dur", np.median(p_done[e] - p_go[e]))
     if n_st > 8:
         e13, e14, e15 = rel(13, n_st), rel(14, n_st), rel(15, n_st)
-        print("widen g0 phases (median clk): LDS+release", np.median(e13[e] - wg[0][e]), "a_empty wait", np.median(e14[e] - e13[e]),
-              "convert+tmem st+wait", np.median(e15[e] - e14[e]), "fence+arrive", np.median(wg[2][e] - e15[e]))
+        print("widen g0 phases (median clk): LDS+release+a_empty wait", np.median(e14[e] - wg[0][e]),
+              "convert+tmem st issue", np.median(e13[e] - e14[e]), "wait::st", np.median(e15[e] - e13[e]),
+              "fence+arrive", np.median(wg[2][e] - e15[e]))
     ep = [(t[10][i] - base, t[11][i] - base if t[11][i] else -1, t[12][i] - base) for i in range(8) if t[10][i]]
     print("epilogues (start, partials ready, done):", ep)
     print("end of last promotion", p_done[-1] if n_st else None)
