@@ -55,6 +55,9 @@ namespace {
 #ifndef COMET_DEC_SX32
 #define COMET_DEC_SX32 4    // X ring depth for NT >= 32 (a shallower X ring leaves room for weights)
 #endif
+#ifndef COMET_DEC_WIDEN_WARPS
+#define COMET_DEC_WIDEN_WARPS 8   // 8: two warps per TMEM lane quadrant (KS/2 K-blocks each); 4: one
+#endif
 #ifndef COMET_DEC_WIDEN_PF
 #define COMET_DEC_WIDEN_PF 0   // 1: widen warps load stage s+1 weights before storing stage s (measured slower)
 #endif
@@ -165,14 +168,14 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
     tma_prefetch(&P.map_s);
     for (int i = 0; i < SW; ++i) {
       mbar_init(&full_w[i], 1);
-      mbar_init(&empty_w[i], 8);
+      mbar_init(&empty_w[i], COMET_DEC_WIDEN_WARPS);
     }
     for (int i = 0; i < SX; ++i) {
       mbar_init(&full_x[i], 1);
       mbar_init(&empty_x[i], 2 + 4);
     }
     for (int i = 0; i < NA; ++i) {
-      mbar_init(&a_full[i], 8);
+      mbar_init(&a_full[i], COMET_DEC_WIDEN_WARPS);
       mbar_init(&a_empty[i], 2);
     }
     for (int i = 0; i < NACC; ++i) {
@@ -344,10 +347,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
       }
 #endif
     }
+  } else if (warp < kPromoWarp0 && warp - kWidenWarp0 >= COMET_DEC_WIDEN_WARPS) {
+    setmaxnreg_dec<112>();                        // spare warps of a 4-warp widen variant
   } else if (warp < kPromoWarp0) {
     setmaxnreg_dec<112>();
     // -------------------------------------------------------------------- widen (W -> TMEM A)
-    constexpr int KH = KS / 2;                    // K-blocks per widen warp and stage
+    constexpr int KH = KS * 4 / COMET_DEC_WIDEN_WARPS;   // K-blocks per widen warp and stage
     const int half = (warp - kWidenWarp0) >> 2;   // K-blocks [half KH, (half+1) KH) of a stage
     const int q = warp & 3;
     const int r = q * 32 + lane;                  // TMEM lane = weight row within the tile
