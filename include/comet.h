@@ -196,7 +196,9 @@ typedef struct {
                          -1 = auto (stream-K when whole tiles fill < 92 % of the last wave) */
   float cost_int4;     /* planner cost of one INT4 K-block unit (default 1.0) */
   float cost_int8;     /* planner cost of one INT8 K-block unit (default 1.0 on B200) */
-  int stages;          /* shared-memory ring depth; 0 = auto */
+  int stages;          /* shared-memory ring depth: 0 = auto; any other value must equal the
+                          depth the plan's kernel is compiled with (reported by
+                          comet_plan_info().stages), else COMET_ERR_INVALID_ARG */
   int device_plan;     /* 1 (default) = upload the work list to the device at create time;
                           0 = host-only plan (comet_plan_describe only; CPU-safe) */
   int orientation;     /* 0 = auto (3 when M >= 256, 2 when M >= 128, else 1);
@@ -257,7 +259,15 @@ comet_status_t comet_plan_describe(comet_plan_t plan, int32_t* items, int64_t ma
  *   debug_acc               NULL, or device [M][N] int32: sum_b acc_b[m,n] in code units
  *                           (bit-exact integer accumulators; slower debug kernel).
  *   debug_acc_blocks        NULL, or device [K/128][M][N] int32 per-block acc_b (tiny shapes).
- *   workspace               device, >= the plan's workspace_bytes (may be NULL if 0).
+ *   workspace               device, >= the plan's workspace_bytes (may be NULL if 0).  Zero it
+ *                           once before its first use; afterwards it may be reused by any
+ *                           later call of any plan without clearing (stream-K flags are
+ *                           compared with a process-wide launch counter), but it must not be
+ *                           used by two GEMMs in flight at the same time.
+ * The persistent grid is sized at plan time to what the occupancy calculator admits as
+ * co-resident (the stream-K owner of a split tile waits for the other units' partials); a
+ * fix-up or pipeline wait that exceeds 4 s (only possible if another kernel holds the SMs that
+ * long) traps, i.e. the launch fails with a CUDA error instead of hanging the device.
  */
 comet_status_t comet_w4ax_gemm(comet_plan_t plan, const void* act_packed, const float* act_scales,
                                const void* w_packed, const float* w_scales, void* y,
@@ -308,6 +318,18 @@ comet_status_t comet_w4ax_linear_host_async(comet_plan_t plan, const void* x_hos
                                             void* workspace, size_t ws_bytes, void* stream);
 /* Block until the downloads of the last comet_w4ax_linear_host(_async) call with `plan` are done. */
 comet_status_t comet_linear_host_wait(comet_plan_t plan);
+
+/* ------------------------------------------------------------------------------------------
+ * Diagnostic: the GEMM kernels' widening step on caller-chosen packed words (P:L202-206
+ * "location switch" + "zero extension"; layout R14 above), for the exhaustive widening pin.
+ * For i in [0, n): word v = (first_word + i) mod 2^32, eight consecutive channels packed as
+ * above; out_dev[2i] = bytes u[0..3], out_dev[2i+1] = bytes u[4..7] (u = nibble value 0..15,
+ * i.e. the E4M3 operand u * 2^-9 of an INT4 block); with int8_block != 0 each byte is instead
+ * the s8 value 16 * (u - 8) of an INT8 block.  out_dev: device [n][2] uint32, 8-byte aligned.
+ * n in [0, 2^32].  Asynchronous on `stream`.
+ * ---------------------------------------------------------------------------------------- */
+comet_status_t comet_debug_widen(uint64_t first_word, int64_t n, int int8_block, uint32_t* out_dev,
+                                 void* stream);
 
 const char* comet_status_string(comet_status_t s);
 const char* comet_last_error(void);

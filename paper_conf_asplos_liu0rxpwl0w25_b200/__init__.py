@@ -97,6 +97,7 @@ def lib():
         "comet_w4ax_linear_host": (I32, [P, P, I32, P, P, P, I32, P, SZ, P, SZ, P]),
         "comet_w4ax_linear_host_async": (I32, [P, P, I32, P, P, P, I32, P, SZ, P, SZ, P]),
         "comet_linear_host_wait": (I32, [P]),
+        "comet_debug_widen": (I32, [ctypes.c_uint64, I64, I32, P, P]),
         "comet_status_string": (ctypes.c_char_p, [I32]),
         "comet_last_error": (ctypes.c_char_p, []),
         "comet_version": (ctypes.c_char_p, []),
@@ -364,6 +365,17 @@ def w4ax_linear(plan: Plan, x, w_packed, w_scales, *, perm=None, out_dtype=None,
     w4ax_gemm."""
     act, sc = quantize_act(x, plan.tags, perm=perm, stream=stream)
     return w4ax_gemm(plan, act, sc, w_packed, w_scales, out_dtype=out_dtype, stream=stream)
+
+
+def debug_widen(first_word: int, n: int, int8_block: bool = False, *, out=None, stream=None):
+    """comet_debug_widen: the GEMM kernels' widening of the packed words first_word ..
+    first_word + n - 1 (mod 2^32) -> [n, 2] int32 CUDA tensor (lo / hi byte words)."""
+    import torch
+    if out is None:
+        out = torch.empty((n, 2), dtype=torch.int32, device="cuda")
+    _check(lib().comet_debug_widen(first_word, n, 1 if int8_block else 0, ctypes.c_void_p(out.data_ptr()),
+                                   _stream(stream)))
+    return out
 
 
 def linear_scratch_bytes(plan: Plan, xdt: int, ydt: int) -> int:

@@ -101,6 +101,21 @@ int comet_last_launch_count(void) { return g_launches; }
  * first two CTAs into buf ([2][8][1024] uint64, device memory); NULL disables. */
 void comet_debug_set_trace(void* buf) { comet::gemm::g_trace = static_cast<unsigned long long*>(buf); }
 
+comet_status_t comet_debug_widen(uint64_t first_word, int64_t n, int int8_block, uint32_t* out_dev,
+                                 void* stream) {
+  g_launches = 0;
+  if (n < 0 || n > ((int64_t)1 << 32)) return fail(COMET_ERR_INVALID_ARG, "n must be in [0, 2^32]");
+  if (n == 0) return COMET_OK;
+  if (!out_dev) return fail(COMET_ERR_INVALID_ARG, "out_dev is NULL");
+  if ((reinterpret_cast<uintptr_t>(out_dev) & 7u) != 0) return fail(COMET_ERR_MISALIGNED, "out_dev must be 8-byte aligned");
+  comet_status_t st = check_device();
+  if (st != COMET_OK) return st;
+  cudaError_t e = gemm::launch_debug_widen(first_word, n, int8_block ? 1 : 0, out_dev, static_cast<cudaStream_t>(stream));
+  if (e != cudaSuccess) return cuda_status(e, "widen launch");
+  g_launches = 1;
+  return COMET_OK;
+}
+
 comet_status_t comet_act_layout(int64_t M, int64_t K, comet_act_layout_t* out) {
   if (!out) return fail(COMET_ERR_INVALID_ARG, "out is NULL");
   comet_status_t st = check_mk(M, K);
@@ -305,6 +320,29 @@ comet_status_t comet_plan_create(int64_t M, int64_t N, int64_t K, const uint8_t*
   p.mask = mask_of(tags_host, K / kBlockK);
   st = build_plan(p, cfg);
   if (st != COMET_OK) { delete h; return st; }
+  p.stages = gemm_stages(p);
+  if (cfg.stages != 0 && cfg.stages != p.stages) {
+    const std::string msg = "stages: the kernel this plan runs is compiled with a ring depth of " +
+                            std::to_string(p.stages) + " (0 = auto)";
+    delete h;
+    return fail(COMET_ERR_INVALID_ARG, msg);
+  }
+  if (cfg.device_plan) {
+    // the persistent grid must be co-resident (stream-K owners wait for other units' partials):
+    // clamp it to what the occupancy calculator admits (e.g. CTA-pair clusters when a GPC has
+    // an odd number of SMs)
+    int sms = 0;
+    check_device(&sms);
+    const int units = max_coresident_units(p, sms);
+    if (units <= 0) { delete h; return fail(COMET_ERR_CUDA, "occupancy query of the GEMM kernel failed"); }
+    if (p.num_ctas > units) {
+      comet_sched_config c2 = cfg;
+      c2.num_sms = p.orientation == 3 ? 2 * units : units;
+      c2.orientation = p.orientation;
+      st = build_plan(p, c2);
+      if (st != COMET_OK) { delete h; return st; }
+    }
+  }
   if (cfg.device_plan) {
     cudaGetDevice(&p.device);
     cudaError_t e = cudaMalloc(&p.d_cta_begin, p.cta_begin.size() * sizeof(int32_t));
@@ -534,9 +572,19 @@ static comet_status_t linear_host(comet_plan_t plan, const void* x_host, comet_d
     const int l2 = g_launches;
     e = cudaMemcpyAsync(y_host, s + lay.y_off, (size_t)(p.M * p.N) * esz, cudaMemcpyDeviceToHost, cs);
     if (e != cudaSuccess) return cuda_status(e, "D2H copy");
+    // completion event of this call's download: comet_linear_host_wait blocks on it
+    if (plan->ev.empty()) {
+      cudaEvent_t ev;
+      e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming);
+      if (e != cudaSuccess) return cuda_status(e, "event create");
+      plan->ev.push_back(ev);
+    }
+    e = cudaEventRecord(plan->ev[0], cs);
+    if (e != cudaSuccess) return cuda_status(e, "event record");
+    plan->prev_call = true;
     if (blocking) {
-      e = cudaStreamSynchronize(cs);
-      if (e != cudaSuccess) return cuda_status(e, "stream synchronize");
+      e = cudaEventSynchronize(plan->ev[0]);
+      if (e != cudaSuccess) return cuda_status(e, "D2H synchronize");
     }
     g_launches = l1 + l2;
     return COMET_OK;
@@ -559,7 +607,7 @@ static comet_status_t linear_host(comet_plan_t plan, const void* x_host, comet_d
   }
   cudaEvent_t ev_quant_last = plan->ev[3 * nch], ev_d2h_last = plan->ev[3 * nch + 1];
   // zero the sub-plans' stream-K flag workspace the first time this scratch is used (flags are
-  // compared with per-plan epochs that start at 1)
+  // compared with process-wide launch epochs, which start at 1)
   if (plan->ws_zeroed != scratch) {
     e = cudaMemsetAsync(s + lay.ws_chunk_off, 0, lay.total - lay.ws_chunk_off, cs);
     if (e != cudaSuccess) return cuda_status(e, "workspace clear");
@@ -614,8 +662,9 @@ static comet_status_t linear_host(comet_plan_t plan, const void* x_host, comet_d
 
 comet_status_t comet_linear_host_wait(comet_plan_t plan) {
   if (!plan) return fail(COMET_ERR_INVALID_ARG, "NULL plan");
-  if (lin_chunks(plan->p) == 1 || !plan->prev_call) return COMET_OK;
-  cudaError_t e = cudaEventSynchronize(plan->ev[3 * lin_chunks(plan->p) + 1]);
+  if (!plan->prev_call) return COMET_OK;
+  const int64_t nch = lin_chunks(plan->p);
+  cudaError_t e = cudaEventSynchronize(plan->ev[nch == 1 ? 0 : 3 * nch + 1]);
   if (e != cudaSuccess) return cuda_status(e, "D2H synchronize");
   return COMET_OK;
 }

@@ -421,12 +421,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
             for (int e = 0; e < 4; ++e) {
               const uint32_t pv = pw[e];
               const int g = 2 * (j * 4 + e);
+              widen_int4(pv, o[g], o[g + 1]);
               if (is8) {
-                o[g] = ((pv << 4) & 0xF0F0F0F0u) ^ 0x80808080u;
-                o[g + 1] = (pv & 0xF0F0F0F0u) ^ 0x80808080u;
-              } else {
-                o[g] = pv & 0x0F0F0F0Fu;
-                o[g + 1] = (pv >> 4) & 0x0F0F0F0Fu;
+                o[g] = int4_to_int8(o[g]);
+                o[g + 1] = int4_to_int8(o[g + 1]);
               }
             }
           }
@@ -481,12 +479,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
               for (int e = 0; e < 4; ++e) {
                 const uint32_t pv = pw[e];
                 const int g = 32 * i + 2 * (j * 4 + e);
+                widen_int4(pv, o[g], o[g + 1]);
                 if (is8) {
-                  o[g] = ((pv << 4) & 0xF0F0F0F0u) ^ 0x80808080u;
-                  o[g + 1] = (pv & 0xF0F0F0F0u) ^ 0x80808080u;
-                } else {
-                  o[g] = pv & 0x0F0F0F0Fu;
-                  o[g + 1] = (pv >> 4) & 0x0F0F0F0Fu;
+                  o[g] = int4_to_int8(o[g]);
+                  o[g + 1] = int4_to_int8(o[g + 1]);
                 }
               }
             }
@@ -507,12 +503,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
               for (int e = 0; e < 4; ++e) {
                 const uint32_t pv = pw[e];
                 const int g = 2 * (j * 4 + e);
+                widen_int4(pv, o[g], o[g + 1]);
                 if (is8) {
-                  o[g] = ((pv << 4) & 0xF0F0F0F0u) ^ 0x80808080u;
-                  o[g + 1] = (pv & 0xF0F0F0F0u) ^ 0x80808080u;
-                } else {
-                  o[g] = pv & 0x0F0F0F0Fu;
-                  o[g + 1] = (pv >> 4) & 0x0F0F0F0Fu;
+                  o[g] = int4_to_int8(o[g]);
+                  o[g + 1] = int4_to_int8(o[g + 1]);
                 }
               }
             }
@@ -744,12 +738,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
 template <int NT, int DEBUG, bool GS = false>
 cudaError_t launch_nt(const GemmParams& prm, int grid, cudaStream_t stream) {
   using C = Cfg<NT, GS>;
-  static bool attr_set = false;
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(k_w4ax<NT, DEBUG, GS>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_BYTES);
-    if (e != cudaSuccess) return e;
-    attr_set = true;
-  }
+  static std::atomic<uint64_t> attr_done{0};
+  cudaError_t ea = set_smem_attr(k_w4ax<NT, DEBUG, GS>, C::SMEM_BYTES, attr_done);
+  if (ea != cudaSuccess) return ea;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)grid);
   cfg.blockDim = dim3(kThreads);
@@ -810,7 +801,68 @@ bool make_map_2d(CUtensorMap* map, const void* base, uint64_t inner, uint64_t ou
 
 unsigned long long* g_trace = nullptr;
 
+uint32_t next_epoch() {
+  static std::atomic<uint32_t> g_epoch{0};
+  uint32_t e = g_epoch.fetch_add(1, std::memory_order_relaxed) + 1;
+  while (e == 0) e = g_epoch.fetch_add(1, std::memory_order_relaxed) + 1;   // 0 = zeroed flag
+  return e;
+}
+
+// Diagnostic: the GEMM kernels' widening (widen_int4 / int4_to_int8) applied to the words
+// first, first + 1, ... (mod 2^32); out[i] = {lo, hi} bytes of word first + i.
+__global__ void k_debug_widen(uint64_t first, int64_t n, int is8, uint2* out) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    uint32_t lo, hi;
+    widen_int4((uint32_t)(first + (uint64_t)i), lo, hi);
+    if (is8) {
+      lo = int4_to_int8(lo);
+      hi = int4_to_int8(hi);
+    }
+    out[i] = make_uint2(lo, hi);
+  }
+}
+
+cudaError_t launch_debug_widen(uint64_t first, int64_t n, int is8, uint32_t* out, cudaStream_t stream) {
+  const int64_t blocks = std::min<int64_t>((n + 255) / 256, 148 * 16);
+  k_debug_widen<<<(unsigned)std::max<int64_t>(blocks, 1), 256, 0, stream>>>(first, n, is8, reinterpret_cast<uint2*>(out));
+  return cudaGetLastError();
+}
+
 }  // namespace gemm
+
+// Persistent units of the plan's production kernel that can be co-resident on the current
+// device: the stream-K fix-up waits of the persistent grid assume every unit is resident.
+int max_coresident_units(const Plan& p, int sms) {
+  using namespace gemm;
+  if (p.orientation >= 2) return max_units_gemm_n(p.tile_w, p.orientation == 3 ? 2 : 1, sms);
+  int b = 0;
+  cudaError_t e = cudaSuccess;
+  auto occ = [&](auto kern, int smem) {   // plan time: set the attribute directly (one lambda
+                                          // instantiation serves every tile_n, so no cached flag)
+    e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kern, kThreads, smem);
+  };
+  switch (p.tile_n) {
+    case 16: occ(k_w4ax<16, 0, false>, Cfg<16>::SMEM_BYTES); break;
+    case 32: occ(k_w4ax<32, 0, false>, Cfg<32>::SMEM_BYTES); break;
+    case 64: occ(k_w4ax<64, 0, false>, Cfg<64>::SMEM_BYTES); break;
+    default: occ(k_w4ax<128, 0, false>, Cfg<128>::SMEM_BYTES); break;
+  }
+  return e == cudaSuccess ? b * sms : -1;
+}
+
+// Shared-memory ring depth of the plan's production kernel (reported as plan_info.stages):
+// prefill kernels: pipeline slots; decode kernel: packed-weight ring slots.
+int gemm_stages(const Plan& p) {
+  using namespace gemm;
+  if (p.orientation >= 2) return stages_gemm_n(p.tile_w, p.orientation == 3 ? 2 : 1);
+  switch (p.tile_n) {
+    case 16: return Cfg<16>::SW;
+    case 32: return Cfg<32>::SW;
+    case 64: return Cfg<64>::SW;
+    default: return Cfg<128>::SW;
+  }
+}
 
 comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_scales,
                            const void* w_packed, const float* w_scales, void* y,
@@ -918,7 +970,7 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
     prm.max_seg = p.max_segments;
     prm.ws_part = static_cast<float*>(workspace);
     prm.ws_flags = reinterpret_cast<uint32_t*>(static_cast<uint8_t*>(workspace) + p.ws_flags_off);
-    prm.epoch = ++p.epoch;
+    prm.epoch = next_epoch();
     grid = p.num_ctas * cg;
   }
   if (normal) {

@@ -43,6 +43,19 @@ struct __align__(64) GemmParams {
   TagMask tags;
 };
 
+// Widening of packed INT4 weights (the B200 form of the paper's "location switch" + "zero
+// extension"; layout R14 in include/comet.h).  One packed 32-bit word holds 8
+// consecutive channels; widen_int4 yields their offset-binary bytes u = w + 8 in channel order
+// (lo = channels 0..3, hi = 4..7) in 3 instructions -- the byte u read as E4M3 is exactly
+// u * 2^-9, the INT4-block MMA operand.  int4_to_int8 turns such a word into the s8 bytes 16 w
+// = (u << 4) ^ 0x80 of an INT8 block.  Every GEMM kernel widens through these two functions;
+// comet_debug_widen runs them on caller-chosen words (exhaustive pin I9).
+__device__ __forceinline__ void widen_int4(uint32_t pv, uint32_t& lo, uint32_t& hi) {
+  lo = pv & 0x0F0F0F0Fu;
+  hi = (pv >> 4) & 0x0F0F0F0Fu;
+}
+__device__ __forceinline__ uint32_t int4_to_int8(uint32_t u4) { return (u4 << 4) ^ 0x80808080u; }
+
 __device__ __forceinline__ void named_bar_sync(int id, int n) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
 }
@@ -117,9 +130,31 @@ bool make_map(CUtensorMap* map, CUtensorMapDataType dt, int rank, const void* ba
 
 extern unsigned long long* g_trace;   // diagnostic timeline buffer (comet_debug_set_trace)
 
+// Stream-K fix-up epoch: one process-wide monotonic counter, so no two launches (of any plan,
+// on any workspace) publish or wait for the same flag value; a zeroed workspace never matches.
+uint32_t next_epoch();
+
+// cudaFuncSetAttribute(MaxDynamicSharedMemorySize) once per (kernel, device): function
+// attributes are per device context, so the flag is a per-device bit (devices 0..63).
+template <typename Kern>
+inline cudaError_t set_smem_attr(Kern kernel, int bytes, std::atomic<uint64_t>& done) {
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  const uint64_t bit = 1ull << (dev & 63);
+  if (done.load(std::memory_order_acquire) & bit) return cudaSuccess;
+  e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+  if (e == cudaSuccess) done.fetch_or(bit, std::memory_order_acq_rel);
+  return e;
+}
+
 // Normal-orientation launcher (gemm_n.cu).  BN = weights per tile (256, or 128 for debug);
 // cg = CTAs per tile (1, or 2 for the tcgen05 CTA pair; grid must then be even).
 cudaError_t launch_gemm_n(const GemmParams& prm, int grid, int bn, int cg, int debug, cudaStream_t stream);
+// Persistent units (CTAs, or pairs for cg = 2) of the production kernel that fit on the device
+// at once (occupancy query; -1 on error).
+int max_units_gemm_n(int bn, int cg, int sms);
+int stages_gemm_n(int bn, int cg);   // pipeline slots S of the production kernel
 
 }  // namespace gemm
 }  // namespace comet

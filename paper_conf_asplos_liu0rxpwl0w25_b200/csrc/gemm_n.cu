@@ -415,13 +415,10 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
               const uint32_t pw[4] = {c[i][q4].x, c[i][q4].y, c[i][q4].z, c[i][q4].w};
               uint32_t o[8];
 #pragma unroll
-              for (int k = 0; k < 4; ++k) {
-                o[2 * k] = pw[k] & 0x0F0F0F0Fu;           // u[8g .. 8g+3]
-                o[2 * k + 1] = (pw[k] >> 4) & 0x0F0F0F0Fu; // u[8g+4 .. 8g+7]
-              }
+              for (int k = 0; k < 4; ++k) widen_int4(pw[k], o[2 * k], o[2 * k + 1]);   // u[8g ..], u[8g+4 ..]
               if (is8) {                                  // warp-uniform: 5 % of blocks
 #pragma unroll
-                for (int k = 0; k < 8; ++k) o[k] = (o[k] << 4) ^ 0x80808080u;
+                for (int k = 0; k < 8; ++k) o[k] = int4_to_int8(o[k]);
               }
               const int oc = 2 * q4;                      // logical 16-byte output chunk
               asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(dst + ((oc ^ sw128) << 4)),
@@ -791,12 +788,9 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
 template <int BN, int CG, int NPW, int NWG, int DEBUG>
 cudaError_t launch_bn(const GemmParams& prm, int grid, cudaStream_t stream) {
   using C = CfgN<BN, CG, NPW, NWG, DEBUG>;
-  static bool attr_set = false;
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(k_w4ax_n<BN, CG, NPW, NWG, DEBUG>, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_BYTES);
-    if (e != cudaSuccess) return e;
-    attr_set = true;
-  }
+  static std::atomic<uint64_t> attr_done{0};
+  cudaError_t ea = set_smem_attr(k_w4ax_n<BN, CG, NPW, NWG, DEBUG>, C::SMEM_BYTES, attr_done);
+  if (ea != cudaSuccess) return ea;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)grid);
   cfg.blockDim = dim3(C::THREADS);
@@ -812,7 +806,59 @@ cudaError_t launch_bn(const GemmParams& prm, int grid, cudaStream_t stream) {
   return cudaLaunchKernelEx(&cfg, k_w4ax_n<BN, CG, NPW, NWG, DEBUG>, prm);
 }
 
+// Persistent units (CTAs, or CTA pairs for CG = 2) of this kernel that can be resident at once.
+template <int BN, int CG, int NPW, int NWG, int DEBUG>
+int max_units_bn(int sms) {
+  using C = CfgN<BN, CG, NPW, NWG, DEBUG>;
+  auto kern = k_w4ax_n<BN, CG, NPW, NWG, DEBUG>;
+  static std::atomic<uint64_t> attr_done{0};
+  if (set_smem_attr(kern, C::SMEM_BYTES, attr_done) != cudaSuccess) return -1;
+  if (CG == 1) {
+    int b = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kern, C::THREADS, C::SMEM_BYTES) != cudaSuccess) return -1;
+    return b * sms;
+  }
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)(CG * sms / CG));
+  cfg.blockDim = dim3(C::THREADS);
+  cfg.dynamicSmemBytes = C::SMEM_BYTES;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = CG;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  int n = 0;
+  if (cudaOccupancyMaxActiveClusters(&n, kern, &cfg) != cudaSuccess) return -1;
+  return n;
+}
+
 }  // namespace
+
+int stages_gemm_n(int bn, int cg) {
+  if (cg == 2) {
+    if (bn == 192) return CfgN<192, 2, 3, 2, 0>::S;
+    if (bn == 160) return CfgN<160, 2, 2, 2, 0>::S;
+    if (bn == 128) return CfgN<128, 2, 2, 2, 0>::S;
+    return CfgN<256, 2, COMET_N256_NPW, COMET_N256_NWG, 0>::S;
+  }
+  if (bn == 192) return CfgN<192, 1, 3, 1, 0>::S;
+  if (bn == 160) return CfgN<160, 1, 2, 1, 0>::S;
+  return CfgN<128, 1, 2, 2, 0>::S;
+}
+
+int max_units_gemm_n(int bn, int cg, int sms) {
+  if (cg == 2) {
+    if (bn == 192) return max_units_bn<192, 2, 3, 2, 0>(sms);
+    if (bn == 160) return max_units_bn<160, 2, 2, 2, 0>(sms);
+    if (bn == 128) return max_units_bn<128, 2, 2, 2, 0>(sms);
+    return max_units_bn<256, 2, COMET_N256_NPW, COMET_N256_NWG, 0>(sms);
+  }
+  if (bn == 192) return max_units_bn<192, 1, 3, 1, 0>(sms);
+  if (bn == 160) return max_units_bn<160, 1, 2, 1, 0>(sms);
+  return max_units_bn<128, 1, 2, 2, 0>(sms);
+}
 
 // bn = 128, 160, 192 or 256; 96 for the debug-accumulator kernels (they need the registers).
 cudaError_t launch_gemm_n(const GemmParams& prm, int grid, int bn, int cg, int debug, cudaStream_t stream) {

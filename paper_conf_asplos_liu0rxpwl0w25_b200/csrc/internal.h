@@ -54,7 +54,6 @@ struct Plan {
   WorkItem* d_items = nullptr;
   size_t ws_bytes = 0;                  // stream-K partials + flags
   size_t ws_flags_off = 0;
-  std::atomic<uint32_t> epoch{0};
   int device = -1;
 };
 
@@ -93,6 +92,11 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
                            comet_dtype_t ydt, int64_t ldy, int32_t* debug_acc,
                            int32_t* debug_acc_blocks, void* workspace, size_t ws_bytes,
                            cudaStream_t stream, int* launches, bool grouped = false);
+int max_coresident_units(const Plan& p, int sms);
+int gemm_stages(const Plan& p);
+namespace gemm {
+cudaError_t launch_debug_widen(uint64_t first, int64_t n, int is8, uint32_t* out, cudaStream_t stream);
+}
 // act layout
 void act_layout(int64_t M, int64_t K, comet_act_layout_t* out);
 

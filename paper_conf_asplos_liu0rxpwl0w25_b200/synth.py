@@ -108,6 +108,86 @@ def make_problem(M: int, K: int, N: int, *, frac: float = 0.05, seed: int = 0,
     return Problem(x=x, tags=tags, w=w, s_w=s_w, bf16=bf16)
 
 
+@dataclass
+class ExactProblem(Problem):
+    """A Problem whose inputs are built from chosen integer codes (see make_exact_problem)."""
+    q: np.ndarray = None      # [M, K] int16: the codes every block is built from
+    e: np.ndarray = None      # [M, nb] int: x[m, block b] = q * 2^e[m, b]
+    f: np.ndarray = None      # [N] int: s_w[n] = 2^f[n]
+
+
+EXACT_SPECIAL_ROWS = ("zero", "all_pos", "alternating", "all_neg")
+
+
+def make_exact_problem(M: int, K: int, N: int, *, frac: float = 0.05, seed: int = 0,
+                       bf16: bool = False, n8: int | None = None,
+                       special_rows: dict | None = None) -> ExactProblem:
+    """Inputs on which the whole W4Ax path is EXACT in binary32, so a GEMM's FP32 output can be
+    compared bit for bit (VERDICT r01 "integer exactness of the production kernels").
+
+    Every (token m, block b) is built from integer codes q in [-qmax_b, qmax_b] (qmax 7 for
+    INT4 blocks, 127 for INT8 blocks) with at least one element equal to +-qmax_b, as
+    x = q * 2^e[m, b]; so amax = qmax_b 2^e, s_a = 2^e exactly and the quantised codes are q.
+    Weight scales are powers of two, s_w[n] = 2^f[n].  Then y[m, n] = sum_b 2^(e[m,b]+f[n])
+    acc_b[m, n] is a sum of integers times powers of two, and the exponents are limited so
+    that sum_b 2^(e_b - min e) * c_b * sum_k |q| < 2^24 per row (c_b = 15 INT4, 8 INT8): every partial sum of every
+    accumulation order (the INT4 blocks' offset-binary operand u = w + 8 included) is exact in
+    binary32.  A single wrong accumulator code unit changes y by >= 2^(min e + f).
+
+    special_rows maps a row index to one of EXACT_SPECIAL_ROWS: "zero" (an all-zero row, s_a =
+    0), "all_pos" / "all_neg" (every code +-qmax: the largest |sum q w| of a block, e.g. 7 * 15
+    * 128 = 13,440 against an all-7 weight row's offset-binary u = 15), "alternating" (codes
+    +-qmax alternating: maximal cancellation).  Weight rows 0, 1, 2 and N-1 are all-7, all -8,
+    alternating 7/-8 and all-7 (their u = 15, 0, 15/0).  Only input values are drawn here --
+    none of the method's arithmetic."""
+    rng = np.random.default_rng(seed)
+    tags = make_tags(K, frac, rng, n8=n8)
+    nb = K // BLOCK
+    qmax = np.where(tags != 0, 127, 7).astype(np.int16)                 # [nb]
+    qm = np.repeat(qmax, BLOCK)                                          # [K]
+    q = (rng.integers(-(1 << 15), 1 << 15, size=(M, K)) % (2 * qm + 1) - qm).astype(np.int16)
+    pos = rng.integers(0, BLOCK, size=(M, nb))
+    sgn = rng.choice(np.array([-1, 1], np.int16), size=(M, nb))
+    rows_i = np.repeat(np.arange(M), nb)
+    cols_i = (np.tile(np.arange(nb), M) * BLOCK + pos.reshape(-1))
+    q[rows_i, cols_i] = (sgn * qmax[None, :]).reshape(-1)
+    special_rows = special_rows or {}
+    for r, kind in special_rows.items():
+        if not 0 <= r < M:
+            continue
+        if kind == "zero":
+            q[r] = 0
+        elif kind == "all_pos":
+            q[r] = qm
+        elif kind == "all_neg":
+            q[r] = -qm
+        elif kind == "alternating":
+            q[r] = qm * np.where(np.arange(K) % 2 == 0, 1, -1).astype(np.int16)
+        else:
+            raise ValueError(kind)
+    # block exponents: random in [e0, e0 + 3], flattened to e0 for rows that would not be exact
+    # (|operand| <= 15 = max u for INT4 blocks, <= 8 = max |w| for INT8 blocks; a binary32 sum
+    # of integers whose magnitudes total < 2^24 is exact in every order)
+    e0 = -2
+    e = rng.integers(e0, e0 + 4, size=(M, nb))
+    absq = np.abs(q.astype(np.int64)).reshape(M, nb, BLOCK).sum(2) * np.where(tags != 0, 8, 15)[None, :]
+    bound = (absq * (2.0 ** (e - e0))).sum(1)
+    e[bound >= 2.0 ** 24] = e0
+    assert np.all(absq.sum(1) < 2 ** 24), "row too large for an exact binary32 sum"
+    xf = q.astype(np.float32) * np.repeat(np.exp2(e).astype(np.float32), BLOCK, axis=1)
+    x = bf16_bits_from_f32(xf) if bf16 else xf.astype(np.float16)
+    w = rng.integers(-8, 8, size=(N, K), dtype=np.int8)
+    w[0] = 7
+    if N > 1:
+        w[1] = -8
+    if N > 2:
+        w[2] = np.where(np.arange(K) % 2 == 0, 7, -8)
+    w[N - 1] = 7
+    f = rng.integers(-7, -4, size=N)
+    s_w = np.exp2(f).astype(np.float32)
+    return ExactProblem(x=x, tags=tags, w=w, s_w=s_w, bf16=bf16, q=q, e=e, f=f)
+
+
 def config1(seed: int = 1) -> Problem:
     """BASELINE config 1: single linear M=16 K=256 N=256, 2 blocks, 1 INT8 outlier block."""
     return make_problem(16, 256, 256, seed=seed, n8=1)

@@ -175,3 +175,55 @@ def test_planner_cover_order_and_balance(M, N, K, frac, P, mode, orientation):
                 seen_owner = True
             elif is_split:
                 assert not seen_owner, "non-owner segment after an owner item"
+
+
+def test_stages_honoured_or_rejected():
+    """comet_sched_config.stages: 0 = auto (the compiled ring depth, reported by plan_info);
+    any other value must equal that depth, else COMET_ERR_INVALID_ARG (ADVICE/VERDICT r01)."""
+    import ctypes
+    L = cb.lib()
+    tags = np.zeros(32, np.uint8)
+    for M, orient in ((4096, 3), (1, 1), (200, 2)):
+        p = cb.Plan(M, 4096, 4096, tags, num_sms=148, device_plan=False, orientation=orient)
+        depth = p.info()["stages"]
+        assert 2 <= depth <= 8
+        cfg = cb.SchedConfig()
+        L.comet_sched_config_default(ctypes.byref(cfg))
+        cfg.num_sms, cfg.device_plan, cfg.orientation = 148, 0, orient
+        for st, ok in ((depth, True), (depth + 1, False), (1, False)):
+            cfg.stages = st
+            h = ctypes.c_void_p()
+            ws = ctypes.c_size_t()
+            rc = L.comet_plan_create(M, 4096, 4096, tags.ctypes.data_as(ctypes.c_void_p), ctypes.byref(cfg),
+                                     ctypes.byref(h), ctypes.byref(ws))
+            assert (rc == 0) == ok, (M, st, rc)
+            if rc == 0:
+                L.comet_plan_destroy(h)
+            else:
+                assert rc == 1 and b"ring depth" in L.comet_last_error()
+
+
+def test_layout_decoder_exhaustive_16bit():
+    """Pin I9 on the host side: the numpy decoder the GPU tests use for packed
+    weights (tests/_layout.py) against the layout definition of include/comet.h, exhaustively
+    over all 65,536 values of the word's low 16 bits (bytes 0 and 1 = channels 0/4 and 1/5),
+    plus a pure-Python packer of the same definition round-tripping every code pair."""
+    from _layout import unpack_weight
+    v = np.arange(1 << 16, dtype=np.uint32)
+    words = v | (0x88 << 16) | (0x88 << 24)            # bytes 2, 3: u = 8 -> w = 0
+    wp = words.view(np.uint8).reshape(-1, 4)          # little-endian bytes of each word
+    codes = unpack_weight(np.ascontiguousarray(wp), len(v), 8)
+    b0, b1 = (v & 0xFF).astype(np.int64), ((v >> 8) & 0xFF).astype(np.int64)
+    want = np.zeros((len(v), 8), np.int64)
+    want[:, 0], want[:, 4] = (b0 & 0xF) - 8, (b0 >> 4) - 8
+    want[:, 1], want[:, 5] = (b1 & 0xF) - 8, (b1 >> 4) - 8
+    assert np.array_equal(codes.astype(np.int64), want)
+
+    def pack_py(w8):   # comet.h: byte i = (u[i] & 0xF) | (u[i+4] << 4), u = w + 8
+        u = [x + 8 for x in w8]
+        return bytes(((u[i] & 0xF) | (u[i + 4] << 4)) for i in range(4))
+    for a in range(-8, 8):
+        for b in range(-8, 8):
+            w8 = [a, -8, 7, 0, b, 3, -1, -5]
+            got = unpack_weight(np.frombuffer(pack_py(w8), np.uint8).reshape(1, 4), 1, 8)
+            assert got.tolist() == [w8]

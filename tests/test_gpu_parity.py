@@ -1,7 +1,8 @@
 """GPU parity: the CUDA path (through the C ABI) against the CPU oracle on the same seeded
 inputs.  Codes, tags, scales, qsum, weight packing and the INT32 debug accumulators are
-compared bit-exactly; the dequantised output within the north-star tolerance
-(rtol 1e-3 / atol 1e-2 for FP16/FP32 outputs, 1 BF16 ulp for BF16 outputs, R10)."""
+compared bit-exactly; the dequantised output within the north-star tolerance, tightened
+(see _close; R10).  The production kernels' bit-exactness at full size is in
+tests/test_gpu_exact.py."""
 import numpy as np
 import pytest
 
@@ -124,15 +125,29 @@ def _run(p: synth.Problem, *, tile_n=0, split_mode=-1, out_dtype=torch.float32, 
 
 
 def _close(y, ref, dtype):
+    """Dequantised output against the binary64 oracle (north star: rtol 1e-3; R10).
+    FP32: |y - ref| <= 1e-3 |ref| + 1e-5 max|ref| (the GPU's binary32 summation of <= 224
+    exact block terms errs by ~1e-6 of the terms; 1e-5 max|ref| still catches one dropped or
+    mis-scaled block partial, ~1e-1).  FP16: within 1 FP16 ulp of ref (+ the same 1e-5 max|ref|
+    binary32 slack).  BF16: within 1 BF16 ulp of the oracle rounded to BF16 (a true 1-ulp bound:
+    the spacing of the binade of max(|r|, |y|))."""
+    got = y.float().cpu().numpy().astype(np.float64)
+    assert np.all(np.isfinite(got)), "non-finite outputs"
+    slack = 1e-5 * float(np.abs(ref).max())
     if dtype == torch.bfloat16:
-        got = y.float().cpu().numpy()
-        r = torch.from_numpy(ref).to(torch.bfloat16).float().numpy()
-        ulp = np.abs(r) * 2.0 ** -7 + 1e-30
-        assert np.all(np.abs(got - r) <= ulp * 1.0001 + 1e-6), "bf16 output off by more than 1 ulp"
+        r = torch.from_numpy(ref.astype(np.float32)).to(torch.bfloat16).double().numpy()
+        mag = np.maximum(np.abs(r), np.abs(got))
+        ulp = np.exp2(np.floor(np.log2(np.maximum(mag, 2.0 ** -126))) - 7)
+        bad = np.abs(got - r) > ulp
+        assert not bad.any(), f"{bad.sum()} bf16 outputs off by more than 1 ulp"
+    elif dtype == torch.float16:
+        mag = np.maximum(np.abs(ref), 2.0 ** -14)
+        ulp = np.exp2(np.floor(np.log2(mag)) - 10)
+        bad = np.abs(got - ref) > ulp + slack
+        assert not bad.any(), f"{bad.sum()} fp16 outputs off by more than 1 ulp; max err {np.abs(got-ref).max()}"
     else:
-        got = y.float().cpu().numpy().astype(np.float64)
-        bad = ~np.isclose(got, ref, rtol=1e-3, atol=1e-2)
-        assert not bad.any(), f"{bad.sum()} outputs outside rtol 1e-3 / atol 1e-2; max err {np.abs(got-ref).max()}"
+        bad = np.abs(got - ref) > 1e-3 * np.abs(ref) + slack
+        assert not bad.any(), f"{bad.sum()} outputs outside 1e-3 |ref| + 1e-5 max|ref|; max err {np.abs(got-ref).max()}"
 
 
 @pytest.mark.parametrize("orientation", [1, 2])
@@ -246,12 +261,28 @@ FULL = [
 
 @pytest.mark.parametrize("name,M,K,N,frac", FULL, ids=[f[0] for f in FULL])
 def test_gemm_full_size(name, M, K, N, frac):
-    """BASELINE sizes, the bench's launch configuration (auto plan), sampled rows vs oracle."""
+    """BASELINE sizes, the bench's launch configuration (auto plan), the synthetic workload
+    (N(0,1) activations with outlier channels), 64 sampled rows vs oracle (bit-exactness on
+    these configurations is tests/test_gpu_exact.py)."""
     p = synth.make_problem(M, K, N, frac=frac, seed=sum(map(ord, name)))
     y, plan = _run(p, out_dtype=torch.float16)
-    rows = synth.sample_rows(M, 8, p.x)
+    rows = synth.sample_rows(M, 64, p.x)
     yref, acc_sum, codes, scales = oracle.w4ax_rows(p.x, p.tags, p.w, p.s_w, rows)
     _close(y[torch.from_numpy(rows).to(DEV)], yref, torch.float16)
+
+
+@pytest.mark.parametrize("M,K,N,mean", [(4096, 28672, 8192, 2.0), (16, 8192, 28672, -1.5), (300, 4096, 1024, 3.0)])
+def test_gemm_nonzero_mean_activations(M, K, N, mean):
+    """Activations with a non-zero mean: large code sums, so the offset-binary correction
+    corr = 8 sum_b s_a qsum cancels a large part of the INT4 blocks' accumulators.
+    FP32 output, tightened tolerance."""
+    p = synth.make_problem(M, K, N, frac=0.05, seed=M + K)
+    x = (p.x.astype(np.float32) + np.float32(mean)).astype(np.float16)
+    p = synth.Problem(x=x, tags=p.tags, w=p.w, s_w=p.s_w)
+    y, plan = _run(p, out_dtype=torch.float32)
+    rows = synth.sample_rows(M, 64, p.x)
+    yref, _, _, _ = oracle.w4ax_rows(p.x, p.tags, p.w, p.s_w, rows)
+    _close(y[torch.from_numpy(rows).to(DEV)], yref, torch.float32)
 
 
 # ------------------------------------------------------------------------------- host-buffer path
