@@ -770,6 +770,36 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
             stage_and_store(pk, q * 32, 2);
             if (q == 1 && threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 15, 4 * (it - it_begin) + 2);
           }
+          if constexpr (COLS % 32 == 16) {
+            // the last 16 columns (tile_w = 160: 80 per warpgroup) do not fill a 64-byte TMA
+            // chunk: each thread stores its row's 32 bytes directly
+            constexpr int c0 = COLS - 16;
+            uint32_t pk[8];
+#pragma unroll
+            for (int i = 0; i < 8; i += 2) {
+              const int c = c0 + 2 * i;
+              const float4 s4 = *reinterpret_cast<const float4*>(sw + c);
+              const float2 y0 = ffma2(make_float2(acc[c], acc[c + 1]), make_float2(s4.x, s4.y),
+                                      make_float2(init * s4.x, init * s4.y));
+              const float2 y1 = ffma2(make_float2(acc[c + 2], acc[c + 3]), make_float2(s4.z, s4.w),
+                                      make_float2(init * s4.z, init * s4.w));
+              if (bf) {
+                __nv_bfloat162 h0 = __floats2bfloat162_rn(y0.x, y0.y), h1 = __floats2bfloat162_rn(y1.x, y1.y);
+                pk[i] = *reinterpret_cast<uint32_t*>(&h0);
+                pk[i + 1] = *reinterpret_cast<uint32_t*>(&h1);
+              } else {
+                __half2 h0 = __floats2half2_rn(y0.x, y0.y), h1 = __floats2half2_rn(y1.x, y1.y);
+                pk[i] = *reinterpret_cast<uint32_t*>(&h0);
+                pk[i + 1] = *reinterpret_cast<uint32_t*>(&h1);
+              }
+            }
+            const int64_t n = (int64_t)n0 + col_n(wg, c0);
+            if (m < P.M && n < P.N) {
+              uint4* dst = reinterpret_cast<uint4*>(reinterpret_cast<uint16_t*>(P.y) + m * P.ldy + n);
+              dst[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+              dst[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+            }
+          }
         }
         if (threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 15, 4 * (it - it_begin) + 3);
       }

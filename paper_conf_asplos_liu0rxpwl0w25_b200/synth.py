@@ -183,7 +183,7 @@ def make_exact_problem(M: int, K: int, N: int, *, frac: float = 0.05, seed: int 
     if N > 2:
         w[2] = np.where(np.arange(K) % 2 == 0, 7, -8)
     w[N - 1] = 7
-    f = rng.integers(-7, -4, size=N)
+    f = rng.integers(-9, -6, size=N)
     s_w = np.exp2(f).astype(np.float32)
     return ExactProblem(x=x, tags=tags, w=w, s_w=s_w, bf16=bf16, q=q, e=e, f=f)
 
