@@ -10,8 +10,18 @@ gate/up and qkv column-parallel (N sharded, no collective), down row-parallel (K
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl comet|reference]
 
-Prints one JSON line on rank 0.  --impl reference times the CPU oracle (oracle/) on a bounded
-sample of the same workload on the host cores (rank 0 only).
+N > 1: under torchrun (RANK / WORLD_SIZE / LOCAL_RANK / MASTER_* in the environment) every
+process is one rank; without them bench.py spawns the N ranks itself (one process per GPU,
+MASTER_ADDR 127.0.0.1) and fails loudly if fewer than N GPUs are visible or fewer than N ranks
+join.  Prints one JSON line on rank 0.  --impl reference times the CPU oracle (oracle/) on a
+bounded sample of the same workload on the host cores (rank 0 only; other ranks exit 0).
+
+Besides the headline (config 4) the line carries, at N = 1: `decode` (config 5, HBM-bound
+sweep), `configs.c2_llama2_7b` (config 2: LLaMA-2-7B shapes x M in {1, 16, 256, 4096}, FP16
+and BF16 inputs), `configs.c3_llama3_8b_mlp_m8192` (config 3: INT8-block fraction sweep
+0/5/25/100 % x scheduler mode, the Fig. 14 analog), `ablation` and
+`next_rows`; at N > 1: per-GPU GEMM TOPS and the all-reduce time of the
+row-parallel layer separately, for configs 4 and 5.
 """
 from __future__ import annotations
 
@@ -172,90 +182,28 @@ def cpu_baseline_sample(budget_s=15.0):
 
 # ---------------------------------------------------------------------------- comet arm
 
-def decode_sweep(cb, torch, dev, peaks, Ms=(1, 4, 8, 32), iters=20):
-    """BASELINE config 5: decode-regime W4Ax GEMM on the LLaMA-3-70B layers (TP1), HBM-bound.
-    Before every timed GEMM a 256 MiB write and a 256 MiB read leave L2 full of clean unrelated
-    lines, so the packed weights stream from HBM (and no dirty write-back competes with them).
-    All launches are queued behind a GPU sleep so host launch latency never appears as GPU idle
-    time inside the events.  Bytes = packed weights + weight scales + activation codes/scales +
-    output."""
-    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
-    flush_rd = torch.ones(64 << 20, dtype=torch.float32, device=dev)
-    out = {}
-    hbm = peaks["hbm_gbs"]
-    for name, K, N, _ in LAYERS:
-        rng = np.random.default_rng(7)
-        tags = synth.make_tags(K, FRAC, rng)
-        w, s_w = synth.make_weights(N, K, rng)
-        wp = cb.pack_weight(torch.from_numpy(w).to(dev))
-        swd = torch.from_numpy(s_w).to(dev)
-        del w
-        for M in Ms:
-            x = torch.from_numpy(synth.make_activations(M, K, tags, rng)).to(dev)
-            plan = cb.Plan(M, N, K, tags)
-            act, sc = cb.quantize_act(x, tags)
-            y = torch.empty((M, N), dtype=torch.float16, device=dev)
-            cb.w4ax_gemm(plan, act, sc, wp, swd, out=y)
-            torch.cuda.synchronize()
-            torch.cuda._sleep(int(4e7))
-            ws = []
-            for i in range(iters + 3):
-                flush.fill_(i & 0xFF)
-                flush_rd.sum()
-                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-                a.record()
-                cb.w4ax_gemm(plan, act, sc, wp, swd, out=y)
-                b.record()
-                ws.append((a, b))
-            torch.cuda.synchronize()
-            us = statistics.median(a.elapsed_time(b) for a, b in ws[3:]) * 1e3
-            # the whole decode layer step: kernel 1 (quantise x) + the GEMM, which launches as
-            # its programmatic dependent and streams weights while kernel 1 runs
-            torch.cuda._sleep(int(4e7))
-            ws2 = []
-            for i in range(iters + 3):
-                flush.fill_(i & 0xFF)
-                flush_rd.sum()
-                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-                a.record()
-                cb.quantize_act(x, tags, out=(act, sc))
-                cb.w4ax_gemm(plan, act, sc, wp, swd, out=y)
-                b.record()
-                ws2.append((a, b))
-            torch.cuda.synchronize()
-            us_step = statistics.median(a.elapsed_time(b) for a, b in ws2[3:]) * 1e3
-            nbytes = N * K // 2 + N * 4 + act.numel() + sc.numel() * 4 + M * N * 2
-            gbs = nbytes / (us * 1e-6) / 1e9
-            out[f"{name}_M{M}"] = {"us": round(us, 2), "GB/s": round(gbs, 1), "frac_hbm": round(gbs / hbm, 3),
-                                   "step_us": round(us_step, 2),
-                                   "step_GB/s": round((nbytes + M * K * 2) / (us_step * 1e-6) / 1e9, 1),
-                                   "orientation": plan.info()["orientation"], "tile_n": plan.info()["tile_n"]}
-        del wp
-    del flush, flush_rd
-    return {"unit": "GB/s", "peak_gbs": hbm, "kernel": "k_w4ax (decode orientation, weights on MMA M)",
-            "l2": "256 MiB write + 256 MiB read before every timed GEMM (clean L2, weights from HBM)",
-            "step": "step_us = kernel 1 (quantise x) + the GEMM as one decode layer step (the GEMM is a programmatic dependent launch)",
-            "layers": out}
+class Timer:
+    """Median device time of a launch sequence, CUDA events on the current stream.  Before every
+    timed iteration a 256 MiB write and a 256 MiB read leave L2 full of clean unrelated lines (so
+    weights and activations stream from HBM and no dirty write-back competes with them); the
+    launches are queued behind a GPU sleep so host launch latency never shows up as GPU idle time
+    inside the events."""
 
+    def __init__(self, torch, dev):
+        self.torch = torch
+        self.flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+        self.flush_rd = torch.ones(64 << 20, dtype=torch.float32, device=dev)
 
-def next_rows(cb, torch, dev, peaks, iters=20):
-    """SURVEY §8(f) rows built beyond the hot path, timed live (L2 left clean before every
-    launch, CUDA events, median): NEXT-1 fused channel permutation in kernel 1 (LLaMA-3-70B
-    layer inputs at M = 4096, permutation calibrated on a separate sample) against the
-    identity kernel, NEXT-3 group-wise weight scales on the decode GEMM against per-channel
-    scales, and NEXT-4 KV4 quantise / dequantise of a LLaMA-3-70B KV cache
-    (8 KV heads x 128 = 1024 channels, 32768 tokens, group 128).  GB/s = algorithmic bytes."""
-    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
-    flush_rd = torch.ones(64 << 20, dtype=torch.float32, device=dev)
-    hbm = peaks["hbm_gbs"]
-
-    def t(fn):
+    def us(self, fn, iters=20, flush=True):
+        torch = self.torch
         fn()
         torch.cuda.synchronize()
+        torch.cuda._sleep(int(4e7))
         ws = []
         for i in range(iters + 3):
-            flush.fill_(i & 0xFF)
-            flush_rd.sum()
+            if flush:
+                self.flush.fill_(i & 0xFF)
+                self.flush_rd.sum()
             a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             a.record()
             fn()
@@ -263,6 +211,220 @@ def next_rows(cb, torch, dev, peaks, iters=20):
             ws.append((a, b))
         torch.cuda.synchronize()
         return statistics.median(a.elapsed_time(b) for a, b in ws[3:]) * 1e3
+
+
+def alg_bytes(M, K, N, frac, out_bytes=2):
+    """SURVEY §8(d) algorithmic bytes of one W4Ax GEMM: activation codes at their packed width
+    (INT4 0.5 B, INT8 1 B) + scales, packed weights + scales, output."""
+    return M * K * (0.5 * (1 - frac) + frac) + 4 * M * (K // 128) + N * K / 2 + 4 * N + out_bytes * M * N
+
+
+def roofline_point(ops, nbytes, us, peaks):
+    """Fraction of the binding roofline: max(ops / tensor peak, bytes / HBM peak) / measured."""
+    t_ops = ops / (2.0 * peaks["bf16_tflops"] * 1e12)
+    t_mem = nbytes / (peaks["hbm_gbs"] * 1e9)
+    bound = "tensor" if t_ops >= t_mem else "hbm"
+    return {"bound": bound, "frac": round(max(t_ops, t_mem) / (us * 1e-6), 3),
+            "TOPS": round(ops / (us * 1e-6) / 1e12, 1), "GB/s": round(nbytes / (us * 1e-6) / 1e9, 1)}
+
+
+def dev_activations(torch, M, K, tags, seed, dev, bf16=False):
+    """synth.make_activations' recipe drawn on the device (fast at 8192 x 14336): N(0,1) with 4
+    channels of every INT8 block scaled by U(20, 100)."""
+    g = torch.Generator(device=dev)
+    g.manual_seed(seed)
+    x = torch.randn(M, K, generator=g, device=dev)
+    for b in np.nonzero(tags)[0]:
+        ch = int(b) * 128 + torch.randperm(128, generator=g, device=dev)[:4]
+        x[:, ch] *= 20.0 + 80.0 * torch.rand(4, generator=g, device=dev)
+    return x.to(torch.bfloat16 if bf16 else torch.float16)
+
+
+def dev_weights(cb, torch, N, K, seed, dev):
+    """synth.make_weights' recipe on the device: INT4 codes U[-8, 7], s_w = U(0.5, 1.5)/(8 sqrt K);
+    returns (packed weights, s_w)."""
+    g = torch.Generator(device=dev)
+    g.manual_seed(seed)
+    w = torch.randint(-8, 8, (N, K), generator=g, device=dev, dtype=torch.int8)
+    s_w = (0.5 + torch.rand(N, generator=g, device=dev)) / (8.0 * K ** 0.5)
+    return cb.pack_weight(w), s_w.float(), w
+
+
+def decode_sweep(cb, torch, dev, peaks, timer, Ms=(1, 4, 8, 32), iters=20, rank=0, world=1, dist=None):
+    """BASELINE config 5: decode-regime W4Ax GEMM on the LLaMA-3-70B layers, HBM-bound; at N GPUs
+    the layers are sharded as in the headline (gate_up / qkv column-parallel, down row-parallel
+    + NCCL all_reduce of FP32 partials, timed separately).  Bytes = packed weights + weight
+    scales + activation codes/scales + output (this rank's shard)."""
+    out = {}
+    hbm = peaks["hbm_gbs"]
+    for li, (name, K, N, kind) in enumerate(LAYERS):
+        rng = np.random.default_rng(7)
+        tags = synth.make_tags(K, FRAC, rng)
+        k0, k1, n0, n1 = shard(K, N, kind, tags, rank, world)
+        Kl, Nl, tl = k1 - k0, n1 - n0, np.ascontiguousarray(tags[k0 // 128:k1 // 128])
+        wp, swd, _ = dev_weights(cb, torch, Nl, Kl, 70 + li + 1000 * rank, dev)
+        for M in Ms:
+            x = dev_activations(torch, M, Kl, tl, 700 + M + rank, dev)
+            plan = cb.Plan(M, Nl, Kl, tl)
+            act, sc = cb.quantize_act(x, tl)
+            ydt = torch.float32 if (kind == "row" and world > 1) else torch.float16
+            y = torch.empty((M, Nl), dtype=ydt, device=dev)
+            us = timer.us(lambda: cb.w4ax_gemm(plan, act, sc, wp, swd, out=y), iters)
+            # the whole decode layer step: kernel 1 (quantise x) + the GEMM, which launches as its
+            # programmatic dependent and streams weights while kernel 1 runs
+            us_step = timer.us(lambda: (cb.quantize_act(x, tl, out=(act, sc)),
+                                        cb.w4ax_gemm(plan, act, sc, wp, swd, out=y)), iters)
+            ar_us = None
+            if kind == "row" and world > 1:
+                ar_us = timer.us(lambda: dist.all_reduce(y, op=dist.ReduceOp.SUM), iters, flush=False)
+            nbytes = Nl * Kl // 2 + Nl * 4 + act.numel() + sc.numel() * 4 + M * Nl * y.element_size()
+            if world > 1:
+                t = torch.tensor([us, us_step, ar_us or 0.0], device=dev, dtype=torch.float64)
+                dist.all_reduce(t, op=dist.ReduceOp.MAX)
+                us, us_step, ar_us = t[0].item(), t[1].item(), (t[2].item() if ar_us is not None else None)
+            gbs = nbytes / (us * 1e-6) / 1e9
+            out[f"{name}_M{M}"] = {"us": round(us, 2), "GB/s": round(gbs, 1), "frac_hbm": round(gbs / hbm, 3),
+                                   "step_us": round(us_step, 2),
+                                   "step_GB/s": round((nbytes + M * Kl * 2) / (us_step * 1e-6) / 1e9, 1),
+                                   "orientation": plan.info()["orientation"], "tile_n": plan.info()["tile_n"]}
+            if ar_us is not None:
+                out[f"{name}_M{M}"]["allreduce_us"] = round(ar_us, 2)
+        del wp
+    return {"unit": "GB/s", "peak_gbs": hbm, "kernel": "k_w4ax (decode orientation, weights on MMA M)",
+            "per_gpu": world > 1, "parallelism": "single GPU" if world == 1 else f"tp{world} (per-rank shard; GB/s per GPU, max over ranks)",
+            "l2": "256 MiB write + 256 MiB read before every timed GEMM (clean L2, weights from HBM)",
+            "step": "step_us = kernel 1 (quantise x) + the GEMM as one decode layer step (the GEMM is a programmatic dependent launch)",
+            "layers": out}
+
+
+LLAMA2_7B = [("qkvo", 4096, 4096), ("gate_up", 4096, 11008), ("down", 11008, 4096)]
+LLAMA3_8B = [("up", 4096, 14336), ("down", 14336, 4096)]
+
+
+def config2_sweep(cb, torch, dev, peaks, timer, iters=20):
+    """BASELINE config 2: LLaMA-2-7B linear layers x M in {1, 16, 256, 4096}, 5 % INT8 blocks,
+    FP16 and BF16 activations.  Per (dtype, M): each layer's GEMM alone, and the step (quantise +
+    GEMM of the three layers) with its roofline fraction (SURVEY §8(d) bytes / ops)."""
+    out = {}
+    wts = []
+    for li, (name, K, N) in enumerate(LLAMA2_7B):
+        tags = synth.make_tags(K, FRAC, np.random.default_rng(200 + li))
+        wp, sw, _ = dev_weights(cb, torch, N, K, 210 + li, dev)
+        wts.append((name, K, N, tags, wp, sw))
+    for bf16 in (False, True):
+        for M in (1, 16, 256, 4096):
+            L = []
+            for li, (name, K, N, tags, wp, sw) in enumerate(wts):
+                x = dev_activations(torch, M, K, tags, 220 + li + M, dev, bf16=bf16)
+                plan = cb.Plan(M, N, K, tags)
+                act, sc = cb.quantize_act(x, tags)
+                y = torch.empty((M, N), dtype=torch.float16, device=dev)
+                L.append((name, K, N, tags, wp, sw, x, plan, act, sc, y))
+            row = {"layers": {}}
+            ops = nbytes = 0.0
+            for (name, K, N, tags, wp, sw, x, plan, act, sc, y) in L:
+                us = timer.us(lambda: cb.w4ax_gemm(plan, act, sc, wp, sw, out=y), iters)
+                o, b = 2.0 * M * N * K, alg_bytes(M, K, N, FRAC)
+                ops += o
+                nbytes += b + 2 * M * K          # + the 16-bit input kernel 1 reads
+                d = roofline_point(o, b, us, peaks)
+                d.update(us=round(us, 2), orientation=plan.info()["orientation"],
+                         tile=[plan.info()["tile_n"], plan.info()["tile_w"]])
+                row["layers"][name] = d
+
+            def step():
+                for (name, K, N, tags, wp, sw, x, plan, act, sc, y) in L:
+                    cb.quantize_act(x, tags, out=(act, sc))
+                    cb.w4ax_gemm(plan, act, sc, wp, sw, out=y)
+            us = timer.us(step, iters)
+            row["step"] = dict(roofline_point(ops, nbytes, us, peaks), us=round(us, 2))
+            out[f"{'bf16' if bf16 else 'f16'}_M{M}"] = row
+            del L
+    return {"workload": "llama2_7b q/k/v/o 4096->4096, gate/up 4096->11008, down 11008->4096; 5 % INT8 blocks",
+            "l2": "clean L2 before every timed launch", "output": "f16",
+            "roofline": "frac = max(ops / (2 x bf16 peak), SURVEY bytes / HBM peak) / measured", "points": out}
+
+
+def config3_sweep(cb, torch, dev, peaks, timer, iters=10):
+    """BASELINE config 3: LLaMA-3-8B MLP (up 4096->14336, down 14336->4096) at M = 8192, INT8-block
+    fraction 0 / 5 / 25 / 100 % x scheduler mode (the Fig. 14 analog: naive ->
+    remapping -> decomposition).  On B200 both block kinds run at the same tensor rate,
+    so the modes differ by wave quantisation and fix-up cost, not INT4/INT8 balance.  Modes:
+    -1 auto, 0 whole-tile remapping, 1 stream-K decomposition, 2 naive unit round-robin, 3 unit
+    remapping (modes 2/3 split every tile across CTAs; refused when the fix-up workspace would
+    exceed 8 GiB)."""
+    M = 8192
+    out = {}
+    for li, (name, K, N) in enumerate(LLAMA3_8B):
+        wp, sw, _ = dev_weights(cb, torch, N, K, 300 + li, dev)
+        for f in (0.0, 0.05, 0.25, 1.0):
+            tags = synth.make_tags(K, f, np.random.default_rng(310 + li))
+            x = dev_activations(torch, M, K, tags, 320 + li, dev)
+            act, sc = cb.quantize_act(x, tags)
+            y = torch.empty((M, N), dtype=torch.float16, device=dev)
+            ops = 2.0 * M * N * K
+            q_us = timer.us(lambda: cb.quantize_act(x, tags, out=(act, sc)), iters)
+            row = {"int8_blocks": int(tags.sum()), "quantize_us": round(q_us, 2), "modes": {}}
+            for mode in (-1, 0, 1, 2, 3):
+                try:
+                    plan = cb.Plan(M, N, K, tags, split_mode=mode)
+                except cb.CometError as e:
+                    row["modes"][str(mode)] = {"refused": str(e)[:120]}
+                    continue
+                if plan.workspace_bytes > (4 << 30):
+                    row["modes"][str(mode)] = {"skipped": f"fix-up workspace {plan.workspace_bytes >> 20} MiB"}
+                    continue
+                us = timer.us(lambda: cb.w4ax_gemm(plan, act, sc, wp, sw, out=y), iters)
+                info = plan.info()
+                d = roofline_point(ops, alg_bytes(M, K, N, f), us, peaks)
+                d.update(us=round(us, 2), split_mode=info["split_mode"], n_split_tiles=info["n_split_tiles"],
+                         balance=round(info["mean_cta_cost"] / info["max_cta_cost"], 3))
+                row["modes"][str(mode)] = d
+                del plan
+                plan = None
+            out[f"{name}_f{int(round(f * 100))}"] = row
+        del wp
+    return {"workload": "llama3_8b MLP up 4096->14336, down 14336->4096, M=8192", "output": "f16",
+            "l2": "clean L2 before every timed launch",
+            "modes": {"-1": "auto", "0": "whole-tile remapping", "1": "stream-K decomposition (Fig. 8e)",
+                      "2": "naive unit round-robin (Fig. 8b/c)", "3": "unit remapping (Fig. 8d)"},
+            "points": out}
+
+
+def ablation(cb, torch, dev, peaks, timer, iters=10):
+    """SURVEY §8(d) ablations on LLaMA-3-70B gate_up (8192 -> 28672, M = 4096): (1) where the INT4
+    weights are widened: shared memory as the MMA B operand (orientation 3, the production
+    prefill kernel) vs tensor memory as the MMA A operand (orientation 1, 128-token tiles);
+    (3) data-parallel whole tiles vs stream-K decomposition."""
+    M, K, N = M_TOKENS, 8192, 28672
+    tags = synth.make_tags(K, FRAC, np.random.default_rng(400))
+    wp, sw, _ = dev_weights(cb, torch, N, K, 401, dev)
+    x = dev_activations(torch, M, K, tags, 402, dev)
+    act, sc = cb.quantize_act(x, tags)
+    y = torch.empty((M, N), dtype=torch.float16, device=dev)
+    ops = 2.0 * M * N * K
+    out = {}
+    for key, kw in (("widen_smem_pair_256x256", dict(orientation=3)),
+                    ("widen_smem_single_128x192", dict(orientation=2)),
+                    ("widen_tmem_A_128x128", dict(orientation=1, tile_n=128)),
+                    ("data_parallel_tiles", dict(orientation=3, split_mode=0)),
+                    ("stream_k", dict(orientation=3, split_mode=1))):
+        plan = cb.Plan(M, N, K, tags, **kw)
+        us = timer.us(lambda: cb.w4ax_gemm(plan, act, sc, wp, sw, out=y), iters)
+        out[key] = dict(roofline_point(ops, alg_bytes(M, K, N, FRAC), us, peaks), us=round(us, 2))
+    return {"layer": "llama3_70b gate_up M=4096", "points": out,
+            "not_live": "promotion variants and pipeline depth are compile-time (tools/gpu_variants.sh; DESIGN §7)"}
+
+
+def next_rows(cb, torch, dev, peaks, timer, iters=20):
+    """SURVEY §8(f) rows built beyond the hot path, timed live (L2 left clean before every
+    launch, CUDA events, median): NEXT-1 fused channel permutation in kernel 1 (LLaMA-3-70B
+    layer inputs at M = 4096, permutation calibrated on a separate sample) against the
+    identity kernel, NEXT-3 group-wise weight scales on the decode GEMM against per-channel
+    scales, and NEXT-4 KV4 quantise / dequantise of a LLaMA-3-70B KV cache
+    (8 KV heads x 128 = 1024 channels, 32768 tokens, group 128).  GB/s = algorithmic bytes."""
+    hbm = peaks["hbm_gbs"]
+    t = lambda fn: timer.us(fn, iters)
 
     out = {}
     for name, K in (("gate_up_qkv_input", 8192), ("down_input", 28672)):
@@ -312,7 +474,6 @@ def next_rows(cb, torch, dev, peaks, iters=20):
         us = t(fn)
         out[f"{nm}_T{T}_C{C}"] = {"us": round(us, 2), "GB/s": round(nbytes / us / 1e3, 1),
                                   "frac_hbm": round(nbytes / us / 1e3 / hbm, 3)}
-    del flush, flush_rd
     return {"unit": "GB/s", "peak_gbs": hbm, "l2": "256 MiB write + 256 MiB read before every launch",
             "rows": out}
 
@@ -339,6 +500,8 @@ def run_comet(args, rank, world, local_rank):
     dev = torch.device("cuda", local_rank)
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
+        if dist.get_world_size() != world:
+            raise SystemExit(f"bench.py: {dist.get_world_size()} ranks joined, expected {world}")
     stream = torch.cuda.current_stream()
 
     # ---- data (synthetic, seeded; identical on every rank, each rank keeps its shard)
@@ -426,9 +589,9 @@ def run_comet(args, rank, world, local_rank):
             if L["kind"] == "row" and world > 1:
                 ar_ms += eva[e][0].elapsed_time(eva[e][1])
     if world > 1:
-        t = torch.tensor([ms_total, sum(gemm_ms), ar_ms], device=dev, dtype=torch.float64)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms_total, gemm_max, ar_ms = t.tolist()
+        ms_total, ar_ms = max_over_ranks([ms_total, ar_ms], dist, torch, dev)
+        gemm_ms = max_over_ranks(gemm_ms, dist, torch, dev)
+        q_ms = max_over_ranks(q_ms, dist, torch, dev)
     ms_step = ms_total / args.steps
     value = total_ops() / (ms_step * 1e-3) / 1e12     # whole-job: all ranks' shards = the full layers
 
@@ -502,8 +665,16 @@ def run_comet(args, rank, world, local_rank):
                        "public API: H2D copy + quantize_act + w4ax_gemm (+ NCCL all_reduce) + D2H copy"}
 
     cpu = cpu_baseline_sample(args.cpu_budget) if (rank == 0 and world == 1 and args.cpu_budget > 0) else None
-    decode = decode_sweep(cb, torch, dev, peaks) if (rank == 0 and world == 1 and args.decode) else None
-    nxt = next_rows(cb, torch, dev, peaks) if (rank == 0 and world == 1 and args.decode) else None
+    timer = Timer(torch, dev) if (args.decode or args.configs) else None
+    # config 5 runs at every N (sharded like the headline); the N = 1-only sweeps after it
+    decode = decode_sweep(cb, torch, dev, peaks, timer, rank=rank, world=world, dist=dist) if args.decode else None
+    solo = rank == 0 and world == 1
+    cfgs = None
+    if solo and args.configs:
+        cfgs = {"c2_llama2_7b": config2_sweep(cb, torch, dev, peaks, timer),
+                "c3_llama3_8b_mlp_m8192": config3_sweep(cb, torch, dev, peaks, timer)}
+    abl = ablation(cb, torch, dev, peaks, timer) if (solo and args.configs) else None
+    nxt = next_rows(cb, torch, dev, peaks, timer) if (solo and args.decode) else None
 
     if rank == 0:
         line = {
@@ -523,9 +694,14 @@ def run_comet(args, rank, world, local_rank):
             "gpu_launches": 2 * len(layers) * args.steps,
             "clocks": clocks,
             "decode": decode,
+            "configs": cfgs,
+            "ablation": abl,
             "next_rows": nxt,
         }
         if world > 1:
+            # per-GPU GEMM throughput (each rank's shard over its own GEMM time, max over ranks)
+            # and the row-parallel all-reduce, reported separately
+            line["per_gpu_gemm_tops"] = gemm_ops_rank / (sum(gemm_ms) / args.steps * 1e-3) / 1e12
             line["allreduce_ms_per_step"] = ar_ms / args.steps
         print(json.dumps(line), flush=True)
     if world > 1:
@@ -533,7 +709,38 @@ def run_comet(args, rank, world, local_rank):
     return 0
 
 
-def main():
+def max_over_ranks(vals, dist, torch, dev):
+    """Element-wise max over ranks of a list of floats (device timings are maxed, never averaged)."""
+    t = torch.tensor([float(v) for v in vals], dtype=torch.float64, device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return t.tolist()
+
+
+def free_port() -> int:
+    import socket
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        return so.getsockname()[1]
+
+
+def _rank_entry(rank, world, port, target, target_args):
+    os.environ.update(RANK=str(rank), LOCAL_RANK=str(rank), WORLD_SIZE=str(world), LOCAL_WORLD_SIZE=str(world),
+                      MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    rc = target(*target_args)
+    if rc:
+        raise SystemExit(rc)
+
+
+def launch_ranks(world: int, target, target_args=()):
+    """One process per rank (spawn), RANK / LOCAL_RANK / WORLD_SIZE / MASTER_ADDR=127.0.0.1 /
+    MASTER_PORT set as torchrun would; raises if any rank fails (so fewer ranks than asked is an
+    error, never a silent single-process run).  target(*target_args) runs in every rank."""
+    import torch.multiprocessing as mp
+    mp.start_processes(_rank_entry, args=(world, free_port(), target, tuple(target_args)), nprocs=world,
+                       join=True, start_method="spawn")
+
+
+def parse_args(argv=None):
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=30)
@@ -545,14 +752,39 @@ def main():
     ap.add_argument("--split-mode", type=int, default=-1)
     ap.add_argument("--orientation", type=int, default=0, help="0 = planner default")
     ap.add_argument("--tile-w", type=int, default=0, help="weights per tile (192/256); 0 = planner default")
-    ap.add_argument("--decode", type=int, default=1, help="1 = add the decode (M<=32) HBM sweep (N=1)")
-    args = ap.parse_args()
+    ap.add_argument("--decode", type=int, default=1, help="1 = add the decode (M<=32) HBM sweep (config 5)")
+    ap.add_argument("--configs", type=int, default=1, help="1 = add configs 2 / 3 and the ablations (N=1)")
+    return ap.parse_args(argv)
+
+
+def rank_main(argv=None):
+    """The work of one rank (RANK / WORLD_SIZE / LOCAL_RANK from the environment)."""
+    args = parse_args(argv)
     rank = int(os.environ.get("RANK", "0"))
-    world = int(os.environ.get("WORLD_SIZE", str(args.gpus if args.gpus == 1 else 1)))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        raise SystemExit(f"bench.py: WORLD_SIZE={world} but --gpus {args.gpus}")
     if args.impl == "reference":
         return run_reference(args, rank, world)
     return run_comet(args, rank, world, local_rank)
+
+
+def main(argv=None):
+    args = parse_args(argv)
+    if "WORLD_SIZE" in os.environ or args.gpus == 1:
+        return rank_main(argv)
+    # --gpus N > 1 without a launcher: spawn the N ranks here
+    if args.impl == "reference":
+        # the reference arm is the host oracle on rank 0; the other ranks would exit without work
+        os.environ.update(RANK="0", LOCAL_RANK="0", WORLD_SIZE=str(args.gpus))
+        return rank_main(argv)
+    import torch
+    n = torch.cuda.device_count()
+    if n < args.gpus:
+        raise SystemExit(f"bench.py: --gpus {args.gpus} but only {n} CUDA device(s) visible")
+    launch_ranks(args.gpus, rank_main, (sys.argv[1:] if argv is None else list(argv),))
+    return 0
 
 
 if __name__ == "__main__":
