@@ -213,6 +213,25 @@ class Timer:
         return statistics.median(a.elapsed_time(b) for a, b in ws[3:]) * 1e3
 
 
+def us_rotating(torch, fns, rounds=10):
+    """Mean device time per launch of a back-to-back sequence cycling through `fns` (each reads
+    its own copy of the weights; together > 2 x L2, so every launch streams from HBM) -- the way
+    consecutive decode layers run.  Amortises the ~1 us event-clock granularity and the fixed
+    cost of an isolated, event-bracketed launch (an empty kernel measures ~6 us that way)."""
+    for f in fns:
+        f()
+    torch.cuda.synchronize()
+    torch.cuda._sleep(int(4e7))
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record()
+    for _ in range(rounds):
+        for f in fns:
+            f()
+    b.record()
+    torch.cuda.synchronize()
+    return a.elapsed_time(b) * 1e3 / (rounds * len(fns))
+
+
 def alg_bytes(M, K, N, frac, out_bytes=2):
     """SURVEY §8(d) algorithmic bytes of one W4Ax GEMM: activation codes at their packed width
     (INT4 0.5 B, INT8 1 B) + scales, packed weights + scales, output."""
@@ -263,37 +282,47 @@ def decode_sweep(cb, torch, dev, peaks, timer, Ms=(1, 4, 8, 32), iters=20, rank=
         k0, k1, n0, n1 = shard(K, N, kind, tags, rank, world)
         Kl, Nl, tl = k1 - k0, n1 - n0, np.ascontiguousarray(tags[k0 // 128:k1 // 128])
         wp, swd, _ = dev_weights(cb, torch, Nl, Kl, 70 + li + 1000 * rank, dev)
+        # weight copies for the back-to-back measurement: > 2 x L2 (126 MB) in total
+        ncopy = max(2, -(-300 * (1 << 20) // (Nl * Kl // 2)))
+        wps = [wp] + [wp.clone() for _ in range(ncopy - 1)]
         for M in Ms:
             x = dev_activations(torch, M, Kl, tl, 700 + M + rank, dev)
             plan = cb.Plan(M, Nl, Kl, tl)
             act, sc = cb.quantize_act(x, tl)
             ydt = torch.float32 if (kind == "row" and world > 1) else torch.float16
             y = torch.empty((M, Nl), dtype=ydt, device=dev)
-            us = timer.us(lambda: cb.w4ax_gemm(plan, act, sc, wp, swd, out=y), iters)
+            # isolated launch (event-bracketed, L2 cleaned before it)
+            us_iso = timer.us(lambda: cb.w4ax_gemm(plan, act, sc, wp, swd, out=y), iters)
+            # back-to-back launches over rotating weight copies (how consecutive decode layers
+            # run; every launch streams its weights from HBM): the number the roofline uses
+            us = us_rotating(torch, [lambda w_=w_: cb.w4ax_gemm(plan, act, sc, w_, swd, out=y) for w_ in wps])
             # the whole decode layer step: kernel 1 (quantise x) + the GEMM, which launches as its
             # programmatic dependent and streams weights while kernel 1 runs
-            us_step = timer.us(lambda: (cb.quantize_act(x, tl, out=(act, sc)),
-                                        cb.w4ax_gemm(plan, act, sc, wp, swd, out=y)), iters)
+            us_step = us_rotating(torch, [lambda w_=w_: (cb.quantize_act(x, tl, out=(act, sc)),
+                                                          cb.w4ax_gemm(plan, act, sc, w_, swd, out=y)) for w_ in wps])
             ar_us = None
             if kind == "row" and world > 1:
                 ar_us = timer.us(lambda: dist.all_reduce(y, op=dist.ReduceOp.SUM), iters, flush=False)
             nbytes = Nl * Kl // 2 + Nl * 4 + act.numel() + sc.numel() * 4 + M * Nl * y.element_size()
             if world > 1:
-                t = torch.tensor([us, us_step, ar_us or 0.0], device=dev, dtype=torch.float64)
+                t = torch.tensor([us, us_step, ar_us or 0.0, us_iso], device=dev, dtype=torch.float64)
                 dist.all_reduce(t, op=dist.ReduceOp.MAX)
-                us, us_step, ar_us = t[0].item(), t[1].item(), (t[2].item() if ar_us is not None else None)
+                us, us_step, ar_us, us_iso = t[0].item(), t[1].item(), (t[2].item() if ar_us is not None else None), t[3].item()
             gbs = nbytes / (us * 1e-6) / 1e9
             out[f"{name}_M{M}"] = {"us": round(us, 2), "GB/s": round(gbs, 1), "frac_hbm": round(gbs / hbm, 3),
+                                   "isolated_us": round(us_iso, 2),
                                    "step_us": round(us_step, 2),
                                    "step_GB/s": round((nbytes + M * Kl * 2) / (us_step * 1e-6) / 1e9, 1),
                                    "orientation": plan.info()["orientation"], "tile_n": plan.info()["tile_n"]}
             if ar_us is not None:
                 out[f"{name}_M{M}"]["allreduce_us"] = round(ar_us, 2)
-        del wp
-    return {"unit": "GB/s", "peak_gbs": hbm, "kernel": "k_w4ax (decode orientation, weights on MMA M)",
+        del wp, wps
+    return {"unit": "GB/s", "peak_gbs": hbm, "kernel": "k_w4ax (decode orientation, weights on MMA M) + k_fixup for split tiles",
             "per_gpu": world > 1, "parallelism": "single GPU" if world == 1 else f"tp{world} (per-rank shard; GB/s per GPU, max over ranks)",
-            "l2": "256 MiB write + 256 MiB read before every timed GEMM (clean L2, weights from HBM)",
-            "step": "step_us = kernel 1 (quantise x) + the GEMM as one decode layer step (the GEMM is a programmatic dependent launch)",
+            "timing": "us / GB/s / frac_hbm: mean per launch of 10 rounds of back-to-back launches cycling over >= 300 MB of "
+                      "weight copies (> 2 x L2: every launch streams from HBM); isolated_us: one event-bracketed launch after a "
+                      "256 MiB write + 256 MiB read (median of 20; includes the ~6 us an empty kernel measures that way)",
+            "step": "step_us = kernel 1 (quantise x) + the GEMM as one decode layer step (the GEMM is a programmatic dependent launch), back to back",
             "layers": out}
 
 

@@ -260,10 +260,12 @@ comet_status_t comet_plan_describe(comet_plan_t plan, int32_t* items, int64_t ma
  *                           (bit-exact integer accumulators; slower debug kernel).
  *   debug_acc_blocks        NULL, or device [K/128][M][N] int32 per-block acc_b (tiny shapes).
  *   workspace               device, >= the plan's workspace_bytes (may be NULL if 0).  Zero it
- *                           once before its first use; afterwards it may be reused by any
- *                           later call of any plan without clearing (stream-K flags are
- *                           compared with a process-wide launch counter), but it must not be
- *                           used by two GEMMs in flight at the same time.
+ *                           once before its first use: every completed launch leaves its
+ *                           flag / counter words zero again, so it may then be reused by any
+ *                           later call of any plan without clearing (flags also carry a
+ *                           process-wide launch counter), but it must not be used by two GEMMs
+ *                           in flight at the same time, and must be re-zeroed after a launch
+ *                           that failed.
  * The persistent grid is sized at plan time to what the occupancy calculator admits as
  * co-resident (the stream-K owner of a split tile waits for the other units' partials); a
  * fix-up or pipeline wait that exceeds 4 s (only possible if another kernel holds the SMs that

@@ -350,9 +350,13 @@ comet_status_t comet_plan_create(int64_t M, int64_t N, int64_t K, const uint8_t*
     if (e == cudaSuccess) e = cudaMemcpy(p.d_cta_begin, p.cta_begin.data(), p.cta_begin.size() * sizeof(int32_t), cudaMemcpyHostToDevice);
     if (e == cudaSuccess && !p.items.empty())
       e = cudaMemcpy(p.d_items, p.items.data(), p.items.size() * sizeof(WorkItem), cudaMemcpyHostToDevice);
+    if (e == cudaSuccess) e = cudaMalloc(&p.d_fix, std::max<size_t>(2, p.fix_info.size()) * sizeof(int32_t));
+    if (e == cudaSuccess && !p.fix_info.empty())
+      e = cudaMemcpy(p.d_fix, p.fix_info.data(), p.fix_info.size() * sizeof(int32_t), cudaMemcpyHostToDevice);
     if (e != cudaSuccess) {
       if (p.d_cta_begin) cudaFree(p.d_cta_begin);
       if (p.d_items) cudaFree(p.d_items);
+      if (p.d_fix) cudaFree(p.d_fix);
       delete h;
       return cuda_status(e, "plan upload");
     }
@@ -371,6 +375,7 @@ comet_status_t comet_plan_destroy(comet_plan_t plan) {
   // s_h2d / s_d2h are the device's shared copy streams (copy_streams), not owned by the plan
   if (plan->p.d_cta_begin) cudaFree(plan->p.d_cta_begin);
   if (plan->p.d_items) cudaFree(plan->p.d_items);
+  if (plan->p.d_fix) cudaFree(plan->p.d_fix);
   delete plan;
   return COMET_OK;
 }

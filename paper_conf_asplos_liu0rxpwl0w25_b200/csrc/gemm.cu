@@ -15,11 +15,10 @@
 // profiles/r01/probe_stream.txt), the two K-blocks' activation codes and their scales.
 //
 // Roles (512 threads, 16 warps):
-//   warp 0       TMA producer: W box [128 rows x 128 B], X boxes [NT x 128 B] per K-block, and
-//                each K-block's scales s_a[b][m0 .. m0+NT) (own ring).
-//   warp 1       MMA issuer (one thread): per K-block 4 x tcgen05.mma (K = 32) into its own TMEM
+//   warp 0       TMA producer of the weight ring (lane 0).
+//   warp 1       MMA issuer: per K-block 4 x tcgen05.mma (K = 32) into its own TMEM
 //                accumulator; INT4 blocks use kind::f8f6f4 (E4M3), INT8 blocks kind::i8.
-//   warp 2       TMEM allocator.
+//   warp 2       TMEM allocator; TMA producer of the activation ring (lane 0): codes + scales.
 //   warps 4-11   widen, two groups of 4 warps taking alternate stages: a packed INT4 weight row
 //                -> 256 bytes in 3 instructions per 8 values (the B200 form of the paper's
 //                location switch + zero extension), tcgen05.st into a TMEM A buffer.
@@ -44,7 +43,8 @@ namespace gemm {
 namespace {
 #ifndef COMET_DEC_ABLATE
 #define COMET_DEC_ABLATE 0      // timing experiments only (wrong results): bit 0 no MMAs, bit 1 no
-#endif                          // TMEM stores of widened weights, bit 2 no accumulator loads
+#endif                          // TMEM stores of widened weights, bit 2 no accumulator loads,
+                                // bit 3 no weight reads by the widen warps, bit 4 no activation loads
 
 #ifndef COMET_DEC_NA
 #define COMET_DEC_NA 2
@@ -61,11 +61,11 @@ namespace {
 #ifndef COMET_DEC_WIDEN_PF
 #define COMET_DEC_WIDEN_PF 0   // 1: widen warps load stage s+1 weights before storing stage s (measured slower)
 #endif
+#ifndef COMET_DEC_SWMAX
+#define COMET_DEC_SWMAX 8   // cap of the packed-weight ring depth (variant experiments)
+#endif
 #ifndef COMET_DEC_PDL
 #define COMET_DEC_PDL 1     // launch as a programmatic dependent of kernel 1 (weights stream early)
-#endif
-#ifndef COMET_DEC_UNIFORM_MMA
-#define COMET_DEC_UNIFORM_MMA 1
 #endif
 constexpr int kWidenWarp0 = 4;
 constexpr int kPromoWarp0 = 12;
@@ -101,7 +101,7 @@ struct Cfg {
   static constexpr int SX = NT >= 32 ? COMET_DEC_SX32 : 4;     // X ring depth
   static constexpr int SMEM_BUDGET = 224 * 1024;            // 227 KB minus alignment, barriers, tags
   static constexpr int SW_RAW = (SMEM_BUDGET - SX * X_STAGE) / W_BYTES;
-  static constexpr int SW = SW_RAW > 8 ? 8 : SW_RAW;           // W ring depth
+  static constexpr int SW = SW_RAW > COMET_DEC_SWMAX ? COMET_DEC_SWMAX : SW_RAW;   // W ring depth
   static constexpr int SMEM_DATA = SW * W_BYTES + SX * X_STAGE;
   static constexpr int N_BARS = 2 * SW + 2 * SX + 2 * NA + 2 * NACC;
   static constexpr int SMEM_BYTES = 1024 + SMEM_DATA + N_BARS * 8 + 16 + kMaxBlocks;
@@ -152,6 +152,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bars + C::N_BARS);
   uint8_t* s_tags = reinterpret_cast<uint8_t*>(tmem_holder + 4);
   const uint32_t s_tags_a = smem_u32(s_tags);
+  // The CTA's work items, staged in shared memory at setup: every role walks the list, and a
+  // global load of the next item at an item boundary costs microseconds once the weight stream
+  // saturates HBM (it stalled the whole pipeline at every boundary).
+  constexpr int kSmemItems = 64;
+  __shared__ WorkItem s_items[kSmemItems];
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
@@ -172,14 +177,14 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
     }
     for (int i = 0; i < SX; ++i) {
       mbar_init(&full_x[i], 1);
-      mbar_init(&empty_x[i], 2 + 4);
+      mbar_init(&empty_x[i], 1 + 4);
     }
     for (int i = 0; i < NA; ++i) {
       mbar_init(&a_full[i], COMET_DEC_WIDEN_WARPS);
-      mbar_init(&a_empty[i], 2);
+      mbar_init(&a_empty[i], 1);
     }
     for (int i = 0; i < NACC; ++i) {
-      mbar_init(&acc_full[i], 2);
+      mbar_init(&acc_full[i], 1);
       mbar_init(&acc_empty[i], 4);
     }
     fence_mbar_init();
@@ -189,10 +194,14 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
     tmem_relinquish();
   }
   for (int i = threadIdx.x; i < nb; i += kThreads) s_tags[i] = P.tags.get(i) ? 1 : 0;
+  for (int i = threadIdx.x; i < min(kSmemItems, it_end - it_begin); i += kThreads) s_items[i] = load_item(P, it_begin + i, debug);
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
   const uint32_t tbase = *tmem_holder;
+  auto item = [&](int it) -> WorkItem {
+    return it - it_begin < kSmemItems ? s_items[it - it_begin] : load_item(P, it, debug);
+  };
   if (tracing && threadIdx.x == 0) P.trace[32768 + blockIdx.x * 4 + 1] = globaltimer_ns();
   int tr = 0;   // trace index (per role)
   // Programmatic dependent launch: the kernel may start while the previous kernel of the stream
@@ -203,13 +212,13 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
   if (!(warp == 0 && lane == 0)) asm volatile("griddepcontrol.wait;" ::: "memory");
 
   if (warp < kWidenWarp0) {
-    setmaxnreg_dec<40>();
+    setmaxnreg_dec<56>();
     if (warp == 0 && lane == 0) {
       // ------------------------------------------------------------------ W producer
       int st = 0;
       uint32_t ph = 0;
       for (int it = it_begin; it < it_end; ++it) {
-        const WorkItem w = load_item(P, it, debug);
+        const WorkItem w = item(it);
         const int n0 = (w.tile / P.n_m_tiles) * kTileW;
         for (int kb = w.kb_begin; kb < w.kb_end; kb += KS) {
           const int npair = (min(KS, w.kb_end - kb) + 1) >> 1;
@@ -226,11 +235,16 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
       int st = 0;
       uint32_t ph = 0;
       for (int it = it_begin; it < it_end; ++it) {
-        const WorkItem w = load_item(P, it, debug);
+        const WorkItem w = item(it);
         const int m0 = (w.tile % P.n_m_tiles) * NT;
         const int n0 = (w.tile / P.n_m_tiles) * kTileW;
         for (int kb = w.kb_begin; kb < w.kb_end; kb += KS) {
           mbar_wait(&empty_x[st], ph ^ 1);
+          if (COMET_DEC_ABLATE & 16) {            // timing experiment: no activation loads
+            mbar_arrive(&full_x[st]);
+            if (++st == SX) { st = 0; ph ^= 1; }
+            continue;
+          }
           mbar_arrive_expect_tx(&full_x[st], KS * C::XKB_BYTES + C::S_BYTES + C::Q_BYTES + C::G_BYTES);
           tma_load_3d(sX(st), &P.map_x, &full_x[st], 0, m0, kb);
           tma_load_2d(sS(st), &P.map_s, &full_x[st], m0, kb);
@@ -241,16 +255,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
           if (++st == SX) { st = 0; ph ^= 1; }
         }
       }
-    } else if (warp == 1 || warp == 3) {
-      // ------------------------------------------------------------------ MMA issuers
-      // Two issuing warps share every stage: warp 1 issues the stage's even K-blocks, warp 3
-      // the odd ones (each K-block has its own accumulator).  tcgen05.commit tracks the
-      // issuing thread's own MMAs, so both commit each stage's barriers (counts 2).
+    } else if (warp == 1) {
+      // ------------------------------------------------------------------ MMA issuer
       // The whole warp runs the loop and every operand is made warp-uniform (shuffle from lane
       // 0), so the compiler keeps the MMA operands in uniform registers; one elected lane
       // issues.  (With a lane-0-only loop every tcgen05.mma went through an R2UR waterfall.)
-#if COMET_DEC_UNIFORM_MMA
-      const int par = warp == 1 ? 0 : 1;
+      // One K-block = 4 x tcgen05.mma (K = 32) into its own accumulator of the stage's set.
       const uint32_t id_f8 = idesc_f8f6f4_e4m3(128, NT);
       const uint32_t id_i8 = idesc_i8(128, NT);
       const uint32_t tb = __shfl_sync(0xffffffffu, tbase, 0);
@@ -258,7 +268,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
       int sx = 0, ab = 0, accs = 0;
       uint32_t xph = 0, aph = 0, accph = 0;
       for (int it = it_begin; it < it_end; ++it) {
-        const WorkItem w = load_item(P, it, debug);
+        const WorkItem w = item(it);
         const int kb_begin = __shfl_sync(0xffffffffu, w.kb_begin, 0);
         const int kb_end = __shfl_sync(0xffffffffu, w.kb_end, 0);
         for (int kb = kb_begin; kb < kb_end; kb += KS) {
@@ -266,16 +276,14 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
           mbar_wait(&full_x[sx], xph);
           mbar_wait(&a_full[ab], aph);
           mbar_wait(&acc_empty[accs], accph ^ 1);
-          if (par == 0 && lane == 0) trace_ev(P, 1, tr);
+          if (lane == 0) trace_ev(P, 1, tr);
           tc_fence_after();
           const uint32_t d0 = tb + C::ACC_COL + accs * C::ACC_SET;
           const uint32_t a0 = tb + ab * C::A_COLS;
           const uint64_t b0 = sdesc_kmajor_sw128(sx0 + sx * C::X_STAGE);
-          const uint32_t tagw = __shfl_sync(0xffffffffu, lane < KS ? lds_u8(s_tags_a + kb + lane) : 0u, 0) |
-                                (__shfl_sync(0xffffffffu, lane < KS ? lds_u8(s_tags_a + kb + lane) : 0u, 1) << 1) |
-                                (__shfl_sync(0xffffffffu, lane < KS ? lds_u8(s_tags_a + kb + lane) : 0u, 2) << 2) |
-                                (__shfl_sync(0xffffffffu, lane < KS ? lds_u8(s_tags_a + kb + lane) : 0u, 3) << 3);
-          for (int c = par; c < nk; c += 2) {
+          const uint32_t tg = lane < KS ? lds_u8(s_tags_a + kb + lane) : 0u;
+          const uint32_t tagw = __ballot_sync(0xffffffffu, tg != 0);
+          for (int c = 0; c < nk; ++c) {
             const uint32_t d = d0 + c * NT, a = a0 + c * 32;
             const uint64_t bd = b0 + (uint64_t)((c * C::XKB_BYTES) >> 4);
             if (COMET_DEC_ABLATE & 1) {
@@ -298,54 +306,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
             tc_commit(&a_empty[ab]);
           }
           __syncwarp();
-          if (par == 0 && lane == 0) trace_ev(P, 2, tr++);
+          if (lane == 0) trace_ev(P, 2, tr++);
           if (++sx == SX) { sx = 0; xph ^= 1; }
           if (++ab == NA) { ab = 0; aph ^= 1; }
           if (++accs == NACC) { accs = 0; accph ^= 1; }
         }
       }
-#else
-      if (lane == 0) {
-      const int par = warp == 1 ? 0 : 1;
-      const uint32_t id_f8 = idesc_f8f6f4_e4m3(128, NT);
-      const uint32_t id_i8 = idesc_i8(128, NT);
-      int sx = 0, ab = 0, accs = 0;
-      uint32_t xph = 0, aph = 0, accph = 0;
-      for (int it = it_begin; it < it_end; ++it) {
-        const WorkItem w = load_item(P, it, debug);
-        for (int kb = w.kb_begin; kb < w.kb_end; kb += KS) {
-          const int nk = min(KS, w.kb_end - kb);
-          mbar_wait(&full_x[sx], xph);
-          mbar_wait(&a_full[ab], aph);
-          mbar_wait(&acc_empty[accs], accph ^ 1);
-          if (par == 0) trace_ev(P, 1, tr);
-          tc_fence_after();
-          const uint32_t d0 = tbase + C::ACC_COL + accs * C::ACC_SET;
-          const uint32_t a0 = tbase + ab * C::A_COLS;
-          const uint64_t b0 = sdesc_kmajor_sw128(smem_u32(sX(sx)));
-          for (int c = par; c < nk; c += 2) {
-            const uint32_t d = d0 + c * NT, a = a0 + c * 32;
-            const uint64_t bd = b0 + (uint64_t)((c * C::XKB_BYTES) >> 4);
-            if (COMET_DEC_ABLATE & 1) {
-            } else if (lds_u8(s_tags_a + kb + c)) {
-#pragma unroll
-              for (int k = 0; k < 4; ++k) mma_i8_ts(d, a + 8 * k, bd + 2 * k, id_i8, k);
-            } else {
-#pragma unroll
-              for (int k = 0; k < 4; ++k) mma_f8_ts(d, a + 8 * k, bd + 2 * k, id_f8, k);
-            }
-          }
-          tc_commit(&acc_full[accs]);
-          tc_commit(&empty_x[sx]);
-          tc_commit(&a_empty[ab]);
-          if (par == 0) trace_ev(P, 2, tr++);
-          if (++sx == SX) { sx = 0; xph ^= 1; }
-          if (++ab == NA) { ab = 0; aph ^= 1; }
-          if (++accs == NACC) { accs = 0; accph ^= 1; }
-        }
-      }
-      }
-#endif
     }
   } else if (warp < kPromoWarp0 && warp - kWidenWarp0 >= COMET_DEC_WIDEN_WARPS) {
     setmaxnreg_dec<112>();                        // spare warps of a 4-warp widen variant
@@ -369,7 +335,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
     int it = it_begin;
     WorkItem w{};
     int kb = 0;
-    if (it < it_end) { w = load_item(P, it, debug); kb = w.kb_begin; }
+    if (it < it_end) { w = item(it); kb = w.kb_begin; }
     uint4 cn[4 * KH];
     int kb_n = 0, nk_n = 0, seq_f = 0;
     auto fetch = [&]() {
@@ -393,7 +359,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
       kb += KS;                                   // advance to the next stage of the work list
       if (kb >= w.kb_end) {
         ++it;
-        if (it < it_end) { w = load_item(P, it, debug); kb = w.kb_begin; }
+        if (it < it_end) { w = item(it); kb = w.kb_begin; }
       }
     };
     bool have = it < it_end;
@@ -444,7 +410,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
     }
 #else
     for (int it = it_begin; it < it_end; ++it) {
-      const WorkItem w = load_item(P, it, debug);
+      const WorkItem w = item(it);
       for (int kb = w.kb_begin; kb < w.kb_end; kb += KS, ++seq) {
         const int nk = min(KS, w.kb_end - kb);
         mbar_wait(&full_w[st], ph);
@@ -495,22 +461,15 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
           const int cb = half * KH + i;
           if (cb < nk) {
             const bool is8 = lds_u8(s_tags_a + kb + cb) != 0;
+            const uint32_t ta = tbase + ab * C::A_COLS + cb * 32 + lane_addr;
             uint32_t o[32];
-#pragma unroll
-            for (int j = 0; j < 4; ++j) {
-              const uint32_t pw[4] = {cc[4 * i + j].x, cc[4 * i + j].y, cc[4 * i + j].z, cc[4 * i + j].w};
-#pragma unroll
-              for (int e = 0; e < 4; ++e) {
-                const uint32_t pv = pw[e];
-                const int g = 2 * (j * 4 + e);
-                widen_int4(pv, o[g], o[g + 1]);
-                if (is8) {
-                  o[g] = int4_to_int8(o[g]);
-                  o[g + 1] = int4_to_int8(o[g + 1]);
-                }
-              }
+            if (is8) {                          // warp-uniform, one branch per K-block
+              widen_kblock_row<true>(&cc[4 * i], o);
+              if (!(COMET_DEC_ABLATE & 2)) tmem_st32(ta, o);
+            } else {
+              widen_kblock_row<false>(&cc[4 * i], o);
+              if (!(COMET_DEC_ABLATE & 2)) tmem_st32(ta, o);
             }
-            if (!(COMET_DEC_ABLATE & 2)) tmem_st32(tbase + ab * C::A_COLS + cb * 32 + lane_addr, o);
           }
         }
         if (lane == 0 && q == 0 && half == 0) trace_ev(P, 13, seq);   // stores issued
@@ -537,25 +496,36 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
     const int ptid = threadIdx.x - kPromoWarp0 * 32;
     int sx = 0, accs = 0;
     uint32_t xph = 0, accph = 0;
+    // Epilogue operands (s_w[n]; corr[m], the offset-binary correction of the owner segment) are
+    // loaded ONE ITEM AHEAD into registers and first used at the next item: a global load
+    // consumed at the start of an item stalls these warps for the load's latency -- microseconds
+    // once the weight stream saturates HBM -- and with them the MMA and the whole stream.
+    constexpr bool kEarlyCorr = NT <= 32 && !GS; // registers: NT > 32 loads corr at the end
+    float sw_nx = 0.f, cr_nx[kEarlyCorr ? NT : 1];
+    auto prefetch_epi = [&](int it2) {
+      if (it2 >= it_end) return;
+      const WorkItem w2 = item(it2);
+      const int64_t n2 = (int64_t)(w2.tile / P.n_m_tiles) * kTileW + row;
+      const int64_t m2 = (int64_t)(w2.tile % P.n_m_tiles) * NT;
+      if (!GS) sw_nx = ldg_nc_f32(P.w_scales + min(n2, P.N - 1));
+      if constexpr (kEarlyCorr) {
+#pragma unroll
+        for (int j = 0; j < NT; ++j) cr_nx[j] = ldg_nc_f32(P.corr + min(m2 + j, P.Mp - 1));
+      }
+    };
+    prefetch_epi(it_begin);
     for (int it = it_begin; it < it_end; ++it) {
-      const WorkItem w = load_item(P, it, debug);
+      const WorkItem w = item(it);
       const int n_tile = w.tile / P.n_m_tiles, m_tile = w.tile % P.n_m_tiles;
       const int m0 = m_tile * NT, n0 = n_tile * kTileW;
       const bool owner = (w.flags & 2) != 0;
       const bool split = (w.flags & 1) != 0;
       const int n = n0 + row;
-      // epilogue operands loaded now (their latency overlaps the K loop): s_w[n] and, for the
-      // owner, corr[m] (the offset-binary weight correction, applied once at the end)
-      const float swv = GS ? 512.f : (n < P.N ? __ldg(P.w_scales + n) * 512.f : 0.f);
-      constexpr bool kEarlyCorr = NT <= 32 && !GS; // registers: NT > 32 loads corr at the end
+      const float sw_raw = sw_nx;
       float cr[kEarlyCorr ? NT : 1];
-      if constexpr (kEarlyCorr) {
 #pragma unroll
-        for (int j = 0; j < NT; ++j) {
-          const int64_t m = m0 + j;
-          cr[j] = (owner && m < P.Mp) ? __ldg(P.corr + m) * 0.001953125f : 0.f;   // 2^-9
-        }
-      }
+      for (int j = 0; j < (kEarlyCorr ? NT : 1); ++j) cr[j] = cr_nx[j];
+      prefetch_epi(it + 1);
       float acc[NT];
       int32_t dacc[DEBUG ? NT : 1];
 #pragma unroll
@@ -663,60 +633,40 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
       }
       // ---------------------------------------------------------------- epilogue
       if (ptid == 0) trace_ev(P, 10, it - it_begin);
+      // the offset-binary correction -corr * 2^-9 belongs to the tile once: the owner segment
+      // (K-block 0) folds it into its own sum
+      const float swv = GS ? 512.f : (n < P.N ? sw_raw * 512.f : 0.f);
+      if (!GS && owner) {
+#pragma unroll
+        for (int j = 0; j < NT; ++j) {
+          if constexpr (kEarlyCorr) acc[j] -= (m0 + j < P.Mp) ? cr[j] * 0.001953125f : 0.f;   // 2^-9
+          else acc[j] -= (m0 + j < P.Mp) ? __ldg(P.corr + m0 + j) * 0.001953125f : 0.f;
+        }
+      }
       if (split) {
+        // Stream-K fix-up off the pipeline: every segment of a split tile stores its
+        // partial, already scaled by s_w (the owner's with the offset correction folded in),
+        // into slot [fix][seg] -- only the tile's real token columns -- and moves on.  No fence,
+        // atomic or wait: under a saturated HBM stream each gpu-scope round trip costs
+        // microseconds and stalled this CTA's whole pipeline (tools/trace_dec.py).  The slots
+        // are summed in segment order (deterministic) by k_fixup, a programmatic dependent launch
+        // that starts when this grid has completed.
         const int seg = (w.flags >> 8) & 0xFF;
-        const int nseg = (w.flags >> 16) & 0xFF;
-        const int64_t part_tile = (int64_t)NT * kTileW;
-        if (!owner) {
-          float4* dst = reinterpret_cast<float4*>(
-              P.ws_part + ((int64_t)w.fix * (P.max_seg - 1) + (seg - 1)) * part_tile);
+        const int64_t part4 = (int64_t)NT * kTileW / 4;
+        const int nq = (int)((min((int64_t)NT, P.M - m0) + 3) / 4);   // float4 token groups stored
+        float4* slot = reinterpret_cast<float4*>(P.ws_part) + ((int64_t)w.fix * P.max_seg + seg) * part4 + ptid;
 #pragma unroll
-          for (int j = 0; j < NT; j += 4) dst[(j / 4) * 128 + ptid] = make_float4(acc[j], acc[j + 1], acc[j + 2], acc[j + 3]);
-          // the 128 threads' partial stores, ordered by the CTA barrier, are published by one
-          // thread's gpu-scope release (cumulative)
-          named_bar_sync(1, 128);
-          if (ptid == 0) {
-            fence_acq_rel_gpu();
-            st_release_gpu(P.ws_flags + (int64_t)w.fix * P.max_seg + seg, P.epoch);
-          }
-          if (ptid == 0) trace_ev(P, 12, it - it_begin);
-          continue;
-        }
-        if (ptid == 0) {
-          for (int sgi = 1; sgi < nseg; ++sgi) {
-            const uint32_t* f = P.ws_flags + (int64_t)w.fix * P.max_seg + sgi;
-            uint64_t t0g = globaltimer_ns();
-            while (ld_acquire_gpu(f) != P.epoch) {
-              if (globaltimer_ns() - t0g > COMET_MBAR_TIMEOUT_NS) {
-                __trap();
-              }
-            }
-          }
-        }
-        named_bar_sync(1, 128);
-        if (ptid == 0) trace_ev(P, 11, it - it_begin);
-        for (int sgi = 1; sgi < nseg; ++sgi) {
-          const float4* src = reinterpret_cast<const float4*>(
-              P.ws_part + ((int64_t)w.fix * (P.max_seg - 1) + (sgi - 1)) * part_tile);
-#pragma unroll
-          for (int j = 0; j < NT; j += 4) {
-            float4 t4;
-            asm volatile("ld.global.cg.v4.f32 {%0,%1,%2,%3}, [%4];"
-                         : "=f"(t4.x), "=f"(t4.y), "=f"(t4.z), "=f"(t4.w) : "l"(src + (j / 4) * 128 + ptid));
-            acc[j] += t4.x; acc[j + 1] += t4.y; acc[j + 2] += t4.z; acc[j + 3] += t4.w;
-          }
-        }
+        for (int j = 0; j < NT; j += 4)
+          if (j / 4 < nq) slot[(j / 4) * 128] = make_float4(acc[j] * swv, acc[j + 1] * swv, acc[j + 2] * swv, acc[j + 3] * swv);
+        if (ptid == 0) trace_ev(P, 12, it - it_begin);
+        continue;
       }
       if (n < P.N) {
 #pragma unroll
         for (int j = 0; j < NT; ++j) {
           const int64_t m = m0 + j;
           if (m < P.M) {
-            float c0;
-            if constexpr (GS) c0 = 0.f;                // the offset term was removed per block
-            else if constexpr (kEarlyCorr) c0 = cr[j];
-            else c0 = owner ? __ldg(P.corr + m) * 0.001953125f : 0.f;
-            const float yv = (acc[j] - c0) * swv;
+            const float yv = acc[j] * swv;
             const int64_t off = m * P.ldy + n;
             if (P.ydt == COMET_F16) reinterpret_cast<__half*>(P.y)[off] = __float2half_rn(yv);
             else if (P.ydt == COMET_BF16) reinterpret_cast<__nv_bfloat16*>(P.y)[off] = __float2bfloat16_rn(yv);
@@ -731,8 +681,64 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
 
   tc_fence_before();
   __syncthreads();
+  // the fix-up kernel (programmatic dependent) may launch once every CTA got here; its
+  // griddepcontrol.wait still waits for this grid's completion and memory flush
+  asm volatile("griddepcontrol.launch_dependents;");
   if (tracing && threadIdx.x == 0) P.trace[32768 + blockIdx.x * 4 + 2] = globaltimer_ns();
   if (warp == 2) tmem_dealloc<512>(tbase);
+}
+
+// Stream-K fix-up of the decode kernel's split tiles: one CTA per split tile, thread = weight
+// row; y[m, n] = sum over the tile's segments (in segment order) of the s_w-scaled partials.
+template <int NT>
+__global__ void __launch_bounds__(128) k_fixup(const __grid_constant__ GemmParams P, const int2* __restrict__ fix_info) {
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  const int2 fi = fix_info[blockIdx.x];                 // {tile, segments}
+  const int m0 = (fi.x % P.n_m_tiles) * NT, n0 = (fi.x / P.n_m_tiles) * kTileW;
+  const int64_t n = n0 + threadIdx.x;
+  const int64_t part4 = (int64_t)NT * kTileW / 4;
+  const int nq = (int)((min((int64_t)NT, P.M - m0) + 3) / 4);
+  const float4* slots = reinterpret_cast<const float4*>(P.ws_part) + (int64_t)blockIdx.x * P.max_seg * part4 + threadIdx.x;
+  float4 acc[NT / 4];
+#pragma unroll
+  for (int j = 0; j < NT / 4; ++j) acc[j] = make_float4(0.f, 0.f, 0.f, 0.f);
+  for (int sg = 0; sg < fi.y; ++sg) {
+#pragma unroll
+    for (int j = 0; j < NT / 4; ++j) {
+      if (j >= nq) break;
+      const float4 t = __ldcg(slots + sg * part4 + j * 128);
+      acc[j].x += t.x; acc[j].y += t.y; acc[j].z += t.z; acc[j].w += t.w;
+    }
+  }
+  if (n >= P.N) return;
+#pragma unroll
+  for (int j = 0; j < NT / 4; ++j) {
+    const float v[4] = {acc[j].x, acc[j].y, acc[j].z, acc[j].w};
+#pragma unroll
+    for (int t = 0; t < 4; ++t) {
+      const int64_t m = m0 + 4 * j + t;
+      if (j >= nq || m >= P.M) continue;
+      const int64_t off = m * P.ldy + n;
+      if (P.ydt == COMET_F16) reinterpret_cast<__half*>(P.y)[off] = __float2half_rn(v[t]);
+      else if (P.ydt == COMET_BF16) reinterpret_cast<__nv_bfloat16*>(P.y)[off] = __float2bfloat16_rn(v[t]);
+      else reinterpret_cast<float*>(P.y)[off] = v[t];
+    }
+  }
+}
+
+template <int NT>
+cudaError_t launch_fixup(const GemmParams& prm, const int2* fix_info, int n_fix, cudaStream_t stream) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)n_fix);
+  cfg.blockDim = dim3(128);
+  cfg.dynamicSmemBytes = 0;
+  cfg.stream = stream;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, k_fixup<NT>, prm, fix_info);
 }
 
 template <int NT, int DEBUG, bool GS = false>
@@ -997,6 +1003,19 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
   }
   if (e != cudaSuccess) return cuda_status(e, "w4ax gemm launch");
   *launches = 1;
+  if (!normal && !dbg && p.n_split_tiles > 0) {
+    // the decode kernel's split tiles are summed by the fix-up kernel
+    const int2* fi = reinterpret_cast<const int2*>(p.d_fix);
+    const int nf = (int)p.n_split_tiles;
+    switch (tile_m) {
+      case 16: e = launch_fixup<16>(prm, fi, nf, stream); break;
+      case 32: e = launch_fixup<32>(prm, fi, nf, stream); break;
+      case 64: e = launch_fixup<64>(prm, fi, nf, stream); break;
+      default: e = launch_fixup<128>(prm, fi, nf, stream); break;
+    }
+    if (e != cudaSuccess) return cuda_status(e, "fix-up launch");
+    *launches = 2;
+  }
   return COMET_OK;
 }
 

@@ -55,6 +55,34 @@ __device__ __forceinline__ void widen_int4(uint32_t pv, uint32_t& lo, uint32_t& 
   hi = (pv >> 4) & 0x0F0F0F0Fu;
 }
 __device__ __forceinline__ uint32_t int4_to_int8(uint32_t u4) { return (u4 << 4) ^ 0x80808080u; }
+// One K-block row of a weight (64 packed bytes = 4 x uint4) -> 128 widened bytes (32 words) in
+// channel order.  The block kind is a template parameter: the caller branches once per K-block
+// (warp-uniform), so an INT4 block costs exactly the 3 instructions per 8 values of widen_int4
+// (a runtime flag inside the loop gets if-converted: both forms computed and selected per word).
+template <bool IS8>
+__device__ __forceinline__ void widen_kblock_row(const uint4* c, uint32_t (&o)[32]) {
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    const uint32_t pw[4] = {c[j].x, c[j].y, c[j].z, c[j].w};
+#pragma unroll
+    for (int e = 0; e < 4; ++e) {
+      const int g = 2 * (j * 4 + e);
+      widen_int4(pw[e], o[g], o[g + 1]);
+      if (IS8) {
+        o[g] = int4_to_int8(o[g]);
+        o[g + 1] = int4_to_int8(o[g + 1]);
+      }
+    }
+  }
+}
+
+// A global load the compiler keeps where it is written (volatile) and whose result is consumed
+// only where the caller first uses it: for operands prefetched a work item ahead.
+__device__ __forceinline__ float ldg_nc_f32(const float* p) {
+  float v;
+  asm volatile("ld.global.nc.f32 %0, [%1];" : "=f"(v) : "l"(p));
+  return v;
+}
 
 __device__ __forceinline__ void named_bar_sync(int id, int n) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");

@@ -654,6 +654,7 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
                 __trap();
               }
             }
+            *const_cast<uint32_t*>(f) = 0u;   // consumed: every launch leaves the flags zeroed
           }
         }
         named_bar_sync(1, 128 * C::NPW);

@@ -52,6 +52,8 @@ struct Plan {
   // device copies
   int32_t* d_cta_begin = nullptr;
   WorkItem* d_items = nullptr;
+  std::vector<int32_t> fix_info;        // [n_split_tiles][2] = {tile, segments} (fix order)
+  int32_t* d_fix = nullptr;
   size_t ws_bytes = 0;                  // stream-K partials + flags
   size_t ws_flags_off = 0;
   int device = -1;

@@ -225,6 +225,7 @@ comet_status_t build_plan(Plan& p, const comet_sched_config& cfg) {
   p.n_split_tiles = 0;
   p.max_segments = 1;
   int32_t fix = 0;
+  p.fix_info.clear();
   for (auto& [tile, segs] : by_tile) {
     std::sort(segs.begin(), segs.end(), [&](const SegRef& a, const SegRef& b) {
       return runs[a.cta][a.idx].kb0 < runs[b.cta][b.idx].kb0;
@@ -241,7 +242,11 @@ comet_status_t build_plan(Plan& p, const comet_sched_config& cfg) {
       w.fix = split ? fix : -1;
       per[segs[s].cta][segs[s].idx] = w;
     }
-    if (split) ++fix;
+    if (split) {
+      p.fix_info.push_back((int32_t)tile);
+      p.fix_info.push_back(nseg);
+      ++fix;
+    }
   }
   p.cta_begin.assign(P + 1, 0);
   p.items.clear();
@@ -255,7 +260,10 @@ comet_status_t build_plan(Plan& p, const comet_sched_config& cfg) {
   p.max_cost = *std::max_element(load.begin(), load.end());
   p.mean_cost = std::accumulate(load.begin(), load.end(), 0.0) / P;
   const size_t part = (size_t)p.tile_n * p.tile_w * sizeof(float);
-  const size_t n_part = (size_t)p.n_split_tiles * (size_t)(p.max_segments - 1);
+  // partial slots: [split tile][segment] (the decode kernel stores every segment's partial and
+  // the last arriver sums them; the prefill kernel uses slots 1.. for the non-owner segments);
+  // flags / arrival counters after them
+  const size_t n_part = (size_t)p.n_split_tiles * (size_t)p.max_segments;
   p.ws_flags_off = n_part * part;
   p.ws_bytes = p.n_split_tiles ? p.ws_flags_off + (size_t)p.n_split_tiles * p.max_segments * 2 * sizeof(uint32_t) : 0;
   p.ws_bytes = (p.ws_bytes + 255) / 256 * 256;

@@ -19,7 +19,8 @@ from paper_conf_asplos_liu0rxpwl0w25_b200 import synth  # noqa: E402
 
 M = int(sys.argv[1]) if len(sys.argv) > 1 else 1
 layer = sys.argv[2] if len(sys.argv) > 2 else "gate_up"
-K, N = {"gate_up": (8192, 28672), "down": (28672, 8192), "qkv": (8192, 10240)}[layer]
+K, N = {"gate_up": (8192, 28672), "down": (28672, 8192), "qkv": (8192, 10240),
+        "l2_qkvo": (4096, 4096), "l2_gate_up": (4096, 11008), "l2_down": (11008, 4096)}[layer]
 rng = np.random.default_rng(0)
 tags = synth.make_tags(K, 0.05, rng)
 x = torch.randn(M, K, device="cuda", dtype=torch.float16)
@@ -46,6 +47,13 @@ info = plan.info()
 print("plan", {k: info[k] for k in ("tile_n", "num_ctas", "split_mode", "n_tiles", "n_items", "n_split_tiles")})
 g = b[32768:32768 + 4 * info["num_ctas"]].reshape(-1, 4)
 t0 = g[:, 0].min()
+ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+flush.fill_(9)
+ev0.record()
+cb.w4ax_gemm(plan, act, sc, wp, sw, out=y)
+ev1.record()
+torch.cuda.synchronize()
+print("event time (us, trace build)", round(ev0.elapsed_time(ev1) * 1e3, 2))
 print("CTA start  (us) min/med/max", *(np.round(np.percentile(g[:, 0] - t0, [0, 50, 100]) / 1e3, 2)))
 print("CTA setup  (us) min/med/max", *(np.round(np.percentile(g[:, 1] - t0, [0, 50, 100]) / 1e3, 2)))
 print("CTA end    (us) min/med/max", *(np.round(np.percentile(g[:, 2] - t0, [0, 50, 100]) / 1e3, 2)))
@@ -93,3 +101,14 @@ for cta in (0, 1):
     ep = [(t[10][i] - base, t[11][i] - base if t[11][i] else -1, t[12][i] - base) for i in range(8) if t[10][i]]
     print("epilogues (start, partials ready, done):", ep)
     print("end of last promotion", p_done[-1] if n_st else None)
+
+# detailed timeline of CTA 1 around its item boundaries: per stage, each role's timestamps
+t = b[:32768].reshape(2, 16, 1024)[1]
+base = t[0][0]
+n_st = int((t[0] > 0).sum())
+print("stage | W-issued widenStart widenDone MMAgo MMAdone promoGo promoDone")
+for i in range(n_st):
+    def g(e, k):
+        return int(t[e][k] - base) if t[e][k] else -1
+    print(f"{i:3d} | {g(0, i):7d} {min(g(3, i), g(4, i)):7d} {max(g(5, i), g(6, i)):7d} {g(1, i):7d} {g(2, i):7d} {g(7, i):7d} {g(8, i):7d}")
+print("epilogue start/last/done per item:", [(int(t[10][i] - base), int(t[11][i] - base) if t[11][i] else -1, int(t[12][i] - base)) for i in range(6) if t[10][i]])
