@@ -40,6 +40,9 @@
 #ifndef COMET_PROMO_SB
 #define COMET_PROMO_SB 1    // single-buffered 32-column promotion batches when they fit
 #endif
+#ifndef COMET_PROMO_W64
+#define COMET_PROMO_W64 1   // 64-column TMEM load rounds in the promotion when the registers allow
+#endif
 #ifndef COMET_WIDEN40
 #define COMET_WIDEN40 1     // widen warpgroups at 40 registers when promotion still fits
 #endif
@@ -53,7 +56,7 @@
 #define COMET_N256_NPW 2   // promotion warpgroups of the 256-wide tile
 #endif
 #ifndef COMET_N256_NWG
-#define COMET_N256_NWG 2   // widen warpgroups of the 256-wide tile
+#define COMET_N256_NWG 1   // widen warpgroups of the 256-wide tile (1: its registers go to promotion)
 #endif
 
 namespace comet {
@@ -103,8 +106,11 @@ struct CfgN {
   static constexpr int REG_PROMO = promo_regs2(REG_LOW, REG_WIDEN);
   // SB: single-buffered 32-column batches (fewer, larger TMEM loads in flight) when the
   // double-buffered 32-column form does not fit (variant experiments: COMET_PROMO_SB)
-  static constexpr bool SB = TIGHT || (!LOADALL && COMET_PROMO_SB && REG_PROMO < ACC_REGS + 2 * 32 + 24 &&
-                             REG_PROMO >= ACC_REGS + 32 + 24 && COLS % 32 == 0);
+  // W64: the accumulator leaves TMEM in 64-column rounds (two 32-column loads in flight, one
+  // wait) -- half the load round trips of 32-column batches before the buffer is released
+  static constexpr bool W64 = !LOADALL && !TIGHT && COLS % 64 == 0 && REG_PROMO >= ACC_REGS + 64 + 24 && COMET_PROMO_W64;
+  static constexpr bool SB = !W64 && (TIGHT || (!LOADALL && COMET_PROMO_SB && REG_PROMO < ACC_REGS + 2 * 32 + 24 &&
+                             REG_PROMO >= ACC_REGS + 32 + 24 && COLS % 32 == 0));
   static constexpr int PB = TIGHT ? 16 : LOADALL ? COLS
                           : ((SB || (REG_PROMO >= ACC_REGS + 2 * 32 + 24 && COLS % 32 == 0)) ? 32 : 16);
   static constexpr int NACC_TMEM = 512 / BN >= 4 ? 4 : 512 / BN;   // accumulators TMEM holds
@@ -525,6 +531,44 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
         // folded in; the accumulator is released once the last load has landed.
         constexpr int PB = C::PB;                         // columns per TMEM load batch
         constexpr int NB_ = COLS / PB;
+        if constexpr (C::W64) {
+          float s;
+          asm volatile("ld.shared.f32 %0, [%1];" : "=f"(s) : "r"(s_scale_r + 4u * BM * sc));
+          if (is8) s *= 1.220703125e-04f;                 // 2^-13: INT8 block acc = 16 sum x w
+          const float2 s2 = make_float2(s, s);
+#pragma unroll
+          for (int b = 0; b < COLS / 64; ++b) {
+            uint32_t v[64];
+            tmem_ld_32x32b<64>(taddr + b * 64, v);
+            tmem_wait_ld();
+            if (b == 0 && threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 9, tr);
+            if (b + 1 == COLS / 64) {
+              // every accumulator column of this thread is in registers: release the buffer
+              tc_fence_before();
+              __syncwarp();
+              if (lane == 0) mbar_arrive_cluster(ready_rel + rs * 8);
+              if (threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 10, tr);
+            }
+            if (is8) {
+#pragma unroll
+              for (int c = 0; c < 64; ++c) v[c] = __float_as_uint(__int2float_rn((int)v[c]));
+            }
+#pragma unroll
+            for (int c = 0; c < 64; c += 2) {
+              const int a = b * 64 + c;
+              float2 y = ffma2(make_float2(__uint_as_float(v[c]), __uint_as_float(v[c + 1])), s2,
+                               make_float2(acc[a], acc[a + 1]));
+              acc[a] = y.x;
+              acc[a + 1] = y.y;
+            }
+          }
+          if (threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 7, tr);
+          ++tr;
+          if (++accb == NACC) { accb = 0; accph ^= 1; }
+          if (++sc == SS) sc = 0;
+          if (++rs == S) rs = 0;
+          continue;
+        }
         if constexpr (C::SB) {
           // single-buffered batches: load, wait, fold; release after the last load landed
           float s;
