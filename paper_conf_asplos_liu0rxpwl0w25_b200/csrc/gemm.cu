@@ -283,24 +283,21 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
           const uint64_t b0 = sdesc_kmajor_sw128(sx0 + sx * C::X_STAGE);
           const uint32_t tg = lane < KS ? lds_u8(s_tags_a + kb + lane) : 0u;
           const uint32_t tagw = __ballot_sync(0xffffffffu, tg != 0);
-          for (int c = 0; c < nk; ++c) {
-            const uint32_t d = d0 + c * NT, a = a0 + c * 32;
-            const uint64_t bd = b0 + (uint64_t)((c * C::XKB_BYTES) >> 4);
-            if (COMET_DEC_ABLATE & 1) {
-            } else if ((tagw >> c) & 1u) {
-              if (elect_one()) {
+          // one elected thread issues the stage's MMAs AND its commits (tcgen05.commit tracks the
+          // issuing thread's MMAs only)
+          if (elect_one()) {
+            for (int c = 0; c < nk; ++c) {
+              const uint32_t d = d0 + c * NT, a = a0 + c * 32;
+              const uint64_t bd = b0 + (uint64_t)((c * C::XKB_BYTES) >> 4);
+              if (COMET_DEC_ABLATE & 1) {
+              } else if ((tagw >> c) & 1u) {
 #pragma unroll
                 for (int k = 0; k < 4; ++k) mma_i8_ts(d, a + 8 * k, bd + 2 * k, id_i8, k);
-              }
-            } else {
-              if (elect_one()) {
+              } else {
 #pragma unroll
                 for (int k = 0; k < 4; ++k) mma_f8_ts(d, a + 8 * k, bd + 2 * k, id_f8, k);
               }
             }
-            __syncwarp();
-          }
-          if (elect_one()) {
             tc_commit(&acc_full[accs]);
             tc_commit(&empty_x[sx]);
             tc_commit(&a_empty[ab]);

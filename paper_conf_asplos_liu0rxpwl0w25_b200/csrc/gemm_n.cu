@@ -32,7 +32,7 @@
 #define COMET_NSTAGE 2   // output staging buffers per promotion warpgroup (TMA-store epilogue)
 #endif
 #ifndef COMET_N_UNIFORM_MMA
-#define COMET_N_UNIFORM_MMA 0   // 1: MMA issue loop on the whole warp with uniform operands (intermittent launch failures under stream-K, tools/stress_gemm.py; no gain here)
+#define COMET_N_UNIFORM_MMA 1   // 1: MMA issue loop on the whole warp with uniform operands, one elected lane issues MMAs + commits
 #endif
 #ifndef COMET_PRODUCERS
 #define COMET_PRODUCERS 1   // TMA-issuing warps (2: K-blocks alternate between them)
@@ -294,27 +294,24 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
           const uint32_t sa = sx0 + s * C::SLOT_BYTES;
           const uint32_t sbv = sa + C::X_BYTES + h * (C::WROWS / NSUB) * 128;
           const bool is8 = __shfl_sync(0xffffffffu, lds_u8(s_tags_a + kb), 0) != 0;
-          if (diag_ablate(P) & 8) {
-            // diagnostic: no MMA
-          } else if (is8) {
-            if (elect_one()) {
+          // one elected thread issues the K-block's four MMAs AND its commits: tcgen05.commit
+          // tracks the MMAs of the issuing thread only, so both must come from the same lane
+          if (elect_one()) {
+            if (diag_ablate(P) & 8) {
+              // diagnostic: no MMA
+            } else if (is8) {
 #pragma unroll
               for (int k = 0; k < 4; ++k) {
                 const uint64_t ad = sdesc_kmajor_sw128(sa + 32 * k), bd = sdesc_kmajor_sw128(sbv + 32 * k);
                 if (CG == 2) mma_i8_ss_cg2(d, ad, bd, id_i8, k); else mma_i8_ss(d, ad, bd, id_i8, k);
               }
-            }
-          } else {
-            if (elect_one()) {
+            } else {
 #pragma unroll
               for (int k = 0; k < 4; ++k) {
                 const uint64_t ad = sdesc_kmajor_sw128(sa + 32 * k), bd = sdesc_kmajor_sw128(sbv + 32 * k);
                 if (CG == 2) mma_f8_ss_cg2(d, ad, bd, id_f8, k); else mma_f8_ss(d, ad, bd, id_f8, k);
               }
             }
-          }
-          __syncwarp();
-          if (elect_one()) {
             if (CG == 2) {
               tc_commit_mc(&acc_full[h * NACC + accb], 3);
               tc_commit_mc(&slot_free[s], 3);
