@@ -290,6 +290,34 @@ comet_status_t comet_w4ax_gemm_grouped(comet_plan_t plan, const void* act_packed
                                        void* workspace, size_t ws_bytes, void* stream);
 
 
+/* ------------------------------------------------------------------------------------------
+ * NEXT-2: the row-parallel layer's reduction fused into the GEMM epilogue (the
+ * paper lists "operator pipelining" as future work).  Under tensor parallelism a
+ * row-parallel layer (e.g. LLaMA down, K sharded over `world` ranks at 128-channel block
+ * boundaries, each rank quantising its own K shard) produces per-rank FP32 partials
+ * Y_r = X_r W_r^T that must be summed.  Instead of writing Y_r and running an all-reduce, the
+ * prefill pair kernel's epilogue stores every finished tile row m straight into the receive
+ * buffer of the rank that owns row m (owner = m / ms, ms = ceil(M / world)) -- peer memory
+ * over NVLink, so the transfer of one tile overlaps the MMAs of the next -- and the owner sums
+ * the `world` slots in rank order (deterministic): a reduce-scatter over token rows.
+ *
+ *   recv buffer of every rank: device [world][ms][N] float (comet_rs_recv_bytes bytes),
+ *     slot [src][m - owner * ms][n] = Y_src[m][n]; recv_bufs_host[i] = rank i's buffer as
+ *     mapped in this process (peer pointers, e.g. from torch symmetric memory).
+ *   comet_w4ax_gemm_rs  this rank's GEMM (plan orientation 3, else COMET_ERR_UNSUPPORTED_SHAPE;
+ *     arguments as comet_w4ax_gemm); writes its slot in every owner's buffer.
+ *   comet_rs_reduce     on the owner, after EVERY rank's comet_w4ax_gemm_rs has completed (the
+ *     caller orders them, e.g. a barrier across ranks): y[i][n] = sum_src recv[src][i][n] for
+ *     this rank's rows i < min(ms, M - rank * ms) (output rows rank * ms + i), into y [rows][ldy]
+ *     of ydt.  world in 1..8.
+ * ---------------------------------------------------------------------------------------- */
+size_t comet_rs_recv_bytes(int64_t M, int64_t N, int world);
+comet_status_t comet_w4ax_gemm_rs(comet_plan_t plan, const void* act_packed, const float* act_scales,
+                                  const void* w_packed, const float* w_scales, float* const* recv_bufs_host,
+                                  int world, int rank, void* workspace, size_t ws_bytes, void* stream);
+comet_status_t comet_rs_reduce(const float* recv_local, int world, int rank, int64_t M, int64_t N, void* y,
+                               comet_dtype_t ydt, int64_t ldy, void* stream);
+
 /*
  * Convenience: the whole hot path for one linear layer with HOST buffers (used for the
  * end-to-end measurement).  Copies x_host [M][K] (F16/BF16, pinned host memory for overlap) to

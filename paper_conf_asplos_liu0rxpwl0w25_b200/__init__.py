@@ -98,6 +98,9 @@ def lib():
         "comet_w4ax_linear_host_async": (I32, [P, P, I32, P, P, P, I32, P, SZ, P, SZ, P]),
         "comet_linear_host_wait": (I32, [P]),
         "comet_debug_widen": (I32, [ctypes.c_uint64, I64, I32, P, P]),
+        "comet_rs_recv_bytes": (SZ, [I64, I64, I32]),
+        "comet_w4ax_gemm_rs": (I32, [P, P, P, P, P, P, I32, I32, P, SZ, P]),
+        "comet_rs_reduce": (I32, [P, I32, I32, I64, I64, P, I32, I64, P]),
         "comet_status_string": (ctypes.c_char_p, [I32]),
         "comet_last_error": (ctypes.c_char_p, []),
         "comet_version": (ctypes.c_char_p, []),
@@ -375,6 +378,36 @@ def debug_widen(first_word: int, n: int, int8_block: bool = False, *, out=None, 
         out = torch.empty((n, 2), dtype=torch.int32, device="cuda")
     _check(lib().comet_debug_widen(first_word, n, 1 if int8_block else 0, ctypes.c_void_p(out.data_ptr()),
                                    _stream(stream)))
+    return out
+
+
+def rs_recv_bytes(M: int, N: int, world: int) -> int:
+    return int(lib().comet_rs_recv_bytes(M, N, world))
+
+
+def w4ax_gemm_rs(plan: Plan, act_packed, act_scales, w_packed, w_scales, recv_ptrs, rank: int, *, stream=None):
+    """comet_w4ax_gemm_rs (NEXT-2): this rank's row-parallel GEMM with the reduce-scatter fused
+    into the epilogue.  recv_ptrs: [world] device addresses (ints) of every rank's receive buffer
+    as mapped in this process (comet_rs_recv_bytes bytes each)."""
+    world = len(recv_ptrs)
+    arr = (ctypes.c_void_p * world)(*[ctypes.c_void_p(int(p)) for p in recv_ptrs])
+    ws = plan.workspace(act_packed.device)
+    _check(lib().comet_w4ax_gemm_rs(plan.handle, ctypes.c_void_p(act_packed.data_ptr()),
+                                    ctypes.c_void_p(act_scales.data_ptr()), ctypes.c_void_p(w_packed.data_ptr()),
+                                    ctypes.c_void_p(w_scales.data_ptr()), arr, world, rank,
+                                    ctypes.c_void_p(ws.data_ptr()), ws.numel(), _stream(stream)))
+
+
+def rs_reduce(recv_local, world: int, rank: int, M: int, N: int, *, out=None, out_dtype=None, stream=None):
+    """comet_rs_reduce (NEXT-2): the owner's sum of the world slots of its receive buffer ->
+    its rows of Y ([min(ms, M - rank*ms), N], ms = ceil(M / world))."""
+    import torch
+    ms = -(-M // world)
+    rows = max(0, min(ms, M - rank * ms))
+    if out is None:
+        out = torch.empty((rows, N), dtype=out_dtype or torch.float16, device=recv_local.device)
+    _check(lib().comet_rs_reduce(ctypes.c_void_p(recv_local.data_ptr()), world, rank, M, N,
+                                 ctypes.c_void_p(out.data_ptr()), _dt(out.dtype), out.stride(0), _stream(stream)))
     return out
 
 

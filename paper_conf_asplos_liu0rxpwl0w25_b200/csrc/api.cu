@@ -467,6 +467,67 @@ comet_status_t comet_w4ax_gemm_grouped(comet_plan_t plan, const void* act_packed
   return st;
 }
 
+static int64_t rs_rows_per_rank(int64_t M, int world) { return ceil_div(M, world); }
+
+size_t comet_rs_recv_bytes(int64_t M, int64_t N, int world) {
+  if (M < 1 || N < 1 || world < 1 || world > 8) return 0;
+  return (size_t)world * (size_t)rs_rows_per_rank(M, world) * (size_t)N * sizeof(float);
+}
+
+comet_status_t comet_w4ax_gemm_rs(comet_plan_t plan, const void* act_packed, const float* act_scales,
+                                  const void* w_packed, const float* w_scales, float* const* recv_bufs_host,
+                                  int world, int rank, void* workspace, size_t ws_bytes, void* stream) {
+  g_launches = 0;
+  if (!plan || !act_packed || !act_scales || !w_packed || !w_scales || !recv_bufs_host)
+    return fail(COMET_ERR_INVALID_ARG, "NULL pointer argument");
+  if (world < 1 || world > 8 || rank < 0 || rank >= world) return fail(COMET_ERR_INVALID_ARG, "world must be 1..8 and 0 <= rank < world");
+  Plan& p = plan->p;
+  if (p.orientation != 3 || p.tile_w != 256)
+    return fail(COMET_ERR_UNSUPPORTED_SHAPE, "the fused reduce-scatter runs on the 256-wide CTA-pair prefill kernel (plan orientation 3, tile_w 256)");
+  RsArgs rs{};
+  rs.world = world;
+  rs.rank = rank;
+  rs.ms = rs_rows_per_rank(p.M, world);
+  for (int i = 0; i < world; ++i) {
+    if (!recv_bufs_host[i]) return fail(COMET_ERR_INVALID_ARG, "NULL receive buffer");
+    if (!aligned16(recv_bufs_host[i])) return fail(COMET_ERR_MISALIGNED, "receive buffers must be 16-byte aligned");
+    rs.dst[i] = recv_bufs_host[i];
+  }
+  if ((reinterpret_cast<uintptr_t>(act_packed) & 255u) != 0) return fail(COMET_ERR_MISALIGNED, "act_packed must be 256-byte aligned");
+  if (!aligned16(act_scales) || !aligned16(w_packed) || !aligned16(w_scales) || (workspace && !aligned16(workspace)))
+    return fail(COMET_ERR_MISALIGNED, "device pointers must be 16-byte aligned");
+  comet_status_t st = check_device();
+  if (st != COMET_OK) return st;
+  int launches = 0;
+  // y is never written on this path (the epilogue stores to the receive buffers); the local
+  // receive buffer stands in for the output tensor map
+  st = launch_gemm(p, act_packed, act_scales, w_packed, w_scales, recv_bufs_host[rank], COMET_F32, p.N, nullptr,
+                   nullptr, workspace, ws_bytes, static_cast<cudaStream_t>(stream), &launches, false, &rs);
+  g_launches = launches;
+  return st;
+}
+
+comet_status_t comet_rs_reduce(const float* recv_local, int world, int rank, int64_t M, int64_t N, void* y,
+                               comet_dtype_t ydt, int64_t ldy, void* stream) {
+  g_launches = 0;
+  if (!recv_local || !y) return fail(COMET_ERR_INVALID_ARG, "NULL pointer argument");
+  if (world < 1 || world > 8 || rank < 0 || rank >= world) return fail(COMET_ERR_INVALID_ARG, "world must be 1..8 and 0 <= rank < world");
+  if (N % 4 != 0) return fail(COMET_ERR_UNSUPPORTED_SHAPE, "N must be a multiple of 4");
+  if (ydt != COMET_F16 && ydt != COMET_BF16 && ydt != COMET_F32) return fail(COMET_ERR_INVALID_ARG, "bad ydt");
+  const int esz = ydt == COMET_F32 ? 4 : 2;
+  if (ldy < N || (ldy * esz) % 16 != 0) return fail(COMET_ERR_MISALIGNED, "ldy must be >= N with ldy*sizeof(y) % 16 == 0");
+  if (!aligned16(recv_local) || !aligned16(y)) return fail(COMET_ERR_MISALIGNED, "device pointers must be 16-byte aligned");
+  const int64_t ms = rs_rows_per_rank(M, world);
+  const int64_t rows = std::max<int64_t>(0, std::min<int64_t>(ms, M - (int64_t)rank * ms));
+  comet_status_t st = check_device();
+  if (st != COMET_OK) return st;
+  // the slots of the source ranks are [src][ms][N]; this rank owns `rows` of them
+  cudaError_t e = launch_rs_reduce(recv_local, world, rows, ms, N, y, (int)ydt, ldy, static_cast<cudaStream_t>(stream));
+  if (e != cudaSuccess) return cuda_status(e, "reduce launch");
+  g_launches = 1;
+  return COMET_OK;
+}
+
 // Pipelined host path: chunks of kLinChunk token rows once M >= 2 kLinChunk.
 static constexpr int64_t kLinChunk = 1024;
 

@@ -871,7 +871,7 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
                            const void* w_packed, const float* w_scales, void* y,
                            comet_dtype_t ydt, int64_t ldy, int32_t* debug_acc,
                            int32_t* debug_acc_blocks, void* workspace, size_t ws_bytes,
-                           cudaStream_t stream, int* launches, bool grouped) {
+                           cudaStream_t stream, int* launches, bool grouped, const RsArgs* rs) {
   using namespace gemm;
   if (grouped && p.orientation != 1)
     return fail(COMET_ERR_UNSUPPORTED_SHAPE, "group-wise weight scales need a plan with orientation 1 (weights on the MMA M side)");
@@ -951,6 +951,12 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
   prm.nb = (int)p.nb;
   prm.ydt = (int)ydt;
   prm.tags = p.mask;
+  if (rs) {
+    prm.rs_world = rs->world;
+    prm.rs_rank = rs->rank;
+    prm.rs_ms = rs->ms;
+    for (int i = 0; i < 8; ++i) prm.rs_dst[i] = i < rs->world ? rs->dst[i] : nullptr;
+  }
   {
     const char* ab = getenv("COMET_ABLATE");
     prm.ablate = ab ? atoi(ab) : 0;
@@ -1014,6 +1020,41 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
     *launches = 2;
   }
   return COMET_OK;
+}
+
+// NEXT-2: the owner's side of the fused reduce-scatter -- y[m][n] = sum over source ranks, in rank
+// order (deterministic), of recv[src][m][n]; FP32 in, F16 / BF16 / F32 out.  HBM-bound.
+__global__ void __launch_bounds__(256) k_rs_reduce(const float4* __restrict__ recv, int world, int64_t rows,
+                                                   int64_t ms, int64_t N, void* y, int ydt, int64_t ldy) {
+  const int64_t n4 = N / 4, total = rows * n4, plane = ms * n4;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    float4 acc = __ldcs(recv + i);
+    for (int s = 1; s < world; ++s) {
+      const float4 t = __ldcs(recv + s * plane + i);
+      acc.x += t.x; acc.y += t.y; acc.z += t.z; acc.w += t.w;
+    }
+    const int64_t m = i / n4, n = (i - m * n4) * 4;
+    if (ydt == COMET_F32) {
+      *reinterpret_cast<float4*>(reinterpret_cast<float*>(y) + m * ldy + n) = acc;
+    } else if (ydt == COMET_BF16) {
+      __nv_bfloat162 a = __floats2bfloat162_rn(acc.x, acc.y), b = __floats2bfloat162_rn(acc.z, acc.w);
+      *reinterpret_cast<uint2*>(reinterpret_cast<__nv_bfloat16*>(y) + m * ldy + n) =
+          make_uint2(*reinterpret_cast<uint32_t*>(&a), *reinterpret_cast<uint32_t*>(&b));
+    } else {
+      __half2 a = __floats2half2_rn(acc.x, acc.y), b = __floats2half2_rn(acc.z, acc.w);
+      *reinterpret_cast<uint2*>(reinterpret_cast<__half*>(y) + m * ldy + n) =
+          make_uint2(*reinterpret_cast<uint32_t*>(&a), *reinterpret_cast<uint32_t*>(&b));
+    }
+  }
+}
+
+cudaError_t launch_rs_reduce(const float* recv, int world, int64_t rows, int64_t ms, int64_t N, void* y, int ydt,
+                             int64_t ldy, cudaStream_t stream) {
+  const int64_t total = rows * (N / 4);
+  if (total == 0) return cudaSuccess;
+  const int64_t blocks = std::min<int64_t>((total + 255) / 256, 148 * 8);
+  k_rs_reduce<<<(unsigned)blocks, 256, 0, stream>>>(reinterpret_cast<const float4*>(recv), world, rows, ms, N, y, ydt, ldy);
+  return cudaGetLastError();
 }
 
 }  // namespace comet

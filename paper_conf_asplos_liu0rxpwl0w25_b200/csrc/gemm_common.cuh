@@ -40,6 +40,12 @@ struct __align__(64) GemmParams {
   unsigned long long* trace;  // diagnostic only (comet_debug_set_trace): [cta<2][event<8][kb<1024] clock64
   int ablate;                // diagnostic only (env COMET_ABLATE): 4 skip widening, 8 skip MMAs
                              // (prefill kernel); the output is invalid under it
+  // NEXT-2 fused reduce-scatter (prefill pair kernel): when rs_world > 0 the epilogue stores
+  // this rank's FP32 partial of output row m straight into the receive buffer of the rank that
+  // owns row m (P2P over NVLink; owner = m / rs_ms), slot [rs_rank][m - owner * rs_ms][N]
+  int rs_world, rs_rank;
+  int64_t rs_ms;
+  float* rs_dst[8];
   TagMask tags;
 };
 

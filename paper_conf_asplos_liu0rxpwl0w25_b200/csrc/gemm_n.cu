@@ -167,7 +167,7 @@ struct CfgN {
 // kb only after slot_free[s] for kb - S; the scales of kb have landed when acc_full(kb) fires
 // (MMA(kb) waited mma_ready(kb) which waited widen(kb) which waited full[s]); the producer may
 // reuse scale slot kb % (S+NACC) because slot_free(kb-S) => MMA(kb-S) => promotion(kb-S-NACC).
-template <int BN, int CG, int NPW, int NWG, int DEBUG>
+template <int BN, int CG, int NPW, int NWG, int DEBUG, bool RS = false>
 __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w4ax_n(const __grid_constant__ GemmParams P) {
   using C = CfgN<BN, CG, NPW, NWG, DEBUG>;
   constexpr int kThreadsN = C::THREADS;
@@ -728,6 +728,26 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
             }
           }
         }
+      } else if constexpr (RS) {
+        // NEXT-2: the row-parallel layer's reduce-scatter fused into the epilogue (P:L373
+        // "operator pipelining"): this rank's FP32 partial y_r = (acc - corr 2^-9) s_w 2^9 of row m
+        // goes straight to the owner of row m over NVLink -- the transfer of tile t overlaps the
+        // MMAs of tile t+1 -- and comet_rs_reduce sums the ranks' slots there in rank order.
+        named_bar_sync(1, 128 * C::NPW);                  // this tile's w_scales are in smem
+        const float* sw = sWs + tp * BN + wg * COLS;
+        if (m < P.M) {
+          const int owner = (int)(m / P.rs_ms);
+          const int64_t ml = m - (int64_t)owner * P.rs_ms;
+          float* dst = P.rs_dst[owner] + ((int64_t)P.rs_rank * P.rs_ms + ml) * P.N + n0;
+#pragma unroll
+          for (int c = 0; c < COLS; c += 4) {
+            const int64_t nc = col_n(wg, c);              // 4 consecutive columns from here
+            if (n0 + nc >= P.N) continue;
+            const float4 v = make_float4((acc[c] + init) * sw[c], (acc[c + 1] + init) * sw[c + 1],
+                                         (acc[c + 2] + init) * sw[c + 2], (acc[c + 3] + init) * sw[c + 3]);
+            asm volatile("st.global.v4.f32 [%0], {%1,%2,%3,%4};" ::"l"(dst + nc), "f"(v.x), "f"(v.y), "f"(v.z), "f"(v.w) : "memory");
+          }
+        }
       } else {
         // TMA-store epilogue.  y = (acc - corr 2^-9) * s_w * 512 (R7).  The
         // WG's COLS columns leave in chunks of 64 bytes per row (32 half / 16 float columns),
@@ -857,11 +877,11 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
   }
 }
 
-template <int BN, int CG, int NPW, int NWG, int DEBUG>
+template <int BN, int CG, int NPW, int NWG, int DEBUG, bool RS = false>
 cudaError_t launch_bn(const GemmParams& prm, int grid, cudaStream_t stream) {
   using C = CfgN<BN, CG, NPW, NWG, DEBUG>;
   static std::atomic<uint64_t> attr_done{0};
-  cudaError_t ea = set_smem_attr(k_w4ax_n<BN, CG, NPW, NWG, DEBUG>, C::SMEM_BYTES, attr_done);
+  cudaError_t ea = set_smem_attr(k_w4ax_n<BN, CG, NPW, NWG, DEBUG, RS>, C::SMEM_BYTES, attr_done);
   if (ea != cudaSuccess) return ea;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)grid);
@@ -875,7 +895,7 @@ cudaError_t launch_bn(const GemmParams& prm, int grid, cudaStream_t stream) {
   attr[0].val.clusterDim.z = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  return cudaLaunchKernelEx(&cfg, k_w4ax_n<BN, CG, NPW, NWG, DEBUG>, prm);
+  return cudaLaunchKernelEx(&cfg, k_w4ax_n<BN, CG, NPW, NWG, DEBUG, RS>, prm);
 }
 
 // Persistent units (CTAs, or CTA pairs for CG = 2) of this kernel that can be resident at once.
@@ -934,6 +954,11 @@ int max_units_gemm_n(int bn, int cg, int sms) {
 
 // bn = 128, 160, 192 or 256; 96 for the debug-accumulator kernels (they need the registers).
 cudaError_t launch_gemm_n(const GemmParams& prm, int grid, int bn, int cg, int debug, cudaStream_t stream) {
+  if (prm.rs_world > 0) {
+    // NEXT-2 fused reduce-scatter: the 256-wide pair kernel with the peer-store epilogue
+    if (cg != 2 || bn != 256 || debug) return cudaErrorInvalidValue;
+    return launch_bn<256, 2, COMET_N256_NPW, COMET_N256_NWG, 0, true>(prm, grid, stream);
+  }
   if (cg == 2) {
     if (debug == 2) return launch_bn<96, 2, 3, 2, 2>(prm, grid, stream);
     if (debug == 1) return launch_bn<96, 2, 3, 2, 1>(prm, grid, stream);

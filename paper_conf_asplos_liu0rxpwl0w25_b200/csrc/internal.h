@@ -89,11 +89,19 @@ cudaError_t launch_kv4_dequantize(const uint8_t* codes, const float* scales, con
 cudaError_t launch_pack_weight(const int8_t* w, int64_t N, int64_t K, void* w_packed,
                                cudaStream_t stream);
 // gemm.cu
+struct RsArgs {            // NEXT-2 fused reduce-scatter of the row-parallel layer
+  int world, rank;
+  int64_t ms;              // output rows per owner rank
+  float* dst[8];           // every rank's receive buffer [world][ms][N] (peer-mapped pointers)
+};
 comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_scales,
                            const void* w_packed, const float* w_scales, void* y,
                            comet_dtype_t ydt, int64_t ldy, int32_t* debug_acc,
                            int32_t* debug_acc_blocks, void* workspace, size_t ws_bytes,
-                           cudaStream_t stream, int* launches, bool grouped = false);
+                           cudaStream_t stream, int* launches, bool grouped = false,
+                           const RsArgs* rs = nullptr);
+cudaError_t launch_rs_reduce(const float* recv, int world, int64_t rows, int64_t ms, int64_t N, void* y, int ydt,
+                             int64_t ldy, cudaStream_t stream);
 int max_coresident_units(const Plan& p, int sms);
 int gemm_stages(const Plan& p);
 namespace gemm {
