@@ -693,6 +693,10 @@ def run_comet(args, rank, world, local_rank):
                "path": "comet_w4ax_linear_host_async x3 + sync (C ABI, pinned host buffers, 1024-row chunk pipeline)" if world == 1 else
                        "public API: H2D copy + quantize_act + w4ax_gemm (+ NCCL all_reduce) + D2H copy"}
 
+    # ---- NEXT-2 at N > 1: the row-parallel layer with its reduction fused into the GEMM epilogue
+    # (peer stores into symmetric-memory receive buffers + owner reduction) against GEMM + NCCL
+    fused = fused_rs_compare(cb, torch, dist, dev, layers, rank, world, args.steps) if world > 1 else None
+
     cpu = cpu_baseline_sample(args.cpu_budget) if (rank == 0 and world == 1 and args.cpu_budget > 0) else None
     timer = Timer(torch, dev) if (args.decode or args.configs) else None
     # config 5 runs at every N (sharded like the headline); the N = 1-only sweeps after it
@@ -732,10 +736,69 @@ def run_comet(args, rank, world, local_rank):
             # and the row-parallel all-reduce, reported separately
             line["per_gpu_gemm_tops"] = gemm_ops_rank / (sum(gemm_ms) / args.steps * 1e-3) / 1e12
             line["allreduce_ms_per_step"] = ar_ms / args.steps
+            line["next2_fused_reduce_scatter"] = fused
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
     return 0
+
+
+def fused_rs_compare(cb, torch, dist, dev, layers, rank, world, steps):
+    """NEXT-2 on the row-parallel layer: (a) the headline path, GEMM writing FP32
+    partials + NCCL all_reduce; (b) GEMM + NCCL reduce_scatter (each rank keeps M / world rows);
+    (c) comet_w4ax_gemm_rs -- the epilogue stores each tile row into its owner's symmetric-memory
+    receive buffer over NVLink -- + a device barrier + comet_rs_reduce.  (b) and (c) produce the
+    same reduce-scatter result.  Device times per step, max over ranks.  Returns a dict (with an
+    "error" entry when symmetric memory is unavailable)."""
+    try:
+        import torch.distributed._symmetric_memory as symm
+        L = next(L for L in layers if L["kind"] == "row")
+        M, N = M_TOKENS, L["N"]
+        n_f = cb.rs_recv_bytes(M, N, world) // 4
+        recv = symm.empty(n_f, dtype=torch.float32, device=dev)
+        h = symm.rendezvous(recv, dist.group.WORLD)
+        ptrs = [int(p) for p in h.buffer_ptrs]
+        ms = -(-M // world)
+        rows = max(0, min(ms, M - rank * ms))
+        y32 = torch.empty((M, N), dtype=torch.float32, device=dev)
+        ys = torch.empty((ms, N), dtype=torch.float32, device=dev)
+        yr = torch.empty((max(rows, 1), N), dtype=torch.float16, device=dev)
+        plan = L["plan"] if L["plan"].info()["orientation"] == 3 else cb.Plan(M, N, L["K"], L["tags"], orientation=3)
+
+        def a():
+            cb.w4ax_gemm(plan, L["act"], L["sc"], L["wp"], L["sw"], out=y32)
+            dist.all_reduce(y32, op=dist.ReduceOp.SUM)
+
+        def b():
+            cb.w4ax_gemm(plan, L["act"], L["sc"], L["wp"], L["sw"], out=y32)
+            if M % world == 0:
+                dist.reduce_scatter_tensor(ys, y32, op=dist.ReduceOp.SUM)
+
+        def c():
+            cb.w4ax_gemm_rs(plan, L["act"], L["sc"], L["wp"], L["sw"], ptrs, rank)
+            h.barrier(channel=0)
+            if rows:
+                cb.rs_reduce(recv, world, rank, M, N, out=yr[:rows])
+
+        out = {}
+        for name, fn in (("gemm_allreduce_ms", a), ("gemm_nccl_reduce_scatter_ms", b), ("fused_gemm_rs_ms", c)):
+            for _ in range(3):
+                fn()
+            torch.cuda.synchronize()
+            dist.barrier()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            for _ in range(steps):
+                fn()
+            e1.record()
+            torch.cuda.synchronize()
+            out[name] = e0.elapsed_time(e1) / steps
+        vals = max_over_ranks([out[k] for k in sorted(out)], dist, torch, dev)
+        return {"layer": f"{L['name']} (row-parallel, K shard {L['K']}, M={M}, N={N})",
+                "timing": "ms per step, device events around `steps` back-to-back calls, max over ranks",
+                **{k: round(v, 4) for k, v in zip(sorted(out), vals)}}
+    except Exception as e:   # noqa: BLE001 -- report, do not fail the bench line
+        return {"error": f"{type(e).__name__}: {str(e)[:200]}"}
 
 
 def max_over_ranks(vals, dist, torch, dev):
