@@ -339,20 +339,22 @@ def config2_sweep(cb, torch, dev, peaks, timer, iters=20):
     for li, (name, K, N) in enumerate(LLAMA2_7B):
         tags = synth.make_tags(K, FRAC, np.random.default_rng(200 + li))
         wp, sw, _ = dev_weights(cb, torch, N, K, 210 + li, dev)
-        wts.append((name, K, N, tags, wp, sw))
+        # weight copies so back-to-back launches stream from HBM (> 300 MB per layer)
+        wps = [wp] + [wp.clone() for _ in range(max(1, -(-300 * (1 << 20) // (N * K // 2))) - 1)]
+        wts.append((name, K, N, tags, wps, sw))
     for bf16 in (False, True):
         for M in (1, 16, 256, 4096):
             L = []
-            for li, (name, K, N, tags, wp, sw) in enumerate(wts):
+            for li, (name, K, N, tags, wps, sw) in enumerate(wts):
                 x = dev_activations(torch, M, K, tags, 220 + li + M, dev, bf16=bf16)
                 plan = cb.Plan(M, N, K, tags)
                 act, sc = cb.quantize_act(x, tags)
                 y = torch.empty((M, N), dtype=torch.float16, device=dev)
-                L.append((name, K, N, tags, wp, sw, x, plan, act, sc, y))
+                L.append((name, K, N, tags, wps, sw, x, plan, act, sc, y))
             row = {"layers": {}}
             ops = nbytes = 0.0
-            for (name, K, N, tags, wp, sw, x, plan, act, sc, y) in L:
-                us = timer.us(lambda: cb.w4ax_gemm(plan, act, sc, wp, sw, out=y), iters)
+            for (name, K, N, tags, wps, sw, x, plan, act, sc, y) in L:
+                us = us_rotating(torch, [lambda w_=w_: cb.w4ax_gemm(plan, act, sc, w_, sw, out=y) for w_ in wps])
                 o, b = 2.0 * M * N * K, alg_bytes(M, K, N, FRAC)
                 ops += o
                 nbytes += b + 2 * M * K          # + the 16-bit input kernel 1 reads
@@ -361,16 +363,19 @@ def config2_sweep(cb, torch, dev, peaks, timer, iters=20):
                          tile=[plan.info()["tile_n"], plan.info()["tile_w"]])
                 row["layers"][name] = d
 
-            def step():
-                for (name, K, N, tags, wp, sw, x, plan, act, sc, y) in L:
+            ncopy = min(len(l[4]) for l in L)
+
+            def step(i):
+                for (name, K, N, tags, wps, sw, x, plan, act, sc, y) in L:
                     cb.quantize_act(x, tags, out=(act, sc))
-                    cb.w4ax_gemm(plan, act, sc, wp, sw, out=y)
-            us = timer.us(step, iters)
+                    cb.w4ax_gemm(plan, act, sc, wps[i], sw, out=y)
+            us = us_rotating(torch, [lambda i=i: step(i) for i in range(ncopy)])
             row["step"] = dict(roofline_point(ops, nbytes, us, peaks), us=round(us, 2))
             out[f"{'bf16' if bf16 else 'f16'}_M{M}"] = row
             del L
     return {"workload": "llama2_7b q/k/v/o 4096->4096, gate/up 4096->11008, down 11008->4096; 5 % INT8 blocks",
-            "l2": "clean L2 before every timed launch", "output": "f16",
+            "timing": "mean per launch (per step) over back-to-back launches cycling through > 300 MB of weight copies per layer",
+            "output": "f16",
             "roofline": "frac = max(ops / (2 x bf16 peak), SURVEY bytes / HBM peak) / measured", "points": out}
 
 
@@ -492,6 +497,22 @@ def next_rows(cb, torch, dev, peaks, timer, iters=20):
         out[f"grouped_scales_gemm_gate_up_M{M}"] = {"us": round(us_g, 2), "GB/s": round(nbytes / us_g / 1e3, 1),
                                                     "frac_hbm": round(nbytes / us_g / 1e3 / hbm, 3),
                                                     "per_channel_us": round(us_c, 2)}
+    # prefill-sized M: group-wise scales run on the weights-on-MMA-M kernel (128-token tiles);
+    # per-channel scales on the production pair kernel -- the measured cost of not building the
+    # grouped promotion into the pair kernel
+    M = M_TOKENS
+    x = dev_activations(torch, M, K, tags, 23, dev)
+    act, sc = cb.quantize_act(x, tags)
+    y = torch.empty((M, N), dtype=torch.float16, device=dev)
+    plan_g = cb.Plan(M, N, K, tags, orientation=1, tile_n=128)
+    plan_c = cb.Plan(M, N, K, tags)
+    us_g = t(lambda: cb.w4ax_gemm_grouped(plan_g, act, sc, wp, swg, out=y))
+    us_c = t(lambda: cb.w4ax_gemm(plan_c, act, sc, wp, swd, out=y))
+    ops = 2.0 * M * N * K
+    out[f"grouped_scales_gemm_gate_up_M{M}"] = {"us": round(us_g, 2), "TOPS": round(ops / us_g / 1e6, 1),
+                                                "per_channel_pair_kernel_us": round(us_c, 2),
+                                                "per_channel_TOPS": round(ops / us_c / 1e6, 1),
+                                                "kernel": "k_w4ax<128, grouped> (weights on MMA M) vs k_w4ax_n pair"}
     del wp, swg
     T, C, G = 32768, 1024, 128
     kv = torch.from_numpy(synth.make_kv(T, C, np.random.default_rng(0))).to(dev)

@@ -595,8 +595,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
               for (int j = 0; j < CH; j += 2) {
                 const int a = ch * CH + j;
                 const float2 s8 = make_float2(sc[j] * 1.220703125e-04f, sc[j + 1] * 1.220703125e-04f);  // 2^-13
-                const float2 y = ffma2(make_float2(__int2float_rn((int)v[j]), __int2float_rn((int)v[j + 1])),
-                                       s8, make_float2(acc[a], acc[a + 1]));
+                const float2 y = ffma2(i2f2_exact(v[j], v[j + 1]), s8, make_float2(acc[a], acc[a + 1]));
                 acc[a] = y.x;
                 acc[a + 1] = y.y;
               }

@@ -82,6 +82,20 @@ __device__ __forceinline__ void widen_kblock_row(const uint4* c, uint32_t (&o)[3
   }
 }
 
+// Exact int32 -> binary32 of two INT8-block accumulators (|v| <= 16 * 128 * 127 * 8 =
+// 2,080,768 < 2^22).  Default: two I2F.  COMET_I2F_MAGIC=1 instead adds 0x4B400000 (the bit
+// pattern of 1.5 * 2^23 + v) and subtracts 1.5 * 2^23 with one exact packed FMA -- no I2F, but
+// measured slower in the prefill promotion (tools/fsweep.py, all-INT8 blocks: 1556 against
+// 1805 TOPS on the same box), so it is off.
+#ifndef COMET_I2F_MAGIC
+#define COMET_I2F_MAGIC 0
+#endif
+__device__ __forceinline__ float2 i2f2_exact(uint32_t a, uint32_t b) {
+  if (!COMET_I2F_MAGIC) return make_float2(__int2float_rn((int)a), __int2float_rn((int)b));
+  const float2 x = make_float2(__uint_as_float(a + 0x4B400000u), __uint_as_float(b + 0x4B400000u));
+  return ffma2(x, make_float2(1.f, 1.f), make_float2(-12582912.f, -12582912.f));
+}
+
 // A global load the compiler keeps where it is written (volatile) and whose result is consumed
 // only where the caller first uses it: for operands prefetched a work item ahead.
 __device__ __forceinline__ float ldg_nc_f32(const float* p) {

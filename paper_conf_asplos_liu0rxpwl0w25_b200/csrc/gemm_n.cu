@@ -546,17 +546,23 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
               if (lane == 0) mbar_arrive_cluster(ready_rel + rs * 8);
               if (threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 10, tr);
             }
-            if (is8) {
+            if (is8) {                                    // warp-uniform (5 % of blocks)
 #pragma unroll
-              for (int c = 0; c < 64; ++c) v[c] = __float_as_uint(__int2float_rn((int)v[c]));
-            }
+              for (int c = 0; c < 64; c += 2) {
+                const int a = b * 64 + c;
+                const float2 y = ffma2(i2f2_exact(v[c], v[c + 1]), s2, make_float2(acc[a], acc[a + 1]));
+                acc[a] = y.x;
+                acc[a + 1] = y.y;
+              }
+            } else {
 #pragma unroll
-            for (int c = 0; c < 64; c += 2) {
-              const int a = b * 64 + c;
-              float2 y = ffma2(make_float2(__uint_as_float(v[c]), __uint_as_float(v[c + 1])), s2,
-                               make_float2(acc[a], acc[a + 1]));
-              acc[a] = y.x;
-              acc[a + 1] = y.y;
+              for (int c = 0; c < 64; c += 2) {
+                const int a = b * 64 + c;
+                const float2 y = ffma2(make_float2(__uint_as_float(v[c]), __uint_as_float(v[c + 1])), s2,
+                                       make_float2(acc[a], acc[a + 1]));
+                acc[a] = y.x;
+                acc[a + 1] = y.y;
+              }
             }
           }
           if (threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 7, tr);
@@ -586,7 +592,11 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
             }
             if (is8) {
 #pragma unroll
-              for (int c = 0; c < PB; ++c) v[c] = __float_as_uint(__int2float_rn((int)v[c]));
+              for (int c = 0; c < PB; c += 2) {
+              const float2 f = i2f2_exact(v[c], v[c + 1]);
+              v[c] = __float_as_uint(f.x);
+              v[c + 1] = __float_as_uint(f.y);
+            }
             }
 #pragma unroll
             for (int c = 0; c < PB; c += 2) {
@@ -634,7 +644,11 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
           }
           if (is8) {
 #pragma unroll
-            for (int c = 0; c < PB; ++c) v[c] = __float_as_uint(__int2float_rn((int)v[c]));
+            for (int c = 0; c < PB; c += 2) {
+              const float2 f = i2f2_exact(v[c], v[c + 1]);
+              v[c] = __float_as_uint(f.x);
+              v[c + 1] = __float_as_uint(f.y);
+            }
           }
 #pragma unroll
           for (int c = 0; c < PB; c += 2) {
