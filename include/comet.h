@@ -281,9 +281,10 @@ comet_status_t comet_w4ax_gemm(comet_plan_t plan, const void* act_packed, const 
  * comparison; reading R18): one scale per (128-channel block b, output channel n),
  *   Y[m,n] = sum_b s_a[m,b] * s_w[b,n] * acc_b[m,n]          (acc_b = sum_{k in b} q w, exact)
  * w_scales_grouped: device [K/128][N] float (block-major).  Arguments otherwise as
- * comet_w4ax_gemm (no per-block debug output).  Runs on the weights-on-MMA-M kernel: the plan
- * must have orientation 1 (the default for M < 128; set comet_sched_config.orientation = 1 for
- * larger M), else COMET_ERR_UNSUPPORTED_SHAPE. */
+ * comet_w4ax_gemm (no per-block debug output).  Runs on the weights-on-MMA-M kernel (plan
+ * orientation 1, the default for M < 128) or on the 256-wide prefill pair kernel (orientation 3,
+ * tile_w 256, the default for M >= 256; no debug accumulators there); other plans get
+ * COMET_ERR_UNSUPPORTED_SHAPE. */
 comet_status_t comet_w4ax_gemm_grouped(comet_plan_t plan, const void* act_packed, const float* act_scales,
                                        const void* w_packed, const float* w_scales_grouped, void* y,
                                        comet_dtype_t ydt, int64_t ldy, int32_t* debug_acc,

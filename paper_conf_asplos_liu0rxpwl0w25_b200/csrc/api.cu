@@ -456,8 +456,8 @@ comet_status_t comet_w4ax_gemm_grouped(comet_plan_t plan, const void* act_packed
   if (!aligned16(act_scales) || !aligned16(w_packed) || !aligned16(w_scales_grouped) || !aligned16(y) ||
       (debug_acc && !aligned16(debug_acc)) || (workspace && !aligned16(workspace)))
     return fail(COMET_ERR_MISALIGNED, "device pointers must be 16-byte aligned");
-  if (p.orientation != 1)
-    return fail(COMET_ERR_UNSUPPORTED_SHAPE, "group-wise weight scales need a plan with orientation 1 (weights on the MMA M side)");
+  if (p.orientation != 1 && !(p.orientation == 3 && p.tile_w == 256))
+    return fail(COMET_ERR_UNSUPPORTED_SHAPE, "group-wise weight scales run on orientation 1 or on the 256-wide pair kernel (orientation 3)");
   comet_status_t st = check_device();
   if (st != COMET_OK) return st;
   int launches = 0;

@@ -872,8 +872,10 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
                            int32_t* debug_acc_blocks, void* workspace, size_t ws_bytes,
                            cudaStream_t stream, int* launches, bool grouped, const RsArgs* rs) {
   using namespace gemm;
-  if (grouped && p.orientation != 1)
-    return fail(COMET_ERR_UNSUPPORTED_SHAPE, "group-wise weight scales need a plan with orientation 1 (weights on the MMA M side)");
+  if (grouped && p.orientation != 1 && !(p.orientation == 3 && p.tile_w == 256))
+    return fail(COMET_ERR_UNSUPPORTED_SHAPE, "group-wise weight scales run on orientation 1 or on the 256-wide pair kernel (orientation 3)");
+  if (grouped && p.orientation == 3 && (debug_acc || debug_acc_blocks))
+    return fail(COMET_ERR_UNSUPPORTED_SHAPE, "group-wise weight scales on the pair kernel have no debug accumulators");
   *launches = 0;
   const bool dbg = debug_acc != nullptr || debug_acc_blocks != nullptr;
   const int debug = debug_acc_blocks ? 2 : (dbg ? 1 : 0);
@@ -982,7 +984,7 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
     grid = p.num_ctas * cg;
   }
   if (normal) {
-    e = launch_gemm_n(prm, grid, tile_w, cg, debug, stream);
+    e = launch_gemm_n(prm, grid, tile_w, cg, debug, stream, grouped);
   } else if (dbg) {
     if (grouped) e = debug == 2 ? launch_nt<32, 2, true>(prm, grid, stream) : launch_nt<32, 1, true>(prm, grid, stream);
     else e = debug == 2 ? launch_nt<32, 2>(prm, grid, stream) : launch_nt<32, 1>(prm, grid, stream);

@@ -82,6 +82,22 @@ __device__ __forceinline__ void widen_kblock_row(const uint4* c, uint32_t (&o)[3
   }
 }
 
+// Packed binary32 pairs, round-to-nearest (FMUL2 / FADD2 on sm_100a).
+__device__ __forceinline__ float2 fmul2_f(float2 a, float2 b) {
+  float2 d;
+  asm("{\n\t.reg .b64 ra, rb, rd;\n\tmov.b64 ra, {%2, %3};\n\tmov.b64 rb, {%4, %5};\n\t"
+      "mul.rn.f32x2 rd, ra, rb;\n\tmov.b64 {%0, %1}, rd;\n\t}\n"
+      : "=f"(d.x), "=f"(d.y) : "f"(a.x), "f"(a.y), "f"(b.x), "f"(b.y));
+  return d;
+}
+__device__ __forceinline__ float2 fadd2_f(float2 a, float2 b) {
+  float2 d;
+  asm("{\n\t.reg .b64 ra, rb, rd;\n\tmov.b64 ra, {%2, %3};\n\tmov.b64 rb, {%4, %5};\n\t"
+      "add.rn.f32x2 rd, ra, rb;\n\tmov.b64 {%0, %1}, rd;\n\t}\n"
+      : "=f"(d.x), "=f"(d.y) : "f"(a.x), "f"(a.y), "f"(b.x), "f"(b.y));
+  return d;
+}
+
 // Exact int32 -> binary32 of two INT8-block accumulators (|v| <= 16 * 128 * 127 * 8 =
 // 2,080,768 < 2^22).  Default: two I2F.  COMET_I2F_MAGIC=1 instead adds 0x4B400000 (the bit
 // pattern of 1.5 * 2^23 + v) and subtracts 1.5 * 2^23 with one exact packed FMA -- no I2F, but
@@ -198,7 +214,8 @@ inline cudaError_t set_smem_attr(Kern kernel, int bytes, std::atomic<uint64_t>& 
 
 // Normal-orientation launcher (gemm_n.cu).  BN = weights per tile (256, or 128 for debug);
 // cg = CTAs per tile (1, or 2 for the tcgen05 CTA pair; grid must then be even).
-cudaError_t launch_gemm_n(const GemmParams& prm, int grid, int bn, int cg, int debug, cudaStream_t stream);
+cudaError_t launch_gemm_n(const GemmParams& prm, int grid, int bn, int cg, int debug, cudaStream_t stream,
+                          bool grouped = false);
 // Persistent units (CTAs, or pairs for cg = 2) of the production kernel that fit on the device
 // at once (occupancy query; -1 on error).
 int max_units_gemm_n(int bn, int cg, int sms);

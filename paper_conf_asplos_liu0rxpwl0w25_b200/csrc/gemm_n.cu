@@ -63,7 +63,7 @@ namespace comet {
 namespace gemm {
 namespace {
 
-template <int BN, int CG, int NPW_, int NWG_, int DEBUG_>
+template <int BN, int CG, int NPW_, int NWG_, int DEBUG_, bool GS_ = false>
 struct CfgN {
   static constexpr int BM = 128;                          // tokens per CTA (TMEM lanes)
   static constexpr int WROWS = BN / CG;                   // weight rows widened by this CTA
@@ -142,7 +142,10 @@ struct CfgN {
   static constexpr int SS = S + NACC;
   static constexpr int PRODUCERS = (COMET_PRODUCERS == 2 && S % 2 == 0 && SS % 2 == 0) ? 2 : 1;
   // [slots][output staging][scale ring SS x BM][w_scales 2 x BN][barriers][tmem][tags]
-  static constexpr int SMEM_DATA = S * SLOT_BYTES + STAGE_BYTES + SS * BM * 4 + 2 * BN * 4;
+  // GS (NEXT-3 group-wise weight scales): per scale-ring slot also the K-block's weight scales
+  // s_w[b][n0 .. n0+BN) (f32) and the tile rows' code sums qsum[b][m] (int16)
+  static constexpr int GS_BYTES = GS_ ? SS * (BN * 4 + BM * 2) : 0;
+  static constexpr int SMEM_DATA = S * SLOT_BYTES + STAGE_BYTES + SS * BM * 4 + 2 * BN * 4 + GS_BYTES;
   static constexpr int N_BARS = 2 * S + NSUB * S + NSUB * NACC;
   static constexpr int SMEM_BYTES = 1024 + SMEM_DATA + N_BARS * 8 + 16 + kMaxBlocks;
   static_assert(S >= 3, "pipeline depth");
@@ -167,9 +170,9 @@ struct CfgN {
 // kb only after slot_free[s] for kb - S; the scales of kb have landed when acc_full(kb) fires
 // (MMA(kb) waited mma_ready(kb) which waited widen(kb) which waited full[s]); the producer may
 // reuse scale slot kb % (S+NACC) because slot_free(kb-S) => MMA(kb-S) => promotion(kb-S-NACC).
-template <int BN, int CG, int NPW, int NWG, int DEBUG, bool RS = false>
-__global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w4ax_n(const __grid_constant__ GemmParams P) {
-  using C = CfgN<BN, CG, NPW, NWG, DEBUG>;
+template <int BN, int CG, int NPW, int NWG, int DEBUG, bool RS = false, bool GS = false>
+__global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG, GS>::THREADS, 1) k_w4ax_n(const __grid_constant__ GemmParams P) {
+  using C = CfgN<BN, CG, NPW, NWG, DEBUG, GS>;
   constexpr int kThreadsN = C::THREADS;
   constexpr int kPromoWarp0 = 4 + 4 * NWG;              // first promotion warp
   constexpr int S = C::S;
@@ -185,6 +188,8 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
   uint8_t* sY = smem + S * C::SLOT_BYTES;                                       // [NPW][2][8 KB]
   float* sS = reinterpret_cast<float*>(sY + C::STAGE_BYTES);                     // [SS][BM]
   float* sWs = sS + SS * BM;                                                     // [2][BN]
+  float* sG = sWs + 2 * BN;                                                      // GS: [SS][BN]
+  int16_t* sQ = reinterpret_cast<int16_t*>(sG + (GS ? SS * BN : 0));             // GS: [SS][BM]
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + C::SMEM_DATA);
   uint64_t* full = bars;                     // [S]
   uint64_t* slot_free = full + S;            // [S]
@@ -248,6 +253,9 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
         const int n_tile = w.tile / P.n_m_tiles, m_tile = w.tile % P.n_m_tiles;
         const int m0 = m_tile * (BM * CG) + BM * rank, n0 = n_tile * BN + C::WROWS * rank;
         const uint32_t sbytes = m0 < P.Mp ? (uint32_t)(min((int64_t)BM, P.Mp - m0) * 4) : 0u;
+        const int64_t ng0 = (int64_t)n_tile * BN;              // GS: the whole tile's columns
+        const uint32_t gbytes = GS ? (uint32_t)(min((int64_t)BN, P.N - ng0) * 4) : 0u;
+        const uint32_t qbytes = GS ? sbytes / 2 : 0u;
         for (int kb = w.kb_begin; kb < w.kb_end; ++kb, ++j) {
           if (C::PRODUCERS == 2 && (j & 1) != par) continue;
           const int s = j % S, sc = j % SS;
@@ -257,10 +265,14 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
           if (diag_ablate(P) & 32) {                       // diagnostic: no global loads
             mbar_arrive(&full[s]);
           } else {
-            mbar_arrive_expect_tx(&full[s], C::X_BYTES + C::WP_BYTES + sbytes);
+            mbar_arrive_expect_tx(&full[s], C::X_BYTES + C::WP_BYTES + sbytes + gbytes + qbytes);
             tma_load_2d(sX(s), &P.map_x, &full[s], kb * 128, m0);
             tma_load_2d(sWp(s), &P.map_w, &full[s], kb * 64, n0);
             if (sbytes) bulk_load(sS + sc * BM, P.scales + (int64_t)kb * P.Mp + m0, sbytes, &full[s]);
+            if (GS) {
+              bulk_load(sG + sc * BN, P.w_scales + (int64_t)kb * P.N + ng0, gbytes, &full[s]);
+              if (qbytes) bulk_load(sQ + sc * BM, P.qsum + (int64_t)kb * P.Mp + m0, qbytes, &full[s]);
+            }
           }
           if (par == 0) trace_ev(P, 0, tr++);
         }
@@ -478,7 +490,8 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
       const bool split = (w.flags & 1) != 0;
       // -corr * 2^-9 (offset-binary weight correction, owner segment only); loaded now, used
       // in the epilogue, so the load latency is off the K-loop's critical path
-      const float init = (owner && m < P.Mp) ? -__ldg(P.corr + m) * 0.001953125f : 0.f;
+      // (GS: the offset term is removed per block instead, and there is no per-channel s_w)
+      const float corr_raw = (!GS && owner && m < P.Mp) ? ldg_nc_f32(P.corr + m) : 0.f;
       // this tile's per-output-channel weight scales: loaded into registers now, written to
       // shared memory after the K-loop (read in the epilogue), so the global-load latency never
       // stalls the start of the tile's promotion
@@ -492,7 +505,7 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
           if (i < BN) {
             const int wgi = i / COLS, c = i % COLS;
             const int64_t n = (int64_t)n0 + col_n(wgi, c);
-            if (n < P.N) wsv[k] = __ldg(P.w_scales + n);
+            if (n < P.N) wsv[k] = GS ? 1.f : __ldg(P.w_scales + n);
           }
         }
       }
@@ -533,6 +546,49 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
           asm volatile("ld.shared.f32 %0, [%1];" : "=f"(s) : "r"(s_scale_r + 4u * BM * sc));
           if (is8) s *= 1.220703125e-04f;                 // 2^-13: INT8 block acc = 16 sum x w
           const float2 s2 = make_float2(s, s);
+          // GS (NEXT-3, reading R18): per column n the K-block's weight scale s_w[b][n] joins
+          // the row's s_a[m,b], and an INT4 block's offset-binary term 2^-6 qsum[b][m] is removed
+          // per block: acc += (s_a v - s_a 2^-6 qsum) * s_w[b][n] -- the bracket is one FFMA2
+          // with row scalars, the s_w product a second: two packed operations per two columns
+          float qc = 0.f;
+          if (GS && !is8) qc = -(float)sQ[sc * BM + r] * 0.015625f * s;   // -s_a 2^-6 qsum
+          const float2 qc2 = make_float2(qc, qc);
+          const float* gsw = sG + sc * BN + col0;
+          if constexpr (GS) {
+#pragma unroll
+            for (int b = 0; b < COLS / 64; ++b) {
+              uint32_t v[64];
+              tmem_ld_32x32b<64>(taddr + b * 64, v);
+              tmem_wait_ld();
+              if (b + 1 == COLS / 64) {
+                tc_fence_before();
+                __syncwarp();
+                if (lane == 0) mbar_arrive_cluster(ready_rel + rs * 8);
+              }
+#pragma unroll
+              for (int c = 0; c < 64; c += 4) {
+                const int a = b * 64 + c;
+                const float4 w4 = *reinterpret_cast<const float4*>(gsw + a);   // broadcast smem load
+                float2 x0, x1;
+                if (is8) {
+                  x0 = i2f2_exact(v[c], v[c + 1]);
+                  x1 = i2f2_exact(v[c + 2], v[c + 3]);
+                } else {
+                  x0 = make_float2(__uint_as_float(v[c]), __uint_as_float(v[c + 1]));
+                  x1 = make_float2(__uint_as_float(v[c + 2]), __uint_as_float(v[c + 3]));
+                }
+                const float2 u0 = ffma2(x0, s2, qc2), u1 = ffma2(x1, s2, qc2);   // s_a v - s_a 2^-6 qsum
+                const float2 y0 = ffma2(u0, make_float2(w4.x, w4.y), make_float2(acc[a], acc[a + 1]));
+                const float2 y1 = ffma2(u1, make_float2(w4.z, w4.w), make_float2(acc[a + 2], acc[a + 3]));
+                acc[a] = y0.x; acc[a + 1] = y0.y; acc[a + 2] = y1.x; acc[a + 3] = y1.y;
+              }
+            }
+            ++tr;
+            if (++accb == NACC) { accb = 0; accph ^= 1; }
+            if (++sc == SS) sc = 0;
+            if (++rs == S) rs = 0;
+            continue;
+          }
 #pragma unroll
           for (int b = 0; b < COLS / 64; ++b) {
             uint32_t v[64];
@@ -684,6 +740,7 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
         }
       }
       // ---------------------------------------------------------------- epilogue
+      const float init = -corr_raw * 0.001953125f;        // -corr * 2^-9 (0 for GS / non-owners)
       if (split) {
         const int seg = (w.flags >> 8) & 0xFF;
         const int nseg = (w.flags >> 16) & 0xFF;
@@ -891,11 +948,11 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG>::THREADS, 1) k_w
   }
 }
 
-template <int BN, int CG, int NPW, int NWG, int DEBUG, bool RS = false>
+template <int BN, int CG, int NPW, int NWG, int DEBUG, bool RS = false, bool GS = false>
 cudaError_t launch_bn(const GemmParams& prm, int grid, cudaStream_t stream) {
-  using C = CfgN<BN, CG, NPW, NWG, DEBUG>;
+  using C = CfgN<BN, CG, NPW, NWG, DEBUG, GS>;
   static std::atomic<uint64_t> attr_done{0};
-  cudaError_t ea = set_smem_attr(k_w4ax_n<BN, CG, NPW, NWG, DEBUG, RS>, C::SMEM_BYTES, attr_done);
+  cudaError_t ea = set_smem_attr(k_w4ax_n<BN, CG, NPW, NWG, DEBUG, RS, GS>, C::SMEM_BYTES, attr_done);
   if (ea != cudaSuccess) return ea;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)grid);
@@ -909,7 +966,7 @@ cudaError_t launch_bn(const GemmParams& prm, int grid, cudaStream_t stream) {
   attr[0].val.clusterDim.z = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  return cudaLaunchKernelEx(&cfg, k_w4ax_n<BN, CG, NPW, NWG, DEBUG, RS>, prm);
+  return cudaLaunchKernelEx(&cfg, k_w4ax_n<BN, CG, NPW, NWG, DEBUG, RS, GS>, prm);
 }
 
 // Persistent units (CTAs, or CTA pairs for CG = 2) of this kernel that can be resident at once.
@@ -967,7 +1024,13 @@ int max_units_gemm_n(int bn, int cg, int sms) {
 }
 
 // bn = 128, 160, 192 or 256; 96 for the debug-accumulator kernels (they need the registers).
-cudaError_t launch_gemm_n(const GemmParams& prm, int grid, int bn, int cg, int debug, cudaStream_t stream) {
+cudaError_t launch_gemm_n(const GemmParams& prm, int grid, int bn, int cg, int debug, cudaStream_t stream,
+                          bool grouped) {
+  if (grouped) {
+    // NEXT-3 group-wise weight scales: the 256-wide pair kernel with the grouped promotion
+    if (cg != 2 || bn != 256 || debug || prm.rs_world > 0) return cudaErrorInvalidValue;
+    return launch_bn<256, 2, COMET_N256_NPW, COMET_N256_NWG, 0, false, true>(prm, grid, stream);
+  }
   if (prm.rs_world > 0) {
     // NEXT-2 fused reduce-scatter: the 256-wide pair kernel with the peer-store epilogue
     if (cg != 2 || bn != 256 || debug) return cudaErrorInvalidValue;
