@@ -680,7 +680,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
   // the fix-up kernel (programmatic dependent) may launch once every CTA got here; its
   // griddepcontrol.wait still waits for this grid's completion and memory flush
   asm volatile("griddepcontrol.launch_dependents;");
-  if (tracing && threadIdx.x == 0) P.trace[32768 + blockIdx.x * 4 + 2] = globaltimer_ns();
+  if (tracing && threadIdx.x == 0) {
+    P.trace[32768 + blockIdx.x * 4 + 2] = globaltimer_ns();
+    uint32_t smid;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    P.trace[32768 + blockIdx.x * 4 + 3] = smid;
+  }
   if (warp == 2) tmem_dealloc<512>(tbase);
 }
 
