@@ -61,6 +61,12 @@ namespace {
 #ifndef COMET_DEC_WIDEN_PF
 #define COMET_DEC_WIDEN_PF 0   // 1: widen warps load stage s+1 weights before storing stage s (measured slower)
 #endif
+#ifndef COMET_DEC_EARLY_TRIGGER
+#define COMET_DEC_EARLY_TRIGGER 0   // 1: trigger dependents at the start (measured slower)
+#endif
+#ifndef COMET_FIXUP_EARLY_TRIGGER
+#define COMET_FIXUP_EARLY_TRIGGER 1
+#endif
 #ifndef COMET_DEC_SWMAX
 #define COMET_DEC_SWMAX 8   // cap of the packed-weight ring depth (variant experiments)
 #endif
@@ -210,6 +216,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
   // ahead and fills the weight ring; every other thread first waits for the predecessor grid
   // to complete and its memory to be visible (a no-op without a programmatic predecessor).
   if (!(warp == 0 && lane == 0)) asm volatile("griddepcontrol.wait;" ::: "memory");
+  // COMET_DEC_EARLY_TRIGGER: the next kernel of the stream (the fix-up kernel, or the next
+  // layer's kernel) may launch now -- its CTAs take SMs as ours retire, so the tail of this grid
+  // overlaps their start; they wait for our completion before touching our outputs
+  if (COMET_DEC_EARLY_TRIGGER && threadIdx.x == 0) asm volatile("griddepcontrol.launch_dependents;");
 
   if (warp < kWidenWarp0) {
     setmaxnreg_dec<56>();
@@ -679,7 +689,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
   __syncthreads();
   // the fix-up kernel (programmatic dependent) may launch once every CTA got here; its
   // griddepcontrol.wait still waits for this grid's completion and memory flush
-  asm volatile("griddepcontrol.launch_dependents;");
+  if (!COMET_DEC_EARLY_TRIGGER) asm volatile("griddepcontrol.launch_dependents;");
   if (tracing && threadIdx.x == 0) {
     P.trace[32768 + blockIdx.x * 4 + 2] = globaltimer_ns();
     uint32_t smid;
@@ -693,6 +703,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
 // row; y[m, n] = sum over the tile's segments (in segment order) of the s_w-scaled partials.
 template <int NT>
 __global__ void __launch_bounds__(128) k_fixup(const __grid_constant__ GemmParams P, const int2* __restrict__ fix_info) {
+  // let the next kernel of the stream (typically the next layer's GEMM, a programmatic
+  // dependent) launch at once: its weight producer streams while this grid and the tail of the
+  // GEMM before it run; its other threads wait for our completion
+  if (COMET_FIXUP_EARLY_TRIGGER) asm volatile("griddepcontrol.launch_dependents;");
   asm volatile("griddepcontrol.wait;" ::: "memory");
   const int2 fi = fix_info[blockIdx.x];                 // {tile, segments}
   const int m0 = (fi.x % P.n_m_tiles) * NT, n0 = (fi.x / P.n_m_tiles) * kTileW;

@@ -40,6 +40,12 @@
 #ifndef COMET_PROMO_SB
 #define COMET_PROMO_SB 1    // single-buffered 32-column promotion batches when they fit
 #endif
+#ifndef COMET_SPIN_MMA
+#define COMET_SPIN_MMA 0    // 1: MMA issuers spin (test_wait) on mma_ready instead of suspending
+#endif
+#ifndef COMET_SPIN_PROMO
+#define COMET_SPIN_PROMO 0  // 1: promotion warps spin on acc_full instead of suspending
+#endif
 #ifndef COMET_PROMO_W64
 #define COMET_PROMO_W64 1   // 64-column TMEM load rounds in the promotion when the registers allow
 #endif
@@ -299,7 +305,7 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG, GS>::THREADS, 1)
           const int s = j % S, accb = j % NACC;
           const uint32_t ph = (uint32_t)(j / S) & 1u;
           if (lane == 0) trace_ev(P, parity ? 13 : 1, tr);
-          mbar_wait(&mma_ready[h * S + s], ph);
+          if (COMET_SPIN_MMA) mbar_wait_spin(&mma_ready[h * S + s], ph); else mbar_wait(&mma_ready[h * S + s], ph);
           if (lane == 0) trace_ev(P, parity ? 11 : 3, tr);
           tc_fence_after();
           const uint32_t d = tb + accb * BN + h * NMMA;
@@ -357,7 +363,7 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG, GS>::THREADS, 1)
           const int s = j % S, accb = j % NACC;
           const uint32_t ph = (uint32_t)(j / S) & 1u;
           trace_ev(P, parity ? 13 : 1, tr);
-          mbar_wait(&mma_ready[h * S + s], ph);
+          if (COMET_SPIN_MMA) mbar_wait_spin(&mma_ready[h * S + s], ph); else mbar_wait(&mma_ready[h * S + s], ph);
           trace_ev(P, parity ? 11 : 3, tr++);
           tc_fence_after();
           const uint32_t d = tbase + accb * BN + h * NMMA;
@@ -521,7 +527,7 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG, GS>::THREADS, 1)
         int qs = 0;
         if (DEBUG && !is8 && m < P.Mp) qs = P.qsum[(int64_t)kb * P.Mp + m];
         if (threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 12, tr);
-        mbar_wait(&acc_full[sub * NACC + accb], accph);
+        if (COMET_SPIN_PROMO) mbar_wait_spin(&acc_full[sub * NACC + accb], accph); else mbar_wait(&acc_full[sub * NACC + accb], accph);
         if (threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 6, tr);
         tc_fence_after();
         if (diag_ablate(P) & 16) {                              // diagnostic: no promotion work

@@ -114,6 +114,34 @@ __device__ __forceinline__ void mbar_wait_addr(uint32_t a, uint32_t parity) {
       "r"(parity), "n"(1000000), "l"((uint64_t)COMET_MBAR_TIMEOUT_NS)
       : "memory");
 }
+// Spin variant: test_wait in a loop (no suspension), for a wait on the critical path whose
+// waiter has nothing else to do; same hang guard.
+__device__ __forceinline__ void mbar_wait_spin(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t"
+      ".reg .pred P, Q;\n\t"
+      ".reg .u32 c;\n\t"
+      ".reg .u64 t0, t1;\n\t"
+      "mov.u64 t0, %%globaltimer;\n"
+      "SPIN_OUTER:\n\t"
+      "mov.u32 c, 256;\n"
+      "SPIN_LOOP:\n\t"
+      "mbarrier.test_wait.parity.shared::cta.b64 P, [%0], %1;\n\t"
+      "@P bra.uni SPIN_DONE;\n\t"
+      "sub.u32 c, c, 1;\n\t"
+      "setp.ne.u32 Q, c, 0;\n\t"
+      "@Q bra.uni SPIN_LOOP;\n\t"
+      "mov.u64 t1, %%globaltimer;\n\t"
+      "sub.u64 t1, t1, t0;\n\t"
+      "setp.lt.u64 Q, t1, %2;\n\t"
+      "@Q bra.uni SPIN_OUTER;\n\t"
+      "trap;\n"
+      "SPIN_DONE:\n\t"
+      "}\n" ::"r"(smem_u32(bar)),
+      "r"(parity), "l"((uint64_t)COMET_MBAR_TIMEOUT_NS)
+      : "memory");
+}
+
 #ifndef COMET_HANG_PRINT
 #define COMET_HANG_PRINT 0
 #endif
