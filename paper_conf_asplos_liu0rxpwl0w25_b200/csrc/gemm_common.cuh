@@ -176,8 +176,11 @@ __device__ __forceinline__ int diag_ablate(const GemmParams& P) {
 }
 
 // Diagnostic timeline: CTA c < 2, event e < 8, K-block index i < 1024 (per-CTA running count).
+#ifndef COMET_TRACE_MASK
+#define COMET_TRACE_MASK 0xFFFF   // events recorded by a trace build (bit e = event e)
+#endif
 __device__ __forceinline__ void trace_ev(const GemmParams& P, int e, int i) {
-  if ((COMET_DIAG || COMET_TRACE) && P.trace != nullptr && blockIdx.x < 2 && i < 1024) {
+  if ((COMET_DIAG || COMET_TRACE) && ((COMET_TRACE_MASK >> e) & 1) && P.trace != nullptr && blockIdx.x < 2 && i < 1024) {
     unsigned long long t;
     asm volatile("mov.u64 %0, %%clock64;" : "=l"(t));
     P.trace[((int)blockIdx.x * 16 + e) * 1024 + i] = t;

@@ -58,6 +58,15 @@
 #ifndef COMET_SMEM_BUDGET_KB
 #define COMET_SMEM_BUDGET_KB 216   // pipeline slots + output staging + scale ring
 #endif
+#ifndef COMET_PROMO_WAIT_PLAIN
+#define COMET_PROMO_WAIT_PLAIN 1   // 1: promotion waits acc_full with a plain try_wait loop (see the wait)
+#endif
+#ifndef COMET_ABLATE_TMA2D
+#define COMET_ABLATE_TMA2D 0   // 1: timing experiment only -- contiguous bulk copies from a small L2-resident buffer replace the 2D TMA loads (wrong results)
+#endif
+#ifndef COMET_STUB
+#define COMET_STUB 0   // timing experiments only (wrong results): 1 MMA kind fixed, 2 promotion scale/kind fixed, 4 no scale loads, 8 no epilogue stores
+#endif
 #ifndef COMET_N256_NPW
 #define COMET_N256_NPW 2   // promotion warpgroups of the 256-wide tile
 #endif
@@ -258,7 +267,7 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG, GS>::THREADS, 1)
         const WorkItem w = load_item(P, it, debug);
         const int n_tile = w.tile / P.n_m_tiles, m_tile = w.tile % P.n_m_tiles;
         const int m0 = m_tile * (BM * CG) + BM * rank, n0 = n_tile * BN + C::WROWS * rank;
-        const uint32_t sbytes = m0 < P.Mp ? (uint32_t)(min((int64_t)BM, P.Mp - m0) * 4) : 0u;
+        const uint32_t sbytes = (m0 < P.Mp && !(COMET_STUB & 4)) ? (uint32_t)(min((int64_t)BM, P.Mp - m0) * 4) : 0u;
         const int64_t ng0 = (int64_t)n_tile * BN;              // GS: the whole tile's columns
         const uint32_t gbytes = GS ? (uint32_t)(min((int64_t)BN, P.N - ng0) * 4) : 0u;
         const uint32_t qbytes = GS ? sbytes / 2 : 0u;
@@ -272,8 +281,11 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG, GS>::THREADS, 1)
             mbar_arrive(&full[s]);
           } else {
             mbar_arrive_expect_tx(&full[s], C::X_BYTES + C::WP_BYTES + sbytes + gbytes + qbytes);
-            tma_load_2d(sX(s), &P.map_x, &full[s], kb * 128, m0);
-            tma_load_2d(sWp(s), &P.map_w, &full[s], kb * 64, n0);
+            const uint8_t* src = reinterpret_cast<const uint8_t*>(P.scales) + ((kb * 7 + m0 / 128) % 32) * 24576;
+            if (COMET_ABLATE_TMA2D & 1) bulk_load(sX(s), src, C::X_BYTES, &full[s]);
+            else tma_load_2d(sX(s), &P.map_x, &full[s], kb * 128, m0);
+            if (COMET_ABLATE_TMA2D & 2) bulk_load(sWp(s), src + C::X_BYTES, C::WP_BYTES, &full[s]);
+            else tma_load_2d(sWp(s), &P.map_w, &full[s], kb * 64, n0);
             if (sbytes) bulk_load(sS + sc * BM, P.scales + (int64_t)kb * P.Mp + m0, sbytes, &full[s]);
             if (GS) {
               bulk_load(sG + sc * BN, P.w_scales + (int64_t)kb * P.N + ng0, gbytes, &full[s]);
@@ -311,7 +323,7 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG, GS>::THREADS, 1)
           const uint32_t d = tb + accb * BN + h * NMMA;
           const uint32_t sa = sx0 + s * C::SLOT_BYTES;
           const uint32_t sbv = sa + C::X_BYTES + h * (C::WROWS / NSUB) * 128;
-          const bool is8 = __shfl_sync(0xffffffffu, lds_u8(s_tags_a + kb), 0) != 0;
+          const bool is8 = (COMET_STUB & 1) ? false : __shfl_sync(0xffffffffu, lds_u8(s_tags_a + kb), 0) != 0;
           // one elected thread issues the K-block's four MMAs AND its commits: tcgen05.commit
           // tracks the MMAs of the issuing thread only, so both must come from the same lane
           if (elect_one()) {
@@ -523,11 +535,17 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG, GS>::THREADS, 1)
         if (DEBUG) dacc[c] = 0;
       }
       for (int kb = w.kb_begin; kb < w.kb_end; ++kb) {
-        const bool is8 = lds_u8(s_tags_a + kb) != 0;
+        const bool is8 = (COMET_STUB & 66) ? false : lds_u8(s_tags_a + kb) != 0;
         int qs = 0;
         if (DEBUG && !is8 && m < P.Mp) qs = P.qsum[(int64_t)kb * P.Mp + m];
         if (threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 12, tr);
-        if (COMET_SPIN_PROMO) mbar_wait_spin(&acc_full[sub * NACC + accb], accph); else mbar_wait(&acc_full[sub * NACC + accb], accph);
+        // Plain try_wait loop (no suspend-time hint, no timer): the hinted, timer-guarded wait
+        // made the wake-up path slower AND kept ptxas from scheduling the post-wait address math
+        // in the wait's shadow (3 % of the prefill GEMM, tools/gpu_pre_variants.sh).  A hang
+        // here is still caught: acc_full(kb) completes unless MMA(kb) was never issued, and the
+        // MMA issuer's own mma_ready wait is guarded (its trap aborts the launch).
+        if (COMET_PROMO_WAIT_PLAIN) { while (!mbar_try_wait(smem_u32(&acc_full[sub * NACC + accb]), accph)) {} }
+        else if (COMET_SPIN_PROMO) mbar_wait_spin(&acc_full[sub * NACC + accb], accph); else mbar_wait(&acc_full[sub * NACC + accb], accph);
         if (threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 6, tr);
         tc_fence_after();
         if (diag_ablate(P) & 16) {                              // diagnostic: no promotion work
@@ -547,10 +565,15 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG, GS>::THREADS, 1)
         // folded in; the accumulator is released once the last load has landed.
         constexpr int PB = C::PB;                         // columns per TMEM load batch
         constexpr int NB_ = COLS / PB;
-        if constexpr (C::W64) {
-          float s;
-          asm volatile("ld.shared.f32 %0, [%1];" : "=f"(s) : "r"(s_scale_r + 4u * BM * sc));
-          if (is8) s *= 1.220703125e-04f;                 // 2^-13: INT8 block acc = 16 sum x w
+        // the row's activation scale of this K-block (shared-memory ring slot sc), times 2^-13 for
+        // an INT8 block (acc = 16 sum x w)
+        auto row_scale = [&]() -> float {
+          float s = 1.0f;
+          if (!(COMET_STUB & 34)) asm volatile("ld.shared.f32 %0, [%1];" : "=f"(s) : "r"(s_scale_r + 4u * BM * sc));
+          return is8 ? s * 1.220703125e-04f : s;
+        };
+        if constexpr (C::W64 && GS) {
+          const float s = row_scale();
           const float2 s2 = make_float2(s, s);
           // GS (NEXT-3, reading R18): per column n the K-block's weight scale s_w[b][n] joins
           // the row's s_a[m,b], and an INT4 block's offset-binary term 2^-6 qsum[b][m] is removed
@@ -595,10 +618,17 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG, GS>::THREADS, 1)
             if (++rs == S) rs = 0;
             continue;
           }
+        }
+        if constexpr (C::W64 && !GS) {
+          float2 s2;
 #pragma unroll
           for (int b = 0; b < COLS / 64; ++b) {
             uint32_t v[64];
             tmem_ld_32x32b<64>(taddr + b * 64, v);
+            if (b == 0) {
+              const float s = row_scale();
+              s2 = make_float2(s, s);
+            }
             tmem_wait_ld();
             if (b == 0 && threadIdx.x == kPromoWarp0 * 32) trace_ev(P, 9, tr);
             if (b + 1 == COLS / 64) {
@@ -825,6 +855,8 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG, GS>::THREADS, 1)
             asm volatile("st.global.v4.f32 [%0], {%1,%2,%3,%4};" ::"l"(dst + nc), "f"(v.x), "f"(v.y), "f"(v.z), "f"(v.w) : "memory");
           }
         }
+      } else if (COMET_STUB & 8) {
+        // timing experiment: no epilogue
       } else {
         // TMA-store epilogue.  y = (acc - corr 2^-9) * s_w * 512 (R7).  The
         // WG's COLS columns leave in chunks of 64 bytes per row (32 half / 16 float columns),

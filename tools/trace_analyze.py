@@ -48,6 +48,9 @@ print("  promo wake -> first load landed  ", med([t[9][j] - t[6][j] for j in js]
 if (t[10] > 0).any():
     print("  promo wake -> released           ", med([t[10][j] - t[6][j] for j in js]))
 print("  promo wake -> done               ", med([t[7][j] - t[6][j] for j in js]))
+if (t[10] > 0).any():
+    print("  released(j) -> MMA issue(j+2)    ", med([issue(j + 2) - t[10][j] for j in js]))
+    print("  released(j) -> promo wait(j+1)   ", med([t[12][j + 1] - t[10][j] for j in js]))
 print("  promo done(j) -> MMA issue(j+2)  ", med([issue(j + 2) - t[7][j] for j in js]))
 print("  MMA issue(j) -> MMA issue(j+2)   ", med([issue(j + 2) - issue(j) for j in js]))
 # tile boundaries (whole 64-K-block tiles, gate_up): promotion gap done(j) -> next wait(j+1) and
