@@ -38,6 +38,32 @@
 #include <cstdlib>
 #include "gemm_common.cuh"
 
+// The pipeline roles' waits (promotion 1, MMA issuer 2, widen 4) are bare try_wait loops: ~2 %
+// faster than the timer-guarded mbar_wait on every decode shape (tools/gpu_decb_variants.sh);
+// even an iteration-count guard (COMET_DEC_GUARD) gave the gain back.  The two producers' waits
+// keep the timer guard: a stalled pipeline stops releasing their ring slots, so their guarded
+// waits trap; the unguarded window is a CTA's last ring-depth of stages, where every load has
+// been issued and only a load that never completes could hang.
+#ifndef COMET_DEC_PLAIN
+#define COMET_DEC_PLAIN 7
+#endif
+#ifndef COMET_DEC_GUARD
+#define COMET_DEC_GUARD 0   // which of them count iterations as a hang guard (experiment)
+#endif
+#define DEC_WAIT(bit, bar, ph)                                                                  \
+  do {                                                                                          \
+    if (COMET_DEC_PLAIN & COMET_DEC_GUARD & (bit)) {                                            \
+      uint32_t n_ = 0;                                                                          \
+      while (!mbar_try_wait(smem_u32(bar), (ph)))                                               \
+        if (++n_ == (1u << 28)) __trap();                                                       \
+    } else if (COMET_DEC_PLAIN & (bit)) {                                                       \
+      while (!mbar_try_wait(smem_u32(bar), (ph))) {}                                            \
+    } else {                                                                                    \
+      mbar_wait((bar), (ph));                                                                   \
+    }                                                                                           \
+  } while (0)
+
+
 namespace comet {
 namespace gemm {
 namespace {
@@ -283,9 +309,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
         const int kb_end = __shfl_sync(0xffffffffu, w.kb_end, 0);
         for (int kb = kb_begin; kb < kb_end; kb += KS) {
           const int nk = min(KS, kb_end - kb);
-          mbar_wait(&full_x[sx], xph);
-          mbar_wait(&a_full[ab], aph);
-          mbar_wait(&acc_empty[accs], accph ^ 1);
+          DEC_WAIT(2, &full_x[sx], xph);
+          DEC_WAIT(2, &a_full[ab], aph);
+          DEC_WAIT(2, &acc_empty[accs], accph ^ 1);
           if (lane == 0) trace_ev(P, 1, tr);
           tc_fence_after();
           const uint32_t d0 = tb + C::ACC_COL + accs * C::ACC_SET;
@@ -348,7 +374,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
     auto fetch = [&]() {
       nk_n = min(KS, w.kb_end - kb);
       kb_n = kb;
-      mbar_wait(&full_w[st], ph);
+      DEC_WAIT(4, &full_w[st], ph);
       if (lane == 0 && q == 0) trace_ev(P, 3 + half, seq_f);
 #pragma unroll
       for (int i = 0; i < KH; ++i) {
@@ -378,7 +404,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
       const int nk = nk_n, kbc = kb_n;
       const bool have_next = it < it_end;
       if (have_next) fetch();
-      mbar_wait(&a_empty[ab], aph ^ 1);
+      DEC_WAIT(4, &a_empty[ab], aph ^ 1);
       if (lane == 0 && q == 0 && half == 0) trace_ev(P, 14, seq);
       tc_fence_after();
 #pragma unroll
@@ -420,7 +446,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
       const WorkItem w = item(it);
       for (int kb = w.kb_begin; kb < w.kb_end; kb += KS, ++seq) {
         const int nk = min(KS, w.kb_end - kb);
-        mbar_wait(&full_w[st], ph);
+        DEC_WAIT(4, &full_w[st], ph);
         if (lane == 0 && q == 0) trace_ev(P, 3 + half, seq);
         // this warp's K-blocks of the stage: 4 x 16 B per K-block (row r, 128B-swizzled chunks)
         uint4 cc[4 * KH];
@@ -435,7 +461,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
         }
         __syncwarp();
         if (lane == 0) mbar_arrive(&empty_w[st]);
-        mbar_wait(&a_empty[ab], aph ^ 1);
+        DEC_WAIT(4, &a_empty[ab], aph ^ 1);
         if (lane == 0 && q == 0 && half == 0) trace_ev(P, 14, seq);
         tc_fence_after();
 #if COMET_DEC_ST64
@@ -542,8 +568,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
       }
       for (int kb0 = w.kb_begin; kb0 < w.kb_end; kb0 += KS) {
         const int nk = min(KS, w.kb_end - kb0);
-        mbar_wait(&full_x[sx], xph);
-        mbar_wait(&acc_full[accs], accph);
+        DEC_WAIT(1, &full_x[sx], xph);
+        DEC_WAIT(1, &acc_full[accs], accph);
         if (ptid == 0) trace_ev(P, 7, tr);
         tc_fence_after();
         const uint32_t sbase = smem_u32(sS(sx));

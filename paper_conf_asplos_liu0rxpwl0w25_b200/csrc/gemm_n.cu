@@ -64,6 +64,12 @@
 #ifndef COMET_ABLATE_TMA2D
 #define COMET_ABLATE_TMA2D 0   // 1: timing experiment only -- contiguous bulk copies from a small L2-resident buffer replace the 2D TMA loads (wrong results)
 #endif
+#ifndef COMET_MMA_WAIT_PLAIN
+#define COMET_MMA_WAIT_PLAIN 1   // 1: MMA issuer waits mma_ready with a plain try_wait loop (iteration-count guard)
+#endif
+#ifndef COMET_WIDEN_WAIT_PLAIN
+#define COMET_WIDEN_WAIT_PLAIN 0   // experiment: plain try_wait loop for the widen warps' full wait
+#endif
 #ifndef COMET_STUB
 #define COMET_STUB 0   // timing experiments only (wrong results): 1 MMA kind fixed, 2 promotion scale/kind fixed, 4 no scale loads, 8 no epilogue stores
 #endif
@@ -317,7 +323,14 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG, GS>::THREADS, 1)
           const int s = j % S, accb = j % NACC;
           const uint32_t ph = (uint32_t)(j / S) & 1u;
           if (lane == 0) trace_ev(P, parity ? 13 : 1, tr);
-          if (COMET_SPIN_MMA) mbar_wait_spin(&mma_ready[h * S + s], ph); else mbar_wait(&mma_ready[h * S + s], ph);
+          if (COMET_MMA_WAIT_PLAIN) {
+            // plain try_wait (no suspend hint); hang guard by iteration count, never read on the
+            // fast path (each try_wait suspends for a hardware window, so 2^28 of them is seconds)
+            uint32_t n = 0;
+            while (!mbar_try_wait(smem_u32(&mma_ready[h * S + s]), ph))
+              if (++n == (1u << 28)) __trap();
+          }
+          else if (COMET_SPIN_MMA) mbar_wait_spin(&mma_ready[h * S + s], ph); else mbar_wait(&mma_ready[h * S + s], ph);
           if (lane == 0) trace_ev(P, parity ? 11 : 3, tr);
           tc_fence_after();
           const uint32_t d = tb + accb * BN + h * NMMA;
@@ -422,7 +435,7 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG, GS>::THREADS, 1)
       for (int kb = w.kb_begin; kb < w.kb_end; ++kb, ++j) {
         if (NWG == 1 || j % NWG == grp) {
           const bool is8 = lds_u8(s_tags_a + kb) != 0;
-          mbar_wait(&full[s], ph);
+          if (COMET_WIDEN_WAIT_PLAIN) { while (!mbar_try_wait(smem_u32(&full[s]), ph)) {} } else mbar_wait(&full[s], ph);
           if (warp == 4 && lane == 0) trace_ev(P, 5, tr);
           uint4 c[RPT][4];
 #pragma unroll

@@ -84,13 +84,15 @@ __device__ __forceinline__ uint64_t globaltimer_ns() {
 }
 // Blocking wait on phase `parity`.  First a non-suspending test_wait: on a phase that has
 // already completed it returns in ~21 clk, where try_wait costs ~165 clk even then
-// (profiles/r01/probe_lat.json).  Otherwise a loop of try_wait with a suspend hint: the thread
-// sleeps in hardware until the phase completes instead of spinning on issue slots.  The whole
+// (profiles/r01/probe_lat.json).  Otherwise a loop of try_wait: the thread is suspended in
+// hardware for a system-defined window instead of spinning on issue slots (COMET_WAIT_MODE 1;
+// mode 0 passes a suspend-time hint, which compiles to NANOSLEEP.SYNCS and measured ~1 % slower
+// on the prefill GEMM, neutral on decode, tools/gpu_pre_variants.sh / decode_bench.py).  The whole
 // loop is one PTX block so the compiler cannot hoist the hang guard into it; the global timer is
 // read once every 64 unsuccessful suspensions, and a wait longer than COMET_MBAR_TIMEOUT_NS
 // traps (the launch fails with an error) instead of hanging the GPU.
 #ifndef COMET_WAIT_MODE
-#define COMET_WAIT_MODE 0
+#define COMET_WAIT_MODE 1
 #endif
 #if COMET_WAIT_MODE == 0        // try_wait with a suspend-time hint (hardware sleep)
 #define COMET_WAIT_INSTR "mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1, %2;\n\t"
