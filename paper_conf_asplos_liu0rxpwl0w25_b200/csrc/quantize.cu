@@ -177,8 +177,12 @@ __device__ __forceinline__ LaneOut quantize32(const float (&v)[32], bool is8) {
 // GATHER: the fused channel permutation (NEXT-1) as direct gathers -- channel k of the row is
 // read from x[m, perm[k]] with 16-bit L1-cached loads (the CTA's rows are re-read sector by
 // sector from L1; calibrated permutations are ascending runs, so a warp's gathers coalesce).
-template <bool BF16, int WPR, bool GATHER = false>
-__global__ void __launch_bounds__(256) k_quantize(const uint16_t* __restrict__ x, int64_t M,
+// PF: the next group's four loads are issued before this group's arithmetic (a warp keeps two
+// groups in flight); it costs 16 registers (80: 3 CTAs per SM instead of 4), so the launcher
+// uses it only when a warp walks >= 3 groups (tools/quant_bench.py: K = 28672 71.3 -> 67.3 us,
+// M = 8192 K = 14336 71.7 -> 66.8 us; at K = 8192, 2 groups per warp, 23.4 -> 24.6 us: off)
+template <bool BF16, int WPR, bool GATHER = false, bool PF = false>
+__global__ void __launch_bounds__(256, PF ? 3 : 4) k_quantize(const uint16_t* __restrict__ x, int64_t M,
                                                   int64_t K, int64_t ldx, int64_t Mp, TagMask tags,
                                                   uint8_t* __restrict__ codes,
                                                   int16_t* __restrict__ qsum,
@@ -200,11 +204,31 @@ __global__ void __launch_bounds__(256) k_quantize(const uint16_t* __restrict__ x
   if (m < M) {
     const uint16_t* xrow = x + m * ldx + sub * 8;
     uint8_t* crow = codes + m * K + sub * 8;
+    uint4 rawn[4];                                    // PF: the next group's loads
+    if (!GATHER && PF && wi < ngroups) {
+      const int b0 = wi * 8 + bl;
+#pragma unroll
+      for (int j = 0; j < 4; ++j)
+        rawn[j] = b0 < nb ? ldg_stream(xrow + b0 * kBlockK + 32 * j) : make_uint4(0, 0, 0, 0);
+    }
     for (int g = wi; g < ngroups; g += WPR) {
       const int b = g * 8 + bl;
       const bool bvalid = b < nb;
       uint4 raw[4];
-      if (GATHER) {
+      if (!GATHER && !PF) {
+#pragma unroll
+        for (int j = 0; j < 4; ++j)
+          raw[j] = bvalid ? ldg_stream(xrow + b * kBlockK + 32 * j) : make_uint4(0, 0, 0, 0);
+      } else if (!GATHER) {
+#pragma unroll
+        for (int j = 0; j < 4; ++j) raw[j] = rawn[j];
+        const int bn_ = (g + WPR) * 8 + bl;
+        if (g + WPR < ngroups) {
+#pragma unroll
+          for (int j = 0; j < 4; ++j)
+            rawn[j] = bn_ < nb ? ldg_stream(xrow + bn_ * kBlockK + 32 * j) : make_uint4(0, 0, 0, 0);
+        }
+      } else {
         const uint16_t* xr = x + m * ldx;
         const int kmax = (int)K - 1;
         int idx[32];
@@ -227,10 +251,6 @@ __global__ void __launch_bounds__(256) k_quantize(const uint16_t* __restrict__ x
         for (int j = 0; j < 4; ++j)
           raw[j] = make_uint4(h[8 * j] | (h[8 * j + 1] << 16), h[8 * j + 2] | (h[8 * j + 3] << 16),
                               h[8 * j + 4] | (h[8 * j + 5] << 16), h[8 * j + 6] | (h[8 * j + 7] << 16));
-      } else {
-#pragma unroll
-        for (int j = 0; j < 4; ++j)
-          raw[j] = bvalid ? ldg_stream(xrow + b * kBlockK + 32 * j) : make_uint4(0, 0, 0, 0);
       }
       float v[32];
 #pragma unroll
@@ -575,10 +595,15 @@ cudaError_t launch_q(const void* x, int64_t M, int64_t K, int64_t ldx, const Tag
   const int rows = 8 / wpr;
   const dim3 grid((unsigned)ceil_div(Mp, rows));
   const uint16_t* xp = static_cast<const uint16_t*>(x);
-  switch (wpr) {
-    case 1: k_quantize<BF16, 1><<<grid, 256, 0, stream>>>(xp, M, K, ldx, Mp, tags, codes, qsum, corr, act_scales); break;
-    case 2: k_quantize<BF16, 2><<<grid, 256, 0, stream>>>(xp, M, K, ldx, Mp, tags, codes, qsum, corr, act_scales); break;
-    case 4: k_quantize<BF16, 4><<<grid, 256, 0, stream>>>(xp, M, K, ldx, Mp, tags, codes, qsum, corr, act_scales); break;
+  const bool pf = ngroups >= 3 * wpr;                // a warp walks >= 3 groups
+  switch (wpr * 2 + (pf ? 1 : 0)) {
+    case 2: k_quantize<BF16, 1><<<grid, 256, 0, stream>>>(xp, M, K, ldx, Mp, tags, codes, qsum, corr, act_scales); break;
+    case 3: k_quantize<BF16, 1, false, true><<<grid, 256, 0, stream>>>(xp, M, K, ldx, Mp, tags, codes, qsum, corr, act_scales); break;
+    case 4: k_quantize<BF16, 2><<<grid, 256, 0, stream>>>(xp, M, K, ldx, Mp, tags, codes, qsum, corr, act_scales); break;
+    case 5: k_quantize<BF16, 2, false, true><<<grid, 256, 0, stream>>>(xp, M, K, ldx, Mp, tags, codes, qsum, corr, act_scales); break;
+    case 8: k_quantize<BF16, 4><<<grid, 256, 0, stream>>>(xp, M, K, ldx, Mp, tags, codes, qsum, corr, act_scales); break;
+    case 9: k_quantize<BF16, 4, false, true><<<grid, 256, 0, stream>>>(xp, M, K, ldx, Mp, tags, codes, qsum, corr, act_scales); break;
+    case 17: k_quantize<BF16, 8, false, true><<<grid, 256, 0, stream>>>(xp, M, K, ldx, Mp, tags, codes, qsum, corr, act_scales); break;
     default: k_quantize<BF16, 8><<<grid, 256, 0, stream>>>(xp, M, K, ldx, Mp, tags, codes, qsum, corr, act_scales); break;
   }
   return cudaGetLastError();
