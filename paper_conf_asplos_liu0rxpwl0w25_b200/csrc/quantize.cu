@@ -592,10 +592,17 @@ cudaError_t launch_q(const void* x, int64_t M, int64_t K, int64_t ldx, const Tag
   }
   int wpr = 1;
   while (wpr < 8 && ceil_div(Mp, 8 / wpr) < target && ngroups >= 2 * wpr) wpr *= 2;
+#ifdef COMET_Q_WPR
+  wpr = COMET_Q_WPR;
+#endif
   const int rows = 8 / wpr;
   const dim3 grid((unsigned)ceil_div(Mp, rows));
   const uint16_t* xp = static_cast<const uint16_t*>(x);
+#ifdef COMET_Q_PF
+  const bool pf = COMET_Q_PF;
+#else
   const bool pf = ngroups >= 3 * wpr;                // a warp walks >= 3 groups
+#endif
   switch (wpr * 2 + (pf ? 1 : 0)) {
     case 2: k_quantize<BF16, 1><<<grid, 256, 0, stream>>>(xp, M, K, ldx, Mp, tags, codes, qsum, corr, act_scales); break;
     case 3: k_quantize<BF16, 1, false, true><<<grid, 256, 0, stream>>>(xp, M, K, ldx, Mp, tags, codes, qsum, corr, act_scales); break;
