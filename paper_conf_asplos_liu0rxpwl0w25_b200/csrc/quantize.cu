@@ -312,7 +312,7 @@ __global__ void __launch_bounds__(256, PF ? 3 : 4) k_quantize(const uint16_t* __
 // blocks (256 B apart, same banks) land in different bank halves.
 __device__ __forceinline__ int64_t swz(int64_t k) { return k ^ (((k >> 7) & 1) << 5); }
 
-template <bool BF16, int NW>
+template <bool BF16, int NW, int R>
 __global__ void __launch_bounds__(NW * 32, 2) k_quantize_perm(const uint16_t* __restrict__ x, int64_t M,
                                                        int64_t K, int64_t ldx, int64_t Mp,
                                                        TagMask tags,
@@ -321,13 +321,16 @@ __global__ void __launch_bounds__(NW * 32, 2) k_quantize_perm(const uint16_t* __
                                                        int16_t* __restrict__ qsum,
                                                        float* __restrict__ corr,
                                                        float* __restrict__ scales) {
+  // R rows per step (R = 2 for K <= 16384): the per-row chain -- gather pass, barrier, FMPQ
+  // pass, barrier -- is latency-bound, and a K = 8192 row has only 8 groups of 8 blocks for 16
+  // warps; two rows per step fill every warp in pass 2 and double the work per barrier
   extern __shared__ __align__(128) uint8_t smem[];
   asm volatile("griddepcontrol.launch_dependents;");                  // see k_quantize
   uint64_t* full = reinterpret_cast<uint64_t*>(smem);                 // [nbuf] (<= 16)
   uint16_t* p16 = reinterpret_cast<uint16_t*>(smem + 128);            // [K] permutation
-  uint16_t* prow = p16 + K;                                           // [K] permuted row (swizzled)
-  uint16_t* rows = prow + K;                                          // [nbuf][K] input rows
-  __shared__ float s_part[NW];
+  uint16_t* prow = p16 + K;                                           // [R][K] permuted rows (swizzled)
+  uint16_t* rows = prow + R * K;                                      // [nbuf][R][K] input rows
+  __shared__ float s_part[R][NW];
   __shared__ uint32_t s_tags[kMaxBlocks / 32];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int bl = lane >> 2, sub = lane & 3;
@@ -346,90 +349,110 @@ __global__ void __launch_bounds__(NW * 32, 2) k_quantize_perm(const uint16_t* __
   __syncthreads();
   // A row arrives as kChunks bulk copies issued by lane 0 of different warps: one issuing
   // thread's bulk copies complete one after another (profiles/r01/probe_stream.txt), several
-  // issuers overlap.  Thread 0 posts the row's byte count; the chunks may land before or after.
+  // issuers overlap.  Thread 0 posts the step's byte count; the chunks may land before or after.
+  // Step i of this CTA holds rows R (blockIdx.x + i gridDim.x) + r, r < R.
   constexpr int kChunks = NW < 8 ? NW : 8;
   const uint32_t chunk = row_bytes / kChunks;          // K % 128 == 0 -> a multiple of 32 B
   const bool issuer = lane == 0 && warp < kChunks;
-  if (issuer) {
-    for (int i = 0; i < nbuf; ++i) {
-      const int64_t m = blockIdx.x + (int64_t)i * gridDim.x;
-      if (m >= M) break;
-      if (warp == 0) sm100::mbar_arrive_expect_tx(&full[i], row_bytes);
-      sm100::bulk_load(reinterpret_cast<uint8_t*>(rows + (int64_t)i * K) + warp * chunk,
-                       reinterpret_cast<const uint8_t*>(x + m * ldx) + warp * chunk, chunk, &full[i]);
-    }
-  }
+  auto load_step = [&](int64_t st, int buf) {          // issuer threads only
+    const int64_t m0 = st * R;
+    const int nr = (int)min((int64_t)R, M - m0);
+    if (nr <= 0) return;
+    if (warp == 0) sm100::mbar_arrive_expect_tx(&full[buf], row_bytes * (uint32_t)nr);
+    for (int r = 0; r < nr; ++r)
+      sm100::bulk_load(reinterpret_cast<uint8_t*>(rows + ((int64_t)buf * R + r) * K) + warp * chunk,
+                       reinterpret_cast<const uint8_t*>(x + (m0 + r) * ldx) + warp * chunk, chunk, &full[buf]);
+  };
+  const int64_t nsteps = (Mp + R - 1) / R;
+  if (issuer)
+    for (int i = 0; i < nbuf; ++i) load_step(blockIdx.x + (int64_t)i * gridDim.x, i);
   int it = 0;
-  for (int64_t m = blockIdx.x; m < Mp; m += gridDim.x, ++it) {
+  for (int64_t st = blockIdx.x; st < nsteps; st += gridDim.x, ++it) {
     const int buf = it % nbuf;
-    float cpart = 0.f;
-    if (m < M) {
+    const int64_t m0 = st * R;
+    const int nr = (int)max((int64_t)0, min((int64_t)R, M - m0));   // real rows of this step
+    float cpart[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) cpart[r] = 0.f;
+    if (nr > 0) {
       sm100::mbar_wait(&full[buf], (uint32_t)((it / nbuf) & 1));
-      // pass 1: gather.  Thread t moves output channels 2t, 2t+1 (+ 2*blockDim.x steps):
-      // consecutive threads read consecutive indices (and, for the mostly ascending calibrated
-      // permutations, consecutive input channels) -- no bank conflicts -- and write the pair
-      // as one word at its swizzled position (see kSwz).
-      const uint16_t* row = rows + (int64_t)buf * K;
+      // pass 1: gather.  Thread t moves output channels 2t, 2t+1 (+ 2*blockDim.x steps) of each
+      // row: consecutive threads read consecutive indices (and, for the mostly ascending
+      // calibrated permutations, consecutive input channels) -- no bank conflicts -- and write
+      // the pair as one word at its swizzled position.
       for (int64_t k = 2 * threadIdx.x; k < K; k += 2 * blockDim.x) {
         const uint32_t pi = *reinterpret_cast<const uint32_t*>(p16 + k);
-        const uint32_t h = (uint32_t)row[pi & 0xFFFFu] | ((uint32_t)row[pi >> 16] << 16);
-        *reinterpret_cast<uint32_t*>(prow + swz(k)) = h;
-      }
-      __syncthreads();   // prow complete; row buffer `buf` free
-      if (issuer) {
-        const int64_t mn = m + (int64_t)nbuf * gridDim.x;   // refill the freed buffer
-        if (mn < M) {
-          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-          if (warp == 0) sm100::mbar_arrive_expect_tx(&full[buf], row_bytes);
-          sm100::bulk_load(reinterpret_cast<uint8_t*>(rows + (int64_t)buf * K) + warp * chunk,
-                           reinterpret_cast<const uint8_t*>(x + mn * ldx) + warp * chunk, chunk, &full[buf]);
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+          if (r >= nr) break;
+          const uint16_t* row = rows + ((int64_t)buf * R + r) * K;
+          const uint32_t h = (uint32_t)row[pi & 0xFFFFu] | ((uint32_t)row[pi >> 16] << 16);
+          *reinterpret_cast<uint32_t*>(prow + (int64_t)r * K + swz(k)) = h;
         }
       }
-      // pass 2: FMPQ on the permuted row, the lane layout of k_quantize (reads conflict-free
-      // thanks to the swizzle: the 8 blocks of a warp step sit 256 B apart)
-      uint8_t* crow = codes + m * K + sub * 8;
-      for (int g = warp; g < ngroups; g += NW) {
-        const int b = g * 8 + bl;
-        const bool bvalid = b < nb;
-        float v[32];
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-          uint4 raw = make_uint4(0, 0, 0, 0);
-          if (bvalid) raw = *reinterpret_cast<const uint4*>(prow + swz((int64_t)b * kBlockK + 32 * j + sub * 8));
-          float t[8];
-          unpack8<BF16>(raw, t);
-#pragma unroll
-          for (int i = 0; i < 8; ++i) v[8 * j + i] = t[i];
+    }
+    __syncthreads();   // prow complete; row buffer `buf` free
+    if (issuer && nr > 0) {
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      load_step(st + (int64_t)nbuf * gridDim.x, buf);   // refill the freed buffer
+    }
+    // pass 2: FMPQ on the permuted rows, the lane layout of k_quantize (reads conflict-free
+    // thanks to the swizzle: the 8 blocks of a warp step sit 256 B apart); padding rows
+    // (M <= m < Mp) get zero scales and code sums
+    for (int gg = warp; gg < R * ngroups; gg += NW) {
+      const int r = gg / ngroups, g = gg % ngroups;
+      const int64_t m = m0 + r;
+      if (m >= Mp) continue;
+      const int b = g * 8 + bl;
+      const bool bvalid = b < nb;
+      if (r >= nr) {
+        if (bvalid && sub == 0) {
+          scales[(int64_t)b * Mp + m] = 0.f;
+          qsum[(int64_t)b * Mp + m] = 0;
         }
-        const bool is8 = bvalid && ((s_tags[b >> 5] >> (b & 31)) & 1u);
-        const LaneOut o = quantize32(v, is8);
-        if (bvalid) {
-          uint8_t* cb = crow + b * kBlockK;
+        continue;
+      }
+      float v[32];
 #pragma unroll
-          for (int j = 0; j < 4; ++j) *reinterpret_cast<uint2*>(cb + 32 * j) = o.c[j];
-          if (sub == 0) {
-            scales[(int64_t)b * Mp + m] = o.s;
-            qsum[(int64_t)b * Mp + m] = (int16_t)o.q;
-            if (!is8) cpart = __fadd_rn(cpart, __fmul_rn(o.s, (float)o.q));
+      for (int j = 0; j < 4; ++j) {
+        uint4 raw = make_uint4(0, 0, 0, 0);
+        if (bvalid) raw = *reinterpret_cast<const uint4*>(prow + (int64_t)r * K + swz((int64_t)b * kBlockK + 32 * j + sub * 8));
+        float t[8];
+        unpack8<BF16>(raw, t);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) v[8 * j + i] = t[i];
+      }
+      const bool is8 = bvalid && ((s_tags[b >> 5] >> (b & 31)) & 1u);
+      const LaneOut o = quantize32(v, is8);
+      if (bvalid) {
+        uint8_t* cb = codes + m * K + sub * 8 + b * kBlockK;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) *reinterpret_cast<uint2*>(cb + 32 * j) = o.c[j];
+        if (sub == 0) {
+          scales[(int64_t)b * Mp + m] = o.s;
+          qsum[(int64_t)b * Mp + m] = (int16_t)o.q;
+          if (!is8) {
+#pragma unroll
+            for (int rr = 0; rr < R; ++rr)
+              if (rr == r) cpart[rr] = __fadd_rn(cpart[rr], __fmul_rn(o.s, (float)o.q));
           }
         }
       }
-    } else {
-      for (int b = threadIdx.x; b < nb; b += blockDim.x) {
-        scales[(int64_t)b * Mp + m] = 0.f;
-        qsum[(int64_t)b * Mp + m] = 0;
-      }
-      __syncthreads();   // matches the pass-1 barrier of the other branch (uniform per CTA)
     }
-    cpart = __fadd_rn(cpart, __shfl_xor_sync(0xffffffffu, cpart, 4));
-    cpart = __fadd_rn(cpart, __shfl_xor_sync(0xffffffffu, cpart, 8));
-    cpart = __fadd_rn(cpart, __shfl_xor_sync(0xffffffffu, cpart, 16));
-    if (lane == 0) s_part[warp] = cpart;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      float c = cpart[r];
+      c = __fadd_rn(c, __shfl_xor_sync(0xffffffffu, c, 4));
+      c = __fadd_rn(c, __shfl_xor_sync(0xffffffffu, c, 8));
+      c = __fadd_rn(c, __shfl_xor_sync(0xffffffffu, c, 16));
+      if (lane == 0) s_part[r][warp] = c;
+    }
     __syncthreads();   // s_part complete; prow free
-    if (threadIdx.x == 0) {
+    if (threadIdx.x < R && m0 + threadIdx.x < Mp) {
+      const int r = threadIdx.x;
       float c = 0.f;
-      for (int i = 0; i < NW; ++i) c = __fadd_rn(c, s_part[i]);
-      corr[m] = __fmul_rn(8.f, c);
+      for (int i = 0; i < NW; ++i) c = __fadd_rn(c, s_part[r][i]);
+      corr[m0 + r] = __fmul_rn(8.f, c);
     }
   }
 }
@@ -677,21 +700,24 @@ static cudaError_t launch_qp(const void* x, int64_t M, int64_t K, int64_t ldx, c
     return cudaGetLastError();
   }
   const int64_t row_bytes = K * 2;
-  // rows in flight per CTA: ~64 KB of staged input, at least 2 (double buffering)
-  int nbuf = (int)std::max<int64_t>(2, std::min<int64_t>(8, (64 << 10) / row_bytes));
+  // R rows per step when two CTAs of 2-row steps with double buffering fit one SM (K <= 8192:
+  // p16 + 2 staged rows + 2 x 2 input rows = 7 rows = 112 KB); else one row per step with
+  // ~64 KB of staged input rows in flight
+  const int R = (128 + (size_t)row_bytes * 7 <= (113u << 10)) ? 2 : 1;
+  int nbuf = R == 2 ? 2 : (int)std::max<int64_t>(2, std::min<int64_t>(8, (64 << 10) / row_bytes));
   const size_t cap = 200u << 10;
-  while (nbuf > 1 && 128 + (size_t)row_bytes * (2 + nbuf) > cap) --nbuf;
-  const size_t smem = 128 + (size_t)row_bytes * (2 + nbuf);
+  while (nbuf > 1 && 128 + (size_t)row_bytes * (1 + R + (size_t)nbuf * R) > cap) --nbuf;
+  const size_t smem = 128 + (size_t)row_bytes * (1 + R + (size_t)nbuf * R);
   int dev = 0, nsm = 148, per_sm = 1;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
   constexpr int NW = 16;   // 16 warps: the gather is latency-bound at one or two CTAs per SM
-  auto kern = k_quantize_perm<BF16, NW>;
+  auto kern = R == 2 ? k_quantize_perm<BF16, NW, 2> : k_quantize_perm<BF16, NW, 1>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, NW * 32, smem);
   if (e != cudaSuccess) return e;
-  const int64_t grid = std::max<int64_t>(1, std::min<int64_t>(L.Mp, (int64_t)nsm * std::max(per_sm, 1)));
+  const int64_t grid = std::max<int64_t>(1, std::min<int64_t>(ceil_div(L.Mp, (int64_t)R), (int64_t)nsm * std::max(per_sm, 1)));
   kern<<<(unsigned)grid, NW * 32, smem, stream>>>(
       static_cast<const uint16_t*>(x), M, K, ldx, L.Mp, tags, perm, nbuf, base + L.codes_off,
       reinterpret_cast<int16_t*>(base + L.qsum_off), reinterpret_cast<float*>(base + L.corr_off),
