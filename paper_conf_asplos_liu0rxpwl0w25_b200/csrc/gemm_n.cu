@@ -70,6 +70,9 @@
 #ifndef COMET_WIDEN_WAIT_PLAIN
 #define COMET_WIDEN_WAIT_PLAIN 0   // experiment: plain try_wait loop for the widen warps' full wait
 #endif
+#ifndef COMET_LDTM_X64
+#define COMET_LDTM_X64 0   // 1: the promotion's 64-column rounds as one 32x32b.x64 load instead of two .x32
+#endif
 #ifndef COMET_STUB
 #define COMET_STUB 0   // timing experiments only (wrong results): 1 MMA kind fixed, 2 promotion scale/kind fixed, 4 no scale loads, 8 no epilogue stores
 #endif
@@ -637,7 +640,7 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG, GS>::THREADS, 1)
 #pragma unroll
           for (int b = 0; b < COLS / 64; ++b) {
             uint32_t v[64];
-            tmem_ld_32x32b<64>(taddr + b * 64, v);
+            if (COMET_LDTM_X64) tmem_ld_32x32b_x64(taddr + b * 64, v); else tmem_ld_32x32b<64>(taddr + b * 64, v);
             if (b == 0) {
               const float s = row_scale();
               s2 = make_float2(s, s);
