@@ -73,8 +73,17 @@
 #ifndef COMET_LDTM_X64
 #define COMET_LDTM_X64 0   // 1: the promotion's 64-column rounds as one 32x32b.x64 load instead of two .x32
 #endif
+#ifndef COMET_PREWIDENED_UB
+#define COMET_PREWIDENED_UB 0   // SURVEY §8(d) ablation, timing only: B arrives pre-widened by TMA (2x weight bytes), no widening work
+#endif
+#ifndef COMET_PROMO_SCALAR
+#define COMET_PROMO_SCALAR 0    // SURVEY §8(d) ablation: scalar FFMA promotion instead of FFMA2
+#endif
 #ifndef COMET_STUB
 #define COMET_STUB 0   // timing experiments only (wrong results): 1 MMA kind fixed, 2 promotion scale/kind fixed, 4 no scale loads, 8 no epilogue stores
+#endif
+#ifndef COMET_N256_SMEM_KB
+#define COMET_N256_SMEM_KB COMET_SMEM_BUDGET_KB
 #endif
 #ifndef COMET_N256_NPW
 #define COMET_N256_NPW 2   // promotion warpgroups of the 256-wide tile
@@ -146,10 +155,13 @@ struct CfgN {
   // the scale ring has S + NACC slots (reuse is implied by the slot-free barrier, see below).
   // output staging for the TMA-store epilogue: per promotion WG two [128 rows][64 B] buffers
   // staging buffers per promotion WG: COMET_NSTAGE when the pipeline keeps >= 4 slots, else 2
-  static constexpr int NSTAGE = (COMET_SMEM_BUDGET_KB * 1024 - NPW * COMET_NSTAGE * 8192) / (SLOT_BYTES + BM * 4) >= 4
+  // shared-memory budget of the pipeline; COMET_N256_SMEM_KB overrides it for the 256-wide pair
+  // tile alone (the pipeline-depth ablation: 160 -> S = 3)
+  static constexpr int BUDGET_KB = (BN == 256 && CG == 2) ? COMET_N256_SMEM_KB : COMET_SMEM_BUDGET_KB;
+  static constexpr int NSTAGE = (BUDGET_KB * 1024 - NPW * COMET_NSTAGE * 8192) / (SLOT_BYTES + BM * 4) >= 4
                                     ? COMET_NSTAGE : 2;
   static constexpr int STAGE_BYTES = NPW * NSTAGE * 8192;
-  static constexpr int S_RAW = (COMET_SMEM_BUDGET_KB * 1024 - STAGE_BYTES) / (SLOT_BYTES + BM * 4);
+  static constexpr int S_RAW = (BUDGET_KB * 1024 - STAGE_BYTES) / (SLOT_BYTES + BM * 4);
   // S must be even when two widen groups or two MMA issuers take alternate K-blocks: a waiter
   // that sees only every other K-block must see every phase of each slot it waits on (parity
   // waits cannot tell phase p from p + 2).  With an odd S a role could pass the wait for
@@ -289,12 +301,20 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG, GS>::THREADS, 1)
           if (diag_ablate(P) & 32) {                       // diagnostic: no global loads
             mbar_arrive(&full[s]);
           } else {
-            mbar_arrive_expect_tx(&full[s], C::X_BYTES + C::WP_BYTES + sbytes + gbytes + qbytes);
+            mbar_arrive_expect_tx(&full[s], C::X_BYTES + (COMET_PREWIDENED_UB ? C::B_BYTES : C::WP_BYTES) + sbytes + gbytes + qbytes);
             const uint8_t* src = reinterpret_cast<const uint8_t*>(P.scales) + ((kb * 7 + m0 / 128) % 32) * 24576;
             if (COMET_ABLATE_TMA2D & 1) bulk_load(sX(s), src, C::X_BYTES, &full[s]);
             else tma_load_2d(sX(s), &P.map_x, &full[s], kb * 128, m0);
-            if (COMET_ABLATE_TMA2D & 2) bulk_load(sWp(s), src + C::X_BYTES, C::WP_BYTES, &full[s]);
-            else tma_load_2d(sWp(s), &P.map_w, &full[s], kb * 64, n0);
+            if (COMET_PREWIDENED_UB) {
+              // the B half arrives as 128 rows x 128 B (an 8-bit weight tile's shape and bytes; the
+              // values are the activation plane's -- timing only) straight into the MMA operand slot
+              const int rb = (int)((n0 % (P.Mp > 256 ? P.Mp - 128 : 128)) & ~127);
+              tma_load_2d(sB(s), &P.map_x, &full[s], kb * 128, rb);
+            } else if (COMET_ABLATE_TMA2D & 2) {
+              bulk_load(sWp(s), src + C::X_BYTES, C::WP_BYTES, &full[s]);
+            } else {
+              tma_load_2d(sWp(s), &P.map_w, &full[s], kb * 64, n0);
+            }
             if (sbytes) bulk_load(sS + sc * BM, P.scales + (int64_t)kb * P.Mp + m0, sbytes, &full[s]);
             if (GS) {
               bulk_load(sG + sc * BN, P.w_scales + (int64_t)kb * P.N + ng0, gbytes, &full[s]);
@@ -444,7 +464,7 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG, GS>::THREADS, 1)
 #pragma unroll
           for (int i = 0; i < RPT; ++i) {
             const int row = t + 128 * i;
-            if (row < C::WROWS && !(diag_ablate(P) & 64)) {   // 64: diagnostic, no widen loads
+            if (row < C::WROWS && !(diag_ablate(P) & 64) && !COMET_PREWIDENED_UB) {   // 64: diagnostic, no widen loads
               const uint32_t src = smem_u32(sWp(s)) + row * 64;
               const int sw64 = (row >> 1) & 3;            // TMA 64-byte swizzle of the packed row
 #pragma unroll
@@ -456,7 +476,7 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG, GS>::THREADS, 1)
 #pragma unroll
           for (int i = 0; i < RPT; ++i) {
             const int row = t + 128 * i;
-            if (row >= C::WROWS || (diag_ablate(P) & 4)) break;
+            if (row >= C::WROWS || (diag_ablate(P) & 4) || COMET_PREWIDENED_UB) break;
             const uint32_t dst = smem_u32(sB(s)) + row * 128;
             const int sw128 = row & 7;                    // UMMA 128-byte swizzle of the widened row
 #pragma unroll
@@ -666,10 +686,15 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG, GS>::THREADS, 1)
 #pragma unroll
               for (int c = 0; c < 64; c += 2) {
                 const int a = b * 64 + c;
-                const float2 y = ffma2(make_float2(__uint_as_float(v[c]), __uint_as_float(v[c + 1])), s2,
-                                       make_float2(acc[a], acc[a + 1]));
-                acc[a] = y.x;
-                acc[a + 1] = y.y;
+                if (COMET_PROMO_SCALAR) {
+                  acc[a] = __fmaf_rn(__uint_as_float(v[c]), s2.x, acc[a]);
+                  acc[a + 1] = __fmaf_rn(__uint_as_float(v[c + 1]), s2.y, acc[a + 1]);
+                } else {
+                  const float2 y = ffma2(make_float2(__uint_as_float(v[c]), __uint_as_float(v[c + 1])), s2,
+                                         make_float2(acc[a], acc[a + 1]));
+                  acc[a] = y.x;
+                  acc[a + 1] = y.y;
+                }
               }
             }
           }
