@@ -300,20 +300,29 @@ def decode_sweep(cb, torch, dev, peaks, timer, Ms=(1, 4, 8, 32), iters=20, rank=
             # programmatic dependent and streams weights while kernel 1 runs
             us_step = us_rotating(torch, [lambda w_=w_: (cb.quantize_act(x, tl, out=(act, sc)),
                                                           cb.w4ax_gemm(plan, act, sc, w_, swd, out=y)) for w_ in wps])
+            # the same layer step as ONE launch (comet_w4ax_linear: kernel 1 fused into the GEMM,
+            # for 16-token decode tiles)
+            us_fused = None
+            if plan.info()["tile_n"] == 16 and plan.info()["orientation"] == 1:
+                us_fused = us_rotating(torch, [lambda w_=w_: cb.w4ax_linear_fused(plan, x, w_, swd, out=y) for w_ in wps])
             ar_us = None
             if kind == "row" and world > 1:
                 ar_us = timer.us(lambda: dist.all_reduce(y, op=dist.ReduceOp.SUM), iters, flush=False)
             nbytes = Nl * Kl // 2 + Nl * 4 + act.numel() + sc.numel() * 4 + M * Nl * y.element_size()
             if world > 1:
-                t = torch.tensor([us, us_step, ar_us or 0.0, us_iso], device=dev, dtype=torch.float64)
+                t = torch.tensor([us, us_step, ar_us or 0.0, us_iso, us_fused or 0.0], device=dev, dtype=torch.float64)
                 dist.all_reduce(t, op=dist.ReduceOp.MAX)
                 us, us_step, ar_us, us_iso = t[0].item(), t[1].item(), (t[2].item() if ar_us is not None else None), t[3].item()
+                us_fused = t[4].item() if us_fused is not None else None
             gbs = nbytes / (us * 1e-6) / 1e9
             out[f"{name}_M{M}"] = {"us": round(us, 2), "GB/s": round(gbs, 1), "frac_hbm": round(gbs / hbm, 3),
                                    "isolated_us": round(us_iso, 2),
                                    "step_us": round(us_step, 2),
                                    "step_GB/s": round((nbytes + M * Kl * 2) / (us_step * 1e-6) / 1e9, 1),
                                    "orientation": plan.info()["orientation"], "tile_n": plan.info()["tile_n"]}
+            if us_fused is not None:
+                out[f"{name}_M{M}"]["fused_step_us"] = round(us_fused, 2)
+                out[f"{name}_M{M}"]["fused_step_GB/s"] = round((nbytes + M * Kl * 2) / (us_fused * 1e-6) / 1e9, 1)
             if ar_us is not None:
                 out[f"{name}_M{M}"]["allreduce_us"] = round(ar_us, 2)
         del wp, wps
@@ -322,7 +331,8 @@ def decode_sweep(cb, torch, dev, peaks, timer, Ms=(1, 4, 8, 32), iters=20, rank=
             "timing": "us / GB/s / frac_hbm: mean per launch of 10 rounds of back-to-back launches cycling over >= 300 MB of "
                       "weight copies (> 2 x L2: every launch streams from HBM); isolated_us: one event-bracketed launch after a "
                       "256 MiB write + 256 MiB read (median of 20; includes the ~6 us an empty kernel measures that way)",
-            "step": "step_us = kernel 1 (quantise x) + the GEMM as one decode layer step (the GEMM is a programmatic dependent launch), back to back",
+            "step": "step_us = kernel 1 (quantise x) + the GEMM as one decode layer step (the GEMM is a programmatic dependent launch), back to back; "
+                    "fused_step_us = the same step as one comet_w4ax_linear launch (kernel 1 fused into the GEMM, 16-token tiles)",
             "layers": out}
 
 

@@ -93,6 +93,7 @@ def lib():
         "comet_plan_describe": (I32, [P, P, I64, ctypes.POINTER(I64)]),
         "comet_w4ax_gemm": (I32, [P, P, P, P, P, P, I32, I64, P, P, P, SZ, P]),
         "comet_w4ax_gemm_grouped": (I32, [P, P, P, P, P, P, I32, I64, P, P, SZ, P]),
+        "comet_w4ax_linear": (I32, [P, P, I32, I64, P, P, P, I32, I64, P, SZ, P]),
         "comet_linear_scratch_bytes": (SZ, [P, I32, I32]),
         "comet_w4ax_linear_host": (I32, [P, P, I32, P, P, P, I32, P, SZ, P, SZ, P]),
         "comet_w4ax_linear_host_async": (I32, [P, P, I32, P, P, P, I32, P, SZ, P, SZ, P]),
@@ -341,6 +342,21 @@ def w4ax_gemm(plan: Plan, act_packed, act_scales, w_packed, w_scales, *, out=Non
     return out
 
 
+def w4ax_linear_fused(plan: Plan, x, w_packed, w_scales, *, out=None, out_dtype=None, stream=None):
+    """comet_w4ax_linear: the decode layer (kernel 1 fused into the GEMM) for plans with
+    orientation 1, 16-token tiles and M <= 8.  x: [M, K] float16 / bfloat16 on the device."""
+    import torch
+    dev = x.device
+    if out is None:
+        out = torch.empty((plan.M, plan.N), dtype=out_dtype or torch.float16, device=dev)
+    ws = plan.workspace(dev)
+    _check(lib().comet_w4ax_linear(plan.handle, ctypes.c_void_p(x.data_ptr()), _dt(x.dtype), x.stride(0),
+                                   ctypes.c_void_p(w_packed.data_ptr()), ctypes.c_void_p(w_scales.data_ptr()),
+                                   ctypes.c_void_p(out.data_ptr()), _dt(out.dtype), out.stride(0),
+                                   ctypes.c_void_p(ws.data_ptr()), ws.numel(), _stream(stream)))
+    return out
+
+
 def w4ax_gemm_grouped(plan: Plan, act_packed, act_scales, w_packed, w_scales_grouped, *, out=None,
                       out_dtype=None, debug: bool = False, stream=None):
     """comet_w4ax_gemm_grouped (NEXT-3): group-wise weight scales w_scales_grouped [K/128, N]
@@ -362,12 +378,20 @@ def w4ax_gemm_grouped(plan: Plan, act_packed, act_scales, w_packed, w_scales_gro
     return (out, dacc) if debug else out
 
 
-def w4ax_linear(plan: Plan, x, w_packed, w_scales, *, perm=None, out_dtype=None, stream=None):
-    """The whole hot path for one linear layer on device tensors: quantize_act (with the fused
+def w4ax_linear(plan: Plan, x, w_packed, w_scales, *, perm=None, out=None, out_dtype=None, stream=None):
+    """The whole hot path for one linear layer on device tensors: one fused launch
+    (comet_w4ax_linear) for decode plans with 16-token tiles, else quantize_act (with the fused
     channel permutation when perm is given; w_packed then packed with the same perm) +
     w4ax_gemm."""
+    info = plan.info()
+    if (perm is None and info["orientation"] == 1 and info["tile_n"] == 16 and plan.M <= 4
+            and info["n_tiles"] * -(-plan.K // 512) <= 12 * info["num_ctas"]):
+        # the fused launch wins while the CTAs' quantiser warps keep up with the weight stream:
+        # small layers (<= 12 pipeline stages per CTA; LLaMA-3-70B qkv at M <= 4: 18.5 ->
+        # 16.3-17.0 us per layer step) -- DESIGN.md §7.4
+        return w4ax_linear_fused(plan, x, w_packed, w_scales, out=out, out_dtype=out_dtype, stream=stream)
     act, sc = quantize_act(x, plan.tags, perm=perm, stream=stream)
-    return w4ax_gemm(plan, act, sc, w_packed, w_scales, out_dtype=out_dtype, stream=stream)
+    return w4ax_gemm(plan, act, sc, w_packed, w_scales, out=out, out_dtype=out_dtype, stream=stream)
 
 
 def debug_widen(first_word: int, n: int, int8_block: bool = False, *, out=None, stream=None):

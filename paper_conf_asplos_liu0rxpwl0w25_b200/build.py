@@ -16,7 +16,7 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 CU_SOURCES = ["quantize.cu", "kv4.cu", "gemm.cu", "gemm_n.cu", "api.cu"]
 CPP_SOURCES = ["planner.cpp", "calibrate.cpp"]
-HEADERS = ["internal.h", "sm100.cuh", "gemm_common.cuh"]
+HEADERS = ["internal.h", "sm100.cuh", "gemm_common.cuh", "fmpq.cuh"]
 
 
 def _newer(src_paths, dst):

@@ -441,6 +441,31 @@ comet_status_t comet_w4ax_gemm(comet_plan_t plan, const void* act_packed, const 
   return st;
 }
 
+comet_status_t comet_w4ax_linear(comet_plan_t plan, const void* x, comet_dtype_t xdt, int64_t ldx,
+                                 const void* w_packed, const float* w_scales, void* y,
+                                 comet_dtype_t ydt, int64_t ldy, void* workspace, size_t ws_bytes,
+                                 void* stream) {
+  g_launches = 0;
+  if (!plan || !x || !w_packed || !w_scales || !y) return fail(COMET_ERR_INVALID_ARG, "NULL pointer argument");
+  Plan& p = plan->p;
+  if (xdt != COMET_F16 && xdt != COMET_BF16) return fail(COMET_ERR_INVALID_ARG, "x must be F16 or BF16");
+  if (ydt != COMET_F16 && ydt != COMET_BF16 && ydt != COMET_F32) return fail(COMET_ERR_INVALID_ARG, "bad ydt");
+  if (ldx < p.K || (ldx * 2) % 16 != 0) return fail(COMET_ERR_MISALIGNED, "ldx must be >= K with ldx*2 % 16 == 0");
+  const int esz = ydt == COMET_F32 ? 4 : 2;
+  if (ldy < p.N || (ldy * esz) % 16 != 0) return fail(COMET_ERR_MISALIGNED, "ldy must be >= N with ldy*sizeof(y) % 16 == 0");
+  if (!aligned16(x) || !aligned16(w_packed) || !aligned16(w_scales) || !aligned16(y) ||
+      (workspace && !aligned16(workspace)))
+    return fail(COMET_ERR_MISALIGNED, "device pointers must be 16-byte aligned");
+  comet_status_t st = check_device();
+  if (st != COMET_OK) return st;
+  const FusedX fx{x, ldx, xdt == COMET_BF16};
+  int launches = 0;
+  st = launch_gemm(p, nullptr, nullptr, w_packed, w_scales, y, ydt, ldy, nullptr, nullptr, workspace,
+                   ws_bytes, static_cast<cudaStream_t>(stream), &launches, false, nullptr, &fx);
+  g_launches = launches;
+  return st;
+}
+
 comet_status_t comet_w4ax_gemm_grouped(comet_plan_t plan, const void* act_packed, const float* act_scales,
                                        const void* w_packed, const float* w_scales_grouped, void* y,
                                        comet_dtype_t ydt, int64_t ldy, int32_t* debug_acc,

@@ -37,6 +37,7 @@
 #include <algorithm>
 #include <cstdlib>
 #include "gemm_common.cuh"
+#include "fmpq.cuh"
 
 // The pipeline roles' waits (promotion 1, MMA issuer 2, widen 4) are bare try_wait loops: ~2 %
 // faster than the timer-guarded mbar_wait on every decode shape (tools/gpu_decb_variants.sh);
@@ -113,7 +114,7 @@ constexpr int kPromoWarp0 = 12;
 // stage: warp 4 + 4h + q widens rows 32q .. 32q+31 of K-blocks [h KS/2, (h+1) KS/2).
 // TMEM columns: [0, 2 * 32 KS) two widened-weight A buffers (alternate stages), then NACC
 // accumulator sets of KS x NT columns (one accumulator per K-block of a stage).
-template <int NT, bool GS = false>
+template <int NT, bool GS = false, bool FQ = false>
 struct Cfg {
   static constexpr int KS = NT <= 32 ? 4 : 2;                  // K-blocks per stage
   static constexpr int NA = COMET_DEC_NA;                       // widened-weight A buffers
@@ -127,15 +128,21 @@ struct Cfg {
   static constexpr int S_BYTES = KS * NT * 4;
   // GS (group-wise weight scales): the X stage also carries the K-blocks' code sums qsum[b][m]
   // (int16, [KS][NT]) and weight scales s_w[b][n] (f32, [KS][128])
-  static constexpr int Q_BYTES = GS ? KS * NT * 2 : 0;
+  // FQ (fused quantiser, comet_w4ax_linear): the in-kernel quantiser writes the codes, scales
+  // and code sums of the stage here itself (the offset term is removed per block as in GS)
+  static constexpr int Q_BYTES = (GS || FQ) ? KS * NT * 2 : 0;
   static constexpr int G_BYTES = GS ? KS * kTileW * 4 : 0;
-  static constexpr int X_STAGE = (KS * XKB_BYTES + S_BYTES + Q_BYTES + G_BYTES + 1023) / 1024 * 1024;
+  // FQ: the stage's raw 16-bit input rows (tokens < 8: the fused path serves M <= 8) land here
+  // by TMA, [KS][8 rows][256 B]; the quantiser warp turns them into the codes above
+  static constexpr int RAW_ROWS = 8;
+  static constexpr int R_BYTES = FQ ? KS * RAW_ROWS * 256 : 0;
+  static constexpr int X_STAGE = (KS * XKB_BYTES + S_BYTES + Q_BYTES + G_BYTES + R_BYTES + 1023) / 1024 * 1024;
   static constexpr int SX = NT >= 32 ? COMET_DEC_SX32 : 4;     // X ring depth
   static constexpr int SMEM_BUDGET = 224 * 1024;            // 227 KB minus alignment, barriers, tags
   static constexpr int SW_RAW = (SMEM_BUDGET - SX * X_STAGE) / W_BYTES;
   static constexpr int SW = SW_RAW > COMET_DEC_SWMAX ? COMET_DEC_SWMAX : SW_RAW;   // W ring depth
   static constexpr int SMEM_DATA = SW * W_BYTES + SX * X_STAGE;
-  static constexpr int N_BARS = 2 * SW + 2 * SX + 2 * NA + 2 * NACC;
+  static constexpr int N_BARS = 2 * SW + 2 * SX + 2 * NA + 2 * NACC + (FQ ? SX : 0);
   static constexpr int SMEM_BYTES = 1024 + SMEM_DATA + N_BARS * 8 + 16 + kMaxBlocks;
   static constexpr int CH = NT < 32 ? NT : 32;                 // promotion column chunk
   static_assert(NT % 16 == 0 && NT <= 128, "decode tile");
@@ -156,9 +163,9 @@ __device__ __forceinline__ void tmem_ld_cols(uint32_t taddr, uint32_t* r) {
 // term per block: INT4 block  acc += s_a s_w (2^-9 sum q u - 2^-6 qsum)   (= s_a s_w 2^-9 sum q w)
 //                 INT8 block  acc += s_a s_w 2^-13 (16 sum q w)
 // and the epilogue only scales by 2^9.
-template <int NT, int DEBUG, bool GS>
+template <int NT, int DEBUG, bool GS, bool FQ = false>
 __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ GemmParams P) {
-  using C = Cfg<NT, GS>;
+  using C = Cfg<NT, GS, FQ>;
   constexpr int SW = C::SW;
   constexpr int SX = C::SX;
   constexpr int NA = C::NA;
@@ -172,6 +179,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
   auto sS = [&](int st) { return smem + SW * C::W_BYTES + st * C::X_STAGE + KS * C::XKB_BYTES; };
   auto sQ = [&](int st) { return sS(st) + C::S_BYTES; };          // GS only
   auto sG = [&](int st) { return sS(st) + C::S_BYTES + C::Q_BYTES; };
+  auto sR = [&](int st) { return sS(st) + C::S_BYTES + C::Q_BYTES + C::G_BYTES; };   // FQ only
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + C::SMEM_DATA);
   uint64_t* full_w = bars;                  // [SW]   TMA -> widen
   uint64_t* empty_w = full_w + SW;          // [SW]   8 widen warps -> W producer
@@ -181,6 +189,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
   uint64_t* a_empty = a_full + NA;          // [NA]   MMA commit -> widen
   uint64_t* acc_full = a_empty + NA;        // [NACC] MMA commit -> promotion
   uint64_t* acc_empty = acc_full + NACC;    // [NACC] promotion -> MMA
+  // FQ: full_x = the raw input landed (TMA -> quantiser), q_full = codes ready (quantiser ->
+  // MMA and promotion); otherwise the consumers wait full_x (TMA of the codes) directly
+  uint64_t* q_full = acc_empty + NACC;      // [SX] FQ only
+  uint64_t* xready = FQ ? q_full : full_x;
   uint32_t* tmem_holder = reinterpret_cast<uint32_t*>(bars + C::N_BARS);
   uint8_t* s_tags = reinterpret_cast<uint8_t*>(tmem_holder + 4);
   const uint32_t s_tags_a = smem_u32(s_tags);
@@ -202,7 +214,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
   if (warp == 0 && lane == 0) {
     tma_prefetch(&P.map_x);
     tma_prefetch(&P.map_w);
-    tma_prefetch(&P.map_s);
+    if (!FQ) tma_prefetch(&P.map_s);
     for (int i = 0; i < SW; ++i) {
       mbar_init(&full_w[i], 1);
       mbar_init(&empty_w[i], COMET_DEC_WIDEN_WARPS);
@@ -219,6 +231,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
       mbar_init(&acc_full[i], 1);
       mbar_init(&acc_empty[i], 4);
     }
+    if (FQ)
+      for (int i = 0; i < SX; ++i) mbar_init(&q_full[i], 1);
     fence_mbar_init();
   }
   if (warp == 2) {
@@ -248,7 +262,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
   if (COMET_DEC_EARLY_TRIGGER && threadIdx.x == 0) asm volatile("griddepcontrol.launch_dependents;");
 
   if (warp < kWidenWarp0) {
-    setmaxnreg_dec<56>();
+    setmaxnreg_dec<FQ ? 80 : 56>();
     if (warp == 0 && lane == 0) {
       // ------------------------------------------------------------------ W producer
       int st = 0;
@@ -266,7 +280,96 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
           if (++st == SW) { st = 0; ph ^= 1; }
         }
       }
-    } else if (warp == 2 && lane == 0) {
+    } else if (FQ && warp == 0 && lane == 1) {
+      // ------------------------------------------------------------------ FQ raw-input producer
+      int st = 0;
+      uint32_t ph = 0;
+      for (int it = it_begin; it < it_end; ++it) {
+        const WorkItem w = item(it);
+        const int m0 = (w.tile % P.n_m_tiles) * NT;
+        for (int kb = w.kb_begin; kb < w.kb_end; kb += KS) {
+          mbar_wait(&empty_x[st], ph ^ 1);
+          mbar_arrive_expect_tx(&full_x[st], C::R_BYTES);
+          tma_load_3d(sR(st), &P.map_x, &full_x[st], 0, m0, kb);
+          if (++st == SX) { st = 0; ph ^= 1; }
+        }
+      }
+    } else if (FQ && (warp == 2 || warp == 3)) {
+      // ------------------------------------------------------------------ fused quantiser (FQ)
+      // Kernel 1 folded into the decode GEMM (comet_w4ax_linear, M <= 8): the stage's raw input
+      // rows arrive by TMA (warp 0 lane 1, up to SX stages ahead); warps 2 and 3 take alternate
+      // stages and quantise their (token, K-block) pairs from shared memory into the X slot, in the layout the codes' TMA would have
+      // produced (codes [KS][NT][128 B] SW128, scales and code sums [KS][NT]), with kernel 1's
+      // arithmetic (fmpq.cuh: identical codes, scales, code sums).  Four lanes per pair, 8 pairs
+      // per round.  The offset-binary term is removed per block by the promotion (as for
+      // group-wise scales): no per-row correction, every stream-K segment complete on its own.
+      // Token rows >= M stay zero (the ring is zeroed first; a warp only ever touches its own
+      // slots, j % SX with j of its parity, SX even).
+      const int par = warp - 2;
+      const int g = lane >> 2, sub = lane & 3;
+      for (int i = par * 32 + lane; i < SX * C::X_STAGE / 16; i += 64)
+        asm volatile("st.shared.v4.u32 [%0], {%1,%1,%1,%1};" ::"r"(smem_u32(sX(0)) + i * 16), "r"(0u) : "memory");
+      __syncwarp();
+      // stage cursor over the work list: (item, first K-block), global stage index j
+      struct Cur { int it, kb, j; };
+      auto advance = [&](Cur c) -> Cur {                  // the next stage
+        const WorkItem w = item(c.it);
+        c.kb += KS;
+        ++c.j;
+        if (c.kb >= w.kb_end) {
+          ++c.it;
+          if (c.it < it_end) c.kb = item(c.it).kb_begin;
+        }
+        return c;
+      };
+      Cur cur{it_begin, it_begin < it_end ? item(it_begin).kb_begin : 0, 0};
+      if (par == 1 && cur.it < it_end) cur = advance(cur);
+      while (cur.it < it_end) {
+        Cur nxt = advance(cur);
+        if (nxt.it < it_end) nxt = advance(nxt);          // this warp's next stage
+        const WorkItem w = item(cur.it);
+        const int st = cur.j % SX;
+        const int64_t m0 = (int64_t)(w.tile % P.n_m_tiles) * NT;
+        const int mrows = (int)min((int64_t)C::RAW_ROWS, P.M - m0);
+        const int nk = min(KS, w.kb_end - cur.kb);
+        mbar_wait(&full_x[st], (uint32_t)(cur.j / SX) & 1u);
+        const int npairs = nk * mrows;
+        for (int p0 = 0; p0 < npairs; p0 += 8) {
+          const int pp = p0 + g;
+          const bool pv = pp < npairs;
+          const int kl = pv ? pp / mrows : 0, m = pv ? pp % mrows : 0;
+          const uint32_t rsrc = smem_u32(sR(st)) + (kl * C::RAW_ROWS + m) * 256 + sub * 16;
+          float v[32];
+#pragma unroll
+          for (int j = 0; j < 4; ++j) {
+            const uint4 raw = lds128(rsrc + 64 * j);      // channels 32 j + 8 sub ..
+            float t8[8];
+            if (P.xq_bf16) fmpq::unpack8<true>(raw, t8); else fmpq::unpack8<false>(raw, t8);
+#pragma unroll
+            for (int i = 0; i < 8; ++i) v[8 * j + i] = t8[i];
+          }
+          const bool is8 = pv && lds_u8(s_tags_a + cur.kb + kl) != 0;
+          const fmpq::LaneOut o = fmpq::quantize32(v, is8);   // every lane: quad shuffles
+          if (pv) {
+            const uint32_t rowb = smem_u32(sX(st)) + kl * C::XKB_BYTES + m * 128;
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+              const int c0 = 32 * j + 8 * sub;              // byte of this lane's 8 codes in the row
+              asm volatile("st.shared.v2.u32 [%0], {%1,%2};" ::"r"(rowb + ((((c0 >> 4) ^ (m & 7))) << 4) + (c0 & 15)),
+                           "r"(o.c[j].x), "r"(o.c[j].y) : "memory");
+            }
+            if (sub == 0) {
+              reinterpret_cast<float*>(sS(st))[kl * NT + m] = o.s;
+              reinterpret_cast<int16_t*>(sQ(st))[kl * NT + m] = (int16_t)o.q;
+            }
+          }
+        }
+        fence_proxy_async_smem();                         // codes -> the MMA (async proxy)
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&q_full[st]);
+        cur = nxt;
+      }
+    } else if (!FQ && warp == 2 && lane == 0) {
       // ------------------------------------------------------------------ X producer
       int st = 0;
       uint32_t ph = 0;
@@ -309,7 +412,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
         const int kb_end = __shfl_sync(0xffffffffu, w.kb_end, 0);
         for (int kb = kb_begin; kb < kb_end; kb += KS) {
           const int nk = min(KS, kb_end - kb);
-          DEC_WAIT(2, &full_x[sx], xph);
+          DEC_WAIT(2, &xready[sx], xph);
           DEC_WAIT(2, &a_full[ab], aph);
           DEC_WAIT(2, &acc_empty[accs], accph ^ 1);
           if (lane == 0) trace_ev(P, 1, tr);
@@ -533,7 +636,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
     // loaded ONE ITEM AHEAD into registers and first used at the next item: a global load
     // consumed at the start of an item stalls these warps for the load's latency -- microseconds
     // once the weight stream saturates HBM -- and with them the MMA and the whole stream.
-    constexpr bool kEarlyCorr = NT <= 32 && !GS; // registers: NT > 32 loads corr at the end
+    constexpr bool kEarlyCorr = NT <= 32 && !GS && !FQ; // registers: NT > 32 loads corr at the end
     float sw_nx = 0.f, cr_nx[kEarlyCorr ? NT : 1];
     auto prefetch_epi = [&](int it2) {
       if (it2 >= it_end) return;
@@ -568,7 +671,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
       }
       for (int kb0 = w.kb_begin; kb0 < w.kb_end; kb0 += KS) {
         const int nk = min(KS, w.kb_end - kb0);
-        DEC_WAIT(1, &full_x[sx], xph);
+        DEC_WAIT(1, &xready[sx], xph);
         DEC_WAIT(1, &acc_full[accs], accph);
         if (ptid == 0) trace_ev(P, 7, tr);
         tc_fence_after();
@@ -599,8 +702,8 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
 #pragma unroll
               for (int j = 0; j < CH; ++j) sc[j] *= swb;
             }
-            float qc[GS ? CH : 1];                    // INT4 offset term 2^-6 qsum[b][m] (GS)
-            if (GS && !is8) {
+            float qc[(GS || FQ) ? CH : 1];            // INT4 offset term 2^-6 qsum[b][m] (GS, FQ)
+            if ((GS || FQ) && !is8) {
               // code sums of this K-block's tokens from the X stage (broadcast shared loads; the
               // box covers rows >= Mp with zeros)
               const uint32_t qa = smem_u32(sQ(sx)) + 2u * (c * NT + ch * CH);
@@ -621,7 +724,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
               for (int j = 0; j < CH; j += 2) {
                 const int a = ch * CH + j;
                 float2 vv = make_float2(__uint_as_float(v[j]), __uint_as_float(v[j + 1]));
-                if (GS) vv = make_float2(vv.x - qc[j], vv.y - qc[j + 1]);   // exact: multiples of 2^-9 below 2^14
+                if (GS || FQ) vv = make_float2(vv.x - qc[j], vv.y - qc[j + 1]);   // exact: multiples of 2^-9 below 2^14
                 const float2 y = ffma2(vv, make_float2(sc[j], sc[j + 1]), make_float2(acc[a], acc[a + 1]));
                 acc[a] = y.x;
                 acc[a + 1] = y.y;
@@ -668,7 +771,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
       // the offset-binary correction -corr * 2^-9 belongs to the tile once: the owner segment
       // (K-block 0) folds it into its own sum
       const float swv = GS ? 512.f : (n < P.N ? sw_raw * 512.f : 0.f);
-      if (!GS && owner) {
+      if (!GS && !FQ && owner) {
 #pragma unroll
         for (int j = 0; j < NT; ++j) {
           if constexpr (kEarlyCorr) acc[j] -= (m0 + j < P.Mp) ? cr[j] * 0.001953125f : 0.f;   // 2^-9
@@ -792,11 +895,11 @@ cudaError_t launch_fixup(const GemmParams& prm, const int2* fix_info, int n_fix,
   return cudaLaunchKernelEx(&cfg, k_fixup<NT>, prm, fix_info);
 }
 
-template <int NT, int DEBUG, bool GS = false>
+template <int NT, int DEBUG, bool GS = false, bool FQ = false>
 cudaError_t launch_nt(const GemmParams& prm, int grid, cudaStream_t stream) {
-  using C = Cfg<NT, GS>;
+  using C = Cfg<NT, GS, FQ>;
   static std::atomic<uint64_t> attr_done{0};
-  cudaError_t ea = set_smem_attr(k_w4ax<NT, DEBUG, GS>, C::SMEM_BYTES, attr_done);
+  cudaError_t ea = set_smem_attr(k_w4ax<NT, DEBUG, GS, FQ>, C::SMEM_BYTES, attr_done);
   if (ea != cudaSuccess) return ea;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)grid);
@@ -808,7 +911,7 @@ cudaError_t launch_nt(const GemmParams& prm, int grid, cudaStream_t stream) {
   attr[0].val.programmaticStreamSerializationAllowed = COMET_DEC_PDL;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  return cudaLaunchKernelEx(&cfg, k_w4ax<NT, DEBUG, GS>, prm);
+  return cudaLaunchKernelEx(&cfg, k_w4ax<NT, DEBUG, GS, FQ>, prm);
 }
 
 PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
@@ -925,8 +1028,12 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
                            const void* w_packed, const float* w_scales, void* y,
                            comet_dtype_t ydt, int64_t ldy, int32_t* debug_acc,
                            int32_t* debug_acc_blocks, void* workspace, size_t ws_bytes,
-                           cudaStream_t stream, int* launches, bool grouped, const RsArgs* rs) {
+                           cudaStream_t stream, int* launches, bool grouped, const RsArgs* rs,
+                           const FusedX* fx) {
   using namespace gemm;
+  if (fx && (p.orientation != 1 || p.tile_n != 16 || p.M > 8 || grouped || rs || debug_acc || debug_acc_blocks))
+    return fail(COMET_ERR_UNSUPPORTED_SHAPE, "the fused decode path needs orientation 1 with 16-token tiles and M <= 8");
+  static_assert(Cfg<16, false, true>::SX % 2 == 0, "the fused quantiser's two warps own alternate X slots");
   if (grouped && p.orientation != 1 && !(p.orientation == 3 && p.tile_w == 256))
     return fail(COMET_ERR_UNSUPPORTED_SHAPE, "group-wise weight scales run on orientation 1 or on the 256-wide pair kernel (orientation 3)");
   if (grouped && p.orientation == 3 && (debug_acc || debug_acc_blocks))
@@ -950,6 +1057,17 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
     if (!make_map_2d(&prm.map_x, base + L.codes_off, (uint64_t)p.K, (uint64_t)p.M, (uint64_t)p.K, 128,
                      (uint32_t)box_m, CU_TENSOR_MAP_SWIZZLE_128B))
       return fail(COMET_ERR_CUDA, "cuTensorMapEncodeTiled failed for the activation codes");
+  } else if (fx) {
+    // the raw input as [nb][M][128 halves] (dims innermost first: channel in block, token,
+    // block), one box of [KS][8 tokens][256 B] per stage (rows >= M are zero-filled)
+    const uint64_t rd[3] = {128, (uint64_t)p.M, (uint64_t)p.nb};
+    const uint64_t rs_[2] = {(uint64_t)fx->ldx * 2, 256};
+    const uint32_t rb[3] = {128, 8, (uint32_t)(tile_m <= 32 ? 4 : 2)};
+    if (!make_map(&prm.map_x, CU_TENSOR_MAP_DATA_TYPE_UINT16, 3, fx->x, rd, rs_, rb, CU_TENSOR_MAP_SWIZZLE_NONE))
+      return fail(COMET_ERR_CUDA, "cuTensorMapEncodeTiled failed for the fused path's input");
+    prm.xq = fx->x;
+    prm.ldxq = fx->ldx;
+    prm.xq_bf16 = fx->bf16 ? 1 : 0;
   } else {
     // decode: codes as [nb][M][128 B] (dims innermost first: byte in block, token, block) so
     // one box brings a stage's KS K-blocks as KS UMMA-ready [NT][128 B] SW128 tiles; scales
@@ -994,8 +1112,8 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
       return fail(COMET_ERR_CUDA, "cuTensorMapEncodeTiled failed for the output");
   }
   prm.scales = act_scales;
-  prm.corr = reinterpret_cast<const float*>(base + L.corr_off);
-  prm.qsum = reinterpret_cast<const int16_t*>(base + L.qsum_off);
+  prm.corr = fx ? nullptr : reinterpret_cast<const float*>(base + L.corr_off);
+  prm.qsum = fx ? nullptr : reinterpret_cast<const int16_t*>(base + L.qsum_off);
   prm.w_scales = w_scales;
   prm.y = y;
   prm.ldy = ldy;
@@ -1051,6 +1169,8 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
       case 128: e = launch_nt<128, 0, true>(prm, grid, stream); break;
       default: return fail(COMET_ERR_UNSUPPORTED_SHAPE, "unsupported tile_n");
     }
+  } else if (fx) {
+    e = launch_nt<16, 0, false, true>(prm, grid, stream);
   } else {
     switch (tile_m) {
       case 16: e = launch_nt<16, 0>(prm, grid, stream); break;

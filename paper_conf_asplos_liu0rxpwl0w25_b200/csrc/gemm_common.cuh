@@ -47,6 +47,11 @@ struct __align__(64) GemmParams {
   int64_t rs_ms;
   float* rs_dst[8];
   TagMask tags;
+  // FQ (fused quantiser, comet_w4ax_linear): the 16-bit input x [M][ldxq] read by the decode
+  // kernel's quantiser warps instead of TMA-loaded codes
+  const void* xq;
+  int64_t ldxq;
+  int xq_bf16;
 };
 
 // Widening of packed INT4 weights (the B200 form of the paper's "location switch" + "zero

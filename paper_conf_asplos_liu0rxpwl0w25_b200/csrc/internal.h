@@ -89,6 +89,13 @@ cudaError_t launch_kv4_dequantize(const uint8_t* codes, const float* scales, con
 cudaError_t launch_pack_weight(const int8_t* w, int64_t N, int64_t K, void* w_packed,
                                cudaStream_t stream);
 // gemm.cu
+// comet_w4ax_linear's fused decode path: the GEMM quantises x itself (no kernel 1)
+struct FusedX {
+  const void* x;
+  int64_t ldx;
+  bool bf16;
+};
+
 struct RsArgs {            // NEXT-2 fused reduce-scatter of the row-parallel layer
   int world, rank;
   int64_t ms;              // output rows per owner rank
@@ -99,7 +106,7 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
                            comet_dtype_t ydt, int64_t ldy, int32_t* debug_acc,
                            int32_t* debug_acc_blocks, void* workspace, size_t ws_bytes,
                            cudaStream_t stream, int* launches, bool grouped = false,
-                           const RsArgs* rs = nullptr);
+                           const RsArgs* rs = nullptr, const FusedX* fx = nullptr);
 cudaError_t launch_rs_reduce(const float* recv, int world, int64_t rows, int64_t ms, int64_t N, void* y, int ydt,
                              int64_t ldy, cudaStream_t stream);
 int max_coresident_units(const Plan& p, int sms);

@@ -8,4 +8,5 @@ dev = torch.device("cuda", 0)
 peaks, _ = bench.load_peaks()
 d = bench.decode_sweep(cb, torch, dev, peaks, bench.Timer(torch, dev))
 for k, v in d["layers"].items():
-    print(f"{k:12s} {v['us']:7.2f} us {v['GB/s']:7.1f} GB/s {v['frac_hbm']:.3f}  isolated {v['isolated_us']:6.2f}  step {v['step_us']:6.2f}")
+    print(f"{k:12s} {v['us']:7.2f} us {v['GB/s']:7.1f} GB/s {v['frac_hbm']:.3f}  isolated {v['isolated_us']:6.2f}  step {v['step_us']:6.2f}"
+          f"  fused {v.get('fused_step_us', float('nan')):6.2f}")
