@@ -305,6 +305,12 @@ def decode_sweep(cb, torch, dev, peaks, timer, Ms=(1, 4, 8, 32), iters=20, rank=
             us_fused = None
             if plan.info()["tile_n"] == 16 and plan.info()["orientation"] == 1:
                 us_fused = us_rotating(torch, [lambda w_=w_: cb.w4ax_linear_fused(plan, x, w_, swd, out=y) for w_ in wps])
+            # SURVEY §8(d) decode ablation: the same GEMM on plan orientation 4 (gemm_v.cu:
+            # mma.sync u8 x s8, weights streamed by cp.async into per-warp rings, no TMEM)
+            us_o4 = None
+            if M <= 8:
+                plan4 = cb.Plan(M, Nl, Kl, tl, orientation=4)
+                us_o4 = us_rotating(torch, [lambda w_=w_: cb.w4ax_gemm(plan4, act, sc, w_, swd, out=y) for w_ in wps])
             ar_us = None
             if kind == "row" and world > 1:
                 ar_us = timer.us(lambda: dist.all_reduce(y, op=dist.ReduceOp.SUM), iters, flush=False)
@@ -320,6 +326,8 @@ def decode_sweep(cb, torch, dev, peaks, timer, Ms=(1, 4, 8, 32), iters=20, rank=
                                    "step_us": round(us_step, 2),
                                    "step_GB/s": round((nbytes + M * Kl * 2) / (us_step * 1e-6) / 1e9, 1),
                                    "orientation": plan.info()["orientation"], "tile_n": plan.info()["tile_n"]}
+            if us_o4 is not None:
+                out[f"{name}_M{M}"]["o4_mma_sync_us"] = round(us_o4, 2)
             if us_fused is not None:
                 out[f"{name}_M{M}"]["fused_step_us"] = round(us_fused, 2)
                 out[f"{name}_M{M}"]["fused_step_GB/s"] = round((nbytes + M * Kl * 2) / (us_fused * 1e-6) / 1e9, 1)
@@ -332,7 +340,8 @@ def decode_sweep(cb, torch, dev, peaks, timer, Ms=(1, 4, 8, 32), iters=20, rank=
                       "weight copies (> 2 x L2: every launch streams from HBM); isolated_us: one event-bracketed launch after a "
                       "256 MiB write + 256 MiB read (median of 20; includes the ~6 us an empty kernel measures that way)",
             "step": "step_us = kernel 1 (quantise x) + the GEMM as one decode layer step (the GEMM is a programmatic dependent launch), back to back; "
-                    "fused_step_us = the same step as one comet_w4ax_linear launch (kernel 1 fused into the GEMM, 16-token tiles)",
+                    "fused_step_us = the same step as one comet_w4ax_linear launch (kernel 1 fused into the GEMM, 16-token tiles); "
+                    "o4_mma_sync_us = the GEMM on plan orientation 4 (gemm_v.cu, warp-level mma.sync, cp.async weight rings; ablation)",
             "layers": out}
 
 

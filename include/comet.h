@@ -207,7 +207,13 @@ typedef struct {
                           2 = tokens on the MMA M side: tile = 128 tokens x tile_w weights
                               (prefill; weights widened into shared memory), tile_n ignored;
                           3 = as 2 on a tcgen05 CTA pair: tile = 256 tokens x tile_w weights,
-                              each SM widens half the weights; num_ctas counts pairs */
+                              each SM widens half the weights; num_ctas counts pairs;
+                          4 = decode, M <= 8, warp-level tensor cores (mma.sync u8 x s8):
+                              weights streamed by cp.async into per-warp rings, units
+                              (128-weight group, K-block) cut into one contiguous range per
+                              CTA, partials summed in CTA order by a second (dependent)
+                              launch; per-channel s_w only, no debug outputs, needs the
+                              plan's workspace; tile_n / tile_w / split_mode ignored */
   int tile_w;          /* orientations 2/3: weights per output tile (MMA N): 128, 160, 192, or
                           256 (orientation 3 only);
                           0 = auto (256 for orientation 3, 192 for 2).  Ignored for

@@ -14,7 +14,7 @@ BUILD = os.path.join(PKG, "build")
 LIB = os.path.join(PKG, "lib", "libcomet.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
-CU_SOURCES = ["quantize.cu", "kv4.cu", "gemm.cu", "gemm_n.cu", "api.cu"]
+CU_SOURCES = ["quantize.cu", "kv4.cu", "gemm.cu", "gemm_n.cu", "gemm_v.cu", "api.cu"]
 CPP_SOURCES = ["planner.cpp", "calibrate.cpp"]
 HEADERS = ["internal.h", "sm100.cuh", "gemm_common.cuh", "fmpq.cuh"]
 

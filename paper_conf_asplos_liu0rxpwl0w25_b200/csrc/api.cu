@@ -299,7 +299,7 @@ comet_status_t comet_plan_create(int64_t M, int64_t N, int64_t K, const uint8_t*
   else comet_sched_config_default(&cfg);
   if (cfg.split_mode < -1 || cfg.split_mode > 3) return fail(COMET_ERR_INVALID_ARG, "split_mode must be -1, 0, 1, 2 or 3");
   if (cfg.cost_int4 < 0 || cfg.cost_int8 < 0) return fail(COMET_ERR_INVALID_ARG, "costs must be >= 0");
-  if (cfg.orientation < 0 || cfg.orientation > 3) return fail(COMET_ERR_INVALID_ARG, "orientation must be 0..3");
+  if (cfg.orientation < 0 || cfg.orientation > 4) return fail(COMET_ERR_INVALID_ARG, "orientation must be 0..4");
   if (cfg.num_sms <= 0) {
     if (!cfg.device_plan) return fail(COMET_ERR_INVALID_ARG, "a host-only plan needs an explicit num_sms");
     int sms = 0;

@@ -994,6 +994,7 @@ cudaError_t launch_debug_widen(uint64_t first, int64_t n, int is8, uint32_t* out
 // device: the stream-K fix-up waits of the persistent grid assume every unit is resident.
 int max_coresident_units(const Plan& p, int sms) {
   using namespace gemm;
+  if (p.orientation == 4) return p.num_ctas;   // no inter-CTA waits: any grid is valid
   if (p.orientation >= 2) return max_units_gemm_n(p.tile_w, p.orientation == 3 ? 2 : 1, sms);
   int b = 0;
   cudaError_t e = cudaSuccess;
@@ -1015,6 +1016,7 @@ int max_coresident_units(const Plan& p, int sms) {
 // prefill kernels: pipeline slots; decode kernel: packed-weight ring slots.
 int gemm_stages(const Plan& p) {
   using namespace gemm;
+  if (p.orientation == 4) return gemv::gemv_stages();
   if (p.orientation >= 2) return stages_gemm_n(p.tile_w, p.orientation == 3 ? 2 : 1);
   switch (p.tile_n) {
     case 16: return Cfg<16>::SW;
@@ -1039,6 +1041,23 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
   if (grouped && p.orientation == 3 && (debug_acc || debug_acc_blocks))
     return fail(COMET_ERR_UNSUPPORTED_SHAPE, "group-wise weight scales on the pair kernel have no debug accumulators");
   *launches = 0;
+  if (p.orientation == 4) {
+    if (grouped || rs || fx || debug_acc || debug_acc_blocks)
+      return fail(COMET_ERR_UNSUPPORTED_SHAPE, "orientation 4 (decode, M <= 8) runs per-channel weight scales without debug outputs");
+    if (p.d_items == nullptr) return fail(COMET_ERR_INVALID_ARG, "plan was created with device_plan = 0");
+    if (workspace == nullptr || ws_bytes < p.ws_bytes)
+      return fail(COMET_ERR_WORKSPACE_TOO_SMALL, "workspace smaller than the plan's workspace_bytes");
+    comet_act_layout_t L;
+    act_layout(p.M, p.K, &L);
+    const uint8_t* base = static_cast<const uint8_t*>(act_packed);
+    cudaError_t e = gemv::launch_gemv(static_cast<const uint8_t*>(w_packed), base + L.codes_off, act_scales,
+                                      reinterpret_cast<const int16_t*>(base + L.qsum_off), w_scales, y, (int)ydt,
+                                      ldy, p.M, p.N, p.K, L.Mp, p.mask, p.num_ctas, p.max_segments,
+                                      p.gemv_nbr, static_cast<float*>(workspace), stream);
+    if (e != cudaSuccess) return cuda_status(e, "w4ax gemv launch");
+    *launches = 2;
+    return COMET_OK;
+  }
   const bool dbg = debug_acc != nullptr || debug_acc_blocks != nullptr;
   const int debug = debug_acc_blocks ? 2 : (dbg ? 1 : 0);
   const bool normal = p.orientation >= 2;

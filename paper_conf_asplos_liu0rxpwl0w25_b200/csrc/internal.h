@@ -41,6 +41,7 @@ struct Plan {
   int orientation = 1;   // 1: weights on MMA M (gemm.cu), 2: tokens on MMA M (gemm_n.cu)
   int tile_w = 128;      // weights per output tile
   int kgran = 1;         // K-blocks per scheduling unit (4 for the decode kernel's stream-K)
+  int gemv_nbr = 0;      // orientation 4: activation K-blocks one CTA stages
   int64_t n_m_tiles, n_n_tiles, n_tiles;
   std::vector<uint8_t> tags;
   TagMask mask;
@@ -111,6 +112,18 @@ cudaError_t launch_rs_reduce(const float* recv, int world, int64_t rows, int64_t
                              int64_t ldy, cudaStream_t stream);
 int max_coresident_units(const Plan& p, int sms);
 int gemm_stages(const Plan& p);
+// gemm_v.cu: the decode-regime kernel of plan orientation 4 (M <= 8)
+namespace gemv {
+int gemv_ctas_per_sm();
+int gemv_stages();
+int gemv_max_segments(int64_t units, int nb, int ctas);
+int gemv_stage_blocks(int64_t units, int nb, int ctas);
+int gemv_pick(int64_t M, int64_t units, int nb, int num_sms, int* nbr_out);
+cudaError_t launch_gemv(const uint8_t* w, const uint8_t* codes, const float* scales, const int16_t* qsum,
+                        const float* w_scales, void* y, int ydt, int64_t ldy, int64_t M, int64_t N,
+                        int64_t K, int64_t Mp, const TagMask& tags, int ctas, int maxseg, int nbr,
+                        float* part, cudaStream_t stream);
+}
 namespace gemm {
 cudaError_t launch_debug_widen(uint64_t first, int64_t n, int is8, uint32_t* out, cudaStream_t stream);
 }

@@ -76,6 +76,38 @@ comet_status_t build_plan(Plan& p, const comet_sched_config& cfg) {
   p.nb = p.K / kBlockK;
   p.Mp = round_up(p.M, COMET_SCALE_PAD);
   p.orientation = cfg.orientation > 0 ? cfg.orientation : (p.M >= 256 ? 3 : (p.M >= 128 ? 2 : 1));
+  if (p.orientation == 4) {
+    // decode on the warp-level tensor-core path (gemm_v.cu): units (128-row group, K-block),
+    // group-major, cut into one contiguous range per CTA (CTA-level stream-K); no work list,
+    // the partials go through the workspace
+    if (p.M > 8) return fail(COMET_ERR_UNSUPPORTED_SHAPE, "orientation 4 takes M <= 8 tokens");
+    p.tile_n = 8;
+    p.tile_w = 128;
+    p.split_mode = 1;
+    p.kgran = 1;
+    if (cfg.num_sms <= 0) return fail(COMET_ERR_INVALID_ARG, "num_sms must be resolved before planning");
+    p.n_m_tiles = 1;
+    p.n_n_tiles = p.N / 128;
+    p.n_tiles = p.n_n_tiles;
+    const int64_t units = p.n_tiles * p.nb;
+    p.num_ctas = gemv::gemv_pick(p.M, units, (int)p.nb, cfg.num_sms, &p.gemv_nbr);
+    if (p.num_ctas < 0) return fail(COMET_ERR_UNSUPPORTED_SHAPE, "orientation 4: a CTA's K range exceeds the activation staging capacity");
+    const int P = p.num_ctas;
+    p.max_segments = gemv::gemv_max_segments(units, (int)p.nb, P);
+    p.n_split_tiles = 0;                       // groups shared by more than one CTA
+    for (int64_t t = 0; t < p.n_tiles; ++t) {
+      const int64_t ua = t * p.nb, ub = ua + p.nb - 1;
+      if (((ua + 1) * P - 1) / units != ((ub + 1) * P - 1) / units) p.n_split_tiles++;
+    }
+    p.cta_begin.assign(P + 1, 0);
+    p.items.clear();
+    p.fix_info.clear();
+    p.max_cost = (double)((units + P - 1) / P);
+    p.mean_cost = (double)units / P;
+    p.ws_flags_off = 0;
+    p.ws_bytes = ((size_t)P * p.max_segments * 128 * 8 * sizeof(float) + 255) / 256 * 256;
+    return COMET_OK;
+  }
   if (p.orientation >= 2) {
     p.tile_n = p.orientation == 3 ? 256 : 128;   // tokens per tile = MMA M (CTA pair: 2 x 128)
     p.tile_w = cfg.tile_w > 0 ? cfg.tile_w : (p.orientation == 3 ? 256 : 192);  // weights per tile = MMA N

@@ -183,7 +183,7 @@ def test_stages_honoured_or_rejected():
     import ctypes
     L = cb.lib()
     tags = np.zeros(32, np.uint8)
-    for M, orient in ((4096, 3), (1, 1), (200, 2)):
+    for M, orient in ((4096, 3), (1, 1), (200, 2), (4, 4)):
         p = cb.Plan(M, 4096, 4096, tags, num_sms=148, device_plan=False, orientation=orient)
         depth = p.info()["stages"]
         assert 2 <= depth <= 8
@@ -227,3 +227,35 @@ def test_layout_decoder_exhaustive_16bit():
             w8 = [a, -8, 7, 0, b, 3, -1, -5]
             got = unpack_weight(np.frombuffer(pack_py(w8), np.uint8).reshape(1, 4), 1, 8)
             assert got.tolist() == [w8]
+
+
+@pytest.mark.parametrize("M,N,K,sms", [(1, 28672, 8192, 148), (8, 8192, 28672, 148), (4, 10240, 8192, 148),
+                                       (3, 128, 28672, 3), (5, 8192, 1024, 2), (8, 1024, 2048, 148)])
+def test_gemv_plan_split(M, N, K, sms):
+    """Orientation 4 (gemm_v.cu): units (128-row group, K-block), group-major, cut into one
+    contiguous range per CTA, equal to within one unit; the reduction kernel finds a group's
+    CTAs with the inverse owner(u) = floor(((u + 1) C - 1) / U).  Checked here against a direct
+    enumeration: every unit owned exactly once, owner() of every unit right, the segment count
+    and the workspace size the plan reports."""
+    tags = np.zeros(K // 128, np.uint8)
+    p = cb.Plan(M, N, K, tags, num_sms=sms, device_plan=False, orientation=4)
+    info = p.info()
+    assert info["orientation"] == 4 and info["tile_w"] == 128 and info["tile_n"] == 8
+    C = info["num_ctas"]
+    assert C % sms == 0 and 1 <= C // sms <= 3
+    nb, G = K // 128, N // 128
+    U = G * nb
+    u0 = [U * c // C for c in range(C + 1)]
+    assert u0[0] == 0 and u0[-1] == U and all(b - a in (U // C, U // C + 1) for a, b in zip(u0, u0[1:]))
+    owner = np.repeat(np.arange(C), np.diff(u0))
+    u = np.arange(U, dtype=np.int64)
+    assert np.array_equal(((u + 1) * C - 1) // U, owner)
+    segs = max([(u0[c + 1] - 1) // nb - u0[c] // nb + 1 for c in range(C) if u0[c + 1] > u0[c]] + [1])
+    assert p.workspace_bytes == -(-(C * segs * 128 * 8 * 4) // 256) * 256
+    split = sum(1 for g in range(G) if owner[g * nb] != owner[g * nb + nb - 1])
+    assert info["n_split_tiles"] == split
+
+
+def test_gemv_plan_rejects_large_m():
+    with pytest.raises(cb.CometError):
+        cb.Plan(9, 1024, 1024, np.zeros(8, np.uint8), num_sms=148, device_plan=False, orientation=4)

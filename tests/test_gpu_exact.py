@@ -157,6 +157,32 @@ def test_decode_tile_widths_exact(tile_n):
     run_exact(100, 4096, 1024, 0.25, seed=tile_n, orientation=1, tile_n=tile_n)
 
 
+GEMV = [(f"o4_l3_70b_{nm}_m{M}", M, K, N, 0.05)
+        for nm, K, N in (("gateup", 8192, 28672), ("down", 28672, 8192), ("qkv", 8192, 10240))
+        for M in (1, 4, 8)] + [(f"o4_l2_7b_{nm}_m1", 1, K, N, 0.05)
+                               for nm, K, N in (("qkvo", 4096, 4096), ("gateup", 4096, 11008), ("down", 11008, 4096))]
+
+
+@pytest.mark.parametrize("name,M,K,N,frac", GEMV, ids=[c[0] for c in GEMV])
+def test_gemv_exact_full_size(name, M, K, N, frac):
+    """Orientation 4 (gemm_v.cu: mma.sync u8 x s8, CTA-level stream-K + ordered reduction) at
+    the decode sizes of configs 2 and 5."""
+    info = run_exact(M, K, N, frac, seed=sum(map(ord, name)), orientation=4,
+                     out_dtypes=(torch.float32, torch.float16, torch.bfloat16))
+    assert info["orientation"] == 4
+
+
+@pytest.mark.parametrize("M,K,N,frac,num_sms", [
+    (3, 28672, 128, 0.25, 3),      # one row group over 6 CTAs: every CTA a segment of one group
+    (5, 1024, 8192, 1.0, 2),       # all INT8 blocks; 4 CTAs: ranges of 16 groups (many segments)
+    (8, 2048, 1024, 0.0, 148),     # more CTAs than units: empty ranges
+    (2, 4096, 2048, 0.5, 7),       # ranges cutting groups at odd K-blocks
+])
+def test_gemv_schedules_exact(M, K, N, frac, num_sms):
+    info = run_exact(M, K, N, frac, seed=M * 7 + num_sms, orientation=4, num_sms=num_sms)
+    assert info["orientation"] == 4
+
+
 def test_bf16_inputs_and_outputs_exact():
     """Config 2's BF16 variant: bf16 activations in, bf16 / fp32 out."""
     run_exact(4096, 4096, 4096, 0.05, seed=77, bf16=True, out_dtypes=(torch.float32, torch.bfloat16))

@@ -63,6 +63,9 @@ def _check_quant(p, act, sc, rows=None):
     (1, 4096, 0.05, False), (16, 4096, 0.05, False), (256, 11008, 0.05, False),   # config 2
     (33, 1024, 0.5, True), (1000, 512, 0.25, False), (7, 14336, 0.05, True),
     (1, 28672, 0.05, False), (32, 28672, 0.05, True), (3, 11008, 0.25, False),   # cluster-split rows
+    # staged-ring kernel (M > 32): ragged groups (71 blocks: a 1-group last chunk of 7 blocks),
+    # a sub-group row, more CTAs than a resident wave holds rows for
+    (300, 9088, 0.25, True), (40, 640, 0.5, False), (777, 3200, 0.05, False), (4100, 1152, 0.05, True),
 ])
 def test_quantize_parity(M, K, frac, bf16):
     if frac is None:
@@ -81,6 +84,12 @@ def test_quantize_edge_cases():
     x[2, 300] = 65504.0
     for tags in (np.array([0, 1, 0, 1], np.uint8), np.zeros(4, np.uint8), np.ones(4, np.uint8)):
         p = synth.Problem(x=x, tags=tags, w=np.zeros((128, 512), np.int8), s_w=np.ones(128, np.float32))
+        act, sc = _quant(p)
+        _check_quant(p, act, sc)
+    # the same rows through the staged-ring kernel (M > 32), tiled to 67 rows
+    xr = np.tile(x, (23, 1))[:67]
+    for tags in (np.array([0, 1, 0, 1], np.uint8), np.ones(4, np.uint8)):
+        p = synth.Problem(x=xr, tags=tags, w=np.zeros((128, 512), np.int8), s_w=np.ones(128, np.float32))
         act, sc = _quant(p)
         _check_quant(p, act, sc)
     xb = np.zeros((2, 128), np.uint16)

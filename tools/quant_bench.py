@@ -16,7 +16,7 @@ from paper_conf_asplos_liu0rxpwl0w25_b200 import synth  # noqa: E402
 
 dev = torch.device("cuda", 0)
 peaks, _ = bench.load_peaks()
-for M, K in [(4096, 8192), (4096, 28672), (8192, 14336), (1, 8192), (32, 28672)]:
+for M, K in [(4096, 8192), (4096, 28672), (8192, 14336), (4096, 11008), (256, 4096), (256, 11008), (1, 8192), (32, 28672)]:
     tags = synth.make_tags(K, 0.05, np.random.default_rng(1))
     x = bench.dev_activations(torch, M, K, tags, 3, dev)
     ncopy = max(2, -(-300 * (1 << 20) // (M * K * 2)))
