@@ -303,14 +303,18 @@ def decode_sweep(cb, torch, dev, peaks, timer, Ms=(1, 4, 8, 32), iters=20, rank=
             # the same layer step as ONE launch (comet_w4ax_linear: kernel 1 fused into the GEMM,
             # for 16-token decode tiles)
             us_fused = None
-            if plan.info()["tile_n"] == 16 and plan.info()["orientation"] == 1:
-                us_fused = us_rotating(torch, [lambda w_=w_: cb.w4ax_linear_fused(plan, x, w_, swd, out=y) for w_ in wps])
-            # SURVEY §8(d) decode ablation: the same GEMM on plan orientation 4 (gemm_v.cu:
-            # mma.sync u8 x s8, weights streamed by cp.async into per-warp rings, no TMEM)
-            us_o4 = None
             if M <= 8:
-                plan4 = cb.Plan(M, Nl, Kl, tl, orientation=4)
-                us_o4 = us_rotating(torch, [lambda w_=w_: cb.w4ax_gemm(plan4, act, sc, w_, swd, out=y) for w_ in wps])
+                plan_f = plan if plan.info()["orientation"] == 1 else cb.Plan(M, Nl, Kl, tl, orientation=1)
+                if plan_f.info()["tile_n"] == 16:
+                    us_fused = us_rotating(torch, [lambda w_=w_: cb.w4ax_linear_fused(plan_f, x, w_, swd, out=y) for w_ in wps])
+            # SURVEY §8(d) decode ablation: the same GEMM on the other decode kernel -- orientation 1
+            # (tcgen05, weights widened into TMEM) or 4 (gemm_v.cu: mma.sync u8 x s8, weights
+            # streamed by cp.async into per-warp rings), whichever the auto plan did not pick
+            alt = None
+            if M <= 8:
+                o_alt = 1 if plan.info()["orientation"] == 4 else 4
+                plan_alt = cb.Plan(M, Nl, Kl, tl, orientation=o_alt)
+                alt = (o_alt, us_rotating(torch, [lambda w_=w_: cb.w4ax_gemm(plan_alt, act, sc, w_, swd, out=y) for w_ in wps]))
             ar_us = None
             if kind == "row" and world > 1:
                 ar_us = timer.us(lambda: dist.all_reduce(y, op=dist.ReduceOp.SUM), iters, flush=False)
@@ -326,8 +330,8 @@ def decode_sweep(cb, torch, dev, peaks, timer, Ms=(1, 4, 8, 32), iters=20, rank=
                                    "step_us": round(us_step, 2),
                                    "step_GB/s": round((nbytes + M * Kl * 2) / (us_step * 1e-6) / 1e9, 1),
                                    "orientation": plan.info()["orientation"], "tile_n": plan.info()["tile_n"]}
-            if us_o4 is not None:
-                out[f"{name}_M{M}"]["o4_mma_sync_us"] = round(us_o4, 2)
+            if alt is not None:
+                out[f"{name}_M{M}"]["o1_tmem_us" if alt[0] == 1 else "o4_mma_sync_us"] = round(alt[1], 2)
             if us_fused is not None:
                 out[f"{name}_M{M}"]["fused_step_us"] = round(us_fused, 2)
                 out[f"{name}_M{M}"]["fused_step_GB/s"] = round((nbytes + M * Kl * 2) / (us_fused * 1e-6) / 1e9, 1)
@@ -341,7 +345,8 @@ def decode_sweep(cb, torch, dev, peaks, timer, Ms=(1, 4, 8, 32), iters=20, rank=
                       "256 MiB write + 256 MiB read (median of 20; includes the ~6 us an empty kernel measures that way)",
             "step": "step_us = kernel 1 (quantise x) + the GEMM as one decode layer step (the GEMM is a programmatic dependent launch), back to back; "
                     "fused_step_us = the same step as one comet_w4ax_linear launch (kernel 1 fused into the GEMM, 16-token tiles); "
-                    "o4_mma_sync_us = the GEMM on plan orientation 4 (gemm_v.cu, warp-level mma.sync, cp.async weight rings; ablation)",
+                    "orientation = the auto plan's decode kernel (1: tcgen05 + TMEM-widened weights, 4: gemm_v.cu warp-level mma.sync "
+                    "with cp.async weight rings); o1_tmem_us / o4_mma_sync_us = the same GEMM on the other one (ablation)",
             "layers": out}
 
 
@@ -508,10 +513,11 @@ def next_rows(cb, torch, dev, peaks, timer, iters=20):
     for M in (1, 32):
         x = torch.from_numpy(synth.make_activations(M, K, tags, rng)).to(dev)
         plan = cb.Plan(M, N, K, tags)
+        plan_g = cb.Plan(M, N, K, tags, orientation=1)   # group-wise scales: the TMEM decode kernel
         act, sc = cb.quantize_act(x, tags)
         y = torch.empty((M, N), dtype=torch.float16, device=dev)
         nbytes = N * K // 2 + swg.numel() * 4 + act.numel() + sc.numel() * 4 + M * N * 2
-        us_g = t(lambda: cb.w4ax_gemm_grouped(plan, act, sc, wp, swg, out=y))
+        us_g = t(lambda: cb.w4ax_gemm_grouped(plan_g, act, sc, wp, swg, out=y))
         us_c = t(lambda: cb.w4ax_gemm(plan, act, sc, wp, swd, out=y))
         out[f"grouped_scales_gemm_gate_up_M{M}"] = {"us": round(us_g, 2), "GB/s": round(nbytes / us_g / 1e3, 1),
                                                     "frac_hbm": round(nbytes / us_g / 1e3 / hbm, 3),

@@ -119,14 +119,18 @@ comet_status_t comet_quantize_act(const void* x, comet_dtype_t xdt, int64_t M, i
 /* ------------------------------------------------------------------------------------------
  * Weight packed layout ("location switch" + "zero extension", reading R14)
  *
- * w_packed [N][K/2] uint8, row-major (row stride K/2 bytes).  For row n and every group of
- * eight consecutive channels k = 8g .. 8g+7, the little-endian 32-bit word at byte offset
- * n*K/2 + 4g has byte i (i = 0..3) equal to
+ * w_packed: N*K/2 bytes in 1 KB tiles of 16 rows x one 128-channel block, the tile of
+ * (row tile n/16, block b) at byte ((n/16) * (K/128) + b) * 1024, inside it row n % 16 at
+ * + (n % 16) * 64 (row-tiled: each 16-row group's K-blocks are contiguous, so a kernel that
+ * walks K for a group of rows streams contiguous memory; N % 16 == 0).  Within a row's 64 B,
+ * for every group of eight consecutive channels k = 8g .. 8g+7 (g relative to the block), the
+ * little-endian 32-bit word at byte 4 (g % 16) has byte i (i = 0..3) equal to
  *        (u[8g+i] & 0xF) | (u[8g+i+4] << 4),      u = w + 8  (offset binary, 0..15).
  * Then (word & 0x0F0F0F0F) holds u[8g..8g+3] and ((word >> 4) & 0x0F0F0F0F) holds
  * u[8g+4..8g+7], one per byte, in channel order: widening costs 3 instructions per 8 values.
  * A byte 0x0u read as E4M3 is exactly u * 2^-9 (subnormal/first binade), so the widened
  * bytes feed the FP8 tensor core directly; (u << 4) ^ 0x80 is the int8 16*w for INT8 blocks.
+ * The layout is opaque to callers beyond its size; comet_pack_weight(_perm) write it.
  * ---------------------------------------------------------------------------------------- */
 size_t comet_weight_packed_bytes(int64_t N, int64_t K);
 /* w_codes_dev: device [N][K] int8 codes in [-8,7] (values outside are masked to 4 bits). */
@@ -201,7 +205,8 @@ typedef struct {
                           comet_plan_info().stages), else COMET_ERR_INVALID_ARG */
   int device_plan;     /* 1 (default) = upload the work list to the device at create time;
                           0 = host-only plan (comet_plan_describe only; CPU-safe) */
-  int orientation;     /* 0 = auto (3 when M >= 256, 2 when M >= 128, else 1);
+  int orientation;     /* 0 = auto (3 when M >= 256, 2 when M >= 128, 4 when M == 1 or M <= 4
+                              with K <= 16384 and the packed weights take >= 96 MiB, else 1);
                           1 = weights on the MMA M side: tile = 128 weights x tile_n tokens
                               (decode-sized M; weights widened into TMEM);
                           2 = tokens on the MMA M side: tile = 128 tokens x tile_w weights
@@ -259,7 +264,7 @@ comet_status_t comet_plan_describe(comet_plan_t plan, int32_t* items, int64_t ma
 /*
  * The W4Ax GEMM.   y[m, n] = s_w[n] * sum_b s_a[m,b] * acc_b[m,n]
  *   act_packed, act_scales  from comet_quantize_act with the plan's M, K and tags.
- *   w_packed                from comet_pack_weight, [N][K/2].
+ *   w_packed                from comet_pack_weight (N*K/2 bytes, row-tiled, see above).
  *   w_scales                device [N] float (per-output-channel, reading R7).
  *   y                       device [M][ldy] of ydt (F16 / BF16 / F32), row-major.
  *   debug_acc               NULL, or device [M][N] int32: sum_b acc_b[m,n] in code units

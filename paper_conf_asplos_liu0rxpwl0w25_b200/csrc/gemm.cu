@@ -275,7 +275,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
           mbar_wait(&empty_w[st], ph ^ 1);
           mbar_arrive_expect_tx(&full_w[st], npair * 2 * kTileW * 64);
           for (int p = 0; p < npair; ++p)
-            tma_load_2d(sW(st) + p * 2 * kTileW * 64, &P.map_w, &full_w[st], (kb + 2 * p) * 64, n0);
+            tma_load_4d(sW(st) + p * 2 * kTileW * 64, &P.map_w, &full_w[st], 0, 0, kb + 2 * p, n0 / kWTileRows);
           trace_ev(P, 0, tr++);
           if (++st == SW) { st = 0; ph ^= 1; }
         }
@@ -459,7 +459,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
     const int q = warp & 3;
     const int r = q * 32 + lane;                  // TMEM lane = weight row within the tile
     const uint32_t lane_addr = (uint32_t)(q * 32) << 16;
-    const int sw = r & 7;                         // TMA 128-byte swizzle: chunk ^= row bits [0:2]
+    // a pair box lands as [8 row tiles][2 K-blocks][16 rows][64 B] (the packed layout's 1 KB
+    // tiles, include/comet.h) with the TMA 64-byte swizzle: chunk ^= (row >> 1) & 3
+    const int sw = (r >> 1) & 3;
+    const uint32_t roff = (uint32_t)((r >> 4) * 2048 + (r & 15) * 64);   // + (cb & 1) KB
     int st = 0, ab = 0;
     uint32_t ph = 0, aph = 0;
     int seq = 0;
@@ -482,10 +485,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
 #pragma unroll
       for (int i = 0; i < KH; ++i) {
         const int cb = half * KH + i;
-        const uint32_t row = smem_u32(sW(st)) + (cb >> 1) * 2 * kTileW * 64 + r * 128;
+        const uint32_t row = smem_u32(sW(st)) + (cb >> 1) * 2 * kTileW * 64 + roff + (cb & 1) * 1024;
 #pragma unroll
         for (int j = 0; j < 4; ++j)
-          cn[4 * i + j] = (cb < nk_n && !(COMET_DEC_ABLATE & 8)) ? lds128(row + ((((cb & 1) * 4 + j) ^ sw) << 4))
+          cn[4 * i + j] = (cb < nk_n && !(COMET_DEC_ABLATE & 8)) ? lds128(row + ((j ^ sw) << 4))
                                                                  : make_uint4(r, j, i, 0);
       }
       __syncwarp();
@@ -556,10 +559,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
 #pragma unroll
         for (int i = 0; i < KH; ++i) {
           const int cb = half * KH + i;
-          const uint32_t row = smem_u32(sW(st)) + (cb >> 1) * 2 * kTileW * 64 + r * 128;
+          const uint32_t row = smem_u32(sW(st)) + (cb >> 1) * 2 * kTileW * 64 + roff + (cb & 1) * 1024;
 #pragma unroll
           for (int j = 0; j < 4; ++j)
-            cc[4 * i + j] = (cb < nk && !(COMET_DEC_ABLATE & 8)) ? lds128(row + ((((cb & 1) * 4 + j) ^ sw) << 4))
+            cc[4 * i + j] = (cb < nk && !(COMET_DEC_ABLATE & 8)) ? lds128(row + ((j ^ sw) << 4))
                                                                  : make_uint4(r, j, i, 0);   // 8: diagnostic, no weight reads
         }
         __syncwarp();
@@ -1016,7 +1019,7 @@ int max_coresident_units(const Plan& p, int sms) {
 // prefill kernels: pipeline slots; decode kernel: packed-weight ring slots.
 int gemm_stages(const Plan& p) {
   using namespace gemm;
-  if (p.orientation == 4) return gemv::gemv_stages();
+  if (p.orientation == 4) return p.gemv_s;
   if (p.orientation >= 2) return stages_gemm_n(p.tile_w, p.orientation == 3 ? 2 : 1);
   switch (p.tile_n) {
     case 16: return Cfg<16>::SW;
@@ -1053,7 +1056,7 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
     cudaError_t e = gemv::launch_gemv(static_cast<const uint8_t*>(w_packed), base + L.codes_off, act_scales,
                                       reinterpret_cast<const int16_t*>(base + L.qsum_off), w_scales, y, (int)ydt,
                                       ldy, p.M, p.N, p.K, L.Mp, p.mask, p.num_ctas, p.max_segments,
-                                      p.gemv_nbr, static_cast<float*>(workspace), stream);
+                                      p.gemv_nbr, p.gemv_s, static_cast<float*>(workspace), stream);
     if (e != cudaSuccess) return cuda_status(e, "w4ax gemv launch");
     *launches = 2;
     return COMET_OK;
@@ -1118,11 +1121,15 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
         return fail(COMET_ERR_CUDA, "cuTensorMapEncodeTiled failed for the group-wise weight scales");
     }
   }
-  // prefill: 64-byte rows (one K-block) with 64B swizzle; decode: 128-byte rows (two K-blocks)
-  if (!make_map_2d(&prm.map_w, w_packed, (uint64_t)(p.K / 2), (uint64_t)p.N, (uint64_t)(p.K / 2),
-                   normal ? 64 : 128, (uint32_t)cta_rows_w,
-                   normal ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B))
-    return fail(COMET_ERR_CUDA, "cuTensorMapEncodeTiled failed for the packed weights");
+  // packed weights as [N/16 row tiles][nb K-blocks][16 rows][64 B] (dims innermost first), 64B
+  // swizzle; prefill: one K-block of the CTA's rows per box, decode: two K-blocks of 128 rows
+  {
+    const uint64_t wd[4] = {64, (uint64_t)kWTileRows, (uint64_t)p.nb, (uint64_t)(p.N / kWTileRows)};
+    const uint64_t ws_[3] = {64, 64 * kWTileRows, (uint64_t)p.nb * 64 * kWTileRows};
+    const uint32_t wb[4] = {64, (uint32_t)kWTileRows, normal ? 1u : 2u, (uint32_t)(cta_rows_w / kWTileRows)};
+    if (!make_map(&prm.map_w, CU_TENSOR_MAP_DATA_TYPE_UINT8, 4, w_packed, wd, ws_, wb, CU_TENSOR_MAP_SWIZZLE_64B))
+      return fail(COMET_ERR_CUDA, "cuTensorMapEncodeTiled failed for the packed weights");
+  }
   if (normal && !dbg) {
     const int esz = ydt == COMET_F32 ? 4 : 2;
     if (!make_map_2d(&prm.map_y, y, (uint64_t)p.N * esz, (uint64_t)p.M, (uint64_t)ldy * esz, 64,

@@ -313,7 +313,7 @@ __global__ void __launch_bounds__(CfgN<BN, CG, NPW, NWG, DEBUG, GS>::THREADS, 1)
             } else if (COMET_ABLATE_TMA2D & 2) {
               bulk_load(sWp(s), src + C::X_BYTES, C::WP_BYTES, &full[s]);
             } else {
-              tma_load_2d(sWp(s), &P.map_w, &full[s], kb * 64, n0);
+              tma_load_4d(sWp(s), &P.map_w, &full[s], 0, 0, kb, n0 / kWTileRows);   // WROWS rows of K-block kb
             }
             if (sbytes) bulk_load(sS + sc * BM, P.scales + (int64_t)kb * P.Mp + m0, sbytes, &full[s]);
             if (GS) {

@@ -34,7 +34,7 @@
 #include "internal.h"
 
 #ifndef COMET_GEMV_S
-#define COMET_GEMV_S 8      // K-blocks in flight per warp (cp.async ring stages of 1 KB)
+#define COMET_GEMV_S 8      // deepest ring (K-blocks in flight per warp, 1 KB stages); gemv_pick may take 6 or 4
 #endif
 #ifndef COMET_GEMV_CPS
 #define COMET_GEMV_CPS 3    // CTAs (8 warps each) per SM, at most (shared memory decides, gemv_pick)
@@ -49,7 +49,7 @@ constexpr int kMaxStageBlocks = 128;   // activation blocks a CTA can stage (M =
 namespace {
 
 struct VParams {
-  const uint8_t* w;        // packed weights [N][K/2]
+  const uint8_t* w;        // packed weights, row-tiled 1 KB tiles (include/comet.h)
   const uint8_t* codes;    // activation codes [M][K]
   const float* scales;     // s_a [nb][Mp]
   const int16_t* qsum;     // code sums [nb][Mp]
@@ -100,7 +100,6 @@ __global__ void __launch_bounds__(256, COMET_GEMV_CPS) k_gemv(const __grid_const
   const int cta = blockIdx.x;
   const int64_t u0 = P.units * cta / P.ctas, u1 = P.units * (cta + 1) / P.ctas;
   const int nb = P.nb;
-  const int64_t rb = P.K / 2;                                          // packed row bytes
   const int kb_s = (int)(u0 % nb);                                     // staging slot j <-> block (kb_s + j) % nb
   const int n_units = (int)(u1 - u0);
   // Weights: each lane copies 16 B of row g and of row g + 8 per unit into the warp's ring
@@ -108,16 +107,18 @@ __global__ void __launch_bounds__(256, COMET_GEMV_CPS) k_gemv(const __grid_const
   // cp.async.wait_group orders them -- no barrier.  Rows are 64 B apart in a stage: a phase of
   // eight lanes reads 128 contiguous bytes.
   const uint32_t ring = (uint32_t)__cvta_generic_to_shared(s_w + warp * S * 1024) + g * 64 + t * 16;
-  const uint8_t* wbase = P.w + (int64_t)(warp * 16 + g) * rb + t * 16;   // + grp * 128 rb + b * 64
-  const int64_t grp_stride = (int64_t)kRowsCta * rb;
+  // rows 16 warp .. of a group are one row tile of the packed layout: tile (grp * 8 + warp, b)
+  // at ((grp * 8 + warp) * nb + b) KB -- each warp streams its tile row contiguously along K
+  const uint8_t* wbase = P.w + (int64_t)warp * nb * 1024 + g * 64 + t * 16;   // + grp * 8 nb KB + b KB
+  const int64_t grp_stride = (int64_t)8 * nb * 1024;
   int64_t lgrp = u0 / nb;
   int lb = (int)(u0 - lgrp * nb);
   int lslot = 0;
   auto issue = [&]() {                       // unit (lgrp, lb) -> ring slot lslot, advance
-    const uint8_t* r0 = wbase + lgrp * grp_stride + lb * 64;
+    const uint8_t* r0 = wbase + lgrp * grp_stride + lb * 1024;
     const uint32_t d = ring + lslot * 1024;
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(d), "l"(r0) : "memory");
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(d + 512), "l"(r0 + 8 * rb) : "memory");
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(d + 512), "l"(r0 + 512) : "memory");
     if (++lb == nb) { lb = 0; ++lgrp; }
     if (++lslot == S) lslot = 0;
   };
@@ -237,6 +238,7 @@ __global__ void __launch_bounds__(256) k_gemv_reduce(const __grid_constant__ VPa
 
 int gemv_ctas_per_sm() { return COMET_GEMV_CPS; }
 int gemv_stages() { return COMET_GEMV_S; }
+constexpr int kStageChoices[3] = {8, 6, 4};   // ring depths instantiated (gemv_pick chooses)
 
 // Plan-time quantities of a grid of `ctas` CTAs: the most groups one CTA touches (workspace
 // slots) and the most K-blocks one CTA stages (its shared memory); -1 when that exceeds the
@@ -249,8 +251,8 @@ int gemv_max_segments(int64_t units, int nb, int ctas) {
   }
   return mx;
 }
-size_t gemv_smem_bytes(int64_t M, int nbr) {
-  return (size_t)8 * COMET_GEMV_S * 1024 + (size_t)nbr * (M * 128 + 8 * 4 + 4 * 4);
+size_t gemv_smem_bytes(int64_t M, int nbr, int S) {
+  return (size_t)8 * S * 1024 + (size_t)nbr * (M * 128 + 8 * 4 + 4 * 4);
 }
 int gemv_stage_blocks(int64_t units, int nb, int ctas) {
   const int64_t len = (units + ctas - 1) / ctas;
@@ -258,25 +260,29 @@ int gemv_stage_blocks(int64_t units, int nb, int ctas) {
   return nbr > kMaxStageBlocks ? -1 : nbr;
 }
 
-// CTAs per SM for this shape: the most (<= COMET_GEMV_CPS) whose shared memory fits an SM.
-// Returns the grid (CTAs) and the K-blocks each stages; -1 when even one CTA per SM does not fit.
-int gemv_pick(int64_t M, int64_t units, int nb, int num_sms, int* nbr_out) {
-  for (int cps = COMET_GEMV_CPS; cps >= 1; --cps) {
-    const int ctas = num_sms * cps;
-    const int nbr = gemv_stage_blocks(units, nb, ctas);
-    if (nbr < 0) continue;
-    if ((size_t)cps * (gemv_smem_bytes(M, nbr) + 1024) <= (size_t)228 * 1024) {
-      *nbr_out = nbr;
-      return ctas;
+// Ring depth S and CTAs per SM for this shape: of the (S, CTAs per SM <= COMET_GEMV_CPS) whose
+// shared memory fits an SM, the one with the most weight bytes in flight per SM (S x CTAs; ties
+// to the deeper ring).  Returns the grid (CTAs), the K-blocks each stages and S; -1 when nothing
+// fits.  (The activation staging grows with M: at M = 4 a 6-deep ring at 3 CTAs per SM keeps
+// more bytes in flight than an 8-deep one at 2.)
+int gemv_pick(int64_t M, int64_t units, int nb, int num_sms, int* nbr_out, int* s_out) {
+  int best = -1, best_ctas = -1;
+  for (int S : kStageChoices)
+    for (int cps = COMET_GEMV_CPS; cps >= 1; --cps) {
+      const int ctas = (int)std::min<int64_t>((int64_t)num_sms * cps, units);   // no empty ranges
+      const int nbr = gemv_stage_blocks(units, nb, ctas);
+      if (nbr < 0) continue;
+      if ((size_t)cps * (gemv_smem_bytes(M, nbr, S) + 1024) > (size_t)228 * 1024) continue;
+      if (S * cps > best) { best = S * cps; best_ctas = ctas; *nbr_out = nbr; *s_out = S; }
+      break;                                                 // fewer CTAs at this S: never better
     }
-  }
-  return -1;
+  return best_ctas;
 }
 
 cudaError_t launch_gemv(const uint8_t* w, const uint8_t* codes, const float* scales, const int16_t* qsum,
                         const float* w_scales, void* y, int ydt, int64_t ldy, int64_t M, int64_t N,
                         int64_t K, int64_t Mp, const TagMask& tags, int ctas, int maxseg, int nbr,
-                        float* part, cudaStream_t stream) {
+                        int S, float* part, cudaStream_t stream) {
   VParams P;
   P.w = w; P.codes = codes; P.scales = scales; P.qsum = qsum; P.part = part; P.w_scales = w_scales;
   P.y = y; P.M = M; P.N = N; P.K = K; P.Mp = Mp; P.ldy = ldy;
@@ -287,17 +293,18 @@ cudaError_t launch_gemv(const uint8_t* w, const uint8_t* codes, const float* sca
   P.nbr = nbr;
   P.ydt = ydt;
   P.tags = tags;
-  const size_t smem = gemv_smem_bytes(M, nbr);
-  auto kern = k_gemv<COMET_GEMV_S>;
-  // the dynamic shared memory this launch needs (set per device when it grows)
-  static std::atomic<int> attr_bytes[64];
+  const size_t smem = gemv_smem_bytes(M, nbr, S);
+  auto kern = S == 8 ? k_gemv<8> : S == 6 ? k_gemv<6> : k_gemv<4>;
+  // the dynamic shared memory this launch needs (set per device and ring depth when it grows)
+  static std::atomic<int> attr_bytes[3][64];
+  const int si = S == 8 ? 0 : S == 6 ? 1 : 2;
   int dev = 0;
   cudaGetDevice(&dev);
-  if ((int)smem > attr_bytes[dev & 63].load()) {
+  if ((int)smem > attr_bytes[si][dev & 63].load()) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e == cudaSuccess) e = cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
     if (e != cudaSuccess) return e;
-    attr_bytes[dev & 63].store((int)smem);
+    attr_bytes[si][dev & 63].store((int)smem);
   }
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)ctas);

@@ -22,6 +22,13 @@ struct TagMask {
   __host__ __device__ bool get(int b) const { return (w[b >> 5] >> (b & 31)) & 1u; }
 };
 
+// Packed weights are row-tiled (include/comet.h): 1 KB tiles of 16 rows x one K-block (64 B
+// per row), tile (n/16, b) at ((n/16) * nb + b) KB.  Word g (channels 8g .. 8g+7) of row n:
+__host__ __device__ inline int64_t packed_word_index(int64_t n, int64_t g, int64_t nb) {
+  return ((((n >> 4) * nb + (g >> 4)) << 4) + (n & 15)) * 16 + (g & 15);
+}
+constexpr int kWTileRows = 16;     // rows per packed-weight tile
+
 inline int64_t round_up(int64_t a, int64_t b) { return (a + b - 1) / b * b; }
 inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
@@ -42,6 +49,7 @@ struct Plan {
   int tile_w = 128;      // weights per output tile
   int kgran = 1;         // K-blocks per scheduling unit (4 for the decode kernel's stream-K)
   int gemv_nbr = 0;      // orientation 4: activation K-blocks one CTA stages
+  int gemv_s = 0;        // orientation 4: weight ring depth (K-blocks in flight per warp)
   int64_t n_m_tiles, n_n_tiles, n_tiles;
   std::vector<uint8_t> tags;
   TagMask mask;
@@ -118,11 +126,11 @@ int gemv_ctas_per_sm();
 int gemv_stages();
 int gemv_max_segments(int64_t units, int nb, int ctas);
 int gemv_stage_blocks(int64_t units, int nb, int ctas);
-int gemv_pick(int64_t M, int64_t units, int nb, int num_sms, int* nbr_out);
+int gemv_pick(int64_t M, int64_t units, int nb, int num_sms, int* nbr_out, int* s_out);
 cudaError_t launch_gemv(const uint8_t* w, const uint8_t* codes, const float* scales, const int16_t* qsum,
                         const float* w_scales, void* y, int ydt, int64_t ldy, int64_t M, int64_t N,
                         int64_t K, int64_t Mp, const TagMask& tags, int ctas, int maxseg, int nbr,
-                        float* part, cudaStream_t stream);
+                        int S, float* part, cudaStream_t stream);
 }
 namespace gemm {
 cudaError_t launch_debug_widen(uint64_t first, int64_t n, int is8, uint32_t* out, cudaStream_t stream);

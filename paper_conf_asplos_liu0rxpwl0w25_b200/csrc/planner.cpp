@@ -76,6 +76,12 @@ comet_status_t build_plan(Plan& p, const comet_sched_config& cfg) {
   p.nb = p.K / kBlockK;
   p.Mp = round_up(p.M, COMET_SCALE_PAD);
   p.orientation = cfg.orientation > 0 ? cfg.orientation : (p.M >= 256 ? 3 : (p.M >= 128 ? 2 : 1));
+  // decode on the warp-level path (gemm_v.cu) where it measured faster than the TMEM kernel:
+  // large layers (>= 96 MiB of packed weights) at M = 1, or M <= 4 with K <= 16384
+  // (tools/gemv_ab.py: LLaMA-3-70B gate/up 23.8 vs 28.1 us at M = 1, 25.9 vs 27.6 at M = 4;
+  // down 26.2 vs 26.6 at M = 1, but 27.4 vs 26.5 at M = 4; qkv, 42 MB, 14.5 vs 14.2)
+  if (cfg.orientation <= 0 && (p.M == 1 || (p.M <= 4 && p.K <= 16384)) && p.N * p.K / 2 >= (96ll << 20))
+    p.orientation = 4;
   if (p.orientation == 4) {
     // decode on the warp-level tensor-core path (gemm_v.cu): units (128-row group, K-block),
     // group-major, cut into one contiguous range per CTA (CTA-level stream-K); no work list,
@@ -90,7 +96,7 @@ comet_status_t build_plan(Plan& p, const comet_sched_config& cfg) {
     p.n_n_tiles = p.N / 128;
     p.n_tiles = p.n_n_tiles;
     const int64_t units = p.n_tiles * p.nb;
-    p.num_ctas = gemv::gemv_pick(p.M, units, (int)p.nb, cfg.num_sms, &p.gemv_nbr);
+    p.num_ctas = gemv::gemv_pick(p.M, units, (int)p.nb, cfg.num_sms, &p.gemv_nbr, &p.gemv_s);
     if (p.num_ctas < 0) return fail(COMET_ERR_UNSUPPORTED_SHAPE, "orientation 4: a CTA's K range exceeds the activation staging capacity");
     const int P = p.num_ctas;
     p.max_segments = gemv::gemv_max_segments(units, (int)p.nb, P);
@@ -104,6 +110,7 @@ comet_status_t build_plan(Plan& p, const comet_sched_config& cfg) {
     p.fix_info.clear();
     p.max_cost = (double)((units + P - 1) / P);
     p.mean_cost = (double)units / P;
+    // partial slots [ctas][max_segments][128][8] f32
     p.ws_flags_off = 0;
     p.ws_bytes = ((size_t)P * p.max_segments * 128 * 8 * sizeof(float) + 255) / 256 * 256;
     return COMET_OK;

@@ -334,7 +334,7 @@ __global__ void __launch_bounds__(256) k_pack_weight_perm(const int8_t* __restri
       const uint32_t hi = ((uint32_t)wr[p1] & 0xFu) ^ 8u;   // u[k0 + j + 4]
       word |= (lo | (hi << 4)) << (8 * j);
     }
-    out[i] = word;
+    out[packed_word_index(n, k0 / 8, K / kBlockK)] = word;
   }
 }
 
@@ -499,14 +499,17 @@ cudaError_t launch_q(const void* x, int64_t M, int64_t K, int64_t ldx, const Tag
 
 // ---------------------------------------------------------------------------- weight packing
 // u = w + 8 = (w & 0xF) ^ 8 per nibble; word byte i = u[i] | u[i+4] << 4 (include/comet.h).
-__global__ void __launch_bounds__(256) k_pack_weight(const uint2* __restrict__ w, int64_t words,
+// Row-tiled placement (include/comet.h): word g of row n goes to 1 KB tile (n/16, g/16), row
+// n % 16, word g % 16.
+__global__ void __launch_bounds__(256) k_pack_weight(const uint2* __restrict__ w, int64_t N, int64_t K,
                                                      uint32_t* __restrict__ out) {
+  const int64_t wpr = K / 8, words = N * wpr, nb = K / kBlockK;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < words;
        i += (int64_t)gridDim.x * blockDim.x) {
     const uint2 v = w[i];
     const uint32_t lo = (v.x & 0x0F0F0F0Fu) ^ 0x08080808u;   // u[k0..k3]
     const uint32_t hi = (v.y & 0x0F0F0F0Fu) ^ 0x08080808u;   // u[k4..k7]
-    out[i] = lo | (hi << 4);
+    out[packed_word_index(i / wpr, i % wpr, nb)] = lo | (hi << 4);
   }
 }
 
@@ -619,7 +622,7 @@ cudaError_t launch_pack_weight(const int8_t* w, int64_t N, int64_t K, void* w_pa
                                cudaStream_t stream) {
   const int64_t words = N * K / 8;
   const int64_t blocks = std::min<int64_t>(ceil_div(words, 256), 148 * 16);
-  k_pack_weight<<<(unsigned)blocks, 256, 0, stream>>>(reinterpret_cast<const uint2*>(w), words,
+  k_pack_weight<<<(unsigned)blocks, 256, 0, stream>>>(reinterpret_cast<const uint2*>(w), N, K,
                                                         static_cast<uint32_t*>(w_packed));
   return cudaGetLastError();
 }

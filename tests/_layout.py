@@ -45,10 +45,24 @@ def decode_act(buf: np.ndarray, scales: np.ndarray, M: int, K: int, tags: np.nda
     return codes.astype(np.int8), sc, qsum, corr
 
 
-def unpack_weight(wp: np.ndarray, N: int, K: int) -> np.ndarray:
-    """w_packed [N][K/2] -> codes int8 [N][K]: word g byte i = u[8g+i] | u[8g+i+4] << 4, u = w+8."""
+def unpack_words(wp: np.ndarray, N: int, K: int) -> np.ndarray:
+    """Row-major packed words [N][K/2] -> codes int8 [N][K]: word g byte i = u[8g+i] | u[8g+i+4] << 4,
+    u = w + 8 (the word format of include/comet.h)."""
     words = wp.reshape(N, K // 8, 4)
     lo = (words & 0x0F).astype(np.int16) - 8      # u[8g + i]
     hi = (words >> 4).astype(np.int16) - 8        # u[8g + 4 + i]
     out = np.concatenate([lo, hi], axis=2).reshape(N, K)
     return out.astype(np.int8)
+
+
+def untile_weight(wp: np.ndarray, N: int, K: int) -> np.ndarray:
+    """The row-tiled w_packed of include/comet.h -- 1 KB tiles [N/16][K/128][16 rows][64 B] --
+    back to row-major [N][K/2] bytes."""
+    nb = K // BLOCK
+    t = np.asarray(wp).reshape(N // 16, nb, 16, 64)
+    return np.ascontiguousarray(t.transpose(0, 2, 1, 3)).reshape(N, K // 2)
+
+
+def unpack_weight(wp: np.ndarray, N: int, K: int) -> np.ndarray:
+    """w_packed (row-tiled, include/comet.h) -> codes int8 [N][K]."""
+    return unpack_words(untile_weight(wp, N, K), N, K)

@@ -56,7 +56,7 @@ def test_grouped_full_size_decode_sampled():
     s_wg = _gs(N, K, 9)
     act, sc = cb.quantize_act(torch.from_numpy(p.x).to(DEV), p.tags)
     wp = cb.pack_weight(torch.from_numpy(p.w).to(DEV))
-    plan = cb.Plan(M, N, K, p.tags)
+    plan = cb.Plan(M, N, K, p.tags, orientation=1)   # group-wise scales run on the TMEM decode kernel
     y = cb.w4ax_gemm_grouped(plan, act, sc, wp, torch.from_numpy(s_wg).to(DEV))
     torch.cuda.synchronize()
     cols = np.random.default_rng(1).choice(N, 512, replace=False)

@@ -45,7 +45,7 @@ def test_linear_exact(M, K, N, frac, split_mode, num_sms, bf16):
                                  special_rows={0: "alternating"} if M > 1 else None)
     wp = cb.pack_weight(torch.from_numpy(p.w).to(DEV))
     sw = torch.from_numpy(p.s_w).to(DEV)
-    plan = cb.Plan(M, N, K, p.tags, split_mode=split_mode, num_sms=num_sms)
+    plan = cb.Plan(M, N, K, p.tags, split_mode=split_mode, num_sms=num_sms, orientation=1)   # the fused path's kernel
     x = _x_dev(p.x, bf16)
     y32 = cb.w4ax_linear_fused(plan, x, wp, sw, out_dtype=torch.float32)
     y16 = cb.w4ax_linear_fused(plan, x, wp, sw, out_dtype=torch.float16)

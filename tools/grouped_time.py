@@ -19,7 +19,7 @@ for name, K, N in (("gate_up", 8192, 28672), ("down", 28672, 8192), ("qkv", 8192
     swg = (sw[None, :] * (0.5 + torch.rand(K // 128, N, device=dev))).contiguous()
     x = bench.dev_activations(torch, M, K, tags, 2, dev)
     act, sc = cb.quantize_act(x, tags)
-    plan = cb.Plan(M, N, K, tags)
+    plan = cb.Plan(M, N, K, tags, **({"orientation": 1} if M < 128 else {}))
     y = torch.empty((M, N), dtype=torch.float16, device=dev)
     us_c = bench.us_rotating(torch, [lambda: cb.w4ax_gemm(plan, act, sc, wp, sw, out=y)], rounds=10)
     us_g = bench.us_rotating(torch, [lambda: cb.w4ax_gemm_grouped(plan, act, sc, wp, swg, out=y)], rounds=10)
