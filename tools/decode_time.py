@@ -1,7 +1,7 @@
 """Time the decode-regime GEMM (BASELINE config 5) alone: LLaMA-3-70B layers at small M, L2
 flushed before every launch.  Prints one line per (layer, M) and a JSON summary on the last line.
 
-  python tools/decode_time.py [--Ms 1,4,8,32] [--tile-n 0] [--split-mode -1] [--iters 20]
+  python tools/decode_time.py [--Ms 1,4,8,32] [--tile-n 0] [--split-mode -1] [--orientation 0] [--iters 20]
 """
 import argparse
 import json
@@ -24,6 +24,7 @@ def main():
     ap.add_argument("--Ms", default="1,4,8,32")
     ap.add_argument("--tile-n", type=int, default=0)
     ap.add_argument("--split-mode", type=int, default=-1)
+    ap.add_argument("--orientation", type=int, default=0, help="0 = auto, 1 = TMEM decode kernel, 4 = warp-level")
     ap.add_argument("--iters", type=int, default=20)
     ap.add_argument("--layers", default="gate_up,down,qkv")
     ap.add_argument("--flush", type=int, default=1, help="1 = write + read 256 MiB before every launch")
@@ -47,7 +48,7 @@ def main():
         swd = torch.from_numpy(s_w).to(dev)
         for M in [int(m) for m in a.Ms.split(",")]:
             x = torch.from_numpy(synth.make_activations(M, K, tags, rng)).to(dev)
-            plan = cb.Plan(M, N, K, tags, tile_n=a.tile_n, split_mode=a.split_mode)
+            plan = cb.Plan(M, N, K, tags, tile_n=a.tile_n, split_mode=a.split_mode, orientation=a.orientation)
             act, sc = cb.quantize_act(x, tags)
             y = torch.empty((M, N), dtype=torch.float16, device=dev)
             evs = []
