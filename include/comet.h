@@ -205,8 +205,8 @@ typedef struct {
                           comet_plan_info().stages), else COMET_ERR_INVALID_ARG */
   int device_plan;     /* 1 (default) = upload the work list to the device at create time;
                           0 = host-only plan (comet_plan_describe only; CPU-safe) */
-  int orientation;     /* 0 = auto (3 when M >= 256, 2 when M >= 128, 4 when M == 1 or M <= 4
-                              with K <= 16384 and the packed weights take >= 96 MiB, else 1);
+  int orientation;     /* 0 = auto (3 when M >= 256, 2 when M >= 128, 4 when M <= 8 and the
+                              packed weights take >= 32 MiB, else 1);
                           1 = weights on the MMA M side: tile = 128 weights x tile_n tokens
                               (decode-sized M; weights widened into TMEM);
                           2 = tokens on the MMA M side: tile = 128 tokens x tile_w weights

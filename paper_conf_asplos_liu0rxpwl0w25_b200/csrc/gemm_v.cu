@@ -209,29 +209,57 @@ __global__ void __launch_bounds__(256, COMET_GEMV_CPS) k_gemv(const __grid_const
 }
 
 // y[m][n] = s_w[n] * sum over the CTAs covering n's row group (in CTA order) of their partials.
-__global__ void __launch_bounds__(256) k_gemv_reduce(const __grid_constant__ VParams P) {
+// One CTA per row group, one thread per row: the group's contributing CTAs and their slots are
+// computed once (the 64-bit divisions off the per-output path), then each thread reads its row's
+// [8 tokens] from every slot with two 16-byte loads, all issued before the in-order sum.
+constexpr int kMaxRed = 64;   // contributing CTAs a group can have (plan: at most one CTA per unit)
+__global__ void __launch_bounds__(kRowsCta) k_gemv_reduce(const __grid_constant__ VParams P) {
   asm volatile("griddepcontrol.launch_dependents;");           // the next layer may start
-  asm volatile("griddepcontrol.wait;" ::: "memory");
-  const int64_t total = P.M * P.N;
-  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (i >= total) return;
-  const int64_t m = i / P.N, n = i - m * P.N;
-  const int64_t grp = n / kRowsCta;
-  const int r = (int)(n - grp * kRowsCta);
-  const int64_t ua = grp * P.nb, ub = ua + P.nb - 1;            // the group's first / last unit
-  // CTA owning unit u: the largest c with floor(units c / ctas) <= u
-  auto owner = [&](int64_t u) { return (int)(((u + 1) * P.ctas - 1) / P.units); };
-  const int ca = owner(ua), cb = owner(ub);
-  float acc = 0.f;
-  for (int c = ca; c <= cb; ++c) {
-    const int64_t first = (P.units * c / P.ctas) / P.nb;         // first group of CTA c
-    const int seg = (int)(grp - first);
-    acc += P.part[((int64_t)(c * P.maxseg + seg) * kRowsCta + r) * 8 + m];
+  __shared__ int s_slot[kMaxRed];
+  __shared__ int s_n;
+  const int64_t grp = blockIdx.x;
+  const int r = threadIdx.x;
+  if (r == 0) {
+    // CTA owning unit u: the largest c with floor(units c / ctas) <= u
+    auto owner = [&](int64_t u) { return (int)(((u + 1) * P.ctas - 1) / P.units); };
+    s_n = owner(grp * P.nb + P.nb - 1) - owner(grp * P.nb) + 1;
+    s_slot[0] = owner(grp * P.nb);
   }
-  const float f = acc * P.w_scales[n];
-  if (P.ydt == COMET_F32) reinterpret_cast<float*>(P.y)[m * P.ldy + n] = f;
-  else if (P.ydt == COMET_BF16) reinterpret_cast<__nv_bfloat16*>(P.y)[m * P.ldy + n] = __float2bfloat16_rn(f);
-  else reinterpret_cast<__half*>(P.y)[m * P.ldy + n] = __float2half_rn(f);
+  __syncthreads();
+  const int nc = s_n, ca = s_slot[0];
+  __syncthreads();
+  for (int c = ca + r; c < ca + nc; c += blockDim.x)            // slot of the group in CTA c
+    s_slot[c - ca] = c * P.maxseg + (int)(grp - (P.units * c / P.ctas) / P.nb);
+  __syncthreads();
+  const int64_t n = grp * kRowsCta + r;
+  const float sw = __ldg(P.w_scales + n);
+  asm volatile("griddepcontrol.wait;" ::: "memory");           // the GEMM's partials are complete
+  float acc[8] = {};
+  constexpr int B = 4;                                          // slots read per batch
+  for (int c0 = 0; c0 < nc; c0 += B) {
+    float4 v[B][2];
+#pragma unroll
+    for (int b = 0; b < B; ++b)
+      if (c0 + b < nc) {
+        const float4* src = reinterpret_cast<const float4*>(P.part + ((int64_t)s_slot[c0 + b] * kRowsCta + r) * 8);
+        v[b][0] = __ldcg(src);
+        v[b][1] = __ldcg(src + 1);
+      }
+#pragma unroll
+    for (int b = 0; b < B; ++b)
+      if (c0 + b < nc) {
+        acc[0] += v[b][0].x; acc[1] += v[b][0].y; acc[2] += v[b][0].z; acc[3] += v[b][0].w;
+        acc[4] += v[b][1].x; acc[5] += v[b][1].y; acc[6] += v[b][1].z; acc[7] += v[b][1].w;
+      }
+  }
+#pragma unroll
+  for (int m = 0; m < 8; ++m) {
+    if (m >= P.M) break;
+    const float f = acc[m] * sw;
+    if (P.ydt == COMET_F32) reinterpret_cast<float*>(P.y)[m * P.ldy + n] = f;
+    else if (P.ydt == COMET_BF16) reinterpret_cast<__nv_bfloat16*>(P.y)[m * P.ldy + n] = __float2bfloat16_rn(f);
+    else reinterpret_cast<__half*>(P.y)[m * P.ldy + n] = __float2half_rn(f);
+  }
 }
 
 }  // namespace
@@ -254,6 +282,11 @@ int gemv_max_segments(int64_t units, int nb, int ctas) {
 size_t gemv_smem_bytes(int64_t M, int nbr, int S) {
   return (size_t)8 * S * 1024 + (size_t)nbr * (M * 128 + 8 * 4 + 4 * 4);
 }
+// CTAs sharing one row group (the reduction reads at most kMaxRed)
+static int gemv_max_group_ctas(int64_t units, int nb, int ctas) {
+  const int64_t per = units / ctas;                             // units per CTA, rounded down
+  return per <= 0 ? nb : (int)std::min<int64_t>(nb, (nb + per - 1) / per + 1);
+}
 int gemv_stage_blocks(int64_t units, int nb, int ctas) {
   const int64_t len = (units + ctas - 1) / ctas;
   const int nbr = (int)std::min<int64_t>(nb, len);
@@ -271,7 +304,7 @@ int gemv_pick(int64_t M, int64_t units, int nb, int num_sms, int* nbr_out, int* 
     for (int cps = COMET_GEMV_CPS; cps >= 1; --cps) {
       const int ctas = (int)std::min<int64_t>((int64_t)num_sms * cps, units);   // no empty ranges
       const int nbr = gemv_stage_blocks(units, nb, ctas);
-      if (nbr < 0) continue;
+      if (nbr < 0 || gemv_max_group_ctas(units, nb, ctas) > kMaxRed) continue;
       if ((size_t)cps * (gemv_smem_bytes(M, nbr, S) + 1024) > (size_t)228 * 1024) continue;
       if (S * cps > best) { best = S * cps; best_ctas = ctas; *nbr_out = nbr; *s_out = S; }
       break;                                                 // fewer CTAs at this S: never better
@@ -318,7 +351,8 @@ cudaError_t launch_gemv(const uint8_t* w, const uint8_t* codes, const float* sca
   cfg.numAttrs = 1;
   cudaError_t e = cudaLaunchKernelEx(&cfg, kern, P);
   if (e != cudaSuccess) return e;
-  cfg.gridDim = dim3((unsigned)ceil_div(M * N, 256));
+  cfg.gridDim = dim3((unsigned)(N / kRowsCta));
+  cfg.blockDim = dim3(kRowsCta);
   cfg.dynamicSmemBytes = 0;
   return cudaLaunchKernelEx(&cfg, k_gemv_reduce, P);
 }

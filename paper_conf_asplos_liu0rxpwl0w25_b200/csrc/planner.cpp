@@ -77,11 +77,15 @@ comet_status_t build_plan(Plan& p, const comet_sched_config& cfg) {
   p.Mp = round_up(p.M, COMET_SCALE_PAD);
   p.orientation = cfg.orientation > 0 ? cfg.orientation : (p.M >= 256 ? 3 : (p.M >= 128 ? 2 : 1));
   // decode on the warp-level path (gemm_v.cu) where it measured faster than the TMEM kernel:
-  // large layers (>= 96 MiB of packed weights) at M = 1, or M <= 4 with K <= 16384
-  // (tools/gemv_ab.py: LLaMA-3-70B gate/up 23.8 vs 28.1 us at M = 1, 25.9 vs 27.6 at M = 4;
-  // down 26.2 vs 26.6 at M = 1, but 27.4 vs 26.5 at M = 4; qkv, 42 MB, 14.5 vs 14.2)
-  if (cfg.orientation <= 0 && (p.M == 1 || (p.M <= 4 && p.K <= 16384)) && p.N * p.K / 2 >= (96ll << 20))
-    p.orientation = 4;
+  // M <= 8 with >= 32 MiB of packed weights (tools/gemv_ab.py, LLaMA-3-70B: gate/up M = 1 / 4 / 8
+  // 22.x / 24.0 / 26.6 vs 28.0 / 27.3 / 27.8 us, down 23.5 / 24.6 / 27.6 vs 26.6 / 26.7 / 27.3,
+  // qkv 12.2 / 12.5 / 12.7 vs 14.2; the 8-22 MB LLaMA-2-7B layers are mixed and stay on 1)
+  bool auto_o4 = false;
+  if (cfg.orientation <= 0 && p.M <= 8 && p.N * p.K / 2 >= (32ll << 20)) {
+    int nbr = 0, s = 0;
+    auto_o4 = gemv::gemv_pick(p.M, (p.N / 128) * (p.K / kBlockK), (int)(p.K / kBlockK), cfg.num_sms, &nbr, &s) > 0;
+    if (auto_o4) p.orientation = 4;
+  }
   if (p.orientation == 4) {
     // decode on the warp-level tensor-core path (gemm_v.cu): units (128-row group, K-block),
     // group-major, cut into one contiguous range per CTA (CTA-level stream-K); no work list,
@@ -97,7 +101,7 @@ comet_status_t build_plan(Plan& p, const comet_sched_config& cfg) {
     p.n_tiles = p.n_n_tiles;
     const int64_t units = p.n_tiles * p.nb;
     p.num_ctas = gemv::gemv_pick(p.M, units, (int)p.nb, cfg.num_sms, &p.gemv_nbr, &p.gemv_s);
-    if (p.num_ctas < 0) return fail(COMET_ERR_UNSUPPORTED_SHAPE, "orientation 4: a CTA's K range exceeds the activation staging capacity");
+    if (p.num_ctas < 0) return fail(COMET_ERR_UNSUPPORTED_SHAPE, "orientation 4: shape unsupported (a CTA's K range exceeds the activation staging capacity, or more than 64 CTAs share a row group)");
     const int P = p.num_ctas;
     p.max_segments = gemv::gemv_max_segments(units, (int)p.nb, P);
     p.n_split_tiles = 0;                       // groups shared by more than one CTA

@@ -123,12 +123,12 @@ ALL = CFG2 + CFG3 + CFG4 + CFG5
 def test_production_exact_full_size(name, M, K, N, frac):
     info = run_exact(M, K, N, frac, seed=sum(map(ord, name)))
     # the launch configuration bench.py times: pair kernel for prefill, a decode kernel below 128
-    # (the warp-level one for the large layers at M = 1, or M <= 4 with K <= 16384)
-    o4 = (M == 1 or (M <= 4 and K <= 16384)) and N * K // 2 >= (96 << 20)
+    # (the warp-level one for M <= 8 on layers of >= 32 MiB of packed weights)
+    o4 = M <= 8 and N * K // 2 >= (32 << 20)
     assert info["orientation"] == (3 if M >= 256 else (2 if M >= 128 else (4 if o4 else 1)))
 
 
-O1_DECODE = [c for c in CFG5 if c[1] <= 4 and c[3] * c[2] // 2 >= (96 << 20)]
+O1_DECODE = [c for c in CFG5 if c[1] <= 8 and c[3] * c[2] // 2 >= (32 << 20)]
 
 
 @pytest.mark.parametrize("name,M,K,N,frac", O1_DECODE, ids=[c[0] + "_o1" for c in O1_DECODE])

@@ -1,7 +1,7 @@
 """Decode GEMM A/B: plan orientation 1 (tcgen05, TMEM-widened weights) against orientation 4
 (gemm_v.cu, mma.sync with register-streamed weights) on the config-5 layers at M = 1, 4, 8.
 Same timing as bench.py's decode sweep: back-to-back launches over weight copies > 2 x L2.
-Usage: python tools/gemv_ab.py [orientations, default 1,4]"""
+Usage: python tools/gemv_ab.py [orientations, default 1,4] [c2: LLaMA-2-7B shapes]"""
 import os
 import sys
 
@@ -16,7 +16,10 @@ from paper_conf_asplos_liu0rxpwl0w25_b200 import synth  # noqa: E402
 dev = torch.device("cuda", 0)
 peaks, _ = bench.load_peaks()
 orients = [int(o) for o in (sys.argv[1] if len(sys.argv) > 1 else "1,4").split(",")]
-for li, (name, K, N, kind) in enumerate(bench.LAYERS):
+layers = bench.LAYERS
+if len(sys.argv) > 2 and sys.argv[2] == "c2":   # LLaMA-2-7B (config 2) shapes
+    layers = [("qkvo", 4096, 4096, "col"), ("gate_up", 4096, 11008, "col"), ("down", 11008, 4096, "row")]
+for li, (name, K, N, kind) in enumerate(layers):
     tags = synth.make_tags(K, bench.FRAC, np.random.default_rng(7))
     wp, swd, _ = bench.dev_weights(cb, torch, N, K, 70 + li, dev)
     ncopy = max(2, -(-300 * (1 << 20) // (N * K // 2)))
