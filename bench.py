@@ -303,10 +303,10 @@ def decode_sweep(cb, torch, dev, peaks, timer, Ms=(1, 4, 8, 32), iters=20, rank=
             # the same layer step as ONE launch (comet_w4ax_linear: kernel 1 fused into the GEMM,
             # for 16-token decode tiles)
             us_fused = None
-            if M <= 8:
-                plan_f = plan if plan.info()["orientation"] == 1 else cb.Plan(M, Nl, Kl, tl, orientation=1)
-                if plan_f.info()["tile_n"] == 16:
-                    us_fused = us_rotating(torch, [lambda w_=w_: cb.w4ax_linear_fused(plan_f, x, w_, swd, out=y) for w_ in wps])
+            # (orientation 4: the warp-level kernel quantises its own K range; orientation 1: the TMEM
+            # kernel's quantiser warps, 16-token tiles)
+            if M <= 8 and plan.info()["orientation"] in (1, 4) and plan.info()["tile_n"] in (8, 16):
+                us_fused = us_rotating(torch, [lambda w_=w_: cb.w4ax_linear_fused(plan, x, w_, swd, out=y) for w_ in wps])
             # SURVEY §8(d) decode ablation: the same GEMM on the other decode kernel -- orientation 1
             # (tcgen05, weights widened into TMEM) or 4 (gemm_v.cu: mma.sync u8 x s8, weights
             # streamed by cp.async into per-warp rings), whichever the auto plan did not pick
@@ -344,7 +344,7 @@ def decode_sweep(cb, torch, dev, peaks, timer, Ms=(1, 4, 8, 32), iters=20, rank=
                       "weight copies (> 2 x L2: every launch streams from HBM); isolated_us: one event-bracketed launch after a "
                       "256 MiB write + 256 MiB read (median of 20; includes the ~6 us an empty kernel measures that way)",
             "step": "step_us = kernel 1 (quantise x) + the GEMM as one decode layer step (the GEMM is a programmatic dependent launch), back to back; "
-                    "fused_step_us = the same step as one comet_w4ax_linear launch (kernel 1 fused into the GEMM, 16-token tiles); "
+                    "fused_step_us = the same step through comet_w4ax_linear (kernel 1 fused into the auto plan's GEMM: no kernel-1 launch); "
                     "orientation = the auto plan's decode kernel (1: tcgen05 + TMEM-widened weights, 4: gemm_v.cu warp-level mma.sync "
                     "with cp.async weight rings); o1_tmem_us / o4_mma_sync_us = the same GEMM on the other one (ablation)",
             "layers": out}

@@ -343,8 +343,9 @@ def w4ax_gemm(plan: Plan, act_packed, act_scales, w_packed, w_scales, *, out=Non
 
 
 def w4ax_linear_fused(plan: Plan, x, w_packed, w_scales, *, out=None, out_dtype=None, stream=None):
-    """comet_w4ax_linear: the decode layer (kernel 1 fused into the GEMM) for plans with
-    orientation 1, 16-token tiles and M <= 8.  x: [M, K] float16 / bfloat16 on the device."""
+    """comet_w4ax_linear: the decode layer with kernel 1 fused into the GEMM, M <= 8, for plans
+    with orientation 4 (the warp-level decode kernel; the reduction is a second launch) or
+    orientation 1 with 16-token tiles.  x: [M, K] float16 / bfloat16 on the device."""
     import torch
     dev = x.device
     if out is None:
@@ -384,6 +385,9 @@ def w4ax_linear(plan: Plan, x, w_packed, w_scales, *, perm=None, out=None, out_d
     channel permutation when perm is given; w_packed then packed with the same perm) +
     w4ax_gemm."""
     info = plan.info()
+    if perm is None and info["orientation"] == 4:
+        # the warp-level decode kernel quantises its own K range: no kernel-1 launch (DESIGN §7.11)
+        return w4ax_linear_fused(plan, x, w_packed, w_scales, out=out, out_dtype=out_dtype, stream=stream)
     if (perm is None and info["orientation"] == 1 and info["tile_n"] == 16 and plan.M <= 4
             and info["n_tiles"] * -(-plan.K // 512) <= 12 * info["num_ctas"]):
         # the fused launch wins while the CTAs' quantiser warps keep up with the weight stream:

@@ -1036,8 +1036,8 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
                            cudaStream_t stream, int* launches, bool grouped, const RsArgs* rs,
                            const FusedX* fx) {
   using namespace gemm;
-  if (fx && (p.orientation != 1 || p.tile_n != 16 || p.M > 8 || grouped || rs || debug_acc || debug_acc_blocks))
-    return fail(COMET_ERR_UNSUPPORTED_SHAPE, "the fused decode path needs orientation 1 with 16-token tiles and M <= 8");
+  if (fx && !(p.orientation == 4 || (p.orientation == 1 && p.tile_n == 16)) || (fx && (p.M > 8 || grouped || rs || debug_acc || debug_acc_blocks)))
+    return fail(COMET_ERR_UNSUPPORTED_SHAPE, "the fused decode path needs M <= 8 and orientation 4, or orientation 1 with 16-token tiles");
   static_assert(Cfg<16, false, true>::SX % 2 == 0, "the fused quantiser's two warps own alternate X slots");
   if (grouped && p.orientation != 1 && !(p.orientation == 3 && p.tile_w == 256))
     return fail(COMET_ERR_UNSUPPORTED_SHAPE, "group-wise weight scales run on orientation 1 or on the 256-wide pair kernel (orientation 3)");
@@ -1045,7 +1045,7 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
     return fail(COMET_ERR_UNSUPPORTED_SHAPE, "group-wise weight scales on the pair kernel have no debug accumulators");
   *launches = 0;
   if (p.orientation == 4) {
-    if (grouped || rs || fx || debug_acc || debug_acc_blocks)
+    if (grouped || rs || debug_acc || debug_acc_blocks)
       return fail(COMET_ERR_UNSUPPORTED_SHAPE, "orientation 4 (decode, M <= 8) runs per-channel weight scales without debug outputs");
     if (p.d_items == nullptr) return fail(COMET_ERR_INVALID_ARG, "plan was created with device_plan = 0");
     if (workspace == nullptr || ws_bytes < p.ws_bytes)
@@ -1053,10 +1053,12 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
     comet_act_layout_t L;
     act_layout(p.M, p.K, &L);
     const uint8_t* base = static_cast<const uint8_t*>(act_packed);
-    cudaError_t e = gemv::launch_gemv(static_cast<const uint8_t*>(w_packed), base + L.codes_off, act_scales,
-                                      reinterpret_cast<const int16_t*>(base + L.qsum_off), w_scales, y, (int)ydt,
-                                      ldy, p.M, p.N, p.K, L.Mp, p.mask, p.num_ctas, p.max_segments,
-                                      p.gemv_nbr, p.gemv_s, static_cast<float*>(workspace), stream);
+    // fx (comet_w4ax_linear): the kernel quantises x itself -- one launch + the reduction
+    cudaError_t e = gemv::launch_gemv(static_cast<const uint8_t*>(w_packed), fx ? nullptr : base + L.codes_off,
+                                      act_scales, fx ? nullptr : reinterpret_cast<const int16_t*>(base + L.qsum_off),
+                                      w_scales, y, (int)ydt, ldy, p.M, p.N, p.K, L.Mp, p.mask, p.num_ctas,
+                                      p.max_segments, p.gemv_nbr, p.gemv_s, static_cast<float*>(workspace), stream,
+                                      fx ? fx->x : nullptr, fx ? fx->ldx : 0, fx ? fx->bf16 : false);
     if (e != cudaSuccess) return cuda_status(e, "w4ax gemv launch");
     *launches = 2;
     return COMET_OK;

@@ -32,6 +32,7 @@
 #include <cuda_fp16.h>
 #include <cuda_bf16.h>
 #include "internal.h"
+#include "fmpq.cuh"
 
 #ifndef COMET_GEMV_S
 #define COMET_GEMV_S 8      // deepest ring (K-blocks in flight per warp, 1 KB stages); gemv_pick may take 6 or 4
@@ -55,6 +56,9 @@ struct VParams {
   const int16_t* qsum;     // code sums [nb][Mp]
   float* part;             // partials [ctas][maxseg][128][8]
   const float* w_scales;   // s_w [N]
+  const uint16_t* x;       // FQ: the layer input [M][ldx] f16 / bf16 (kernel 1 fused into the staging)
+  int64_t ldx;
+  int xbf16;
   void* y;
   int64_t M, N, K, Mp, ldy, units;
   int nb, maxseg, ctas, nbr, ydt;
@@ -88,7 +92,7 @@ __device__ __forceinline__ uint32_t e4m3x4_to_s8(uint32_t e) {
   return __byte_perm(h0, h1, 0x6420);
 }
 
-template <int S>
+template <int S, bool FQ>
 __global__ void __launch_bounds__(256, COMET_GEMV_CPS) k_gemv(const __grid_constant__ VParams P) {
   extern __shared__ __align__(16) uint8_t smem[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, g = lane >> 2, t = lane & 3;
@@ -129,6 +133,49 @@ __global__ void __launch_bounds__(256, COMET_GEMV_CPS) k_gemv(const __grid_const
   }
   asm volatile("griddepcontrol.wait;" ::: "memory");
   // ---- stage the range's activation codes (s8), scales and code sums
+  if constexpr (FQ) {
+    // kernel 1 fused (comet_w4ax_linear): each lane quad quantises one (K-block, token) of the
+    // range from x with kernel 1's own arithmetic (fmpq.cuh: the same codes, scales and code
+    // sums bit for bit); INT4 codes go to shared memory as s8.  Tokens >= M keep s_a = qsum = 0.
+    for (int i = threadIdx.x; i < P.nbr * 8; i += blockDim.x) {
+      s_s[i] = 0.f;
+      if ((i & 1) == 0) s_q[i >> 1] = 0;
+    }
+    __syncthreads();
+    const int quad = threadIdx.x >> 2, sub = threadIdx.x & 3;
+    const int npairs = P.nbr * M;
+    for (int base = 0; base < npairs; base += 64) {              // warp-uniform trip count
+      const int pr = base + quad;
+      const bool ok = pr < npairs;
+      const int j = ok ? pr / M : 0, m = ok ? pr - j * M : 0;
+      const int kb = (kb_s + j) % nb;
+      float v[32];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        uint4 raw = make_uint4(0, 0, 0, 0);
+        if (ok) raw = __ldg(reinterpret_cast<const uint4*>(P.x + m * P.ldx + kb * 128 + 32 * q + 8 * sub));
+        float tq[8];
+        if (P.xbf16) fmpq::unpack8<true>(raw, tq); else fmpq::unpack8<false>(raw, tq);
+#pragma unroll
+        for (int e = 0; e < 8; ++e) v[8 * q + e] = tq[e];
+      }
+      const bool is8 = ok && ((P.tags.w[kb >> 5] >> (kb & 31)) & 1u);
+      const fmpq::LaneOut o = fmpq::quantize32(v, is8);
+      if (ok) {
+        uint8_t* row = s_x + (j * M + m) * 128;
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {            // channels 32q + 8 sub .. + 7: chunk 2q + sub/2, half sub&1
+          uint2 c = o.c[q];
+          if (!is8) { c.x = e4m3x4_to_s8(c.x); c.y = e4m3x4_to_s8(c.y); }
+          *reinterpret_cast<uint2*>(row + (((2 * q + (sub >> 1)) ^ (m & 1)) << 4) + (sub & 1) * 8) = c;
+        }
+        if (sub == 0) {
+          s_s[j * 8 + m] = o.s;
+          reinterpret_cast<int16_t*>(s_q)[j * 8 + m] = (int16_t)o.q;
+        }
+      }
+    }
+  } else {
   for (int i = threadIdx.x; i < P.nbr * M * 8; i += blockDim.x) {   // 16-byte chunks
     const int j = i / (M * 8), r = i - j * (M * 8), m = r >> 3, ch = r & 7;
     const int kb = (kb_s + j) % nb;
@@ -145,6 +192,7 @@ __global__ void __launch_bounds__(256, COMET_GEMV_CPS) k_gemv(const __grid_const
     const int kb = (kb_s + j) % nb;
     s_s[i] = P.scales[(int64_t)kb * P.Mp + m];                       // rows >= M: 0 (kernel 1)
     if ((m & 1) == 0) s_q[i >> 1] = *reinterpret_cast<const int*>(P.qsum + (int64_t)kb * P.Mp + m);
+  }
   }
   __syncthreads();
 
@@ -315,7 +363,7 @@ int gemv_pick(int64_t M, int64_t units, int nb, int num_sms, int* nbr_out, int* 
 cudaError_t launch_gemv(const uint8_t* w, const uint8_t* codes, const float* scales, const int16_t* qsum,
                         const float* w_scales, void* y, int ydt, int64_t ldy, int64_t M, int64_t N,
                         int64_t K, int64_t Mp, const TagMask& tags, int ctas, int maxseg, int nbr,
-                        int S, float* part, cudaStream_t stream) {
+                        int S, float* part, cudaStream_t stream, const void* x, int64_t ldx, bool xbf16) {
   VParams P;
   P.w = w; P.codes = codes; P.scales = scales; P.qsum = qsum; P.part = part; P.w_scales = w_scales;
   P.y = y; P.M = M; P.N = N; P.K = K; P.Mp = Mp; P.ldy = ldy;
@@ -326,11 +374,16 @@ cudaError_t launch_gemv(const uint8_t* w, const uint8_t* codes, const float* sca
   P.nbr = nbr;
   P.ydt = ydt;
   P.tags = tags;
+  P.x = static_cast<const uint16_t*>(x);
+  P.ldx = ldx;
+  P.xbf16 = xbf16 ? 1 : 0;
   const size_t smem = gemv_smem_bytes(M, nbr, S);
-  auto kern = S == 8 ? k_gemv<8> : S == 6 ? k_gemv<6> : k_gemv<4>;
+  const bool fq = x != nullptr;
+  auto kern = S == 8 ? (fq ? k_gemv<8, true> : k_gemv<8, false>)
+            : S == 6 ? (fq ? k_gemv<6, true> : k_gemv<6, false>) : (fq ? k_gemv<4, true> : k_gemv<4, false>);
   // the dynamic shared memory this launch needs (set per device and ring depth when it grows)
-  static std::atomic<int> attr_bytes[3][64];
-  const int si = S == 8 ? 0 : S == 6 ? 1 : 2;
+  static std::atomic<int> attr_bytes[6][64];
+  const int si = (S == 8 ? 0 : S == 6 ? 1 : 2) + (fq ? 3 : 0);
   int dev = 0;
   cudaGetDevice(&dev);
   if ((int)smem > attr_bytes[si][dev & 63].load()) {

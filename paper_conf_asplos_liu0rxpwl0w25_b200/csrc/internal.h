@@ -130,7 +130,8 @@ int gemv_pick(int64_t M, int64_t units, int nb, int num_sms, int* nbr_out, int* 
 cudaError_t launch_gemv(const uint8_t* w, const uint8_t* codes, const float* scales, const int16_t* qsum,
                         const float* w_scales, void* y, int ydt, int64_t ldy, int64_t M, int64_t N,
                         int64_t K, int64_t Mp, const TagMask& tags, int ctas, int maxseg, int nbr,
-                        int S, float* part, cudaStream_t stream);
+                        int S, float* part, cudaStream_t stream, const void* x = nullptr, int64_t ldx = 0,
+                        bool xbf16 = false);
 }
 namespace gemm {
 cudaError_t launch_debug_widen(uint64_t first, int64_t n, int is8, uint32_t* out, cudaStream_t stream);

@@ -40,12 +40,15 @@ def _x_dev(x, bf16=False):
     (5, 1152, 256, 1.0, 0, 0, False),           # all INT8 blocks, whole tiles
     (2, 2048, 640, 0.0, 1, 37, True),           # all INT4 blocks
 ])
-def test_linear_exact(M, K, N, frac, split_mode, num_sms, bf16):
+@pytest.mark.parametrize("orientation", [1, 4])
+def test_linear_exact(M, K, N, frac, split_mode, num_sms, bf16, orientation):
+    """Both fused decode paths: the TMEM kernel's quantiser warps (orientation 1) and the
+    warp-level kernel's fused staging (orientation 4)."""
     p = synth.make_exact_problem(M, K, N, frac=frac, seed=M * 7 + K, bf16=bf16,
                                  special_rows={0: "alternating"} if M > 1 else None)
     wp = cb.pack_weight(torch.from_numpy(p.w).to(DEV))
     sw = torch.from_numpy(p.s_w).to(DEV)
-    plan = cb.Plan(M, N, K, p.tags, split_mode=split_mode, num_sms=num_sms, orientation=1)   # the fused path's kernel
+    plan = cb.Plan(M, N, K, p.tags, split_mode=split_mode, num_sms=num_sms, orientation=orientation)
     x = _x_dev(p.x, bf16)
     y32 = cb.w4ax_linear_fused(plan, x, wp, sw, out_dtype=torch.float32)
     y16 = cb.w4ax_linear_fused(plan, x, wp, sw, out_dtype=torch.float16)
