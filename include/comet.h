@@ -288,18 +288,21 @@ comet_status_t comet_w4ax_gemm(comet_plan_t plan, const void* act_packed, const 
                                int32_t* debug_acc_blocks, void* workspace, size_t ws_bytes,
                                void* stream);
 
-/* The decode layer in one launch (kernel 1 fused into the GEMM, the per-token
- * quantisation of P:L126 / P:L136-138 as comet_quantize_act defines it):
- *   Y = W4Ax(FMPQ(x), W)      for plans with orientation 1, 16-token tiles and M <= 8
- * x: device [M][ldx] F16 or BF16 (ldx >= K, x and ldx*2 16-byte aligned).  Each pipeline stage's
- * input rows arrive by TMA and one warp per CTA quantises them into the MMA's operand slot with
- * comet_quantize_act's arithmetic -- identical codes, scales and code sums -- so there is no
- * activation buffer and no kernel-1 launch; the offset-binary weight term is removed per block
- * (every block sum is exact), so outputs equal the two-launch path's within FP32
- * reassociation, and bit for bit when every partial sum is exact.  Other arguments as
- * comet_w4ax_gemm; other plans get COMET_ERR_UNSUPPORTED_SHAPE.  Launched as a programmatic
- * dependent of the preceding kernel on the stream (its weight stream starts while that kernel
- * finishes; x is read only after it completed). */
+/* The decode layer without a kernel-1 launch (kernel 1 fused into the GEMM, the
+ * per-token quantisation of P:L126 / P:L136-138 as comet_quantize_act defines it):
+ *   Y = W4Ax(FMPQ(x), W)      for M <= 8 and plans with orientation 4, or orientation 1 with
+ *                              16-token tiles
+ * x: device [M][ldx] F16 or BF16 (ldx >= K, x and ldx*2 16-byte aligned).  Orientation 1: each
+ * pipeline stage's input rows arrive by TMA and one warp per CTA quantises them into the MMA's
+ * operand slot (one launch).  Orientation 4: every CTA quantises the K-blocks of its range from
+ * x into shared memory before its weight loop (the GEMM launch, plus the plan's reduction
+ * launch).  Both use comet_quantize_act's arithmetic -- identical codes, scales and code sums --
+ * so there is no activation buffer; the offset-binary weight term is removed per block (every
+ * block sum is exact), so outputs equal the two-launch path's within FP32 reassociation, and bit
+ * for bit when every partial sum is exact.  Other arguments as comet_w4ax_gemm; other plans get
+ * COMET_ERR_UNSUPPORTED_SHAPE.  Launched as a programmatic dependent of the preceding kernel on
+ * the stream (its weight stream starts while that kernel finishes; x is read only after it
+ * completed). */
 comet_status_t comet_w4ax_linear(comet_plan_t plan, const void* x, comet_dtype_t xdt, int64_t ldx,
                                  const void* w_packed, const float* w_scales, void* y,
                                  comet_dtype_t ydt, int64_t ldy, void* workspace, size_t ws_bytes,
