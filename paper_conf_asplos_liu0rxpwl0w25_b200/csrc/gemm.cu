@@ -271,11 +271,12 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
         const WorkItem w = item(it);
         const int n0 = (w.tile / P.n_m_tiles) * kTileW;
         for (int kb = w.kb_begin; kb < w.kb_end; kb += KS) {
-          const int npair = (min(KS, w.kb_end - kb) + 1) >> 1;
+          // one box per stage: KS K-blocks of the 128 rows, landing as [8 row tiles][KS][16][64 B]
+          // (each row tile's KS K-blocks are contiguous in the packed layout: 8 requests of KS KB;
+          // K-blocks past the tensor are zero-filled and counted)
           mbar_wait(&empty_w[st], ph ^ 1);
-          mbar_arrive_expect_tx(&full_w[st], npair * 2 * kTileW * 64);
-          for (int p = 0; p < npair; ++p)
-            tma_load_4d(sW(st) + p * 2 * kTileW * 64, &P.map_w, &full_w[st], 0, 0, kb + 2 * p, n0 / kWTileRows);
+          mbar_arrive_expect_tx(&full_w[st], C::W_BYTES);
+          tma_load_4d(sW(st), &P.map_w, &full_w[st], 0, 0, kb, n0 / kWTileRows);
           trace_ev(P, 0, tr++);
           if (++st == SW) { st = 0; ph ^= 1; }
         }
@@ -459,10 +460,10 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
     const int q = warp & 3;
     const int r = q * 32 + lane;                  // TMEM lane = weight row within the tile
     const uint32_t lane_addr = (uint32_t)(q * 32) << 16;
-    // a pair box lands as [8 row tiles][2 K-blocks][16 rows][64 B] (the packed layout's 1 KB
+    // a stage's box lands as [8 row tiles][KS K-blocks][16 rows][64 B] (the packed layout's 1 KB
     // tiles, include/comet.h) with the TMA 64-byte swizzle: chunk ^= (row >> 1) & 3
     const int sw = (r >> 1) & 3;
-    const uint32_t roff = (uint32_t)((r >> 4) * 2048 + (r & 15) * 64);   // + (cb & 1) KB
+    const uint32_t roff = (uint32_t)((r >> 4) * KS * 1024 + (r & 15) * 64);   // + cb KB
     int st = 0, ab = 0;
     uint32_t ph = 0, aph = 0;
     int seq = 0;
@@ -485,7 +486,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
 #pragma unroll
       for (int i = 0; i < KH; ++i) {
         const int cb = half * KH + i;
-        const uint32_t row = smem_u32(sW(st)) + (cb >> 1) * 2 * kTileW * 64 + roff + (cb & 1) * 1024;
+        const uint32_t row = smem_u32(sW(st)) + roff + cb * 1024;
 #pragma unroll
         for (int j = 0; j < 4; ++j)
           cn[4 * i + j] = (cb < nk_n && !(COMET_DEC_ABLATE & 8)) ? lds128(row + ((j ^ sw) << 4))
@@ -559,7 +560,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_w4ax(const __grid_constant__ Ge
 #pragma unroll
         for (int i = 0; i < KH; ++i) {
           const int cb = half * KH + i;
-          const uint32_t row = smem_u32(sW(st)) + (cb >> 1) * 2 * kTileW * 64 + roff + (cb & 1) * 1024;
+          const uint32_t row = smem_u32(sW(st)) + roff + cb * 1024;
 #pragma unroll
           for (int j = 0; j < 4; ++j)
             cc[4 * i + j] = (cb < nk && !(COMET_DEC_ABLATE & 8)) ? lds128(row + ((j ^ sw) << 4))
@@ -1124,11 +1125,13 @@ comet_status_t launch_gemm(Plan& p, const void* act_packed, const float* act_sca
     }
   }
   // packed weights as [N/16 row tiles][nb K-blocks][16 rows][64 B] (dims innermost first), 64B
-  // swizzle; prefill: one K-block of the CTA's rows per box, decode: two K-blocks of 128 rows
+  // swizzle; prefill: one K-block of the CTA's rows per box, decode: a stage's KS K-blocks of 128
+  // rows (KS = 4 for tiles of <= 32 tokens, else 2)
   {
     const uint64_t wd[4] = {64, (uint64_t)kWTileRows, (uint64_t)p.nb, (uint64_t)(p.N / kWTileRows)};
     const uint64_t ws_[3] = {64, 64 * kWTileRows, (uint64_t)p.nb * 64 * kWTileRows};
-    const uint32_t wb[4] = {64, (uint32_t)kWTileRows, normal ? 1u : 2u, (uint32_t)(cta_rows_w / kWTileRows)};
+    const uint32_t wb[4] = {64, (uint32_t)kWTileRows, normal ? 1u : (tile_m <= 32 ? 4u : 2u),
+                            (uint32_t)(cta_rows_w / kWTileRows)};
     if (!make_map(&prm.map_w, CU_TENSOR_MAP_DATA_TYPE_UINT8, 4, w_packed, wd, ws_, wb, CU_TENSOR_MAP_SWIZZLE_64B))
       return fail(COMET_ERR_CUDA, "cuTensorMapEncodeTiled failed for the packed weights");
   }
