@@ -113,3 +113,27 @@ def test_linear_rejects_other_plans(M):
     y = cb.w4ax_linear(plan, x, wp, sw, out_dtype=torch.float32)
     yref, _, _, _ = oracle.w4ax(p.x, p.tags, p.w, p.s_w)
     _close(y, yref, torch.float32)
+
+
+@pytest.mark.parametrize("orientation", [1, 4])
+@pytest.mark.parametrize("bf16", [False, True])
+def test_linear_strided_input_exact(orientation, bf16):
+    """x with a row stride ldx > K (a view into a wider activation buffer) on both fused paths,
+    and the warp-level path's auto plan through cb.w4ax_linear (no kernel-1 launch)."""
+    M, K, N = 5, 4096, 8192
+    p = synth.make_exact_problem(M, K, N, frac=0.25, seed=41 + orientation, bf16=bf16,
+                                 special_rows={1: "alternating"})
+    wp = cb.pack_weight(torch.from_numpy(p.w).to(DEV))
+    sw = torch.from_numpy(p.s_w).to(DEV)
+    wide = torch.zeros((M, K + 384), dtype=torch.bfloat16 if bf16 else torch.float16, device=DEV)
+    wide[:, 128:128 + K] = _x_dev(p.x, bf16)
+    x = wide[:, 128:128 + K]                      # ldx = K + 384, 256-byte offset
+    assert x.stride(0) == K + 384
+    plan = cb.Plan(M, N, K, p.tags, orientation=orientation)
+    y = cb.w4ax_linear_fused(plan, x, wp, sw, out_dtype=torch.float32)
+    y2 = cb.w4ax_linear(plan, x, wp, sw, out_dtype=torch.float32)
+    torch.cuda.synchronize()
+    yref, _, _, _ = oracle.w4ax_rows(p.x, p.tags, p.w, p.s_w, np.arange(M), bf16_bits=bf16)
+    r32 = yref.astype(np.float32)
+    assert np.array_equal(y.cpu().numpy(), r32)
+    assert np.array_equal(y2.cpu().numpy(), r32)
