@@ -270,3 +270,14 @@ def test_gemv_plan_split(M, N, K, sms):
 def test_gemv_plan_rejects_large_m():
     with pytest.raises(cb.CometError):
         cb.Plan(9, 1024, 1024, np.zeros(8, np.uint8), num_sms=148, device_plan=False, orientation=4)
+
+
+@pytest.mark.parametrize("M,N,K,want", [
+    (1, 28672, 8192, 4), (8, 8192, 28672, 4), (4, 10240, 8192, 4),   # >= 32 MiB packed: warp-level decode
+    (9, 28672, 8192, 1), (32, 28672, 8192, 1),                        # M > 8: TMEM decode kernel
+    (1, 4096, 4096, 1), (8, 11008, 4096, 1),                          # < 32 MiB (LLaMA-2-7B): TMEM decode kernel
+    (128, 4096, 4096, 2), (256, 4096, 4096, 3), (4096, 28672, 8192, 3)])
+def test_auto_orientation(M, N, K, want):
+    """The auto plan's kernel choice (include/comet.h, comet_sched_config.orientation = 0)."""
+    p = cb.Plan(M, N, K, np.zeros(K // 128, np.uint8), num_sms=148, device_plan=False)
+    assert p.info()["orientation"] == want
