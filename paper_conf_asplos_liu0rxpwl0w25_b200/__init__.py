@@ -385,10 +385,11 @@ def w4ax_linear(plan: Plan, x, w_packed, w_scales, *, perm=None, out=None, out_d
     channel permutation when perm is given; w_packed then packed with the same perm) +
     w4ax_gemm."""
     info = plan.info()
-    if perm is None and info["orientation"] == 4:
+    aligned = x.data_ptr() % 16 == 0 and (x.stride(0) * x.element_size()) % 16 == 0
+    if perm is None and info["orientation"] == 4 and aligned:
         # the warp-level decode kernel quantises its own K range: no kernel-1 launch (DESIGN §7.11)
         return w4ax_linear_fused(plan, x, w_packed, w_scales, out=out, out_dtype=out_dtype, stream=stream)
-    if (perm is None and info["orientation"] == 1 and info["tile_n"] == 16 and plan.M <= 4
+    if (perm is None and aligned and info["orientation"] == 1 and info["tile_n"] == 16 and plan.M <= 4
             and info["n_tiles"] * -(-plan.K // 512) <= 12 * info["num_ctas"]):
         # the fused launch wins while the CTAs' quantiser warps keep up with the weight stream:
         # small layers (<= 12 pipeline stages per CTA; LLaMA-3-70B qkv at M <= 4: 18.5 ->
