@@ -10,9 +10,9 @@
 // become the MMA N dimension and decode-sized M still fills an instruction.
 //
 // At decode sizes the kernel is a weight stream: the packed weights (N*K/2 bytes) dominate the
-// traffic.  A pipeline stage therefore carries TWO K-blocks: a 128-row x 128-byte box of packed
-// weights (16 KB; 128-byte rows stream from HBM at ~4.6 TB/s where 64-byte rows reach ~3.8,
-// profiles/r01/probe_stream.txt), the two K-blocks' activation codes and their scales.
+// traffic.  A pipeline stage therefore carries several K-blocks (KS): one 4D TMA box of the 128
+// rows' KS K-blocks of packed weights (the row-tiled layout makes each 16-row tile's KS K-blocks
+// one contiguous KS-KB run, include/comet.h), the K-blocks' activation codes and their scales.
 //
 // Roles (512 threads, 16 warps):
 //   warp 0       TMA producer of the weight ring (lane 0).
@@ -105,8 +105,8 @@ constexpr int kPromoWarp0 = 12;
 
 // One pipeline stage = KS consecutive K-blocks of one tile (KS = 4 for NT <= 32, else 2), in
 // two rings with their own barriers so the big weight slot is recycled as soon as it is read:
-//   W ring  KS/2 boxes of 128 weight rows x 128 B (two K-blocks of packed nibbles per row),
-//           SW128; released by the 8 widen warps right after their shared-memory loads.
+//   W ring  one box [8 row tiles][KS K-blocks][16 rows][64 B] of packed nibbles (64B swizzle);
+//           released by the 8 widen warps right after their shared-memory loads.
 //   X ring  one 3D box [KS K-blocks][NT tokens][128 B] of activation codes (SW128, the UMMA B
 //           operand) + one 2D box [KS][NT] of per-token scales; released by the MMA commit and
 //           the 4 promotion warps (which read the scales).
