@@ -190,6 +190,8 @@ def test_gemv_exact_full_size(name, M, K, N, frac):
     (5, 1024, 8192, 1.0, 2),       # all INT8 blocks; 4 CTAs: ranges of 16 groups (many segments)
     (8, 2048, 1024, 0.0, 148),     # more CTAs than units: empty ranges
     (2, 4096, 2048, 0.5, 7),       # ranges cutting groups at odd K-blocks
+    (1, 128, 128, 0.0, 148),       # one unit: one CTA
+    (7, 256, 128, 1.0, 148),       # one K-block, two groups, all INT8
 ])
 def test_gemv_schedules_exact(M, K, N, frac, num_sms):
     info = run_exact(M, K, N, frac, seed=M * 7 + num_sms, orientation=4, num_sms=num_sms)
