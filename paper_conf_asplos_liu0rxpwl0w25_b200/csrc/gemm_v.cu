@@ -1,5 +1,6 @@
-// gemm_v.cu -- the decode-regime W4Ax GEMM (plan orientation 4, M <= 8): weights streamed with
-// plain 128-bit loads, the product on the warp-level tensor-core path (mma.sync m16n8k32).
+// gemm_v.cu -- the decode-regime W4Ax GEMM (plan orientation 4, M <= 8): weights streamed by
+// cp.async into per-warp shared-memory rings, the product on the warp-level tensor-core path
+// (mma.sync m16n8k32), partials of shared row groups summed by a dependent reduction launch.
 //
 //   Y[m, n] = s_w[n] * sum_b s_a[m,b] * acc_b[m,n],  acc_b = sum_{k in b} w[n,k] q[m,k]
 //
@@ -8,17 +9,20 @@
 // M x K codes): HBM-bound, with ~1 MAC per weight byte per token.  The tcgen05 decode kernel
 // (gemm.cu, orientation 1) stages weights through TMA rings, widens them into TMEM and pays a
 // barrier protocol per stage; its skeleton alone streams below the copy rate.
-// Here every warp is its own weight pipeline: it keeps U K-blocks of its 16 weight rows in
-// flight in registers (2 x 16 B per lane per K-block), widens a K-block in registers (3
-// instructions per 8 nibbles) and feeds 4 mma.sync per K-block -- no barriers in the loop.
+// Here every warp is its own weight pipeline: each lane cp.asyncs 16 B of row g and of row
+// g + 8 per K-block (its warp's 16 rows = one 1 KB tile of the row-tiled layout, contiguous
+// along K) into an S-deep ring it alone reads back -- no barrier in the loop -- widens in
+// registers (3 instructions per 8 nibbles) and feeds 4 mma.sync per K-block.
 //
 // Work split (CTA-level stream-K): units = (group of 128 weight rows, K-block),
 // group-major, cut into one contiguous range per CTA, equal to within one unit; warp w of the
 // CTA takes rows 16 w .. 16 w + 15 of the group in every unit, so the CTA's 8 warps walk the
 // same K-blocks and share one shared-memory copy of the activation codes of its range (staged
-// once in the prologue, converted to s8).  Each CTA stores one FP32 partial per group it
+// once in the prologue as s8: from kernel 1's output, or -- FQ, comet_w4ax_linear -- quantised
+// from x right there with kernel 1's arithmetic).  Each CTA stores one FP32 partial per group it
 // touches ([128 rows][8 tokens] workspace slots); k_gemv_reduce -- a programmatic dependent
-// launch -- sums each group's partials in CTA order (deterministic), applies s_w and converts.
+// launch, one CTA per group -- sums each group's partials in CTA order (deterministic), applies
+// s_w and converts.
 //
 // Product per K-block (128 channels), one path for both block kinds: A = the weight nibbles
 // u = w + 8 zero-extended to u8, B = the activation codes as s8 (INT8 blocks as stored, INT4
