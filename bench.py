@@ -395,10 +395,19 @@ def config2_sweep(cb, torch, dev, peaks, timer, iters=20):
                     cb.w4ax_gemm(plan, act, sc, wps[i], sw, out=y)
             us = us_rotating(torch, [lambda i=i: step(i) for i in range(ncopy)])
             row["step"] = dict(roofline_point(ops, nbytes, us, peaks), us=round(us, 2))
+            if M <= 8:
+                # the same three layers through the library's layer call (cb.w4ax_linear:
+                # comet_w4ax_linear, kernel 1 fused into the decode GEMM where the plan allows)
+                def lstep(i):
+                    for (name, K, N, tags, wps, sw, x, plan, act, sc, y) in L:
+                        cb.w4ax_linear(plan, x, wps[i], sw, out=y)
+                us_l = us_rotating(torch, [lambda i=i: lstep(i) for i in range(ncopy)])
+                row["linear_step"] = dict(roofline_point(ops, nbytes, us_l, peaks), us=round(us_l, 2))
             out[f"{'bf16' if bf16 else 'f16'}_M{M}"] = row
             del L
     return {"workload": "llama2_7b q/k/v/o 4096->4096, gate/up 4096->11008, down 11008->4096; 5 % INT8 blocks",
             "timing": "mean per launch (per step) over back-to-back launches cycling through > 300 MB of weight copies per layer",
+            "step": "step = comet_quantize_act + comet_w4ax_gemm per layer; linear_step (M <= 8) = cb.w4ax_linear per layer (kernel 1 fused where the plan allows)",
             "output": "f16",
             "roofline": "frac = max(ops / (2 x bf16 peak), SURVEY bytes / HBM peak) / measured", "points": out}
 

@@ -206,7 +206,7 @@ typedef struct {
   int device_plan;     /* 1 (default) = upload the work list to the device at create time;
                           0 = host-only plan (comet_plan_describe only; CPU-safe) */
   int orientation;     /* 0 = auto (3 when M >= 256, 2 when M >= 128, 4 when M <= 8 and the
-                              packed weights take >= 32 MiB, else 1);
+                              packed weights take >= 32 MiB, or >= 8 MiB with N >= K, else 1);
                           1 = weights on the MMA M side: tile = 128 weights x tile_n tokens
                               (decode-sized M; weights widened into TMEM);
                           2 = tokens on the MMA M side: tile = 128 tokens x tile_w weights

@@ -76,12 +76,14 @@ comet_status_t build_plan(Plan& p, const comet_sched_config& cfg) {
   p.nb = p.K / kBlockK;
   p.Mp = round_up(p.M, COMET_SCALE_PAD);
   p.orientation = cfg.orientation > 0 ? cfg.orientation : (p.M >= 256 ? 3 : (p.M >= 128 ? 2 : 1));
-  // decode on the warp-level path (gemm_v.cu) where it measured faster than the TMEM kernel:
-  // M <= 8 with >= 32 MiB of packed weights (tools/gemv_ab.py, LLaMA-3-70B: gate/up M = 1 / 4 / 8
-  // 22.x / 24.0 / 26.6 vs 28.0 / 27.3 / 27.8 us, down 23.5 / 24.6 / 27.6 vs 26.6 / 26.7 / 27.3,
-  // qkv 12.2 / 12.5 / 12.7 vs 14.2; the 8-22 MB LLaMA-2-7B layers are mixed and stay on 1)
+  // decode on the warp-level path (gemm_v.cu) where it measured faster than the TMEM kernel
+  // (tools/gemv_ab.py): M <= 8 with >= 32 MiB of packed weights (LLaMA-3-70B: gate/up M = 1 / 4 / 8
+  // 23.3 / 24.0 / 26.7 vs 28.0 / 27.3 / 27.8 us, down 23.6 / 24.6 / 27.6 vs 26.6 / 26.7 / 27.3,
+  // qkv 11.7 / 12.1 / 11.9 vs 14.2), or >= 8 MiB when N >= K (LLaMA-2-7B q/k/v/o 7.2 vs 7.5 us,
+  // gate/up 9.4 vs 10.5; its down, K = 11008 > N, 10.5-11.0 vs 10.4-10.5, stays on 1)
   bool auto_o4 = false;
-  if (cfg.orientation <= 0 && p.M <= 8 && p.N * p.K / 2 >= (32ll << 20)) {
+  if (cfg.orientation <= 0 && p.M <= 8 &&
+      (p.N * p.K / 2 >= (32ll << 20) || (p.N * p.K / 2 >= (8ll << 20) && p.N >= p.K))) {
     int nbr = 0, s = 0;
     auto_o4 = gemv::gemv_pick(p.M, (p.N / 128) * (p.K / kBlockK), (int)(p.K / kBlockK), cfg.num_sms, &nbr, &s) > 0;
     if (auto_o4) p.orientation = 4;

@@ -275,7 +275,8 @@ def test_gemv_plan_rejects_large_m():
 @pytest.mark.parametrize("M,N,K,want", [
     (1, 28672, 8192, 4), (8, 8192, 28672, 4), (4, 10240, 8192, 4),   # >= 32 MiB packed: warp-level decode
     (9, 28672, 8192, 1), (32, 28672, 8192, 1),                        # M > 8: TMEM decode kernel
-    (1, 4096, 4096, 1), (8, 11008, 4096, 1),                          # < 32 MiB (LLaMA-2-7B): TMEM decode kernel
+    (1, 4096, 4096, 4), (8, 11008, 4096, 4),                          # >= 8 MiB with N >= K (LLaMA-2-7B q/k/v/o, gate/up)
+    (1, 4096, 11008, 1), (4, 1024, 4096, 1),                          # LLaMA-2-7B down (K > N); < 8 MiB
     (128, 4096, 4096, 2), (256, 4096, 4096, 3), (4096, 28672, 8192, 3)])
 def test_auto_orientation(M, N, K, want):
     """The auto plan's kernel choice (include/comet.h, comet_sched_config.orientation = 0)."""

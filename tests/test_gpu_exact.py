@@ -124,7 +124,7 @@ def test_production_exact_full_size(name, M, K, N, frac):
     info = run_exact(M, K, N, frac, seed=sum(map(ord, name)))
     # the launch configuration bench.py times: pair kernel for prefill, a decode kernel below 128
     # (the warp-level one for M <= 8 on layers of >= 32 MiB of packed weights)
-    o4 = M <= 8 and N * K // 2 >= (32 << 20)
+    o4 = M <= 8 and (N * K // 2 >= (32 << 20) or (N * K // 2 >= (8 << 20) and N >= K))
     assert info["orientation"] == (3 if M >= 256 else (2 if M >= 128 else (4 if o4 else 1)))
 
 
