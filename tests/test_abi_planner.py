@@ -265,6 +265,8 @@ def test_gemv_plan_split(M, N, K, sms):
     assert p.workspace_bytes == -(-(C * segs * 128 * 8 * 4) // 256) * 256
     split = sum(1 for g in range(G) if owner[g * nb] != owner[g * nb + nb - 1])
     assert info["n_split_tiles"] == split
+    # the reduction kernel reads at most 64 partial slots per group (kMaxRed in gemm_v.cu)
+    assert max(owner[g * nb + nb - 1] - owner[g * nb] + 1 for g in range(G)) <= 64
 
 
 def test_gemv_plan_rejects_large_m():
